@@ -1,0 +1,222 @@
+"""Seeded synthetic workload generators shared by the oracle side and the CUDA side.
+
+This module holds NO arithmetic of the method (no key canonicalisation, no tree
+logic, no lookup/update semantics): it only draws numbers.  Both the oracle
+(``oracle/``) and the product binding consume its arrays; neither imports the
+other.  Every draw is a pure function of (stream seed, counter) through the
+counter-based splitmix64 mixer, so any element of any stream can be recomputed
+on its own (the full-size parity tests sample single elements this way).
+
+Workload recipes follow SURVEY.md §8(d) ("Synthetic inputs") and are restated in
+DESIGN.md §"Input recipe".  Key shapes mirror the paper's workloads: random
+integer keys ("synthetic random test data"), dense sequential
+keys, and variable-length byte strings up to the compile-time maximum of 32 B
+(P:110).
+"""
+from __future__ import annotations
+
+import dataclasses
+import numpy as np
+
+MASK64 = (1 << 64) - 1
+GOLDEN = np.uint64(0x9E3779B97F4A7C15)
+_M1 = np.uint64(0xBF58476D1CE4E5B9)
+_M2 = np.uint64(0x94D049BB133111EB)
+#: Reserved "absent" value (SURVEY §8(b) CUART_MISS); generated values avoid it.
+RESERVED_VALUE = np.uint64(0xFFFFFFFFFFFFFFFF)
+
+# Stream seeds per config c: keys 1000+c, values 1500+c,
+# queries 2000+c, updates 3000+c, update values 3500+c.
+SEED_KEYS, SEED_VALUES, SEED_QUERIES, SEED_UPDATES, SEED_UVALUES = 1000, 1500, 2000, 3000, 3500
+
+
+def splitmix64(seed: int, counter) -> np.ndarray:
+    """Counter-based splitmix64: mix(seed + (counter+1)*golden).
+
+    For a fixed seed this is a bijection of the counter on [0, 2^64), so draws at
+    distinct counters are distinct — used to build key sets with guaranteed
+    distinct members and guaranteed-absent miss keys without any membership test.
+    """
+    c = np.asarray(counter, dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        z = np.uint64(seed & MASK64) + (c + np.uint64(1)) * GOLDEN
+        z = (z ^ (z >> np.uint64(30))) * _M1
+        z = (z ^ (z >> np.uint64(27))) * _M2
+        z = z ^ (z >> np.uint64(31))
+    return z
+
+
+def splitmix64_scalar(seed: int, counter: int) -> int:
+    z = (seed + (counter + 1) * 0x9E3779B97F4A7C15) & MASK64
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & MASK64
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & MASK64
+    return z ^ (z >> 31)
+
+
+def values_for(seed: int, counter) -> np.ndarray:
+    """u64 payloads, remapped away from the reserved miss value."""
+    v = splitmix64(seed, counter)
+    v[v == RESERVED_VALUE] = np.uint64(0)
+    return v
+
+
+@dataclasses.dataclass(frozen=True)
+class Config:
+    name: str
+    kind: str              # "u64" | "u32" | "bytes"
+    n_keys: int
+    n_lookups: int
+    n_updates: int
+    hit_ratio: float       # fraction of lookups drawn from the key set
+    description: str
+
+
+# BASELINE.json "configs" (sizes read as powers of two where the text says M/B).
+CONFIGS = {
+    "c1": Config("c1", "u64", 65_536, 1 << 20, 100_000, 0.5,
+                 "65,536 random 64-bit keys, 1M point lookups (50% hit) + 100K value updates"),
+    "c2": Config("c2", "u32", 1 << 24, 1 << 28, 0, 1.0,
+                 "16M dense sequential 32-bit keys, 256M lookups (100% hit)"),
+    "c3": Config("c3", "u64", 1 << 26, 1 << 30, 1 << 26, 0.5,
+                 "64M sparse uniform-random 64-bit keys, 1B lookups at 50% hit + 64M update batch"),
+    "c4": Config("c4", "bytes", 1 << 25, 1 << 29, 0, 1.0,
+                 "32M variable-length byte-string keys (8-32 B), 512M Zipf lookups"),
+}
+
+
+def config_id(cfg: Config) -> int:
+    return int(cfg.name[1:])
+
+
+# ----------------------------------------------------------------------------- keys
+def u64_keys(c: int, n: int) -> np.ndarray:
+    """n distinct uniform-random u64 keys (bijective counter draw, no dedupe needed)."""
+    return splitmix64(SEED_KEYS + c, np.arange(n, dtype=np.uint64))
+
+
+def u64_absent_keys(c: int, n_keys: int, start: int, m: int) -> np.ndarray:
+    """m u64 keys guaranteed NOT in u64_keys(c, n_keys): counters >= n_keys of the same bijection."""
+    return splitmix64(SEED_KEYS + c, np.arange(n_keys + start, n_keys + start + m, dtype=np.uint64))
+
+
+def build_set(cfg: Config):
+    """(keys, values) for the build call, in generator order (unsorted)."""
+    c = config_id(cfg)
+    vals = values_for(SEED_VALUES + c, np.arange(cfg.n_keys, dtype=np.uint64))
+    if cfg.kind == "u64":
+        return u64_keys(c, cfg.n_keys), vals
+    if cfg.kind == "u32":
+        return np.arange(cfg.n_keys, dtype=np.uint32), vals
+    if cfg.kind == "bytes":
+        slots, lens = string_keys(c, cfg.n_keys)
+        return (slots, lens), vals[: lens.shape[0]]
+    raise ValueError(cfg.kind)
+
+
+def lookup_batch(cfg: Config, keys, start: int = 0, m: int | None = None):
+    """Lookup queries [start, start+m) of the config's stream.
+
+    u64: query j is a hit (uniform key of the set) when the top bit of draw 2j is
+    clear and hit_ratio == 0.5, otherwise a guaranteed-absent key.  u32 (c2):
+    uniform over [0, 2^24) => 100% hit.
+    """
+    c = config_id(cfg)
+    m = cfg.n_lookups - start if m is None else m
+    j = np.arange(start, start + m, dtype=np.uint64)
+    if cfg.kind == "u32":
+        return (splitmix64(SEED_QUERIES + c, j) >> np.uint64(40)).astype(np.uint32)
+    if cfg.kind == "u64":
+        n = keys.shape[0]
+        sel = splitmix64(SEED_QUERIES + c, np.uint64(2) * j)
+        pick = splitmix64(SEED_QUERIES + c, np.uint64(2) * j + np.uint64(1))
+        if cfg.hit_ratio >= 1.0:
+            hit = np.ones(m, dtype=bool)
+        else:
+            thresh = np.uint64(int(cfg.hit_ratio * 2**64) & MASK64)
+            hit = sel < thresh
+        out = splitmix64(SEED_KEYS + c, (np.uint64(n) + np.uint64(1 << 40) + j))  # absent: counters >= n
+        hk = keys[(pick % np.uint64(n)).astype(np.int64)]
+        out[hit] = hk[hit]
+        return out
+    raise ValueError(cfg.kind)
+
+
+def update_batch(cfg: Config, keys, start: int = 0, m: int | None = None):
+    """Update ops [start, start+m): 90% keys drawn with replacement from the set
+    (duplicates exercise last-writer-wins), 10% guaranteed-absent keys."""
+    c = config_id(cfg)
+    m = cfg.n_updates - start if m is None else m
+    j = np.arange(start, start + m, dtype=np.uint64)
+    n = keys.shape[0]
+    sel = splitmix64(SEED_UPDATES + c, np.uint64(2) * j)
+    pick = splitmix64(SEED_UPDATES + c, np.uint64(2) * j + np.uint64(1))
+    present = sel < np.uint64(int(0.9 * 2**64))
+    if cfg.kind == "u64":
+        out = splitmix64(SEED_KEYS + c, (np.uint64(n) + np.uint64(1 << 41) + j))
+    elif cfg.kind == "u32":
+        out = (np.uint64(n) + j).astype(np.uint32)  # dense set is [0, n): n+j is absent
+        keys = keys.astype(np.uint32)
+    else:
+        raise ValueError(cfg.kind)
+    hk = keys[(pick % np.uint64(n)).astype(np.int64)]
+    out[present] = hk[present]
+    vals = values_for(SEED_UVALUES + c, j)
+    return out, vals
+
+
+# ----------------------------------------------------------------------------- strings
+ALPHABET = np.frombuffer(b"abcdefghijklmnopqrstuvwxyz0123456789/.:_-#", dtype=np.uint8)  # 42 symbols
+MAX_KEY = 32
+
+
+def _zipf_index(u01: np.ndarray, n: int, s: float) -> np.ndarray:
+    """Inverse-CDF Zipf(s) over ranks [0, n) from uniforms in [0,1)."""
+    w = 1.0 / np.arange(1, n + 1, dtype=np.float64) ** s
+    cdf = np.cumsum(w)
+    cdf /= cdf[-1]
+    return np.minimum(np.searchsorted(cdf, u01, side="right"), n - 1)
+
+
+def _u01(seed: int, counter) -> np.ndarray:
+    return (splitmix64(seed, counter) >> np.uint64(11)).astype(np.float64) * (1.0 / (1 << 53))
+
+
+def string_keys(c: int, n: int, max_len: int = MAX_KEY, min_len: int = 8):
+    """n distinct, prefix-free byte-string keys as (slots uint8[n,32], lens uint8[n]).
+
+    Recipe: content = level-1 segment (16 choices, Zipf 1.2) +
+    level-2 segment (256 choices, Zipf 1.0), 6 symbols each from a 42-symbol
+    alphabet, then random suffix symbols; total length L ~ U{min_len..max_len}
+    INCLUDING a 0x00 terminator, so the set is prefix-free (no content byte is 0).
+    Duplicates are rejected by drawing extra candidates and keeping the first
+    occurrence (order of first appearance is preserved).
+    """
+    seed = SEED_KEYS + c
+    seg1 = ALPHABET[(splitmix64(seed + 11, np.arange(16 * 6, dtype=np.uint64)) % np.uint64(42)).astype(np.int64)].reshape(16, 6)
+    seg2 = ALPHABET[(splitmix64(seed + 12, np.arange(256 * 6, dtype=np.uint64)) % np.uint64(42)).astype(np.int64)].reshape(256, 6)
+    out_slots, out_lens, have = [], [], 0
+    seen = set() if n <= 1 << 16 else None
+    base = 0
+    while have < n:
+        m = int((n - have) * 1.3) + 1024
+        j = np.arange(base, base + m, dtype=np.uint64)
+        base += m
+        L = (min_len + (splitmix64(seed + 1, j) % np.uint64(max_len - min_len + 1))).astype(np.int64)
+        i1 = _zipf_index(_u01(seed + 2, j), 16, 1.2)
+        i2 = _zipf_index(_u01(seed + 3, j), 256, 1.0)
+        content = np.empty((m, max_len), dtype=np.uint8)
+        content[:, 0:6] = seg1[i1]
+        content[:, 6:12] = seg2[i2]
+        for col in range(12, max_len):
+            content[:, col] = ALPHABET[(splitmix64(seed + 100 + col, j) % np.uint64(42)).astype(np.int64)]
+        pos = np.arange(max_len)[None, :]
+        slots = np.where(pos < (L - 1)[:, None], content, 0).astype(np.uint8)  # terminator + zero pad
+        out_slots.append(slots)
+        out_lens.append(L.astype(np.uint8))
+        allslots = np.concatenate(out_slots)
+        alllens = np.concatenate(out_lens)
+        _, first = np.unique(allslots.view(np.dtype((np.void, max_len))).ravel(), return_index=True)
+        first.sort()
+        out_slots, out_lens = [allslots[first]], [alllens[first]]
+        have = first.shape[0]
+    return out_slots[0][:n].copy(), out_lens[0][:n].copy()
