@@ -1,0 +1,364 @@
+#!/usr/bin/env python
+"""Benchmark of the CuART hot path on B200 (device-timed), one JSON line on rank 0.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--impl cuart|reference]
+
+A "step" = one pass of the whole hot path over one batch of the workload:
+cuart_lookup over the lookup batch, then cuart_update over the update batch
+(the build rows a2-a3 are host-side setup, untimed).
+Default workload: BASELINE config 3 (2^26 random u64 keys, 2^30 lookups at 50%
+hit + a 2^26-op update batch) — the config that carries both halves of the
+metric ("Mlookups/s and Mupdates/s") at 1 and 8 GPUs and fits one B200.
+
+Inputs are resident in HBM before the timed region and are far larger than the
+126 MB L2 (8 GiB of queries), so no explicit L2 flush is needed between steps.
+
+N > 1 (torchrun, one process per GPU, NCCL): replica mode — every rank holds the
+full index, looks up its own 2^30-query shard of the global stream (weak scaling)
+and applies the all-gathered update batches of all ranks in rank-major global
+order, so the replicas stay identical.
+
+--impl reference times the CPU oracle (oracle/, single-threaded pointer ART) on
+a bounded sample of the same workload: the reference arm for this tier.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+METRIC = "Mlookups/s and Mupdates/s (device-timed)"
+
+
+def _args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=10)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--config", default="c3", choices=["c1", "c2", "c3"])
+    p.add_argument("--impl", default="cuart", choices=["cuart", "reference"])
+    p.add_argument("--lut", type=int, default=3)
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--e2e-steps", type=int, default=2)
+    return p.parse_args()
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi sampling of SM clocks + throttle reasons during the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, dev_index: int):
+        self.dev = dev_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                          "-i", str(self.dev), "-lms", "100"], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ oracle timing (CPU)
+def oracle_timing(cfg, keys, vals, n_lookup_sample, n_update_sample, reps=1):
+    """The oracle as it stands, single-threaded on a host core: (Mops/s, detail)."""
+    from oracle import ArtOracle
+    t0 = time.perf_counter()
+    o = ArtOracle(keys, vals)
+    build_s = time.perf_counter() - t0
+    q = W.lookup_batch(cfg, keys, 0, n_lookup_sample)
+    uk, uv = W.update_batch(cfg, keys, 0, n_update_sample) if cfg.n_updates else (None, None)
+    times = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        o.lookup(q)
+        if uk is not None:
+            o.update(uk, uv)
+        times.append(time.perf_counter() - t0)
+    o.close()
+    dt = min(times)
+    ops = n_lookup_sample + (n_update_sample if uk is not None else 0)
+    return ops / dt / 1e6, {"build_s": round(build_s, 2), "sample_lookups": n_lookup_sample,
+                            "sample_updates": n_update_sample if uk is not None else 0, "seconds": round(dt, 3)}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    cfg = W.CONFIGS[args.config]
+    keys, vals = W.build_set(cfg)
+    from oracle import ArtOracle
+    t0 = time.perf_counter()
+    o = ArtOracle(np.sort(keys) if keys.dtype != object else keys, vals[np.argsort(keys)])
+    build_s = time.perf_counter() - t0
+    # bounded sample per step, same lookup:update mix as the workload
+    nl = min(cfg.n_lookups, 1 << 20)
+    nu = min(cfg.n_updates, max(1, nl * cfg.n_updates // cfg.n_lookups)) if cfg.n_updates else 0
+    times = []
+    for s in range(args.warmup + args.steps):
+        q = W.lookup_batch(cfg, keys, s * nl, nl)
+        uk, uv = W.update_batch(cfg, keys, s * nu, nu) if nu else (None, None)
+        t0 = time.perf_counter()
+        o.lookup(q)
+        if nu:
+            o.update(uk, uv)
+        dt = time.perf_counter() - t0
+        if s >= args.warmup:
+            times.append(dt)
+    ms = 1e3 * float(np.mean(times))
+    val = (nl + nu) / (ms * 1e-3) / 1e6
+    line = {"impl": "reference", "metric": METRIC, "value": round(val, 3), "unit": "Mops/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic (seeded splitmix64, SURVEY §8(d) recipe)",
+            "config": {"workload": f"{args.config}: {cfg.description}", "sample_per_step":
+                       {"lookups": nl, "updates": nu}},
+            "cpu_baseline": {"value": round(val, 3), "unit": "Mops/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{nl} lookups + {nu} updates per step of the {args.config} stream, "
+                                       f"pointer-ART oracle built over all {keys.shape[0]} keys "
+                                       f"({build_s:.1f} s, untimed)"},
+            "e2e": {"value": round(val, 3), "unit": "Mops/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ main (GPU)
+def main():
+    args = _args()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_koppehelggp21_b200 as C
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    cfg = W.CONFIGS[args.config]
+    t0 = time.perf_counter()
+    if cfg.kind == "u64":
+        keys_d = W.u64_keys_torch(W.config_id(cfg), cfg.n_keys, dev)
+        keys = keys_d.cpu().numpy().view(np.uint64)
+    else:
+        keys = np.arange(cfg.n_keys, dtype=np.uint32)
+        keys_d = torch.from_numpy(keys.view(np.int32)).to(dev)
+    vals = W.values_for(W.SEED_VALUES + W.config_id(cfg), np.arange(cfg.n_keys, dtype=np.uint64))
+    layout = C.Layout(keys, vals, lut_bytes=args.lut)
+    ix = C.Index.from_layout(layout, device=local)
+    build_s = time.perf_counter() - t0
+    stats = ix.stats()
+
+    # resident inputs: this rank's shard of the global lookup stream, its update batch
+    nl = cfg.n_lookups
+    q = W.lookup_batch_torch(cfg, keys_d, rank * nl, nl, device=dev)
+    out = torch.empty(nl, dtype=torch.int64, device=dev)
+    nu = cfg.n_updates
+    if nu:
+        uk, uv = W.update_batch_torch(cfg, keys_d, rank * nu, nu)
+        if world > 1:   # replica mode: every replica applies all ranks' updates in global order
+            gk = torch.empty(world * nu, dtype=torch.int64, device=dev)
+            gv = torch.empty_like(gk)
+            dist.all_gather_into_tensor(gk, uk)
+            dist.all_gather_into_tensor(gv, uv)
+            uk, uv = gk, gv
+    torch.cuda.synchronize()
+
+    # algorithmic bytes of the dominant kernel (k_lookup): exact sector count of the
+    # lookup path for a 2^20-query sample (host walker over the same layout) + I/O
+    samp = q[: 1 << 20].cpu().numpy()
+    samp = samp.view(np.uint64) if cfg.kind == "u64" else samp.view(np.uint32)
+    sec = layout.sectors(samp).astype(np.float64)
+    io_bytes = (8 if cfg.kind == "u64" else 4) + 8
+    bytes_per_lookup = 32.0 * sec.mean() + io_bytes
+    del samp
+
+    stream = torch.cuda.current_stream()
+
+    def step(ev=None):
+        if ev is not None:
+            ev[0].record(stream)
+        ix.lookup(q, out, stream)
+        if ev is not None:
+            ev[1].record(stream)
+        if nu:
+            ix.update(uk, uv, stream)
+        if ev is not None:
+            ev[2].record(stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    launches0 = C.cuart_launch_count()
+    torch.cuda.synchronize()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(stream)
+    for s in range(args.steps):
+        step(evs[s])
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    launches = C.cuart_launch_count() - launches0
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    total_ms = t_start.elapsed_time(t_end)
+    look_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in evs]))
+    upd_ms = float(np.mean([e[1].elapsed_time(e[2]) for e in evs])) if nu else 0.0
+    tt = torch.tensor([total_ms, look_ms, upd_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    total_ms, look_ms, upd_ms = tt.tolist()
+    ms_step = total_ms / args.steps
+    n_upd_applied = uk.shape[0] if nu else 0
+    # whole job: every rank's lookups + the update ops (each op counted once)
+    ops_per_step = world * nl + (world * nu if nu else 0)
+    value = ops_per_step / (ms_step * 1e-3) / 1e6
+
+    # roofline of the dominant kernel (k_lookup), HBM-bound random gathers
+    peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
+    if os.path.exists(peaks_path):
+        with open(peaks_path) as f:
+            peak = float(json.load(f)["hbm_gbs"])
+        peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)"
+    achieved = nl * bytes_per_lookup / (look_ms * 1e-3) / 1e9
+    hit = float((out[: 1 << 24] != -1).float().mean().item())
+
+    # end-to-end through the public API with HOST buffers (pinned), copies inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        qh = torch.empty(nl, dtype=q.dtype, pin_memory=True)
+        qh.copy_(q)
+        oh = torch.empty(nl, dtype=torch.int64, pin_memory=True)
+        ukh = uvh = None
+        if nu:
+            ukh = torch.empty(uk.shape[0], dtype=torch.int64, pin_memory=True)
+            uvh = torch.empty_like(ukh)
+            ukh.copy_(uk)
+            uvh.copy_(uv)
+        qn = qh.numpy()
+        on = oh.numpy()
+        C.cuart_lookup_host(ix.h, qn, on)    # warm-up
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ts = []
+        for _ in range(args.e2e_steps):
+            t0 = time.perf_counter()
+            C.cuart_lookup_host(ix.h, qn, on)
+            if nu:
+                C.cuart_update_host(ix.h, ukh.numpy(), uvh.numpy())
+            ts.append(time.perf_counter() - t0)
+        et = torch.tensor([float(np.mean(ts))], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        e_s = et.item()
+        ks = q.element_size()
+        e2e = {"value": round(ops_per_step / e_s / 1e6, 3), "unit": "Mops/s",
+               "h2d_bytes_per_step": int(nl * ks + (n_upd_applied * 16 if nu else 0)),
+               "d2h_bytes_per_step": int(nl * 8), "ms_per_step": round(e_s * 1e3, 3),
+               "api": "cuart_lookup_host + cuart_update_host (pinned host buffers, chunked H2D/kernel/D2H)"}
+        del qh, oh, ukh, uvh
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        nls = min(nl, 1 << 22)
+        nus = min(nu, nls * nu // nl) if nu else 0
+        v, det = oracle_timing(cfg, keys, vals, nls, nus)
+        cpu = {"value": round(v, 3), "unit": "Mops/s", "cores": 1, "kind": "oracle",
+               "sample": f"{nls} lookups + {nus} updates of the {args.config} stream (same mix), "
+                         f"single-threaded pointer ART built over all {cfg.n_keys} keys "
+                         f"(build {det['build_s']} s untimed, timed {det['seconds']} s)"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 3), "unit": "Mops/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 4),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic (seeded splitmix64 keys/queries/updates, SURVEY §8(d) recipe)",
+            "config": {"workload": f"{args.config}: {cfg.description}", "keys": cfg.n_keys,
+                       "lookups_per_rank": nl, "updates_per_rank": nu, "key_kind": cfg.kind,
+                       "lut_bytes": args.lut, "mode": "single" if world == 1 else "replica",
+                       "l2": "inputs (8 GiB queries) larger than L2; no flush",
+                       "measured_hit_ratio": round(hit, 4), "build_s": round(build_s, 2)},
+            "lookup": {"mlookups_per_s": round(world * nl / (look_ms * 1e-3) / 1e6, 3), "ms": round(look_ms, 4)},
+            "update": {"mupdates_per_s": round(world * nu / (upd_ms * 1e-3) / 1e6, 3) if nu else None,
+                       "ms": round(upd_ms, 4), "ops_applied_per_rank": n_upd_applied},
+            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(achieved / peak, 4), "traffic": None,
+                         "kernel": "k_lookup<KeyU64>" if cfg.kind == "u64" else "k_lookup<KeyU32>",
+                         "bytes_per_lookup": round(bytes_per_lookup, 3),
+                         "sectors_per_lookup": round(float(sec.mean()), 4), "peak_source": peak_src},
+            "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": int(launches), "clocks": clk,
+            "index": {k: stats[k] for k in ("n4", "n16", "n48", "n256", "leaf8", "arena_bytes", "max_depth")},
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    ix.close()
+
+
+if __name__ == "__main__":
+    main()

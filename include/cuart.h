@@ -1,0 +1,174 @@
+/*
+ * cuart.h — C ABI of the B200-native CuART hot path.
+ *
+ * CuART (Koppehel, Pionteck, Groth, Groppe; ICPP'21).  Citations "P:<n>" are
+ * line numbers of the paper text with the section they fall in.
+ *
+ *  - cuart_build   : populate + map a host ART into the per-node-type device
+ *                    buffers (§4.1 "Populating the ART index /
+ *                    Mapping the CPU ART into the buffer structure"; layout
+ *                    P:108-110 §3.2.1; root lookup table P:112/§3.2.2).
+ *  - cuart_lookup  : batched exact-match lookups on the GPU (Fig. 3, P:98;
+ *                    P:108 §3.2.1).
+ *  - cuart_update  : batched in-place value replacement, two stages with
+ *                    highest-op-index-wins conflict resolution (P:141-143
+ *                    §3.4, Fig. 6).
+ *  - cuart_destroy : free everything the library owns.
+ *
+ * Conventions (all calls):
+ *  - Every call returns cuart_status; no C++ exception crosses the ABI.
+ *  - Keys: CUART_KEY_U64 = uint64_t[n] and CUART_KEY_U32 = uint32_t[n] in the
+ *    machine's native byte order; the library orders them numerically (they
+ *    are indexed as big-endian byte strings, the binary-comparable form of
+ *    ART [17]).  CUART_KEY_BYTES = n slots of CUART_MAX_KEY (32) bytes plus
+ *    lengths[n] in [1, 32]; bytes past the length are ignored.  The maximum key
+ *    length is the paper's compile-time constant (§3.2.1).  A byte-string
+ *    key set must be prefix-free (no stored key is a proper prefix of another).
+ *  - Values are uint64_t.  CUART_MISS (UINT64_MAX) is the lookup result for
+ *    an absent key and is therefore reserved: it may not be stored.
+ *  - Ownership: the caller owns every input/output buffer; the library owns
+ *    the index arena and its scratch and frees them in cuart_destroy.
+ *  - Pointers: cuart_build takes HOST pointers and is synchronous.
+ *    cuart_lookup / cuart_update take DEVICE pointers (on the index's device),
+ *    only enqueue work on `stream` (a cudaStream_t passed as void*, NULL =
+ *    legacy default stream) and never synchronise the host.
+ *    cuart_lookup_host / cuart_update_host take HOST pointers (pinned for full
+ *    speed) and run a chunked H2D -> kernel -> D2H pipeline; they return when
+ *    the results are in host memory.
+ *  - Ordering: lookups may run concurrently on several streams; updates on
+ *    one index must not overlap each other (the conflict scratch is per index).
+ *    A lookup concurrent with an update sees the old or the new 8-byte value
+ *    ("atomically replace values", §1.1) — outside parity guarantees.
+ *  - n == 0 is a no-op returning CUART_OK.
+ */
+#ifndef CUART_H
+#define CUART_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CUART_MAX_KEY 32
+#define CUART_MISS UINT64_MAX
+
+typedef enum {
+    CUART_OK = 0,
+    CUART_ERR_INVALID_ARGUMENT = 1, /* NULL with n > 0, bad kind, bad option    */
+    CUART_ERR_KEY_LENGTH = 2,       /* key length 0 or > 32                      */
+    CUART_ERR_NOT_PREFIX_FREE = 3,  /* build: a key is a proper prefix of another */
+    CUART_ERR_RESERVED_VALUE = 4,   /* build: value == CUART_MISS; update: sticky */
+    CUART_ERR_OOM = 5,              /* host or device allocation failed          */
+    CUART_ERR_CUDA = 6,             /* a CUDA runtime call / launch failed        */
+    CUART_ERR_NCCL = 7,             /* reserved for the multi-GPU layer          */
+    CUART_ERR_NO_DEVICE = 8,        /* no CUDA device / wrong device             */
+    CUART_ERR_TOO_LARGE = 9,        /* a node buffer exceeds the 52-bit link index */
+    CUART_ERR_INTERNAL = 10
+} cuart_status;
+
+typedef enum { CUART_KEY_U32 = 1, CUART_KEY_U64 = 2, CUART_KEY_BYTES = 3 } cuart_key_kind;
+
+typedef struct {
+    cuart_key_kind kind;
+    const void* data;        /* U32: uint32_t[n]; U64: uint64_t[n]; BYTES: uint8_t[n][32] */
+    const uint8_t* lengths;  /* BYTES only: lengths[n] in [1,32]; NULL otherwise          */
+} cuart_keys;
+
+/* Build options.  Zero-initialised = defaults.  All of them change performance
+ * only, never results. */
+typedef struct {
+    uint32_t lut_bytes;          /* 0..3: dense root lookup table over the first k key bytes
+                                    (§3.2.2, 2^(8k) links; k=3 -> 128 MiB).
+                                    CUART_LUT_AUTO (0xFFFFFFFF) = library choice.          */
+    uint32_t l2_persist;         /* 1: request a persisting L2 access-policy window over the
+                                    LUT / top levels (cudaAccessPolicyWindow).               */
+    int32_t device;              /* CUDA device ordinal; -1 = current device                */
+    uint32_t reserved;
+} cuart_build_opts;
+#define CUART_LUT_AUTO 0xFFFFFFFFu
+
+/* Per-node-type counts and bytes of an index (type codes P:108). */
+typedef struct {
+    uint64_t count[8];           /* [1]=N4 [2]=N16 [3]=N48 [4]=N256 [5]=leaf8 [6]=leaf16 [7]=leaf32 */
+    uint64_t bytes[8];
+    uint64_t n_keys;
+    uint64_t lut_entries;        /* 2^(8*lut_bytes) or 0 */
+    uint64_t lut_bytes_total;
+    uint64_t arena_bytes;        /* device bytes held by the index (arena + LUT + scratch) */
+    uint32_t lut_bytes;
+    uint32_t key_kind;
+    uint64_t root;               /* packed root link */
+    uint32_t max_depth;          /* longest root-to-leaf node chain */
+    uint32_t reserved;
+} cuart_stats_t;
+
+typedef struct cuart_index cuart_index;    /* device-resident index (opaque) */
+typedef struct cuart_layout cuart_layout;  /* host-resident flattened layout (opaque) */
+
+/* Read-only view of a host layout's arrays. */
+typedef struct {
+    const uint8_t* buf[8];       /* [1..7] raw records of each type, index order     */
+    uint64_t count[8];
+    uint64_t record_bytes[8];    /* 64, 160, 672, 2080, 16, 32, 48                   */
+    const uint64_t* lut;         /* NULL if lut_bytes == 0                            */
+    uint64_t lut_entries;
+    uint64_t root;
+    uint32_t lut_bytes;
+    uint32_t key_kind;
+    uint64_t n_keys;
+} cuart_layout_view;
+
+/* ---- the hot path -------------------------------------------------------- */
+cuart_status cuart_build(const cuart_keys* keys, const uint64_t* values, size_t n,
+                         const cuart_build_opts* opts, cuart_index** out);
+cuart_status cuart_lookup(const cuart_index* h, const cuart_keys* queries, size_t n,
+                          uint64_t* out, void* stream);
+cuart_status cuart_update(cuart_index* h, const cuart_keys* keys, const uint64_t* new_values,
+                          size_t n, void* stream);
+cuart_status cuart_destroy(cuart_index* h);   /* NULL ok */
+
+/* Host-buffer variants: chunked, stream-pipelined H2D -> kernel -> D2H (P:151
+ * §4.1: batches, several command streams).  Synchronous. */
+cuart_status cuart_lookup_host(const cuart_index* h, const cuart_keys* queries, size_t n,
+                               uint64_t* out);
+cuart_status cuart_update_host(cuart_index* h, const cuart_keys* keys, const uint64_t* new_values,
+                               size_t n);
+
+/* ---- introspection ------------------------------------------------------- */
+cuart_status cuart_stats(const cuart_index* h, cuart_stats_t* out);
+/* Synchronous device->host copy of every array (a snapshot; P:102 the buffers
+ * are regenerated from the host ART).  Free with cuart_layout_free. */
+cuart_status cuart_dump(const cuart_index* h, cuart_layout** out);
+/* Sticky device-side error flag (e.g. an update carried CUART_MISS); reading
+ * synchronises the index's device and clears the flag. */
+cuart_status cuart_get_error(cuart_index* h);
+const char* cuart_status_string(cuart_status s);
+/* Kernel launches issued by this library since load (for launch accounting). */
+uint64_t cuart_launch_count(void);
+
+/* ---- host layout (no GPU needed) ----------------------------------------- */
+/* The canonical ART of the key set flattened into the per-type buffers
+ * (one buffer per node type, packed 64-bit type+index links; P:110:
+ * fixed-size leaves of 8/16/32-byte keys in lexicographic order). */
+cuart_status cuart_layout_build(const cuart_keys* keys, const uint64_t* values, size_t n,
+                                const cuart_build_opts* opts, cuart_layout** out);
+cuart_status cuart_layout_view_get(const cuart_layout* l, cuart_layout_view* out);
+/* CPU lookup engine over the flat layout (§4.2, Fig. 7: the CuART
+ * layout used by a multi-threaded CPU lookup).  A separate engine, never a
+ * fallback of cuart_lookup. */
+cuart_status cuart_layout_lookup(const cuart_layout* l, const cuart_keys* queries, size_t n,
+                                 uint64_t* out, int threads);
+/* Per-query number of distinct 32-byte sectors the GPU lookup kernel reads on the
+ * path of each query (the algorithmic traffic behind the roofline numbers;
+ * DESIGN.md "Roofline").  sectors: host uint32_t[n]. */
+cuart_status cuart_layout_sectors(const cuart_layout* l, const cuart_keys* queries, size_t n,
+                                  uint32_t* sectors, int threads);
+cuart_status cuart_upload(const cuart_layout* l, const cuart_build_opts* opts, cuart_index** out);
+cuart_status cuart_layout_free(cuart_layout* l);  /* NULL ok */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CUART_H */

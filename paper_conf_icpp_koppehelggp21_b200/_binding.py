@@ -1,0 +1,360 @@
+"""ctypes marshalling for libcuart.so (see include/cuart.h for the contract)."""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libcuart.so")
+CUART_MISS = 0xFFFFFFFFFFFFFFFF
+CUART_MAX_KEY = 32
+KIND_U32, KIND_U64, KIND_BYTES = 1, 2, 3
+CUART_LUT_AUTO = 0xFFFFFFFF
+
+
+class CuartError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        super().__init__(f"{where}: cuart status {status} ({cuart_status_string(status)})")
+
+
+class _Keys(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int), ("data", ctypes.c_void_p), ("lengths", ctypes.c_void_p)]
+
+
+class _Opts(ctypes.Structure):
+    _fields_ = [("lut_bytes", ctypes.c_uint32), ("l2_persist", ctypes.c_uint32),
+                ("device", ctypes.c_int32), ("reserved", ctypes.c_uint32)]
+
+
+class _Stats(ctypes.Structure):
+    _fields_ = [("count", ctypes.c_uint64 * 8), ("bytes", ctypes.c_uint64 * 8), ("n_keys", ctypes.c_uint64),
+                ("lut_entries", ctypes.c_uint64), ("lut_bytes_total", ctypes.c_uint64),
+                ("arena_bytes", ctypes.c_uint64), ("lut_bytes", ctypes.c_uint32), ("key_kind", ctypes.c_uint32),
+                ("root", ctypes.c_uint64), ("max_depth", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+
+
+class _View(ctypes.Structure):
+    _fields_ = [("buf", ctypes.c_void_p * 8), ("count", ctypes.c_uint64 * 8), ("record_bytes", ctypes.c_uint64 * 8),
+                ("lut", ctypes.c_void_p), ("lut_entries", ctypes.c_uint64), ("root", ctypes.c_uint64),
+                ("lut_bytes", ctypes.c_uint32), ("key_kind", ctypes.c_uint32), ("n_keys", ctypes.c_uint64)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libcuart.so; raises if it was not built (no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run `python -m paper_conf_icpp_koppehelggp21_b200.build`")
+        L = ctypes.CDLL(LIB_PATH)
+        P, S, I = ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int
+        sig = {
+            "cuart_build": [P, P, S, P, P], "cuart_lookup": [P, P, S, P, P], "cuart_update": [P, P, P, S, P],
+            "cuart_destroy": [P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
+            "cuart_stats": [P, P], "cuart_dump": [P, P], "cuart_get_error": [P],
+            "cuart_layout_build": [P, P, S, P, P], "cuart_layout_view_get": [P, P],
+            "cuart_layout_lookup": [P, P, S, P, I], "cuart_layout_sectors": [P, P, S, P, I], "cuart_upload": [P, P, P], "cuart_layout_free": [P],
+        }
+        for name, args in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = ctypes.c_int
+        L.cuart_status_string.argtypes = [ctypes.c_int]
+        L.cuart_status_string.restype = ctypes.c_char_p
+        L.cuart_launch_count.argtypes = []
+        L.cuart_launch_count.restype = ctypes.c_uint64
+        _lib = L
+    return _lib
+
+
+def cuart_status_string(s: int) -> str:
+    return lib().cuart_status_string(int(s)).decode()
+
+
+def cuart_launch_count() -> int:
+    return int(lib().cuart_launch_count())
+
+
+def _check(rc, where):
+    if rc != 0:
+        raise CuartError(rc, where)
+
+
+# ------------------------------------------------------------------ marshalling
+def _is_torch(x):
+    return type(x).__module__.startswith("torch")
+
+
+def _ptr(x):
+    if x is None:
+        return None
+    if _is_torch(x):
+        return x.data_ptr()
+    return x.ctypes.data
+
+
+def _kind_of(x):
+    dt = str(x.dtype)
+    if dt.endswith(("uint64", "int64")):
+        return KIND_U64
+    if dt.endswith(("uint32", "int32")):
+        return KIND_U32
+    if dt.endswith("uint8") and len(x.shape) == 2:
+        return KIND_BYTES
+    raise TypeError(f"unsupported key array dtype/shape {x.dtype} {tuple(x.shape)}")
+
+
+def _contig(x):
+    if _is_torch(x):
+        return x.contiguous()
+    return np.ascontiguousarray(x)
+
+
+def make_keys(keys, lengths=None):
+    """keys: u64/u32 array, or (slots uint8[n,32], lengths uint8[n]) / slots + lengths."""
+    if isinstance(keys, tuple):
+        keys, lengths = keys
+    keys = _contig(keys)
+    kind = _kind_of(keys)
+    if kind == KIND_BYTES:
+        if lengths is None:
+            raise ValueError("byte-string keys need lengths")
+        if keys.shape[1] != CUART_MAX_KEY:
+            raise ValueError("byte-string keys must be 32-byte slots")
+        lengths = _contig(lengths)
+    n = int(keys.shape[0])
+    st = _Keys(kind, _ptr(keys), _ptr(lengths) if kind == KIND_BYTES else None)
+    return st, n, (keys, lengths)
+
+
+def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1):
+    return _Opts(lut_bytes, l2_persist, device, 0)
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+# ------------------------------------------------------------------ hot path
+def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1):
+    """Build + upload (host buffers).  Returns an opaque handle (int)."""
+    k, n, keep = make_keys(keys)
+    v = np.ascontiguousarray(values, dtype=np.uint64)
+    if v.shape[0] != n:
+        raise ValueError("values length mismatch")
+    h = ctypes.c_void_p()
+    o = _opts(lut_bytes, l2_persist, device)
+    _check(lib().cuart_build(ctypes.byref(k), _ptr(v), n, ctypes.byref(o), ctypes.byref(h)), "cuart_build")
+    return h.value
+
+
+def cuart_lookup(h, queries, out, stream=None):
+    """Device buffers (torch CUDA tensors); async on `stream` (default: current)."""
+    q, n, keep = make_keys(queries)
+    if out.shape[0] < n:
+        raise ValueError("out too small")
+    _check(lib().cuart_lookup(h, ctypes.byref(q), n, _ptr(out), _stream_ptr(stream)), "cuart_lookup")
+    return out
+
+
+def cuart_update(h, keys, new_values, stream=None):
+    k, n, keep = make_keys(keys)
+    if new_values.shape[0] != n:
+        raise ValueError("values length mismatch")
+    _check(lib().cuart_update(h, ctypes.byref(k), _ptr(_contig(new_values)), n, _stream_ptr(stream)), "cuart_update")
+
+
+def cuart_lookup_host(h, queries, out=None):
+    q, n, keep = make_keys(queries)
+    if out is None:
+        out = np.empty(n, dtype=np.uint64)
+    _check(lib().cuart_lookup_host(h, ctypes.byref(q), n, _ptr(out)), "cuart_lookup_host")
+    return out
+
+
+def cuart_update_host(h, keys, new_values):
+    k, n, keep = make_keys(keys)
+    v = _contig(new_values)
+    _check(lib().cuart_update_host(h, ctypes.byref(k), _ptr(v), n), "cuart_update_host")
+
+
+def cuart_destroy(h):
+    if h:
+        _check(lib().cuart_destroy(h), "cuart_destroy")
+
+
+def cuart_get_error(h) -> int:
+    return int(lib().cuart_get_error(h))
+
+
+def cuart_stats(h) -> dict:
+    s = _Stats()
+    _check(lib().cuart_stats(h, ctypes.byref(s)), "cuart_stats")
+    return _stats_dict(s)
+
+
+def _stats_dict(s):
+    names = {1: "n4", 2: "n16", 3: "n48", 4: "n256", 5: "leaf8", 6: "leaf16", 7: "leaf32"}
+    d = {names[t]: int(s.count[t]) for t in names}
+    d.update({f"{names[t]}_bytes": int(s.bytes[t]) for t in names})
+    d.update(n_keys=int(s.n_keys), lut_bytes=int(s.lut_bytes), lut_entries=int(s.lut_entries),
+             arena_bytes=int(s.arena_bytes), root=int(s.root), max_depth=int(s.max_depth), key_kind=int(s.key_kind))
+    return d
+
+
+# ------------------------------------------------------------------ host layout
+def cuart_layout_build(keys, values, lut_bytes=0):
+    k, n, keep = make_keys(keys)
+    v = np.ascontiguousarray(values, dtype=np.uint64)
+    if v.shape[0] != n:
+        raise ValueError("values length mismatch")
+    h = ctypes.c_void_p()
+    o = _opts(lut_bytes)
+    _check(lib().cuart_layout_build(ctypes.byref(k), _ptr(v), n, ctypes.byref(o), ctypes.byref(h)), "cuart_layout_build")
+    return h.value
+
+
+def cuart_layout_free(l):
+    if l:
+        lib().cuart_layout_free(l)
+
+
+def cuart_layout_view_get(l) -> dict:
+    """Copies of the layout's arrays as numpy (record bytes per type code, LUT, root)."""
+    v = _View()
+    _check(lib().cuart_layout_view_get(l, ctypes.byref(v)), "cuart_layout_view_get")
+    bufs = {}
+    for t in range(1, 8):
+        nbytes = int(v.count[t]) * int(v.record_bytes[t])
+        if nbytes:
+            bufs[t] = np.ctypeslib.as_array((ctypes.c_uint8 * nbytes).from_address(v.buf[t])).copy()
+        else:
+            bufs[t] = np.zeros(0, np.uint8)
+    lut = None
+    if v.lut:
+        lut = np.ctypeslib.as_array((ctypes.c_uint64 * int(v.lut_entries)).from_address(v.lut)).copy()
+    return {"buf": bufs, "count": [int(v.count[t]) for t in range(8)],
+            "record_bytes": [int(v.record_bytes[t]) for t in range(8)], "lut": lut, "root": int(v.root),
+            "lut_bytes": int(v.lut_bytes), "key_kind": int(v.key_kind), "n_keys": int(v.n_keys)}
+
+
+def cuart_layout_lookup(l, queries, threads=0):
+    q, n, keep = make_keys(queries)
+    out = np.empty(n, dtype=np.uint64)
+    _check(lib().cuart_layout_lookup(l, ctypes.byref(q), n, _ptr(out), threads), "cuart_layout_lookup")
+    return out
+
+
+def cuart_layout_sectors(l, queries, threads=0):
+    q, n, keep = make_keys(queries)
+    out = np.empty(n, dtype=np.uint32)
+    _check(lib().cuart_layout_sectors(l, ctypes.byref(q), n, _ptr(out), threads), "cuart_layout_sectors")
+    return out
+
+
+def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1):
+    h = ctypes.c_void_p()
+    o = _opts(lut_bytes, l2_persist, device)
+    _check(lib().cuart_upload(l, ctypes.byref(o), ctypes.byref(h)), "cuart_upload")
+    return h.value
+
+
+def cuart_dump(h):
+    """Device -> host snapshot of every array; returns a layout handle (free with cuart_layout_free)."""
+    l = ctypes.c_void_p()
+    _check(lib().cuart_dump(h, ctypes.byref(l)), "cuart_dump")
+    return l.value
+
+
+# ------------------------------------------------------------------ object wrappers
+class Layout:
+    """Host-resident flattened layout (no GPU needed)."""
+
+    def __init__(self, keys, values, lut_bytes=0):
+        self.h = cuart_layout_build(keys, values, lut_bytes)
+
+    def lookup(self, queries, threads=0):
+        return cuart_layout_lookup(self.h, queries, threads)
+
+    def view(self):
+        return cuart_layout_view_get(self.h)
+
+    def sectors(self, queries, threads=0):
+        return cuart_layout_sectors(self.h, queries, threads)
+
+    def close(self):
+        cuart_layout_free(self.h)
+        self.h = None
+
+    def __del__(self):
+        try:
+            if self.h:
+                self.close()
+        except Exception:
+            pass
+
+
+class Index:
+    """Device-resident CuART index on one GPU."""
+
+    def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1):
+        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device)
+
+    @classmethod
+    def from_layout(cls, layout: "Layout", l2_persist=0, device=-1):
+        """Upload an already-built host layout (keeps the host copy usable)."""
+        self = cls.__new__(cls)
+        self.h = cuart_upload(layout.h, 0, l2_persist, device)
+        return self
+
+    def lookup(self, queries, out=None, stream=None):
+        import torch
+        if out is None:
+            q = queries[0] if isinstance(queries, tuple) else queries
+            out = torch.empty(q.shape[0], dtype=torch.uint64, device=q.device)
+        return cuart_lookup(self.h, queries, out, stream)
+
+    def update(self, keys, new_values, stream=None):
+        cuart_update(self.h, keys, new_values, stream)
+
+    def lookup_host(self, queries, out=None):
+        return cuart_lookup_host(self.h, queries, out)
+
+    def update_host(self, keys, new_values):
+        cuart_update_host(self.h, keys, new_values)
+
+    def stats(self):
+        return cuart_stats(self.h)
+
+    def dump(self):
+        l = cuart_dump(self.h)
+        try:
+            return cuart_layout_view_get(l)
+        finally:
+            cuart_layout_free(l)
+
+    def dump_layout(self):
+        return cuart_dump(self.h)
+
+    def get_error(self):
+        return cuart_get_error(self.h)
+
+    def close(self):
+        if self.h:
+            cuart_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

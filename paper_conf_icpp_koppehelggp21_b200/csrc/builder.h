@@ -1,0 +1,34 @@
+// builder.h — host-side canonical ART build + flattening into the CuART layout.
+#pragma once
+#include <stdint.h>
+
+#include <vector>
+
+#include "layout.h"
+
+namespace cuart {
+
+struct HostLayout {
+    uint32_t key_kind = 0;                 // cuart_key_kind
+    std::vector<uint8_t> buf[8];           // raw records per type code (1..7)
+    uint64_t count[8] = {0};
+    uint64_t root = 0;                     // packed root link (0 = empty tree)
+    uint32_t lut_bytes = 0;
+    std::vector<uint64_t> lut;             // 2^(8*lut_bytes) links, or empty
+    uint64_t n_keys = 0;
+    uint32_t max_depth = 0;
+};
+
+// Status codes mirror cuart_status (include/cuart.h).
+int build_host_layout(uint32_t kind, const void* data, const uint8_t* lengths, const uint64_t* values,
+                      uint64_t n, uint32_t lut_bytes, HostLayout& out);
+
+// Multi-threaded CPU walk over the flat layout (§4.2, Fig. 7).
+void host_layout_lookup(const HostLayout& L, uint32_t kind, const void* queries, const uint8_t* lengths,
+                        uint64_t n, uint64_t* out, int threads);
+
+// Per-query count of the 32-byte sectors the GPU lookup reads (algorithmic bytes).
+void host_layout_sectors(const HostLayout& L, uint32_t kind, const void* queries, const uint8_t* lengths,
+                         uint64_t n, uint32_t* sectors, int threads);
+
+}  // namespace cuart

@@ -1,0 +1,535 @@
+// capi.cu — the C ABI (include/cuart.h): device index, lookup / update kernels
+// for sm_100a, host-buffer pipelines, introspection.
+//
+// Kernels:
+//   k_lookup<Key>  : PAPER.md Fig. 3 lookup within the per-type buffers.
+//   k_upd1<Key>    : update stage 1 (§3.4): lookup returning the leaf
+//                    location, then register the op index as the leaf's writer
+//                    if it is larger than the registered one.
+//   k_upd2         : update stage 2: after the grid-wide synchronisation
+//                    (the kernel boundary, reading C13), the op whose index is
+//                    the registered maximum stores its value.
+// Conflict registration (B200 reading of the paper's atomic hash table, P:143,
+// ref. [4]): a dense per-leaf 64-bit word winner[leaf] updated with atomicMax of
+// (epoch << 32 | op index).  Same semantics as the hash table keyed by leaf
+// location storing the maximum op index: the highest op index per leaf wins.
+// The epoch in the high half makes every earlier batch's entries smaller, so no
+// reset pass is needed between batches (reading C12/§8(a) a9).
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include <atomic>
+#include <new>
+
+#include "../../include/cuart.h"
+#include "builder.h"
+#include "kernels.cuh"
+
+using namespace cuart;
+
+struct cuart_layout {
+    HostLayout L;
+};
+
+struct cuart_index {
+    int device = 0;
+    int num_sms = 148;
+    uint32_t key_kind = 0;
+    uint32_t lut_bytes = 0;
+    uint64_t root = 0;
+    uint64_t count[8] = {0};
+    uint64_t n_keys = 0;
+    uint32_t max_depth = 0;
+    uint8_t* arena = nullptr;          // all record buffers + winner words + LUT + error flag
+    size_t arena_bytes = 0;
+    uint64_t off[8] = {0};
+    uint64_t lut_off = 0, winner_off = 0, err_off = 0;
+    uint64_t total_leaves = 0;
+    DevIndex dix{};
+    uint32_t epoch = 0;                // update batch epoch (high half of winner words)
+    // update scratch (leaf links of the current batch)
+    uint64_t* leafref = nullptr;
+    size_t leafref_cap = 0;
+    // host-pipeline staging
+    void* stage[2] = {nullptr, nullptr};
+    uint64_t* stage_out[2] = {nullptr, nullptr};
+    uint8_t* stage_len[2] = {nullptr, nullptr};
+    uint64_t* stage_val[2] = {nullptr, nullptr};
+    size_t stage_cap = 0;
+    cudaStream_t streams[2] = {nullptr, nullptr};
+    bool l2_window = false;
+    size_t l2_window_bytes = 0;
+};
+
+static std::atomic<uint64_t> g_launches{0};
+
+#define CU_TRY(x)                                   \
+    do {                                            \
+        cudaError_t e_ = (x);                       \
+        if (e_ != cudaSuccess) {                    \
+            return e_ == cudaErrorMemoryAllocation ? CUART_ERR_OOM : CUART_ERR_CUDA; \
+        }                                           \
+    } while (0)
+
+// ============================================================================ kernels
+template <class Key>
+__global__ void __launch_bounds__(256) k_lookup(DevIndex ix, const void* __restrict__ q,
+                                                const uint8_t* __restrict__ lens, uint64_t n,
+                                                uint64_t* __restrict__ out) {
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const Key key = Key::load(q, lens, i);
+        uint64_t val = kMiss;
+        const uint64_t leaf = find_leaf(ix, key, start_link(ix, key), val);
+        out[i] = leaf ? val : kMiss;
+    }
+}
+
+__device__ __forceinline__ uint64_t global_leaf_id(const DevIndex& ix, uint64_t leaf) {
+    const uint32_t t = link_type(leaf);
+    return (t == T_LEAF8 ? ix.leaf_base[5] : t == T_LEAF16 ? ix.leaf_base[6] : ix.leaf_base[7]) + link_index(leaf);
+}
+
+template <class Key>
+__global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restrict__ q, const uint8_t* __restrict__ lens,
+                                              const uint64_t* __restrict__ vals, uint64_t n, uint64_t epoch_hi,
+                                              uint64_t* __restrict__ leafref) {
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const Key key = Key::load(q, lens, i);
+        uint64_t val;
+        uint64_t leaf = find_leaf(ix, key, start_link(ix, key), val);
+        if (vals[i] == kMiss) {            // reserved value: op rejected, sticky error
+            atomicOr(ix.err, 1u);
+            leaf = 0;
+        }
+        leafref[i] = leaf;
+        if (leaf) atomicMax((unsigned long long*)&ix.winner[global_leaf_id(ix, leaf)], (unsigned long long)(epoch_hi | i));
+    }
+}
+
+__global__ void __launch_bounds__(256) k_upd2(DevIndex ix, const uint64_t* __restrict__ vals, uint64_t n,
+                                              uint64_t epoch_hi, const uint64_t* __restrict__ leafref) {
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const uint64_t leaf = leafref[i];
+        if (!leaf) continue;
+        if (__ldcg(&ix.winner[global_leaf_id(ix, leaf)]) != (epoch_hi | i)) continue;
+        const uint32_t t = link_type(leaf);
+        uint64_t* dst = (uint64_t*)(ix.base[t] + link_index(leaf) * record_bytes(t) + leaf_value_off(t));
+        *dst = vals[i];                    // one aligned 8-byte store ("atomically replace")
+    }
+}
+
+// ============================================================================ helpers
+static int grid_for(const cuart_index* h, uint64_t n) {
+    uint64_t blocks = (n + 255) / 256;
+    uint64_t cap = uint64_t(h->num_sms) * 8 * 16;   // 8 resident 256-thread CTAs per SM, 16 waves
+    if (blocks > cap) blocks = cap;
+    return int(blocks < 1 ? 1 : blocks);
+}
+
+static cuart_status check_keys(const cuart_index* h, const cuart_keys* k, size_t n) {
+    if (!h || !k) return CUART_ERR_INVALID_ARGUMENT;
+    if (n > 0 && k->data == nullptr) return CUART_ERR_INVALID_ARGUMENT;
+    if (uint32_t(k->kind) != h->key_kind) return CUART_ERR_INVALID_ARGUMENT;
+    if (k->kind == CUART_KEY_BYTES && n > 0 && k->lengths == nullptr) return CUART_ERR_INVALID_ARGUMENT;
+    return CUART_OK;
+}
+
+static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens, uint64_t n,
+                                  uint64_t* out, cudaStream_t s) {
+    if (n == 0) return CUART_OK;
+    const int grid = grid_for(h, n);
+    switch (kind) {
+    case CUART_KEY_U64: k_lookup<KeyU64><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out); break;
+    case CUART_KEY_U32: k_lookup<KeyU32><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out); break;
+    default: k_lookup<KeyBytes><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out); break;
+    }
+    g_launches++;
+    CU_TRY(cudaGetLastError());
+    return CUART_OK;
+}
+
+static cuart_status ensure_leafref(cuart_index* h, size_t n) {
+    if (h->leafref_cap >= n) return CUART_OK;
+    if (h->leafref) cudaFree(h->leafref);
+    h->leafref = nullptr;
+    h->leafref_cap = 0;
+    CU_TRY(cudaMalloc(&h->leafref, n * sizeof(uint64_t)));
+    h->leafref_cap = n;
+    return CUART_OK;
+}
+
+static constexpr uint64_t kUpdateChunk = uint64_t(1) << 30;   // op index must fit the low 32 bits
+
+static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, const uint8_t* lens,
+                                  const uint64_t* vals, uint64_t n, cudaStream_t s) {
+    for (uint64_t base = 0; base < n; base += kUpdateChunk) {
+        const uint64_t m = (n - base) < kUpdateChunk ? (n - base) : kUpdateChunk;
+        cuart_status rc = ensure_leafref(h, m);
+        if (rc != CUART_OK) return rc;
+        if (++h->epoch == 0xFFFFFFFFu) {        // epoch wrap: clear the conflict words
+            CU_TRY(cudaMemsetAsync(h->dix.winner, 0, h->total_leaves * 8, s));
+            h->epoch = 1;
+        }
+        const uint64_t epoch_hi = uint64_t(h->epoch) << 32;
+        const int grid = grid_for(h, m);
+        const size_t kstride = kind == CUART_KEY_U64 ? 8 : kind == CUART_KEY_U32 ? 4 : 32;
+        const void* kb = (const uint8_t*)k + base * kstride;
+        const uint8_t* lb = lens ? lens + base : nullptr;
+        switch (kind) {
+        case CUART_KEY_U64: k_upd1<KeyU64><<<grid, 256, 0, s>>>(h->dix, kb, lb, vals + base, m, epoch_hi, h->leafref); break;
+        case CUART_KEY_U32: k_upd1<KeyU32><<<grid, 256, 0, s>>>(h->dix, kb, lb, vals + base, m, epoch_hi, h->leafref); break;
+        default: k_upd1<KeyBytes><<<grid, 256, 0, s>>>(h->dix, kb, lb, vals + base, m, epoch_hi, h->leafref); break;
+        }
+        g_launches++;
+        CU_TRY(cudaGetLastError());
+        k_upd2<<<grid, 256, 0, s>>>(h->dix, vals + base, m, epoch_hi, h->leafref);
+        g_launches++;
+        CU_TRY(cudaGetLastError());
+    }
+    return CUART_OK;
+}
+
+// ============================================================================ C ABI
+extern "C" {
+
+const char* cuart_status_string(cuart_status s) {
+    switch (s) {
+    case CUART_OK: return "ok";
+    case CUART_ERR_INVALID_ARGUMENT: return "invalid argument";
+    case CUART_ERR_KEY_LENGTH: return "key length must be 1..32";
+    case CUART_ERR_NOT_PREFIX_FREE: return "key set is not prefix-free";
+    case CUART_ERR_RESERVED_VALUE: return "value is the reserved CUART_MISS";
+    case CUART_ERR_OOM: return "out of memory";
+    case CUART_ERR_CUDA: return "CUDA error";
+    case CUART_ERR_NCCL: return "NCCL error";
+    case CUART_ERR_NO_DEVICE: return "no CUDA device";
+    case CUART_ERR_TOO_LARGE: return "node buffer exceeds the link index range";
+    case CUART_ERR_INTERNAL: return "internal error";
+    }
+    return "unknown status";
+}
+
+uint64_t cuart_launch_count(void) { return g_launches.load(); }
+
+cuart_status cuart_layout_build(const cuart_keys* keys, const uint64_t* values, size_t n,
+                                const cuart_build_opts* opts, cuart_layout** out) {
+    if (!out || (!keys && n > 0)) return CUART_ERR_INVALID_ARGUMENT;
+    *out = nullptr;
+    uint32_t lut = opts ? opts->lut_bytes : 0;
+    const uint32_t kind = keys ? uint32_t(keys->kind) : uint32_t(CUART_KEY_U64);
+    if (lut == CUART_LUT_AUTO) lut = (kind == CUART_KEY_BYTES) ? 0 : (n >= (1u << 22) ? 3 : 0);
+    cuart_layout* l = new (std::nothrow) cuart_layout();
+    if (!l) return CUART_ERR_OOM;
+    int rc;
+    try {
+        rc = build_host_layout(kind, keys ? keys->data : nullptr, keys ? keys->lengths : nullptr, values, n, lut, l->L);
+    } catch (const std::bad_alloc&) {
+        rc = CUART_ERR_OOM;
+    } catch (...) {
+        rc = CUART_ERR_INTERNAL;
+    }
+    if (rc != CUART_OK) {
+        delete l;
+        return cuart_status(rc);
+    }
+    *out = l;
+    return CUART_OK;
+}
+
+cuart_status cuart_layout_free(cuart_layout* l) {
+    delete l;
+    return CUART_OK;
+}
+
+cuart_status cuart_layout_view_get(const cuart_layout* l, cuart_layout_view* v) {
+    if (!l || !v) return CUART_ERR_INVALID_ARGUMENT;
+    memset(v, 0, sizeof(*v));
+    for (int t = 1; t < 8; t++) {
+        v->buf[t] = l->L.buf[t].data();
+        v->count[t] = l->L.count[t];
+        v->record_bytes[t] = record_bytes(t);
+    }
+    v->lut = l->L.lut.empty() ? nullptr : l->L.lut.data();
+    v->lut_entries = l->L.lut.size();
+    v->root = l->L.root;
+    v->lut_bytes = l->L.lut_bytes;
+    v->key_kind = l->L.key_kind;
+    v->n_keys = l->L.n_keys;
+    return CUART_OK;
+}
+
+cuart_status cuart_layout_lookup(const cuart_layout* l, const cuart_keys* q, size_t n, uint64_t* out, int threads) {
+    if (!l || !q || (n > 0 && (!q->data || !out))) return CUART_ERR_INVALID_ARGUMENT;
+    if (uint32_t(q->kind) != l->L.key_kind) return CUART_ERR_INVALID_ARGUMENT;
+    if (q->kind == CUART_KEY_BYTES && n > 0 && !q->lengths) return CUART_ERR_INVALID_ARGUMENT;
+    host_layout_lookup(l->L, l->L.key_kind, q->data, q->lengths, n, out, threads);
+    return CUART_OK;
+}
+
+cuart_status cuart_layout_sectors(const cuart_layout* l, const cuart_keys* q, size_t n, uint32_t* sectors, int threads) {
+    if (!l || !q || (n > 0 && (!q->data || !sectors))) return CUART_ERR_INVALID_ARGUMENT;
+    if (uint32_t(q->kind) != l->L.key_kind) return CUART_ERR_INVALID_ARGUMENT;
+    if (q->kind == CUART_KEY_BYTES && n > 0 && !q->lengths) return CUART_ERR_INVALID_ARGUMENT;
+    host_layout_sectors(l->L, l->L.key_kind, q->data, q->lengths, n, sectors, threads);
+    return CUART_OK;
+}
+
+cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts, cuart_index** out) {
+    if (!lay || !out) return CUART_ERR_INVALID_ARGUMENT;
+    *out = nullptr;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return CUART_ERR_NO_DEVICE;
+    int dev = (opts && opts->device >= 0) ? opts->device : -1;
+    if (dev < 0) CU_TRY(cudaGetDevice(&dev));
+    if (dev >= ndev) return CUART_ERR_NO_DEVICE;
+    CU_TRY(cudaSetDevice(dev));
+    const HostLayout& L = lay->L;
+    cuart_index* h = new (std::nothrow) cuart_index();
+    if (!h) return CUART_ERR_OOM;
+    h->device = dev;
+    cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, dev);
+    h->key_kind = L.key_kind;
+    h->lut_bytes = L.lut_bytes;
+    h->root = L.root;
+    h->n_keys = L.n_keys;
+    h->max_depth = L.max_depth;
+    // arena: [N4 | N16 | N48 | N256 | leaf8 | leaf16 | leaf32 | winner | LUT | err], 256-B aligned
+    auto align = [](uint64_t x) { return (x + 255) & ~uint64_t(255); };
+    uint64_t off = 0;
+    for (int t = 1; t < 8; t++) {
+        h->count[t] = L.count[t];
+        h->off[t] = off;
+        off = align(off + L.buf[t].size());
+    }
+    h->total_leaves = L.count[5] + L.count[6] + L.count[7];
+    h->winner_off = off;
+    off = align(off + h->total_leaves * 8);
+    h->lut_off = off;
+    off = align(off + L.lut.size() * 8);
+    h->err_off = off;
+    off = align(off + 256);
+    h->arena_bytes = off;
+    cudaError_t e = cudaMalloc(&h->arena, off);
+    if (e != cudaSuccess) {
+        delete h;
+        return e == cudaErrorMemoryAllocation ? CUART_ERR_OOM : CUART_ERR_CUDA;
+    }
+    cuart_status rc = CUART_OK;
+    for (int t = 1; t < 8 && rc == CUART_OK; t++)
+        if (!L.buf[t].empty() && cudaMemcpy(h->arena + h->off[t], L.buf[t].data(), L.buf[t].size(), cudaMemcpyHostToDevice) != cudaSuccess)
+            rc = CUART_ERR_CUDA;
+    if (rc == CUART_OK && !L.lut.empty() &&
+        cudaMemcpy(h->arena + h->lut_off, L.lut.data(), L.lut.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
+        rc = CUART_ERR_CUDA;
+    if (rc == CUART_OK && h->total_leaves && cudaMemset(h->arena + h->winner_off, 0, h->total_leaves * 8) != cudaSuccess)
+        rc = CUART_ERR_CUDA;
+    if (rc == CUART_OK && cudaMemset(h->arena + h->err_off, 0, 256) != cudaSuccess) rc = CUART_ERR_CUDA;
+    if (rc != CUART_OK) {
+        cudaFree(h->arena);
+        delete h;
+        return rc;
+    }
+    DevIndex& d = h->dix;
+    for (int t = 1; t < 8; t++) d.base[t] = h->arena + h->off[t];
+    d.base[0] = nullptr;
+    d.root = L.root;
+    d.lut = L.lut.empty() ? nullptr : (const uint64_t*)(h->arena + h->lut_off);
+    d.lut_bytes = L.lut_bytes;
+    d.key_kind = L.key_kind;
+    d.winner = (uint64_t*)(h->arena + h->winner_off);
+    d.leaf_base[5] = 0;
+    d.leaf_base[6] = L.count[5];
+    d.leaf_base[7] = L.count[5] + L.count[6];
+    d.err = (uint32_t*)(h->arena + h->err_off);
+    *out = h;
+    return CUART_OK;
+}
+
+cuart_status cuart_build(const cuart_keys* keys, const uint64_t* values, size_t n, const cuart_build_opts* opts,
+                         cuart_index** out) {
+    if (!out) return CUART_ERR_INVALID_ARGUMENT;
+    *out = nullptr;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return CUART_ERR_NO_DEVICE;
+    cuart_layout* l = nullptr;
+    cuart_status rc = cuart_layout_build(keys, values, n, opts, &l);
+    if (rc != CUART_OK) return rc;
+    rc = cuart_upload(l, opts, out);
+    cuart_layout_free(l);
+    return rc;
+}
+
+cuart_status cuart_destroy(cuart_index* h) {
+    if (!h) return CUART_OK;
+    cudaSetDevice(h->device);
+    cudaDeviceSynchronize();
+    cudaFree(h->arena);
+    if (h->leafref) cudaFree(h->leafref);
+    for (int i = 0; i < 2; i++) {
+        if (h->stage[i]) cudaFree(h->stage[i]);
+        if (h->stage_out[i]) cudaFree(h->stage_out[i]);
+        if (h->stage_len[i]) cudaFree(h->stage_len[i]);
+        if (h->stage_val[i]) cudaFree(h->stage_val[i]);
+        if (h->streams[i]) cudaStreamDestroy(h->streams[i]);
+    }
+    delete h;
+    return CUART_OK;
+}
+
+cuart_status cuart_lookup(const cuart_index* h, const cuart_keys* q, size_t n, uint64_t* out, void* stream) {
+    cuart_status rc = check_keys(h, q, n);
+    if (rc != CUART_OK) return rc;
+    if (n == 0) return CUART_OK;
+    if (!out) return CUART_ERR_INVALID_ARGUMENT;
+    return launch_lookup(h, h->key_kind, q->data, q->lengths, n, out, (cudaStream_t)stream);
+}
+
+cuart_status cuart_update(cuart_index* h, const cuart_keys* k, const uint64_t* v, size_t n, void* stream) {
+    cuart_status rc = check_keys(h, k, n);
+    if (rc != CUART_OK) return rc;
+    if (n == 0) return CUART_OK;
+    if (!v) return CUART_ERR_INVALID_ARGUMENT;
+    return launch_update(h, h->key_kind, k->data, k->lengths, v, n, (cudaStream_t)stream);
+}
+
+// ---------------------------------------------------------------- host-buffer pipelines
+static constexpr size_t kStageChunk = size_t(1) << 23;   // ops per pipeline chunk
+
+static cuart_status ensure_stage(cuart_index* h) {
+    if (h->stage_cap) return CUART_OK;
+    for (int i = 0; i < 2; i++) {
+        CU_TRY(cudaMalloc(&h->stage[i], kStageChunk * 32));
+        CU_TRY(cudaMalloc(&h->stage_out[i], kStageChunk * 8));
+        CU_TRY(cudaMalloc(&h->stage_len[i], kStageChunk));
+        CU_TRY(cudaMalloc(&h->stage_val[i], kStageChunk * 8));
+        CU_TRY(cudaStreamCreateWithFlags(&h->streams[i], cudaStreamNonBlocking));
+    }
+    h->stage_cap = kStageChunk;
+    return CUART_OK;
+}
+
+static size_t key_stride(uint32_t kind) { return kind == CUART_KEY_U64 ? 8 : kind == CUART_KEY_U32 ? 4 : 32; }
+
+cuart_status cuart_lookup_host(const cuart_index* hc, const cuart_keys* q, size_t n, uint64_t* out) {
+    cuart_index* h = const_cast<cuart_index*>(hc);
+    cuart_status rc = check_keys(h, q, n);
+    if (rc != CUART_OK) return rc;
+    if (n == 0) return CUART_OK;
+    if (!out) return CUART_ERR_INVALID_ARGUMENT;
+    CU_TRY(cudaSetDevice(h->device));
+    if ((rc = ensure_stage(h)) != CUART_OK) return rc;
+    const size_t ks = key_stride(h->key_kind);
+    size_t c = 0;
+    for (size_t base = 0; base < n; base += kStageChunk, c++) {
+        const size_t m = (n - base) < kStageChunk ? (n - base) : kStageChunk;
+        const int s = int(c & 1);
+        cudaStream_t st = h->streams[s];
+        CU_TRY(cudaMemcpyAsync(h->stage[s], (const uint8_t*)q->data + base * ks, m * ks, cudaMemcpyHostToDevice, st));
+        if (q->lengths) CU_TRY(cudaMemcpyAsync(h->stage_len[s], q->lengths + base, m, cudaMemcpyHostToDevice, st));
+        rc = launch_lookup(h, h->key_kind, h->stage[s], q->lengths ? h->stage_len[s] : nullptr, m, h->stage_out[s], st);
+        if (rc != CUART_OK) return rc;
+        CU_TRY(cudaMemcpyAsync(out + base, h->stage_out[s], m * 8, cudaMemcpyDeviceToHost, st));
+    }
+    CU_TRY(cudaStreamSynchronize(h->streams[0]));
+    CU_TRY(cudaStreamSynchronize(h->streams[1]));
+    return CUART_OK;
+}
+
+cuart_status cuart_update_host(cuart_index* h, const cuart_keys* k, const uint64_t* v, size_t n) {
+    cuart_status rc = check_keys(h, k, n);
+    if (rc != CUART_OK) return rc;
+    if (n == 0) return CUART_OK;
+    if (!v) return CUART_ERR_INVALID_ARGUMENT;
+    CU_TRY(cudaSetDevice(h->device));
+    if ((rc = ensure_stage(h)) != CUART_OK) return rc;
+    const size_t ks = key_stride(h->key_kind);
+    // chunks are applied in op order on ONE stream: sequential semantics across chunks
+    cudaStream_t st = h->streams[0];
+    size_t c = 0;
+    for (size_t base = 0; base < n; base += kStageChunk, c++) {
+        const size_t m = (n - base) < kStageChunk ? (n - base) : kStageChunk;
+        const int s = int(c & 1);
+        CU_TRY(cudaMemcpyAsync(h->stage[s], (const uint8_t*)k->data + base * ks, m * ks, cudaMemcpyHostToDevice, st));
+        if (k->lengths) CU_TRY(cudaMemcpyAsync(h->stage_len[s], k->lengths + base, m, cudaMemcpyHostToDevice, st));
+        CU_TRY(cudaMemcpyAsync(h->stage_val[s], v + base, m * 8, cudaMemcpyHostToDevice, st));
+        rc = launch_update(h, h->key_kind, h->stage[s], k->lengths ? h->stage_len[s] : nullptr, h->stage_val[s], m, st);
+        if (rc != CUART_OK) return rc;
+    }
+    CU_TRY(cudaStreamSynchronize(st));
+    return CUART_OK;
+}
+
+// ---------------------------------------------------------------- introspection
+cuart_status cuart_stats(const cuart_index* h, cuart_stats_t* s) {
+    if (!h || !s) return CUART_ERR_INVALID_ARGUMENT;
+    memset(s, 0, sizeof(*s));
+    for (int t = 1; t < 8; t++) {
+        s->count[t] = h->count[t];
+        s->bytes[t] = h->count[t] * record_bytes(t);
+    }
+    s->n_keys = h->n_keys;
+    s->lut_bytes = h->lut_bytes;
+    s->lut_entries = h->lut_bytes ? (uint64_t(1) << (8 * h->lut_bytes)) : 0;
+    s->lut_bytes_total = s->lut_entries * 8;
+    s->arena_bytes = h->arena_bytes + h->leafref_cap * 8;
+    s->key_kind = h->key_kind;
+    s->root = h->root;
+    s->max_depth = h->max_depth;
+    return CUART_OK;
+}
+
+cuart_status cuart_dump(const cuart_index* h, cuart_layout** out) {
+    if (!h || !out) return CUART_ERR_INVALID_ARGUMENT;
+    *out = nullptr;
+    CU_TRY(cudaSetDevice(h->device));
+    CU_TRY(cudaDeviceSynchronize());
+    cuart_layout* l = new (std::nothrow) cuart_layout();
+    if (!l) return CUART_ERR_OOM;
+    HostLayout& L = l->L;
+    L.key_kind = h->key_kind;
+    L.root = h->root;
+    L.lut_bytes = h->lut_bytes;
+    L.n_keys = h->n_keys;
+    L.max_depth = h->max_depth;
+    try {
+        for (int t = 1; t < 8; t++) {
+            L.count[t] = h->count[t];
+            L.buf[t].resize(h->count[t] * record_bytes(t));
+            if (!L.buf[t].empty() &&
+                cudaMemcpy(L.buf[t].data(), h->arena + h->off[t], L.buf[t].size(), cudaMemcpyDeviceToHost) != cudaSuccess) {
+                delete l;
+                return CUART_ERR_CUDA;
+            }
+        }
+        if (h->lut_bytes) {
+            L.lut.resize(uint64_t(1) << (8 * h->lut_bytes));
+            if (cudaMemcpy(L.lut.data(), h->arena + h->lut_off, L.lut.size() * 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+                delete l;
+                return CUART_ERR_CUDA;
+            }
+        }
+    } catch (...) {
+        delete l;
+        return CUART_ERR_OOM;
+    }
+    *out = l;
+    return CUART_OK;
+}
+
+cuart_status cuart_get_error(cuart_index* h) {
+    if (!h) return CUART_ERR_INVALID_ARGUMENT;
+    CU_TRY(cudaSetDevice(h->device));
+    CU_TRY(cudaDeviceSynchronize());
+    uint32_t flag = 0;
+    CU_TRY(cudaMemcpy(&flag, h->dix.err, 4, cudaMemcpyDeviceToHost));
+    if (flag) {
+        CU_TRY(cudaMemset(h->dix.err, 0, 4));
+        return CUART_ERR_RESERVED_VALUE;
+    }
+    return CUART_OK;
+}
+
+}  // extern "C"

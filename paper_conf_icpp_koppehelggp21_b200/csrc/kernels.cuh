@@ -1,0 +1,204 @@
+// kernels.cuh — device-side traversal of the CuART layout (sm_100a).
+//
+// Lookup algorithm of PAPER.md Fig. 3 within the type-segregated buffers
+// (§3.2.1): decode the packed link (type in the MSBs, index in the LSBs),
+// read a record of a size known before the request, search the child on the key
+// byte, repeat; compare the full key at the leaf.  B200 reading: the branch depth
+// rides in the link (layout.h), so no node header is read on the path, the
+// compressed prefix is skipped optimistically and the leaf compare decides.
+#pragma once
+#include <stdint.h>
+
+#include "layout.h"
+
+namespace cuart {
+
+struct DevIndex {
+    const uint8_t* base[8];       // record buffers per type code
+    uint64_t root;                // packed root link
+    const uint64_t* lut;          // root lookup table, or nullptr
+    uint32_t lut_bytes;
+    uint32_t key_kind;
+    uint64_t* winner;             // per-leaf conflict word for updates (global leaf id)
+    uint64_t leaf_base[8];        // global leaf id = leaf_base[type] + index
+    uint32_t* err;                // sticky device error flag
+};
+
+// ----------------------------------------------------------------------------- loads
+__device__ __forceinline__ uint64_t ld_nc_u64(const void* p) {
+    uint64_t v;
+    asm volatile("ld.global.nc.u64 %0, [%1];" : "=l"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_nc_u8(const void* p) {
+    uint16_t v;
+    asm volatile("ld.global.nc.u8 %0, [%1];" : "=h"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ uint4 ld_nc_v4(const void* p) {
+    uint4 v;
+    asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+}
+// Leaf values are rewritten by the update kernels: read them through L2 (coherent path).
+__device__ __forceinline__ uint64_t ld_cg_u64(const void* p) {
+    uint64_t v;
+    asm volatile("ld.global.cg.u64 %0, [%1];" : "=l"(v) : "l"(p));
+    return v;
+}
+
+__device__ __forceinline__ uint64_t bswap64(uint64_t x) {
+    uint32_t lo = uint32_t(x), hi = uint32_t(x >> 32);
+    return (uint64_t(__byte_perm(lo, 0, 0x0123)) << 32) | __byte_perm(hi, 0, 0x0123);
+}
+
+// ----------------------------------------------------------------------------- key views
+// U64: numeric key, canonical bytes are big-endian (reading C2).
+struct KeyU64 {
+    uint64_t k;
+    static constexpr uint32_t kKind = 2;
+    __device__ __forceinline__ static KeyU64 load(const void* q, const uint8_t*, uint64_t i) {
+        return KeyU64{((const uint64_t*)q)[i]};
+    }
+    __device__ __forceinline__ uint32_t len() const { return 8; }
+    __device__ __forceinline__ uint32_t byte(uint32_t d) const { return uint32_t(k >> (56 - 8 * d)) & 0xFF; }
+    __device__ __forceinline__ uint64_t prefix(uint32_t nb) const { return k >> (64 - 8 * nb); }
+    // One 16-byte load brings key and value of a leaf8 record.
+    __device__ __forceinline__ bool leaf_match(const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
+        const uint4 r = ld_nc_v4(rec);
+        val = uint64_t(r.z) | (uint64_t(r.w) << 32);
+        return aux == 8 && (uint64_t(r.x) | (uint64_t(r.y) << 32)) == bswap64(k);
+    }
+};
+
+struct KeyU32 {
+    uint32_t k;
+    static constexpr uint32_t kKind = 1;
+    __device__ __forceinline__ static KeyU32 load(const void* q, const uint8_t*, uint64_t i) {
+        return KeyU32{((const uint32_t*)q)[i]};
+    }
+    __device__ __forceinline__ uint32_t len() const { return 4; }
+    __device__ __forceinline__ uint32_t byte(uint32_t d) const { return (k >> (24 - 8 * d)) & 0xFF; }
+    __device__ __forceinline__ uint64_t prefix(uint32_t nb) const { return uint64_t(k) >> (32 - 8 * nb); }
+    __device__ __forceinline__ bool leaf_match(const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
+        const uint4 r = ld_nc_v4(rec);
+        val = uint64_t(r.z) | (uint64_t(r.w) << 32);
+        return aux == 4 && r.y == 0 && r.x == __byte_perm(k, 0, 0x0123);
+    }
+};
+
+// BYTES: 32-byte slot + length; bytes past the length are masked to zero.
+struct KeyBytes {
+    uint64_t w[4];   // little-endian words of the zero-padded slot
+    uint32_t l;
+    static constexpr uint32_t kKind = 3;
+    __device__ __forceinline__ static KeyBytes load(const void* q, const uint8_t* lens, uint64_t i) {
+        KeyBytes kb;
+        const uint4 a = *((const uint4*)q + 2 * i);
+        const uint4 b = *((const uint4*)q + 2 * i + 1);
+        kb.w[0] = uint64_t(a.x) | (uint64_t(a.y) << 32);
+        kb.w[1] = uint64_t(a.z) | (uint64_t(a.w) << 32);
+        kb.w[2] = uint64_t(b.x) | (uint64_t(b.y) << 32);
+        kb.w[3] = uint64_t(b.z) | (uint64_t(b.w) << 32);
+        kb.l = lens[i];
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            const int lo = 8 * j;
+            const int keep = int(kb.l) - lo;   // bytes of word j inside the key
+            uint64_t m = keep >= 8 ? ~0ull : (keep <= 0 ? 0ull : ((1ull << (8 * keep)) - 1));
+            kb.w[j] &= m;
+        }
+        return kb;
+    }
+    __device__ __forceinline__ uint32_t len() const { return l; }
+    __device__ __forceinline__ uint64_t word(uint32_t j) const {
+        return j == 0 ? w[0] : j == 1 ? w[1] : j == 2 ? w[2] : w[3];
+    }
+    __device__ __forceinline__ uint32_t byte(uint32_t d) const { return uint32_t(word(d >> 3) >> (8 * (d & 7))) & 0xFF; }
+    __device__ __forceinline__ uint64_t prefix(uint32_t nb) const {
+        uint64_t p = 0;
+        for (uint32_t b = 0; b < nb; b++) p = (p << 8) | byte(b);
+        return p;
+    }
+    __device__ __forceinline__ bool leaf_match(const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
+        const uint4 a = ld_nc_v4(rec);
+        const uint64_t a0 = uint64_t(a.x) | (uint64_t(a.y) << 32), a1 = uint64_t(a.z) | (uint64_t(a.w) << 32);
+        if (t == T_LEAF8) {
+            val = a1;
+            return aux == l && a0 == w[0];
+        }
+        const uint4 b = ld_nc_v4(rec + 16);
+        const uint64_t b0 = uint64_t(b.x) | (uint64_t(b.y) << 32), b1 = uint64_t(b.z) | (uint64_t(b.w) << 32);
+        if (t == T_LEAF16) {
+            val = b0;
+            return aux == l && a0 == w[0] && a1 == w[1];
+        }
+        const uint4 c = ld_nc_v4(rec + 32);
+        val = uint64_t(c.x) | (uint64_t(c.y) << 32);
+        return aux == l && a0 == w[0] && a1 == w[1] && b0 == w[2] && b1 == w[3];
+    }
+};
+
+// Count of key bytes < b among 4 packed bytes (sorted keys; padding repeats the last key).
+__device__ __forceinline__ void search4(uint32_t keys, uint32_t bb, uint32_t& less, uint32_t& eq) {
+    less = __popc(__vcmpltu4(keys, bb)) >> 3;
+    eq = __vcmpeq4(keys, bb);
+}
+
+// Walk from `link` to a leaf.  Returns the leaf link on a full-key match (its value
+// in `val`), 0 otherwise.
+template <class Key>
+__device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Key& key, uint64_t link, uint64_t& val) {
+    const uint32_t len = key.len();
+#pragma unroll 1
+    for (;;) {
+        const uint32_t t = link_type(link);
+        const uint64_t idx = link_index(link);
+        const uint32_t aux = link_aux(link);
+        if (t >= T_LEAF8) {
+            const uint8_t* rec = ix.base[t] + idx * record_bytes(t);
+            return key.leaf_match(rec, t, aux, val) ? link : 0;
+        }
+        if (t == T_NULL || aux >= len) return 0;
+        const uint32_t b = key.byte(aux);
+        const uint8_t* rec = ix.base[t] + idx * record_bytes(t);
+        if (t == T_N256) {
+            link = ld_nc_u64(rec + kN256Child + 8 * b);
+        } else if (t == T_N48) {
+            const uint32_t s = ld_nc_u8(rec + kN48Index + b);
+            if (s == kN48Empty) return 0;
+            link = ld_nc_u64(rec + kN48Child + 8 * s);
+        } else if (t == T_N16) {
+            const uint4 k4 = ld_nc_v4(rec + kN16Keys);
+            const uint32_t bb = b * 0x01010101u;
+            uint32_t l0, l1, l2, l3, e0, e1, e2, e3;
+            search4(k4.x, bb, l0, e0);
+            search4(k4.y, bb, l1, e1);
+            search4(k4.z, bb, l2, e2);
+            search4(k4.w, bb, l3, e3);
+            if ((e0 | e1 | e2 | e3) == 0) return 0;
+            link = ld_nc_u64(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
+        } else {  // N4: whole 64-byte record in one round trip
+            const uint4 h = ld_nc_v4(rec + 16);          // keys[4] | pad | child[0]
+            const uint4 c12 = ld_nc_v4(rec + 32);        // child[1], child[2]
+            const uint64_t c3 = ld_nc_u64(rec + 48);     // child[3]
+            uint32_t less, eq;
+            search4(h.x, b * 0x01010101u, less, eq);
+            if (eq == 0) return 0;
+            const uint64_t c0 = uint64_t(h.z) | (uint64_t(h.w) << 32);
+            const uint64_t c1 = uint64_t(c12.x) | (uint64_t(c12.y) << 32);
+            const uint64_t c2 = uint64_t(c12.z) | (uint64_t(c12.w) << 32);
+            link = less == 0 ? c0 : less == 1 ? c1 : less == 2 ? c2 : c3;
+        }
+    }
+}
+
+template <class Key>
+__device__ __forceinline__ uint64_t start_link(const DevIndex& ix, const Key& key) {
+    if (ix.lut_bytes && key.len() >= ix.lut_bytes) return ld_nc_u64(ix.lut + key.prefix(ix.lut_bytes));
+    return ix.root;
+}
+
+
+}  // namespace cuart

@@ -1,0 +1,89 @@
+"""Test-side decoder of the CuART flat layout.
+
+Independent reading of the layout spec used to turn a host layout or a device
+dump into the oracle's pre-order structure records, so builder/device results
+can be compared with the oracle's pointer ART structure.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+REC = {1: 64, 2: 160, 3: 672, 4: 2080, 5: 16, 6: 32, 7: 48}
+VALOFF = {5: 8, 6: 16, 7: 32}
+IDX_MASK = (1 << 52) - 1
+
+
+def split_link(link: int):
+    return link >> 60, (link >> 52) & 0xFF, link & IDX_MASK
+
+
+def _u64(buf, off):
+    return int(np.frombuffer(bytes(buf[off: off + 8]), dtype="<u8")[0])
+
+
+def children(view, t, idx):
+    """[(byte, child_link)] in byte order."""
+    b = view["buf"][t]
+    o = idx * REC[t]
+    if t == 1 or t == 2:
+        cnt = int(b[o + 1]) + 1
+        ko, co = (16, 24) if t == 1 else (16, 32)
+        return [(int(b[o + ko + j]), _u64(b, o + co + 8 * j)) for j in range(cnt)]
+    if t == 3:
+        out = []
+        for byte in range(256):
+            s = int(b[o + 16 + byte])
+            if s != 0xFF:
+                out.append((byte, _u64(b, o + 272 + 8 * s)))
+        return out
+    out = []
+    for byte in range(256):
+        c = _u64(b, o + 16 + 8 * byte)
+        if c:
+            out.append((byte, c))
+    return out
+
+
+def leaf(view, link):
+    t, ln, idx = split_link(link)
+    b = view["buf"][t]
+    o = idx * REC[t]
+    return bytes(b[o: o + ln]), _u64(b, o + VALOFF[t]), bytes(b[o + ln: o + {5: 8, 6: 16, 7: 32}[t]])
+
+
+def to_records(view) -> list[int]:
+    """Pre-order records in the oracle dump format; asserts layout-internal consistency."""
+    out: list[int] = []
+
+    def first_leaf(link):
+        while split_link(link)[0] < 5:
+            t, _, idx = split_link(link)
+            link = children(view, t, idx)[0][1]
+        return leaf(view, link)[0]
+
+    def rec(link, depth):
+        t, aux, idx = split_link(link)
+        assert t != 0
+        if t >= 5:
+            k, v, pad = leaf(view, link)
+            assert pad == b"\0" * len(pad), "leaf key padding must be zero"
+            assert t == (5 if len(k) <= 8 else 6 if len(k) <= 16 else 7), "leaf class by key length (P:110)"
+            out.extend([0, len(k), *k, v])
+            return
+        b = view["buf"][t]
+        o = idx * REC[t]
+        plen = int(b[o])
+        assert aux == depth + plen, "branch depth in the link = depth + prefix length"
+        kids = children(view, t, idx)
+        assert int(b[o + 1]) + 1 == len(kids), "header count"
+        fl = first_leaf(link)
+        prefix = fl[depth: depth + plen]
+        stored = bytes(b[o + 2: o + 2 + min(plen, 14)])
+        assert stored == prefix[:14], "header stores the first 14 prefix bytes"
+        out.extend([t, plen, *prefix, len(kids), *[k for k, _ in kids]])
+        for _, c in kids:
+            rec(c, depth + plen + 1)
+
+    if view["root"]:
+        rec(view["root"], 0)
+    return out

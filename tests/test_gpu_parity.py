@@ -1,0 +1,273 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, bit-exact.
+
+All results are integers (u64 values / CUART_MISS), so the bar is element-wise
+equality.  Small configs are compared element by element with the pointer-ART
+oracle; full-size configs are compared on sampled outputs with the plain-map
+oracle and on properties that hold at any size.
+"""
+import random
+
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_icpp_koppehelggp21_b200 as C
+import workloads as W
+from oracle import ArtOracle, MapOracle, OART_MISS
+from tests.artspec import golden_key, load_golden
+from tests.layout_decode import to_records
+
+pytestmark = pytest.mark.gpu
+MISS = int(OART_MISS)
+DEV = "cuda:0"
+
+
+def _t(a):
+    """numpy -> CUDA tensor with the same bits (uint64 -> int64 view)."""
+    if isinstance(a, tuple):
+        return (_t(a[0]), _t(a[1]))
+    if a.dtype == np.uint64:
+        return torch.from_numpy(a.view(np.int64)).to(DEV)
+    if a.dtype == np.uint32:
+        return torch.from_numpy(a.view(np.int32)).to(DEV)
+    return torch.from_numpy(a).to(DEV)
+
+
+def _u64(t):
+    return t.cpu().numpy().view(np.uint64)
+
+
+def _strings(keys):
+    slots = np.zeros((len(keys), 32), np.uint8)
+    lens = np.zeros(len(keys), np.uint8)
+    for i, k in enumerate(keys):
+        slots[i, : len(k)] = np.frombuffer(k, np.uint8)
+        lens[i] = len(k)
+    return slots, lens
+
+
+def _as_input(kind, keys):
+    if kind == "u64":
+        return np.array([int.from_bytes(k, "big") for k in keys], np.uint64)
+    if kind == "u32":
+        return np.array([int.from_bytes(k, "big") for k in keys], np.uint32)
+    return _strings(keys)
+
+
+def _lookup(ix, q):
+    qt = _t(q)
+    n = (qt[0] if isinstance(qt, tuple) else qt).shape[0]
+    out = torch.empty(n, dtype=torch.int64, device=DEV)
+    ix.lookup(qt, out)
+    torch.cuda.synchronize()
+    return _u64(out)
+
+
+@pytest.mark.parametrize("name", ["ex_a_u64.json", "ex_d_strings.json", "ex_e_prefix_split.json", "ex_f_long_prefix.json"])
+@pytest.mark.parametrize("lut", [0, 1, 3])
+def test_golden_gpu(name, lut):
+    g = load_golden(name)
+    kind = g["kind"]
+    inp = _as_input(kind, [golden_key(kind, k) for k in g["keys"]])
+    ix = C.Index(inp, np.array(g["values"], np.uint64), lut_bytes=lut)
+    qs = [golden_key(kind, q) for q, _ in g["lookups"]]
+    exp = [MISS if v is None else v for _, v in g["lookups"]]
+    assert _lookup(ix, _as_input(kind, qs) if kind != "bytes" else _strings(qs)).tolist() == exp
+    uk = [golden_key(kind, k) for k, _ in g["update_ops"]]
+    ix.update(_t(_as_input(kind, uk) if kind != "bytes" else _strings(uk)),
+              _t(np.array([v for _, v in g["update_ops"]], np.uint64)))
+    ak = [golden_key(kind, k) for k, _ in g["after_update"]]
+    got = _lookup(ix, _as_input(kind, ak) if kind != "bytes" else _strings(ak)).tolist()
+    assert got == [v for _, v in g["after_update"]]
+    ix.close()
+
+
+@pytest.mark.parametrize("lut", [0, 2, 3])
+def test_c1_full_parity(lut):
+    """Config 1 at full size, element by element against the pointer-ART oracle:
+    1M lookups (50% hit), 100K updates, then the post-update dump."""
+    cfg = W.CONFIGS["c1"]
+    keys, vals = W.build_set(cfg)
+    o = ArtOracle(keys, vals)
+    ix = C.Index(keys, vals, lut_bytes=lut)
+    st = ix.stats()
+    os_ = o.stats()
+    assert (st["n4"], st["n16"], st["n48"], st["n256"], st["leaf8"]) == (os_["n4"], os_["n16"], os_["n48"], os_["n256"], os_["leaves"])
+    q = W.lookup_batch(cfg, keys)
+    got = _lookup(ix, q)
+    exp = o.lookup(q)
+    assert np.array_equal(got, exp)
+    assert abs((exp != OART_MISS).mean() - 0.5) < 0.01
+    uk, uv = W.update_batch(cfg, keys)
+    ix.update(_t(uk), _t(uv))
+    o.update(uk, uv)
+    torch.cuda.synchronize()
+    assert ix.get_error() == 0
+    assert np.array_equal(_lookup(ix, keys), o.lookup(keys))
+    assert np.array_equal(_lookup(ix, q), o.lookup(q))
+    # full post-update tree state: device dump decoded == oracle structure (incl. values)
+    assert to_records(ix.dump()) == o.dump_structure().tolist()
+    ix.close()
+
+
+@pytest.mark.parametrize("mode", ["u64", "u64_shared", "u32", "bytes"])
+@pytest.mark.parametrize("seed", range(3))
+def test_random_sets_gpu(mode, seed):
+    rng = random.Random(seed * 7 + len(mode))
+    n = rng.choice([1, 2, 5, 17, 49, 257, 5000, 40_000])
+    s = set()
+    while len(s) < n:
+        if mode == "u64":
+            s.add(rng.getrandbits(64).to_bytes(8, "big"))
+        elif mode == "u64_shared":
+            k = bytearray(8)
+            for i in range(rng.randrange(0, 8), 8):
+                k[i] = rng.choice([0, 0xFF, rng.randrange(256), rng.randrange(3)])
+            s.add(bytes(k))
+        elif mode == "u32":
+            s.add(rng.choice([rng.getrandbits(32), rng.getrandbits(14)]).to_bytes(4, "big"))
+        else:
+            stem = rng.choice([b"", b"a", b"q" * 14, b"r" * 15, b"s" * 16, b"t" * 24])
+            body = bytes(rng.choice(b"abz\x01\xff") for _ in range(rng.randrange(0, 31 - len(stem) + 1)))
+            s.add((stem + body)[:31] + b"\x00")
+    keys = sorted(s)
+    rng.shuffle(keys)
+    kind = "bytes" if mode == "bytes" else ("u32" if mode == "u32" else "u64")
+    vals = np.array([rng.getrandbits(63) for _ in keys], np.uint64)
+    inp = _as_input(kind, keys)
+    o = ArtOracle(inp, vals)
+    probes = list(keys)
+    for k in keys[:2000]:
+        f = bytearray(k)
+        f[rng.randrange(len(k))] ^= 1 << rng.randrange(8)
+        probes.append(bytes(f))
+        if kind == "bytes":
+            probes += [k[:-1] or b"\x01", k + b"\x01" if len(k) < 32 else k]
+    if kind != "bytes":
+        L = 8 if kind == "u64" else 4
+        probes = [p for p in probes if len(p) == L] + [rng.getrandbits(8 * L).to_bytes(L, "big") for _ in range(999)]
+    pin = _as_input(kind, probes)
+    exp = o.lookup(pin)
+    for lut in (0, 2, 3):
+        ix = C.Index(inp, vals, lut_bytes=lut)
+        assert np.array_equal(_lookup(ix, pin), exp)
+        assert to_records(ix.dump()) == o.dump_structure().tolist()
+        ix.close()
+    # updates with heavy duplication (last writer wins) + absent keys
+    ix = C.Index(inp, vals, lut_bytes=2)
+    m = 3 * len(probes)
+    pick = [rng.randrange(len(probes)) for _ in range(m)]
+    ukeys = [probes[i] for i in pick]
+    uvals = np.array([rng.getrandbits(63) for _ in range(m)], np.uint64)
+    uin = _as_input(kind, ukeys)
+    ix.update(_t(uin), _t(uvals))
+    o.update(uin, uvals)
+    assert np.array_equal(_lookup(ix, pin), o.lookup(pin))
+    assert to_records(ix.dump()) == o.dump_structure().tolist()
+    ix.close()
+
+
+def test_edge_cases():
+    # empty index: everything misses; n = 0 calls are no-ops
+    ix = C.Index(np.zeros(0, np.uint64), np.zeros(0, np.uint64), lut_bytes=0)
+    assert _lookup(ix, np.array([0, 1, 2**63], np.uint64)).tolist() == [MISS] * 3
+    ix.lookup(_t(np.zeros(0, np.uint64)), torch.empty(0, dtype=torch.int64, device=DEV))
+    ix.update(_t(np.zeros(0, np.uint64)), _t(np.zeros(0, np.uint64)))
+    ix.close()
+    # single key: root is a leaf
+    ix = C.Index(np.array([42], np.uint64), np.array([7], np.uint64), lut_bytes=3)
+    assert _lookup(ix, np.array([42, 43, 0], np.uint64)).tolist() == [7, MISS, MISS]
+    ix.close()
+    # ragged batch sizes around the CTA size
+    cfg = W.CONFIGS["c1"]
+    keys, vals = W.build_set(cfg)
+    ix = C.Index(keys, vals)
+    mp = MapOracle(keys, vals)
+    for m in (1, 255, 256, 257, 1000, 65_537):
+        q = W.lookup_batch(cfg, keys, 11, m)
+        assert np.array_equal(_lookup(ix, q), mp.lookup(q))
+    ix.close()
+
+
+def test_reserved_value_update_sets_sticky_error():
+    keys = np.array([1, 2, 3], np.uint64)
+    ix = C.Index(keys, np.array([10, 20, 30], np.uint64))
+    ix.update(_t(np.array([1, 2], np.uint64)), _t(np.array([MISS, 5], np.uint64)))
+    torch.cuda.synchronize()
+    assert ix.get_error() == 4
+    assert ix.get_error() == 0                       # cleared on read
+    assert _lookup(ix, keys).tolist() == [10, 5, 30]  # the rejected op is a no-op
+    ix.close()
+
+
+def test_host_buffer_paths_match_device():
+    cfg = W.CONFIGS["c1"]
+    keys, vals = W.build_set(cfg)
+    ix = C.Index(keys, vals, lut_bytes=3)
+    mp = MapOracle(keys, vals)
+    q = W.lookup_batch(cfg, keys)
+    assert np.array_equal(ix.lookup_host(q), mp.lookup(q))
+    uk, uv = W.update_batch(cfg, keys)
+    ix.update_host(uk, uv)
+    mp.update(uk, uv)
+    assert np.array_equal(ix.lookup_host(keys), mp.lookup(keys))
+    ix.close()
+
+
+def test_c2_full_size_sampled():
+    """Config 2 at full size (2^24 dense u32 keys, LUT over the first 3 bytes):
+    2^28 lookups in the bench's launch configuration; sampled outputs vs the
+    plain map, and the any-size property out[i] == value(q[i]) (100% hit)."""
+    cfg = W.CONFIGS["c2"]
+    keys, vals = W.build_set(cfg)
+    ix = C.Index(keys, vals, lut_bytes=3)
+    st = ix.stats()
+    assert st["n256"] == 1 + 256 + 65_536 and st["leaf8"] == 1 << 24   # Ex-C closed form
+    qd = W.lookup_batch_torch(cfg, torch.zeros(1, dtype=torch.int64, device=DEV), 0, cfg.n_lookups, device=DEV)
+    out = torch.empty(cfg.n_lookups, dtype=torch.int64, device=DEV)
+    ix.lookup(qd, out)
+    torch.cuda.synchronize()
+    # property at full size: value table gathered by key (dense keys: value index = key)
+    vt = torch.from_numpy(vals.view(np.int64)).to(DEV)
+    assert torch.equal(out, vt[qd.long()])
+    # sampled, element by element vs the plain-map oracle
+    idx = np.sort(np.random.default_rng(5).choice(cfg.n_lookups, 200_000, replace=False))
+    qs = W.lookup_at(cfg, None, idx)
+    assert np.array_equal(qd[torch.from_numpy(idx).to(DEV)].cpu().numpy().view(np.uint32), qs)
+    mp = MapOracle(keys, vals)
+    assert np.array_equal(_u64(out[torch.from_numpy(idx).to(DEV)]), mp.lookup(qs))
+    ix.close()
+
+
+@pytest.mark.slow
+def test_c3_full_size_sampled():
+    """Config 3 at full size: 2^26 random u64 keys, 2^30 lookups at 50% hit and
+    the 2^26-op update batch, in the bench's launch configuration; sampled
+    outputs vs the plain-map oracle (the generator recomputes any element)."""
+    cfg = W.CONFIGS["c3"]
+    keys_d = W.u64_keys_torch(3, cfg.n_keys, DEV)
+    keys = _u64(keys_d)
+    _, vals = W.build_set(W.Config("c3", "u64", cfg.n_keys, 0, 0, 0.5, ""))
+    ix = C.Index(keys, vals, lut_bytes=3)
+    n = cfg.n_lookups
+    out = torch.empty(n, dtype=torch.int64, device=DEV)
+    qd = W.lookup_batch_torch(cfg, keys_d, 0, n)
+    ix.lookup(qd, out)
+    uk, uv = W.update_batch_torch(cfg, keys_d)
+    ix.update(uk, uv)
+    out2 = torch.empty(1 << 22, dtype=torch.int64, device=DEV)
+    ix.lookup(keys_d[: 1 << 22], out2)
+    torch.cuda.synchronize()
+    assert ix.get_error() == 0
+    mp = MapOracle(keys, vals)
+    idx = np.sort(np.random.default_rng(3).choice(n, 300_000, replace=False))
+    qs = W.lookup_at(cfg, keys, idx)
+    ti = torch.from_numpy(idx).to(DEV)
+    assert np.array_equal(_u64(qd[ti]), qs)
+    got = _u64(out[ti])
+    assert np.array_equal(got, mp.lookup(qs))
+    hit = (out != -1).float().mean().item()
+    assert abs(hit - 0.5) < 0.001
+    mp.update(_u64(uk), _u64(uv))
+    assert np.array_equal(_u64(out2), mp.lookup(keys[: 1 << 22]))
+    ix.close()

@@ -114,15 +114,21 @@ def build_set(cfg: Config):
 
 
 def lookup_batch(cfg: Config, keys, start: int = 0, m: int | None = None):
-    """Lookup queries [start, start+m) of the config's stream.
+    """Lookup queries [start, start+m) of the config's stream (see lookup_at)."""
+    m = cfg.n_lookups - start if m is None else m
+    return lookup_at(cfg, keys, np.arange(start, start + m, dtype=np.uint64))
 
-    u64: query j is a hit (uniform key of the set) when the top bit of draw 2j is
-    clear and hit_ratio == 0.5, otherwise a guaranteed-absent key.  u32 (c2):
-    uniform over [0, 2^24) => 100% hit.
+
+def lookup_at(cfg: Config, keys, j) -> np.ndarray:
+    """Lookup queries at absolute stream positions j (any order, any subset).
+
+    u64: query j is a hit (uniform key of the set) when draw 2j < hit_ratio*2^64,
+    otherwise a guaranteed-absent key (counter >= n of the key bijection).
+    u32 (c2): uniform over [0, 2^24) => 100% hit.
     """
     c = config_id(cfg)
-    m = cfg.n_lookups - start if m is None else m
-    j = np.arange(start, start + m, dtype=np.uint64)
+    j = np.asarray(j, dtype=np.uint64)
+    m = j.shape[0]
     if cfg.kind == "u32":
         return (splitmix64(SEED_QUERIES + c, j) >> np.uint64(40)).astype(np.uint32)
     if cfg.kind == "u64":
@@ -220,3 +226,88 @@ def string_keys(c: int, n: int, max_len: int = MAX_KEY, min_len: int = 8):
         out_slots, out_lens = [allslots[first]], [alllens[first]]
         have = first.shape[0]
     return out_slots[0][:n].copy(), out_lens[0][:n].copy()
+
+
+# ----------------------------------------------------------------------------- torch twins
+# The same counter-based draws on torch tensors (CPU or CUDA), for generating the
+# full-size batches where they are consumed (device memory) without a host round
+# trip.  int64 arithmetic wraps modulo 2^64 exactly like uint64; logical right
+# shifts are emulated with a mask.  tests/test_workloads.py pins these to the
+# numpy versions bit for bit.
+def _t_srl(x, k):
+    import torch
+    return (x >> k) & ((1 << (64 - k)) - 1)
+
+
+def _t_const(v):
+    return v - (1 << 64) if v >= 1 << 63 else v
+
+
+def splitmix64_torch(seed: int, counter):
+    """torch int64 tensor of splitmix64(seed, counter) bit patterns."""
+    z = counter + 1
+    z = z * _t_const(0x9E3779B97F4A7C15) + _t_const(seed & MASK64)
+    z = (z ^ _t_srl(z, 30)) * _t_const(0xBF58476D1CE4E5B9)
+    z = (z ^ _t_srl(z, 27)) * _t_const(0x94D049BB133111EB)
+    return z ^ _t_srl(z, 31)
+
+
+def _t_ult(a, b_const: int):
+    """unsigned a < b for int64 bit patterns (b a Python int in [0, 2^64))."""
+    import torch
+    return (a ^ (-(1 << 63))) < _t_const(b_const ^ (1 << 63))
+
+
+def _t_umod(a, n: int):
+    """unsigned a mod n (n < 2^62) for int64 bit patterns."""
+    hi = _t_srl(a, 32)
+    lo = a & 0xFFFFFFFF
+    return (((hi % n) * ((1 << 32) % n)) % n + lo % n) % n
+
+
+def u64_keys_torch(c: int, n: int, device):
+    import torch
+    return splitmix64_torch(SEED_KEYS + c, torch.arange(n, dtype=torch.int64, device=device))
+
+
+def lookup_batch_torch(cfg: Config, keys, start: int = 0, m: int | None = None, device=None):
+    """torch twin of lookup_batch (u64 / u32 configs); returns int64 (u64) or int32 (u32) bits."""
+    import torch
+    c = config_id(cfg)
+    m = cfg.n_lookups - start if m is None else m
+    device = keys.device if device is None else device
+    j = torch.arange(start, start + m, dtype=torch.int64, device=device)
+    if cfg.kind == "u32":
+        return _t_srl(splitmix64_torch(SEED_QUERIES + c, j), 40).to(torch.int32)
+    n = keys.shape[0]
+    sel = splitmix64_torch(SEED_QUERIES + c, 2 * j)
+    pick = splitmix64_torch(SEED_QUERIES + c, 2 * j + 1)
+    del j
+    if cfg.hit_ratio >= 1.0:
+        hit = torch.ones(m, dtype=torch.bool, device=device)
+    else:
+        hit = _t_ult(sel, int(cfg.hit_ratio * 2**64) & MASK64)
+    del sel
+    out = splitmix64_torch(SEED_KEYS + c, torch.arange(start, start + m, dtype=torch.int64, device=device) + (n + (1 << 40)))
+    hk = keys[_t_umod(pick, n)]
+    del pick
+    return torch.where(hit, hk, out)
+
+
+def update_batch_torch(cfg: Config, keys, start: int = 0, m: int | None = None):
+    import torch
+    c = config_id(cfg)
+    m = cfg.n_updates - start if m is None else m
+    device = keys.device
+    j = torch.arange(start, start + m, dtype=torch.int64, device=device)
+    n = keys.shape[0]
+    sel = splitmix64_torch(SEED_UPDATES + c, 2 * j)
+    pick = splitmix64_torch(SEED_UPDATES + c, 2 * j + 1)
+    present = _t_ult(sel, int(0.9 * 2**64))
+    if cfg.kind != "u64":
+        raise ValueError(cfg.kind)
+    out = splitmix64_torch(SEED_KEYS + c, j + (n + (1 << 41)))
+    out = torch.where(present, keys[_t_umod(pick, n)], out)
+    vals = splitmix64_torch(SEED_UVALUES + c, j)
+    vals = torch.where(vals == -1, torch.zeros_like(vals), vals)
+    return out, vals
