@@ -85,7 +85,8 @@ typedef struct {
     uint32_t l2_persist;         /* 1: request a persisting L2 access-policy window over the
                                     LUT / top levels (cudaAccessPolicyWindow).               */
     int32_t device;              /* CUDA device ordinal; -1 = current device                */
-    uint32_t reserved;
+    uint32_t lut_entry_bytes;    /* 0 = auto, 8 = packed 64-bit links, 4 = compact 32-bit
+                                    entries (integer keys only; "compacted pointers") */
 } cuart_build_opts;
 #define CUART_LUT_AUTO 0xFFFFFFFFu
 

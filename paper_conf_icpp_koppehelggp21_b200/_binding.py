@@ -25,7 +25,7 @@ class _Keys(ctypes.Structure):
 
 class _Opts(ctypes.Structure):
     _fields_ = [("lut_bytes", ctypes.c_uint32), ("l2_persist", ctypes.c_uint32),
-                ("device", ctypes.c_int32), ("reserved", ctypes.c_uint32)]
+                ("device", ctypes.c_int32), ("lut_entry_bytes", ctypes.c_uint32)]
 
 
 class _Stats(ctypes.Structure):
@@ -131,8 +131,8 @@ def make_keys(keys, lengths=None):
     return st, n, (keys, lengths)
 
 
-def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1):
-    return _Opts(lut_bytes, l2_persist, device, 0)
+def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_entry_bytes=0):
+    return _Opts(lut_bytes, l2_persist, device, lut_entry_bytes)
 
 
 def _stream_ptr(stream):
@@ -145,14 +145,14 @@ def _stream_ptr(stream):
 
 
 # ------------------------------------------------------------------ hot path
-def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1):
+def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_entry_bytes=0):
     """Build + upload (host buffers).  Returns an opaque handle (int)."""
     k, n, keep = make_keys(keys)
     v = np.ascontiguousarray(values, dtype=np.uint64)
     if v.shape[0] != n:
         raise ValueError("values length mismatch")
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device)
+    o = _opts(lut_bytes, l2_persist, device, lut_entry_bytes)
     _check(lib().cuart_build(ctypes.byref(k), _ptr(v), n, ctypes.byref(o), ctypes.byref(h)), "cuart_build")
     return h.value
 
@@ -261,9 +261,9 @@ def cuart_layout_sectors(l, queries, threads=0):
     return out
 
 
-def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1):
+def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_entry_bytes=0):
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device)
+    o = _opts(lut_bytes, l2_persist, device, lut_entry_bytes)
     _check(lib().cuart_upload(l, ctypes.byref(o), ctypes.byref(h)), "cuart_upload")
     return h.value
 
@@ -306,14 +306,14 @@ class Layout:
 class Index:
     """Device-resident CuART index on one GPU."""
 
-    def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1):
-        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device)
+    def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_entry_bytes=0):
+        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_entry_bytes)
 
     @classmethod
-    def from_layout(cls, layout: "Layout", l2_persist=0, device=-1):
+    def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_entry_bytes=0):
         """Upload an already-built host layout (keeps the host copy usable)."""
         self = cls.__new__(cls)
-        self.h = cuart_upload(layout.h, 0, l2_persist, device)
+        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_entry_bytes)
         return self
 
     def lookup(self, queries, out=None, stream=None):

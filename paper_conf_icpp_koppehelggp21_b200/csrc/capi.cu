@@ -18,7 +18,10 @@
 #include <cuda_runtime.h>
 #include <string.h>
 
+#include <stdlib.h>
+
 #include <atomic>
+#include <vector>
 #include <new>
 
 #include "../../include/cuart.h"
@@ -57,8 +60,8 @@ struct cuart_index {
     uint64_t* stage_val[2] = {nullptr, nullptr};
     size_t stage_cap = 0;
     cudaStream_t streams[2] = {nullptr, nullptr};
-    bool l2_window = false;
-    size_t l2_window_bytes = 0;
+    int policy = 1;                    // cache-policy variant of the kernels (kernels.cuh Loader)
+    uint32_t lut_entry_bytes = 8;      // 8 = packed links, 4 = compact entries
 };
 
 static std::atomic<uint64_t> g_launches{0};
@@ -72,16 +75,19 @@ static std::atomic<uint64_t> g_launches{0};
     } while (0)
 
 // ============================================================================ kernels
-template <class Key>
+template <class Key, int POL>
 __global__ void __launch_bounds__(256) k_lookup(DevIndex ix, const void* __restrict__ q,
                                                 const uint8_t* __restrict__ lens, uint64_t n,
                                                 uint64_t* __restrict__ out) {
+    const Loader<POL> ld;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
-        const Key key = Key::load(q, lens, i);
+        const Key key = Key::template load<POL != 0>(q, lens, i);
         uint64_t val = kMiss;
-        const uint64_t leaf = find_leaf(ix, key, start_link(ix, key), val);
-        out[i] = leaf ? val : kMiss;
+        const uint64_t leaf = find_leaf(ix, ld, key, start_link(ix, ld, key), val);
+        const uint64_t r = leaf ? val : kMiss;
+        if (POL != 0) __stcs((unsigned long long*)out + i, (unsigned long long)r);
+        else out[i] = r;
     }
 }
 
@@ -90,15 +96,16 @@ __device__ __forceinline__ uint64_t global_leaf_id(const DevIndex& ix, uint64_t 
     return (t == T_LEAF8 ? ix.leaf_base[5] : t == T_LEAF16 ? ix.leaf_base[6] : ix.leaf_base[7]) + link_index(leaf);
 }
 
-template <class Key>
+template <class Key, int POL>
 __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restrict__ q, const uint8_t* __restrict__ lens,
                                               const uint64_t* __restrict__ vals, uint64_t n, uint64_t epoch_hi,
                                               uint64_t* __restrict__ leafref) {
+    const Loader<POL> ld;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
-        const Key key = Key::load(q, lens, i);
+        const Key key = Key::template load<POL != 0>(q, lens, i);
         uint64_t val;
-        uint64_t leaf = find_leaf(ix, key, start_link(ix, key), val);
+        uint64_t leaf = find_leaf(ix, ld, key, start_link(ix, ld, key), val);
         if (vals[i] == kMiss) {            // reserved value: op rejected, sticky error
             atomicOr(ix.err, 1u);
             leaf = 0;
@@ -141,11 +148,21 @@ static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const voi
                                   uint64_t* out, cudaStream_t s) {
     if (n == 0) return CUART_OK;
     const int grid = grid_for(h, n);
-    switch (kind) {
-    case CUART_KEY_U64: k_lookup<KeyU64><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out); break;
-    case CUART_KEY_U32: k_lookup<KeyU32><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out); break;
-    default: k_lookup<KeyBytes><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out); break;
+#define CUART_LOOKUP(K, P) k_lookup<K, P><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out)
+#define CUART_LOOKUP_POL(K)                          \
+    switch (h->policy) {                             \
+    case 0: CUART_LOOKUP(K, 0); break;               \
+    case 2: CUART_LOOKUP(K, 2); break;               \
+    case 3: CUART_LOOKUP(K, 3); break;               \
+    default: CUART_LOOKUP(K, 1); break;              \
     }
+    switch (kind) {
+    case CUART_KEY_U64: CUART_LOOKUP_POL(KeyU64); break;
+    case CUART_KEY_U32: CUART_LOOKUP_POL(KeyU32); break;
+    default: CUART_LOOKUP_POL(KeyBytes); break;
+    }
+#undef CUART_LOOKUP_POL
+#undef CUART_LOOKUP
     g_launches++;
     CU_TRY(cudaGetLastError());
     return CUART_OK;
@@ -178,11 +195,17 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
         const size_t kstride = kind == CUART_KEY_U64 ? 8 : kind == CUART_KEY_U32 ? 4 : 32;
         const void* kb = (const uint8_t*)k + base * kstride;
         const uint8_t* lb = lens ? lens + base : nullptr;
+#define CUART_UPD1(K, P) k_upd1<K, P><<<grid, 256, 0, s>>>(h->dix, kb, lb, vals + base, m, epoch_hi, h->leafref)
+#define CUART_UPD1_POL(K)                            \
+    if (h->policy == 0) CUART_UPD1(K, 0);            \
+    else CUART_UPD1(K, 1);
         switch (kind) {
-        case CUART_KEY_U64: k_upd1<KeyU64><<<grid, 256, 0, s>>>(h->dix, kb, lb, vals + base, m, epoch_hi, h->leafref); break;
-        case CUART_KEY_U32: k_upd1<KeyU32><<<grid, 256, 0, s>>>(h->dix, kb, lb, vals + base, m, epoch_hi, h->leafref); break;
-        default: k_upd1<KeyBytes><<<grid, 256, 0, s>>>(h->dix, kb, lb, vals + base, m, epoch_hi, h->leafref); break;
+        case CUART_KEY_U64: CUART_UPD1_POL(KeyU64); break;
+        case CUART_KEY_U32: CUART_UPD1_POL(KeyU32); break;
+        default: CUART_UPD1_POL(KeyBytes); break;
         }
+#undef CUART_UPD1_POL
+#undef CUART_UPD1
         g_launches++;
         CU_TRY(cudaGetLastError());
         k_upd2<<<grid, 256, 0, s>>>(h->dix, vals + base, m, epoch_hi, h->leafref);
@@ -277,6 +300,34 @@ cuart_status cuart_layout_sectors(const cuart_layout* l, const cuart_keys* q, si
     return CUART_OK;
 }
 
+// Compact 32-bit LUT (kernels.cuh expand_lut32): integer keys only, every entry must fit.
+static bool compact_lut(const HostLayout& L, std::vector<uint32_t>& out) {
+    if (L.lut.empty() || L.key_kind == CUART_KEY_BYTES) return false;
+    out.resize(L.lut.size());
+    for (size_t i = 0; i < L.lut.size(); i++) {
+        const uint64_t l = L.lut[i];
+        const uint32_t t = link_type(l);
+        const uint64_t idx = link_index(l);
+        if (t == T_NULL) { out[i] = 0; continue; }
+        if (t >= T_LEAF8) {
+            if (idx > 0x1FFFFFFFull) return false;
+            out[i] = (t << 29) | uint32_t(idx);
+        } else {
+            const uint32_t rel = link_aux(l) - L.lut_bytes;
+            if (link_aux(l) < L.lut_bytes || rel > 6 || idx > 0x3FFFFFFull) return false;
+            out[i] = (t << 29) | (rel << 26) | uint32_t(idx);
+        }
+    }
+    return true;
+}
+
+static uint64_t expand_lut32_host(uint32_t e, uint32_t k, uint32_t leaf_len) {
+    const uint32_t t = e >> 29;
+    if (t == T_NULL) return 0;
+    if (t >= T_LEAF8) return make_link(t, leaf_len, e & 0x1FFFFFFFu);
+    return make_link(t, k + ((e >> 26) & 7u), e & 0x3FFFFFFu);
+}
+
 cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts, cuart_index** out) {
     if (!lay || !out) return CUART_ERR_INVALID_ARGUMENT;
     *out = nullptr;
@@ -307,8 +358,14 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     h->total_leaves = L.count[5] + L.count[6] + L.count[7];
     h->winner_off = off;
     off = align(off + h->total_leaves * 8);
+    std::vector<uint32_t> lut32;
+    const uint32_t want = opts ? opts->lut_entry_bytes : 0;
+    if (want != 8 && compact_lut(L, lut32)) h->lut_entry_bytes = 4;
+    else if (want == 4 && !L.lut.empty()) { delete h; return CUART_ERR_INVALID_ARGUMENT; }
+    else lut32.clear();
+    if (const char* pe = getenv("CUART_POLICY")) h->policy = atoi(pe);
     h->lut_off = off;
-    off = align(off + L.lut.size() * 8);
+    off = align(off + (lut32.empty() ? L.lut.size() * 8 : lut32.size() * 4));
     h->err_off = off;
     off = align(off + 256);
     h->arena_bytes = off;
@@ -321,7 +378,10 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     for (int t = 1; t < 8 && rc == CUART_OK; t++)
         if (!L.buf[t].empty() && cudaMemcpy(h->arena + h->off[t], L.buf[t].data(), L.buf[t].size(), cudaMemcpyHostToDevice) != cudaSuccess)
             rc = CUART_ERR_CUDA;
-    if (rc == CUART_OK && !L.lut.empty() &&
+    if (rc == CUART_OK && !lut32.empty() &&
+        cudaMemcpy(h->arena + h->lut_off, lut32.data(), lut32.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)
+        rc = CUART_ERR_CUDA;
+    if (rc == CUART_OK && lut32.empty() && !L.lut.empty() &&
         cudaMemcpy(h->arena + h->lut_off, L.lut.data(), L.lut.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && h->total_leaves && cudaMemset(h->arena + h->winner_off, 0, h->total_leaves * 8) != cudaSuccess)
@@ -336,8 +396,10 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     for (int t = 1; t < 8; t++) d.base[t] = h->arena + h->off[t];
     d.base[0] = nullptr;
     d.root = L.root;
-    d.lut = L.lut.empty() ? nullptr : (const uint64_t*)(h->arena + h->lut_off);
+    d.lut = (L.lut.empty() || !lut32.empty()) ? nullptr : (const uint64_t*)(h->arena + h->lut_off);
+    d.lut32 = lut32.empty() ? nullptr : (const uint32_t*)(h->arena + h->lut_off);
     d.lut_bytes = L.lut_bytes;
+    d.fixed_len = L.key_kind == CUART_KEY_U64 ? 8 : L.key_kind == CUART_KEY_U32 ? 4 : 0;
     d.key_kind = L.key_kind;
     d.winner = (uint64_t*)(h->arena + h->winner_off);
     d.leaf_base[5] = 0;
@@ -473,7 +535,7 @@ cuart_status cuart_stats(const cuart_index* h, cuart_stats_t* s) {
     s->n_keys = h->n_keys;
     s->lut_bytes = h->lut_bytes;
     s->lut_entries = h->lut_bytes ? (uint64_t(1) << (8 * h->lut_bytes)) : 0;
-    s->lut_bytes_total = s->lut_entries * 8;
+    s->lut_bytes_total = s->lut_entries * h->lut_entry_bytes;
     s->arena_bytes = h->arena_bytes + h->leafref_cap * 8;
     s->key_kind = h->key_kind;
     s->root = h->root;
@@ -506,7 +568,14 @@ cuart_status cuart_dump(const cuart_index* h, cuart_layout** out) {
         }
         if (h->lut_bytes) {
             L.lut.resize(uint64_t(1) << (8 * h->lut_bytes));
-            if (cudaMemcpy(L.lut.data(), h->arena + h->lut_off, L.lut.size() * 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+            if (h->lut_entry_bytes == 4) {
+                std::vector<uint32_t> c(L.lut.size());
+                if (cudaMemcpy(c.data(), h->arena + h->lut_off, c.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
+                    delete l;
+                    return CUART_ERR_CUDA;
+                }
+                for (size_t i = 0; i < c.size(); i++) L.lut[i] = expand_lut32_host(c[i], h->lut_bytes, h->dix.fixed_len);
+            } else if (cudaMemcpy(L.lut.data(), h->arena + h->lut_off, L.lut.size() * 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
                 delete l;
                 return CUART_ERR_CUDA;
             }

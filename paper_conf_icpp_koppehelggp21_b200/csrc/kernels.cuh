@@ -17,7 +17,9 @@ struct DevIndex {
     const uint8_t* base[8];       // record buffers per type code
     uint64_t root;                // packed root link
     const uint64_t* lut;          // root lookup table, or nullptr
+    const uint32_t* lut32;        // compact 32-bit root lookup table, or nullptr
     uint32_t lut_bytes;
+    uint32_t fixed_len;           // key length of integer kinds (4 / 8), 0 for byte strings
     uint32_t key_kind;
     uint64_t* winner;             // per-leaf conflict word for updates (global leaf id)
     uint64_t leaf_base[8];        // global leaf id = leaf_base[type] + index
@@ -58,15 +60,18 @@ __device__ __forceinline__ uint64_t bswap64(uint64_t x) {
 struct KeyU64 {
     uint64_t k;
     static constexpr uint32_t kKind = 2;
+    template <bool STREAM>
     __device__ __forceinline__ static KeyU64 load(const void* q, const uint8_t*, uint64_t i) {
-        return KeyU64{((const uint64_t*)q)[i]};
+        const unsigned long long* p = (const unsigned long long*)q + i;
+        return KeyU64{STREAM ? uint64_t(__ldcs(p)) : uint64_t(*p)};
     }
     __device__ __forceinline__ uint32_t len() const { return 8; }
     __device__ __forceinline__ uint32_t byte(uint32_t d) const { return uint32_t(k >> (56 - 8 * d)) & 0xFF; }
     __device__ __forceinline__ uint64_t prefix(uint32_t nb) const { return k >> (64 - 8 * nb); }
     // One 16-byte load brings key and value of a leaf8 record.
-    __device__ __forceinline__ bool leaf_match(const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
-        const uint4 r = ld_nc_v4(rec);
+    template <class LD>
+    __device__ __forceinline__ bool leaf_match(const LD& ld, const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
+        const uint4 r = ld.leafv4(rec);
         val = uint64_t(r.z) | (uint64_t(r.w) << 32);
         return aux == 8 && (uint64_t(r.x) | (uint64_t(r.y) << 32)) == bswap64(k);
     }
@@ -75,14 +80,17 @@ struct KeyU64 {
 struct KeyU32 {
     uint32_t k;
     static constexpr uint32_t kKind = 1;
+    template <bool STREAM>
     __device__ __forceinline__ static KeyU32 load(const void* q, const uint8_t*, uint64_t i) {
-        return KeyU32{((const uint32_t*)q)[i]};
+        const unsigned int* p = (const unsigned int*)q + i;
+        return KeyU32{STREAM ? uint32_t(__ldcs(p)) : uint32_t(*p)};
     }
     __device__ __forceinline__ uint32_t len() const { return 4; }
     __device__ __forceinline__ uint32_t byte(uint32_t d) const { return (k >> (24 - 8 * d)) & 0xFF; }
     __device__ __forceinline__ uint64_t prefix(uint32_t nb) const { return uint64_t(k) >> (32 - 8 * nb); }
-    __device__ __forceinline__ bool leaf_match(const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
-        const uint4 r = ld_nc_v4(rec);
+    template <class LD>
+    __device__ __forceinline__ bool leaf_match(const LD& ld, const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
+        const uint4 r = ld.leafv4(rec);
         val = uint64_t(r.z) | (uint64_t(r.w) << 32);
         return aux == 4 && r.y == 0 && r.x == __byte_perm(k, 0, 0x0123);
     }
@@ -93,10 +101,12 @@ struct KeyBytes {
     uint64_t w[4];   // little-endian words of the zero-padded slot
     uint32_t l;
     static constexpr uint32_t kKind = 3;
+    template <bool STREAM>
     __device__ __forceinline__ static KeyBytes load(const void* q, const uint8_t* lens, uint64_t i) {
         KeyBytes kb;
-        const uint4 a = *((const uint4*)q + 2 * i);
-        const uint4 b = *((const uint4*)q + 2 * i + 1);
+        const uint4* pq = (const uint4*)q + 2 * i;
+        const uint4 a = STREAM ? __ldcs(pq) : pq[0];
+        const uint4 b = STREAM ? __ldcs(pq + 1) : pq[1];
         kb.w[0] = uint64_t(a.x) | (uint64_t(a.y) << 32);
         kb.w[1] = uint64_t(a.z) | (uint64_t(a.w) << 32);
         kb.w[2] = uint64_t(b.x) | (uint64_t(b.y) << 32);
@@ -121,20 +131,21 @@ struct KeyBytes {
         for (uint32_t b = 0; b < nb; b++) p = (p << 8) | byte(b);
         return p;
     }
-    __device__ __forceinline__ bool leaf_match(const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
-        const uint4 a = ld_nc_v4(rec);
+    template <class LD>
+    __device__ __forceinline__ bool leaf_match(const LD& ld, const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
+        const uint4 a = ld.leafv4(rec);
         const uint64_t a0 = uint64_t(a.x) | (uint64_t(a.y) << 32), a1 = uint64_t(a.z) | (uint64_t(a.w) << 32);
         if (t == T_LEAF8) {
             val = a1;
             return aux == l && a0 == w[0];
         }
-        const uint4 b = ld_nc_v4(rec + 16);
+        const uint4 b = ld.leafv4(rec + 16);
         const uint64_t b0 = uint64_t(b.x) | (uint64_t(b.y) << 32), b1 = uint64_t(b.z) | (uint64_t(b.w) << 32);
         if (t == T_LEAF16) {
             val = b0;
             return aux == l && a0 == w[0] && a1 == w[1];
         }
-        const uint4 c = ld_nc_v4(rec + 32);
+        const uint4 c = ld.leafv4(rec + 32);
         val = uint64_t(c.x) | (uint64_t(c.y) << 32);
         return aux == l && a0 == w[0] && a1 == w[1] && b0 == w[2] && b1 == w[3];
     }
@@ -146,10 +157,61 @@ __device__ __forceinline__ void search4(uint32_t keys, uint32_t bb, uint32_t& le
     eq = __vcmpeq4(keys, bb);
 }
 
+// Cache policy for the three kinds of dependent loads (B200 L2 is 126 MB; the
+// structure of a large index is not).  POL 0: plain ld.global.nc everywhere.
+// POL 1: LUT evict_last (keep the root table L2-resident), leaves evict_first.
+// POL 2: as 1 and inner nodes evict_first too.  POL 3: LUT evict_last only.
+template <int POL>
+struct Loader {
+    uint64_t keep, drop;
+    __device__ __forceinline__ Loader() {
+        if (POL != 0) {
+            asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(keep));
+            asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(drop));
+        }
+    }
+    __device__ __forceinline__ static uint64_t u64(const void* p, uint64_t pol) {
+        uint64_t v;
+        asm volatile("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+        return v;
+    }
+    __device__ __forceinline__ static uint32_t u32(const void* p, uint64_t pol) {
+        uint32_t v;
+        asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+        return v;
+    }
+    __device__ __forceinline__ static uint32_t u8(const void* p, uint64_t pol) {
+        uint16_t v;
+        asm volatile("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol));
+        return v;
+    }
+    __device__ __forceinline__ static uint4 v4(const void* p, uint64_t pol) {
+        uint4 v;
+        asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                     : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol));
+        return v;
+    }
+    // LUT entries
+    __device__ __forceinline__ uint64_t lut64(const void* p) const { return POL ? u64(p, keep) : ld_nc_u64(p); }
+    __device__ __forceinline__ uint32_t lut32(const void* p) const {
+        if (POL) return u32(p, keep);
+        uint32_t v;
+        asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(v) : "l"(p));
+        return v;
+    }
+    // inner nodes
+    __device__ __forceinline__ uint64_t node64(const void* p) const { return POL == 2 ? u64(p, drop) : ld_nc_u64(p); }
+    __device__ __forceinline__ uint32_t node8(const void* p) const { return POL == 2 ? u8(p, drop) : ld_nc_u8(p); }
+    __device__ __forceinline__ uint4 nodev4(const void* p) const { return POL == 2 ? v4(p, drop) : ld_nc_v4(p); }
+    // leaves
+    __device__ __forceinline__ uint4 leafv4(const void* p) const { return (POL == 1 || POL == 2) ? v4(p, drop) : ld_nc_v4(p); }
+};
+
 // Walk from `link` to a leaf.  Returns the leaf link on a full-key match (its value
 // in `val`), 0 otherwise.
-template <class Key>
-__device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Key& key, uint64_t link, uint64_t& val) {
+template <class Key, int POL>
+__device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Loader<POL>& ld, const Key& key, uint64_t link,
+                                              uint64_t& val) {
     const uint32_t len = key.len();
 #pragma unroll 1
     for (;;) {
@@ -158,19 +220,19 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Key& key
         const uint32_t aux = link_aux(link);
         if (t >= T_LEAF8) {
             const uint8_t* rec = ix.base[t] + idx * record_bytes(t);
-            return key.leaf_match(rec, t, aux, val) ? link : 0;
+            return key.leaf_match(ld, rec, t, aux, val) ? link : 0;
         }
         if (t == T_NULL || aux >= len) return 0;
         const uint32_t b = key.byte(aux);
         const uint8_t* rec = ix.base[t] + idx * record_bytes(t);
         if (t == T_N256) {
-            link = ld_nc_u64(rec + kN256Child + 8 * b);
+            link = ld.node64(rec + kN256Child + 8 * b);
         } else if (t == T_N48) {
-            const uint32_t s = ld_nc_u8(rec + kN48Index + b);
+            const uint32_t s = ld.node8(rec + kN48Index + b);
             if (s == kN48Empty) return 0;
-            link = ld_nc_u64(rec + kN48Child + 8 * s);
+            link = ld.node64(rec + kN48Child + 8 * s);
         } else if (t == T_N16) {
-            const uint4 k4 = ld_nc_v4(rec + kN16Keys);
+            const uint4 k4 = ld.nodev4(rec + kN16Keys);
             const uint32_t bb = b * 0x01010101u;
             uint32_t l0, l1, l2, l3, e0, e1, e2, e3;
             search4(k4.x, bb, l0, e0);
@@ -178,11 +240,11 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Key& key
             search4(k4.z, bb, l2, e2);
             search4(k4.w, bb, l3, e3);
             if ((e0 | e1 | e2 | e3) == 0) return 0;
-            link = ld_nc_u64(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
+            link = ld.node64(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
         } else {  // N4: whole 64-byte record in one round trip
-            const uint4 h = ld_nc_v4(rec + 16);          // keys[4] | pad | child[0]
-            const uint4 c12 = ld_nc_v4(rec + 32);        // child[1], child[2]
-            const uint64_t c3 = ld_nc_u64(rec + 48);     // child[3]
+            const uint4 h = ld.nodev4(rec + 16);          // keys[4] | pad | child[0]
+            const uint4 c12 = ld.nodev4(rec + 32);        // child[1], child[2]
+            const uint64_t c3 = ld.node64(rec + 48);      // child[3]
             uint32_t less, eq;
             search4(h.x, b * 0x01010101u, less, eq);
             if (eq == 0) return 0;
@@ -194,11 +256,23 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Key& key
     }
 }
 
-template <class Key>
-__device__ __forceinline__ uint64_t start_link(const DevIndex& ix, const Key& key) {
-    if (ix.lut_bytes && key.len() >= ix.lut_bytes) return ld_nc_u64(ix.lut + key.prefix(ix.lut_bytes));
-    return ix.root;
+// Compact 32-bit LUT entry (integer keys only; layout.h): [31:29] type; leaves
+// [28:0] index; inner nodes [28:26] branch depth - k, [25:0] index.
+__device__ __forceinline__ uint64_t expand_lut32(uint32_t e, uint32_t k, uint32_t leaf_len) {
+    const uint32_t t = e >> 29;
+    if (t == T_NULL) return 0;
+    if (t >= T_LEAF8) return make_link(t, leaf_len, e & 0x1FFFFFFFu);
+    return make_link(t, k + ((e >> 26) & 7u), e & 0x3FFFFFFu);
 }
 
+template <class Key, int POL>
+__device__ __forceinline__ uint64_t start_link(const DevIndex& ix, const Loader<POL>& ld, const Key& key) {
+    if (ix.lut_bytes && key.len() >= ix.lut_bytes) {
+        const uint64_t p = key.prefix(ix.lut_bytes);
+        if (ix.lut32) return expand_lut32(ld.lut32(ix.lut32 + p), ix.lut_bytes, ix.fixed_len);
+        return ld.lut64(ix.lut + p);
+    }
+    return ix.root;
+}
 
 }  // namespace cuart

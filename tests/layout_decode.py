@@ -68,7 +68,7 @@ def to_records(view) -> list[int]:
             k, v, pad = leaf(view, link)
             assert pad == b"\0" * len(pad), "leaf key padding must be zero"
             assert t == (5 if len(k) <= 8 else 6 if len(k) <= 16 else 7), "leaf class by key length (P:110)"
-            out.extend([0, len(k), *k, v])
+            out.extend([0, len(k), *k, v - (1 << 64) if v >= 1 << 63 else v])   # oracle dumps int64
             return
         b = view["buf"][t]
         o = idx * REC[t]
