@@ -85,9 +85,17 @@ typedef struct {
     uint32_t l2_persist;         /* 1: request a persisting L2 access-policy window over the
                                     LUT / top levels (cudaAccessPolicyWindow).               */
     int32_t device;              /* CUDA device ordinal; -1 = current device                */
-    uint32_t lut_entry_bytes;    /* 0 = auto, 8 = packed 64-bit links, 4 = compact 32-bit
-                                    entries (integer keys only; "compacted pointers") */
+    uint32_t lut_format;         /* device form of the root table ("compacted pointers"):
+                                    CUART_LUT_FORMAT_AUTO, CUART_LUT_LINKS (8-B links),
+                                    CUART_LUT_COMPACT32 (4-B entries), CUART_LUT_RANK (64-B
+                                    blocks per 64 entries: type bit-planes + per-type base
+                                    index + rank; 1 B/entry, sized for L2 residency).
+                                    COMPACT32 / RANK need integer keys (else LINKS).        */
 } cuart_build_opts;
+#define CUART_LUT_FORMAT_AUTO 0u
+#define CUART_LUT_LINKS 1u
+#define CUART_LUT_COMPACT32 2u
+#define CUART_LUT_RANK 3u
 #define CUART_LUT_AUTO 0xFFFFFFFFu
 
 /* Per-node-type counts and bytes of an index (type codes P:108). */
@@ -102,7 +110,8 @@ typedef struct {
     uint32_t key_kind;
     uint64_t root;               /* packed root link */
     uint32_t max_depth;          /* longest root-to-leaf node chain */
-    uint32_t reserved;
+    uint32_t lut_format;         /* CUART_LUT_* in use on the device */
+    uint64_t lut_exceptions;     /* RANK: entries served by the 64-bit link table */
 } cuart_stats_t;
 
 typedef struct cuart_index cuart_index;    /* device-resident index (opaque) */

@@ -11,6 +11,7 @@ CUART_MISS = 0xFFFFFFFFFFFFFFFF
 CUART_MAX_KEY = 32
 KIND_U32, KIND_U64, KIND_BYTES = 1, 2, 3
 CUART_LUT_AUTO = 0xFFFFFFFF
+LUT_FORMAT_AUTO, LUT_LINKS, LUT_COMPACT32, LUT_RANK = 0, 1, 2, 3
 
 
 class CuartError(RuntimeError):
@@ -25,14 +26,15 @@ class _Keys(ctypes.Structure):
 
 class _Opts(ctypes.Structure):
     _fields_ = [("lut_bytes", ctypes.c_uint32), ("l2_persist", ctypes.c_uint32),
-                ("device", ctypes.c_int32), ("lut_entry_bytes", ctypes.c_uint32)]
+                ("device", ctypes.c_int32), ("lut_format", ctypes.c_uint32)]
 
 
 class _Stats(ctypes.Structure):
     _fields_ = [("count", ctypes.c_uint64 * 8), ("bytes", ctypes.c_uint64 * 8), ("n_keys", ctypes.c_uint64),
                 ("lut_entries", ctypes.c_uint64), ("lut_bytes_total", ctypes.c_uint64),
                 ("arena_bytes", ctypes.c_uint64), ("lut_bytes", ctypes.c_uint32), ("key_kind", ctypes.c_uint32),
-                ("root", ctypes.c_uint64), ("max_depth", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+                ("root", ctypes.c_uint64), ("max_depth", ctypes.c_uint32), ("lut_format", ctypes.c_uint32),
+                ("lut_exceptions", ctypes.c_uint64)]
 
 
 class _View(ctypes.Structure):
@@ -131,8 +133,8 @@ def make_keys(keys, lengths=None):
     return st, n, (keys, lengths)
 
 
-def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_entry_bytes=0):
-    return _Opts(lut_bytes, l2_persist, device, lut_entry_bytes)
+def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0):
+    return _Opts(lut_bytes, l2_persist, device, lut_format)
 
 
 def _stream_ptr(stream):
@@ -145,14 +147,14 @@ def _stream_ptr(stream):
 
 
 # ------------------------------------------------------------------ hot path
-def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_entry_bytes=0):
+def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0):
     """Build + upload (host buffers).  Returns an opaque handle (int)."""
     k, n, keep = make_keys(keys)
     v = np.ascontiguousarray(values, dtype=np.uint64)
     if v.shape[0] != n:
         raise ValueError("values length mismatch")
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_entry_bytes)
+    o = _opts(lut_bytes, l2_persist, device, lut_format)
     _check(lib().cuart_build(ctypes.byref(k), _ptr(v), n, ctypes.byref(o), ctypes.byref(h)), "cuart_build")
     return h.value
 
@@ -207,7 +209,8 @@ def _stats_dict(s):
     d = {names[t]: int(s.count[t]) for t in names}
     d.update({f"{names[t]}_bytes": int(s.bytes[t]) for t in names})
     d.update(n_keys=int(s.n_keys), lut_bytes=int(s.lut_bytes), lut_entries=int(s.lut_entries),
-             arena_bytes=int(s.arena_bytes), root=int(s.root), max_depth=int(s.max_depth), key_kind=int(s.key_kind))
+             arena_bytes=int(s.arena_bytes), root=int(s.root), max_depth=int(s.max_depth), key_kind=int(s.key_kind),
+             lut_format=int(s.lut_format), lut_exceptions=int(s.lut_exceptions))
     return d
 
 
@@ -261,9 +264,9 @@ def cuart_layout_sectors(l, queries, threads=0):
     return out
 
 
-def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_entry_bytes=0):
+def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_format=0):
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_entry_bytes)
+    o = _opts(lut_bytes, l2_persist, device, lut_format)
     _check(lib().cuart_upload(l, ctypes.byref(o), ctypes.byref(h)), "cuart_upload")
     return h.value
 
@@ -306,14 +309,14 @@ class Layout:
 class Index:
     """Device-resident CuART index on one GPU."""
 
-    def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_entry_bytes=0):
-        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_entry_bytes)
+    def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0):
+        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_format)
 
     @classmethod
-    def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_entry_bytes=0):
+    def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_format=0):
         """Upload an already-built host layout (keeps the host copy usable)."""
         self = cls.__new__(cls)
-        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_entry_bytes)
+        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format)
         return self
 
     def lookup(self, queries, out=None, stream=None):

@@ -61,7 +61,9 @@ struct cuart_index {
     size_t stage_cap = 0;
     cudaStream_t streams[2] = {nullptr, nullptr};
     int policy = 1;                    // cache-policy variant of the kernels (kernels.cuh Loader)
-    uint32_t lut_entry_bytes = 8;      // 8 = packed links, 4 = compact entries
+    uint32_t lut_format = CUART_LUT_LINKS;
+    uint64_t lutc_off = 0;             // compact / rank LUT region
+    uint64_t lut_exceptions = 0;       // RANK: entries served by the 64-bit table
 };
 
 static std::atomic<uint64_t> g_launches{0};
@@ -328,6 +330,54 @@ static uint64_t expand_lut32_host(uint32_t e, uint32_t k, uint32_t leaf_len) {
     return make_link(t, k + ((e >> 26) & 7u), e & 0x3FFFFFFu);
 }
 
+// Rank LUT (kernels.cuh expand_lut_rank): 64-entry blocks of 64 B —
+//   u64 plane[3] (type code bits of each entry), u64 exc (entry lives in the 64-bit
+//   link table), u32 base[8] (index of the first entry of each type in the block).
+// An entry is encoded in the block when its target's index is base[type] + (number
+// of earlier entries of that type in the block), its branch depth is k (inner) and
+// its key length is the index's fixed length (leaves).  Everything else is marked
+// as an exception and read from the full 64-bit table.  Integer keys only.
+static bool rank_lut(const HostLayout& L, std::vector<uint64_t>& blocks, uint64_t& n_exc) {
+    if (L.lut.empty() || L.key_kind == CUART_KEY_BYTES) return false;
+    const uint32_t k = L.lut_bytes;
+    const uint32_t flen = L.key_kind == CUART_KEY_U64 ? 8 : 4;
+    const uint64_t nb = L.lut.size() / 64;
+    blocks.assign(nb * 8, 0);
+    n_exc = 0;
+    for (uint64_t bi = 0; bi < nb; bi++) {
+        uint64_t plane[3] = {0, 0, 0}, exc = 0;
+        uint32_t base[8] = {0};
+        uint64_t cnt[8] = {0};
+        for (uint32_t j = 0; j < 64; j++) {
+            const uint64_t l = L.lut[bi * 64 + j];
+            const uint32_t t = link_type(l);
+            if (t == T_NULL) continue;
+            const uint64_t idx = link_index(l);
+            bool ok = (t >= T_LEAF8) ? (link_aux(l) == flen) : (link_aux(l) == k);
+            if (ok && cnt[t] == 0) {
+                if (idx > 0xFFFFFFFFull) ok = false;
+                else base[t] = uint32_t(idx);
+            }
+            if (ok && idx != uint64_t(base[t]) + cnt[t]) ok = false;
+            if (!ok) {
+                exc |= 1ull << j;
+                n_exc++;
+                continue;
+            }
+            cnt[t]++;
+            for (int pb = 0; pb < 3; pb++)
+                if (t & (1u << pb)) plane[pb] |= 1ull << j;
+        }
+        uint64_t* blk = &blocks[bi * 8];
+        blk[0] = plane[0];
+        blk[1] = plane[1];
+        blk[2] = plane[2];
+        blk[3] = exc;
+        for (int t = 0; t < 8; t += 2) blk[4 + t / 2] = uint64_t(base[t]) | (uint64_t(base[t + 1]) << 32);
+    }
+    return true;
+}
+
 cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts, cuart_index** out) {
     if (!lay || !out) return CUART_ERR_INVALID_ARGUMENT;
     *out = nullptr;
@@ -359,13 +409,24 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     h->winner_off = off;
     off = align(off + h->total_leaves * 8);
     std::vector<uint32_t> lut32;
-    const uint32_t want = opts ? opts->lut_entry_bytes : 0;
-    if (want != 8 && compact_lut(L, lut32)) h->lut_entry_bytes = 4;
-    else if (want == 4 && !L.lut.empty()) { delete h; return CUART_ERR_INVALID_ARGUMENT; }
-    else lut32.clear();
+    std::vector<uint64_t> lutr;
+    uint32_t fmt = opts ? opts->lut_format : CUART_LUT_FORMAT_AUTO;
+    if (L.lut.empty()) fmt = CUART_LUT_LINKS;
+    if (fmt == CUART_LUT_FORMAT_AUTO) fmt = (L.key_kind == CUART_KEY_BYTES) ? CUART_LUT_LINKS : CUART_LUT_RANK;
+    if (fmt == CUART_LUT_RANK && !rank_lut(L, lutr, h->lut_exceptions)) fmt = CUART_LUT_LINKS;
+    if (fmt == CUART_LUT_COMPACT32 && !compact_lut(L, lut32)) fmt = CUART_LUT_LINKS;
+    if (fmt < CUART_LUT_LINKS || fmt > CUART_LUT_RANK) {
+        delete h;
+        return CUART_ERR_INVALID_ARGUMENT;
+    }
+    h->lut_format = fmt;
     if (const char* pe = getenv("CUART_POLICY")) h->policy = atoi(pe);
+    // LUT region: 64-bit links (LINKS, and the exception table of RANK) then the compact form
     h->lut_off = off;
-    off = align(off + (lut32.empty() ? L.lut.size() * 8 : lut32.size() * 4));
+    const bool need_links = fmt == CUART_LUT_LINKS || fmt == CUART_LUT_RANK;
+    if (need_links) off = align(off + L.lut.size() * 8);
+    h->lutc_off = off;
+    off = align(off + lut32.size() * 4 + lutr.size() * 8);
     h->err_off = off;
     off = align(off + 256);
     h->arena_bytes = off;
@@ -378,11 +439,14 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     for (int t = 1; t < 8 && rc == CUART_OK; t++)
         if (!L.buf[t].empty() && cudaMemcpy(h->arena + h->off[t], L.buf[t].data(), L.buf[t].size(), cudaMemcpyHostToDevice) != cudaSuccess)
             rc = CUART_ERR_CUDA;
-    if (rc == CUART_OK && !lut32.empty() &&
-        cudaMemcpy(h->arena + h->lut_off, lut32.data(), lut32.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)
-        rc = CUART_ERR_CUDA;
-    if (rc == CUART_OK && lut32.empty() && !L.lut.empty() &&
+    if (rc == CUART_OK && need_links && !L.lut.empty() &&
         cudaMemcpy(h->arena + h->lut_off, L.lut.data(), L.lut.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
+        rc = CUART_ERR_CUDA;
+    if (rc == CUART_OK && !lut32.empty() &&
+        cudaMemcpy(h->arena + h->lutc_off, lut32.data(), lut32.size() * 4, cudaMemcpyHostToDevice) != cudaSuccess)
+        rc = CUART_ERR_CUDA;
+    if (rc == CUART_OK && !lutr.empty() &&
+        cudaMemcpy(h->arena + h->lutc_off, lutr.data(), lutr.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && h->total_leaves && cudaMemset(h->arena + h->winner_off, 0, h->total_leaves * 8) != cudaSuccess)
         rc = CUART_ERR_CUDA;
@@ -396,8 +460,9 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     for (int t = 1; t < 8; t++) d.base[t] = h->arena + h->off[t];
     d.base[0] = nullptr;
     d.root = L.root;
-    d.lut = (L.lut.empty() || !lut32.empty()) ? nullptr : (const uint64_t*)(h->arena + h->lut_off);
-    d.lut32 = lut32.empty() ? nullptr : (const uint32_t*)(h->arena + h->lut_off);
+    d.lut = need_links ? (const uint64_t*)(h->arena + h->lut_off) : nullptr;
+    d.lut32 = lut32.empty() ? nullptr : (const uint32_t*)(h->arena + h->lutc_off);
+    d.lutr = lutr.empty() ? nullptr : (const uint4*)(h->arena + h->lutc_off);
     d.lut_bytes = L.lut_bytes;
     d.fixed_len = L.key_kind == CUART_KEY_U64 ? 8 : L.key_kind == CUART_KEY_U32 ? 4 : 0;
     d.key_kind = L.key_kind;
@@ -535,7 +600,10 @@ cuart_status cuart_stats(const cuart_index* h, cuart_stats_t* s) {
     s->n_keys = h->n_keys;
     s->lut_bytes = h->lut_bytes;
     s->lut_entries = h->lut_bytes ? (uint64_t(1) << (8 * h->lut_bytes)) : 0;
-    s->lut_bytes_total = s->lut_entries * h->lut_entry_bytes;
+    s->lut_bytes_total = h->lut_format == CUART_LUT_COMPACT32 ? s->lut_entries * 4
+                       : h->lut_format == CUART_LUT_RANK ? s->lut_entries * 9 : s->lut_entries * 8;
+    s->lut_format = h->lut_format;
+    s->lut_exceptions = h->lut_exceptions;
     s->arena_bytes = h->arena_bytes + h->leafref_cap * 8;
     s->key_kind = h->key_kind;
     s->root = h->root;
@@ -568,9 +636,9 @@ cuart_status cuart_dump(const cuart_index* h, cuart_layout** out) {
         }
         if (h->lut_bytes) {
             L.lut.resize(uint64_t(1) << (8 * h->lut_bytes));
-            if (h->lut_entry_bytes == 4) {
+            if (h->lut_format == CUART_LUT_COMPACT32) {
                 std::vector<uint32_t> c(L.lut.size());
-                if (cudaMemcpy(c.data(), h->arena + h->lut_off, c.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
+                if (cudaMemcpy(c.data(), h->arena + h->lutc_off, c.size() * 4, cudaMemcpyDeviceToHost) != cudaSuccess) {
                     delete l;
                     return CUART_ERR_CUDA;
                 }

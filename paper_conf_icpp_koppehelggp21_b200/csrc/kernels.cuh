@@ -18,6 +18,7 @@ struct DevIndex {
     uint64_t root;                // packed root link
     const uint64_t* lut;          // root lookup table, or nullptr
     const uint32_t* lut32;        // compact 32-bit root lookup table, or nullptr
+    const uint4* lutr;            // rank-form root lookup table (64-B blocks), or nullptr
     uint32_t lut_bytes;
     uint32_t fixed_len;           // key length of integer kinds (4 / 8), 0 for byte strings
     uint32_t key_kind;
@@ -199,6 +200,7 @@ struct Loader {
         asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(v) : "l"(p));
         return v;
     }
+    __device__ __forceinline__ uint4 lutv4(const void* p) const { return POL ? v4(p, keep) : ld_nc_v4(p); }
     // inner nodes
     __device__ __forceinline__ uint64_t node64(const void* p) const { return POL == 2 ? u64(p, drop) : ld_nc_u64(p); }
     __device__ __forceinline__ uint32_t node8(const void* p) const { return POL == 2 ? u8(p, drop) : ld_nc_u8(p); }
@@ -265,10 +267,32 @@ __device__ __forceinline__ uint64_t expand_lut32(uint32_t e, uint32_t k, uint32_
     return make_link(t, k + ((e >> 26) & 7u), e & 0x3FFFFFFu);
 }
 
+// Rank-form LUT entry p (capi.cu rank_lut): one 64-B block read (one L2 line,
+// sized so the whole table stays L2-resident), type from three bit-planes, index
+// = per-type base + popcount of earlier same-type entries; exceptions go to the
+// 64-bit link table.
+template <int POL>
+__device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Loader<POL>& ld, uint64_t p) {
+    const uint4* blk = ix.lutr + (p >> 6) * 4;
+    const uint4 a = ld.lutv4(blk), b = ld.lutv4(blk + 1);
+    const uint32_t j = uint32_t(p & 63);
+    const uint64_t p0 = uint64_t(a.x) | (uint64_t(a.y) << 32), p1 = uint64_t(a.z) | (uint64_t(a.w) << 32);
+    const uint64_t p2 = uint64_t(b.x) | (uint64_t(b.y) << 32), ex = uint64_t(b.z) | (uint64_t(b.w) << 32);
+    if ((ex >> j) & 1) return ld.lut64(ix.lut + p);
+    const uint32_t t = uint32_t((p0 >> j) & 1) | (uint32_t((p1 >> j) & 1) << 1) | (uint32_t((p2 >> j) & 1) << 2);
+    if (t == T_NULL) return 0;
+    const uint64_t m = ((t & 1) ? p0 : ~p0) & ((t & 2) ? p1 : ~p1) & ((t & 4) ? p2 : ~p2) & ((1ull << j) - 1);
+    const uint4 c = ld.lutv4(blk + 2 + (t >> 2));      // bases 0..3 | 4..7
+    const uint32_t tt = t & 3;
+    const uint32_t base = tt == 0 ? c.x : tt == 1 ? c.y : tt == 2 ? c.z : c.w;
+    return make_link(t, t >= T_LEAF8 ? ix.fixed_len : ix.lut_bytes, uint64_t(base) + __popcll(m));
+}
+
 template <class Key, int POL>
 __device__ __forceinline__ uint64_t start_link(const DevIndex& ix, const Loader<POL>& ld, const Key& key) {
     if (ix.lut_bytes && key.len() >= ix.lut_bytes) {
         const uint64_t p = key.prefix(ix.lut_bytes);
+        if (ix.lutr) return expand_lut_rank(ix, ld, p);
         if (ix.lut32) return expand_lut32(ld.lut32(ix.lut32 + p), ix.lut_bytes, ix.fixed_len);
         return ld.lut64(ix.lut + p);
     }

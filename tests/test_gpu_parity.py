@@ -82,15 +82,16 @@ def test_golden_gpu(name, lut):
     ix.close()
 
 
-@pytest.mark.parametrize("lut", [0, 2, 3])
-def test_c1_full_parity(lut):
+@pytest.mark.parametrize("lut,fmt", [(0, 1), (2, 1), (3, 1), (3, 2), (3, 3), (2, 3)])
+def test_c1_full_parity(lut, fmt):
     """Config 1 at full size, element by element against the pointer-ART oracle:
     1M lookups (50% hit), 100K updates, then the post-update dump."""
     cfg = W.CONFIGS["c1"]
     keys, vals = W.build_set(cfg)
     o = ArtOracle(keys, vals)
-    ix = C.Index(keys, vals, lut_bytes=lut)
+    ix = C.Index(keys, vals, lut_bytes=lut, lut_format=fmt)
     st = ix.stats()
+    assert lut == 0 or st["lut_format"] == fmt
     os_ = o.stats()
     assert (st["n4"], st["n16"], st["n48"], st["n256"], st["leaf8"]) == (os_["n4"], os_["n16"], os_["n48"], os_["n256"], os_["leaves"])
     q = W.lookup_batch(cfg, keys)
@@ -148,13 +149,13 @@ def test_random_sets_gpu(mode, seed):
         probes = [p for p in probes if len(p) == L] + [rng.getrandbits(8 * L).to_bytes(L, "big") for _ in range(999)]
     pin = _as_input(kind, probes)
     exp = o.lookup(pin)
-    for lut in (0, 2, 3):
-        ix = C.Index(inp, vals, lut_bytes=lut)
-        assert np.array_equal(_lookup(ix, pin), exp)
+    for lut, fmt in ((0, 1), (1, 3), (2, 1), (2, 2), (2, 3), (3, 1), (3, 2), (3, 3)):
+        ix = C.Index(inp, vals, lut_bytes=lut, lut_format=fmt)
+        assert np.array_equal(_lookup(ix, pin), exp), (lut, fmt)
         assert to_records(ix.dump()) == o.dump_structure().tolist()
         ix.close()
     # updates with heavy duplication (last writer wins) + absent keys
-    ix = C.Index(inp, vals, lut_bytes=2)
+    ix = C.Index(inp, vals, lut_bytes=2, lut_format=3)
     m = 3 * len(probes)
     pick = [rng.randrange(len(probes)) for _ in range(m)]
     ukeys = [probes[i] for i in pick]
@@ -220,9 +221,10 @@ def test_c2_full_size_sampled():
     plain map, and the any-size property out[i] == value(q[i]) (100% hit)."""
     cfg = W.CONFIGS["c2"]
     keys, vals = W.build_set(cfg)
-    ix = C.Index(keys, vals, lut_bytes=3)
+    ix = C.Index(keys, vals, lut_bytes=3, lut_format=3)
     st = ix.stats()
     assert st["n256"] == 1 + 256 + 65_536 and st["leaf8"] == 1 << 24   # Ex-C closed form
+    assert st["lut_format"] == 3 and st["lut_exceptions"] == 0
     qd = W.lookup_batch_torch(cfg, torch.zeros(1, dtype=torch.int64, device=DEV), 0, cfg.n_lookups, device=DEV)
     out = torch.empty(cfg.n_lookups, dtype=torch.int64, device=DEV)
     ix.lookup(qd, out)

@@ -98,6 +98,35 @@ __global__ void __launch_bounds__(256) pair(const uint8_t* __restrict__ buf, uin
     if (acc == 0x1234567) out[0] = acc;
 }
 
+// random 8-B stores (V=0 plain, 1 .cs streaming, 2 atomicMax u64, 3 red.max (no return))
+template <int V>
+__global__ void __launch_bounds__(256) scatter(uint8_t* __restrict__ buf, uint64_t slots, uint64_t n) {
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += stride) {
+        const uint64_t s = mix(i) % slots;
+        uint64_t* p = (uint64_t*)(buf + s * 64);
+        if (V == 0) *p = i;
+        if (V == 1) __stcs((unsigned long long*)p, (unsigned long long)i);
+        if (V == 2) atomicMax((unsigned long long*)p, (unsigned long long)i);
+        if (V == 3) asm volatile("red.global.max.u64 [%0], %1;" :: "l"(p), "l"(i));
+    }
+}
+
+template <int V>
+void run_scatter(uint8_t* buf, uint64_t bytes, uint64_t n, int grid, const char* name) {
+    cudaEvent_t a, b;
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+    scatter<V><<<grid, 256>>>(buf, bytes / 64, n / 8);
+    cudaEventRecord(a);
+    scatter<V><<<grid, 256>>>(buf, bytes / 64, n);
+    cudaEventRecord(b);
+    cudaEventSynchronize(b);
+    float ms;
+    cudaEventElapsedTime(&ms, a, b);
+    printf("{\"variant\": \"%s\", \"ms\": %.3f, \"Gops_s\": %.2f}\n", name, ms, n / (ms * 1e-3) / 1e9);
+}
+
 template <int D>
 void run_pair(const uint8_t* buf, uint64_t bytes, uint64_t n, uint64_t* out, int grid) {
     cudaEvent_t a, b;
@@ -191,6 +220,14 @@ int main(int argc, char** argv) {
         run_pair<512>(buf, bytes, n, out, grid);
         run_pair<1024>(buf, bytes, n, out, grid);
         run_pair<2048>(buf, bytes, n, out, grid);
+    }
+    if (all || only[0] == 's') {
+        run_scatter<0>(buf, bytes, n, grid, "store8_random");
+        run_scatter<1>(buf, bytes, n, grid, "store8_random_cs");
+        run_scatter<2>(buf, bytes, n, grid, "atomicMax64_random");
+        run_scatter<3>(buf, bytes, n, grid, "red.max64_random");
+        run_scatter<0>(buf, 64ull << 20, n, grid, "store8_random_64MiB");
+        run_scatter<2>(buf, 64ull << 20, n, grid, "atomicMax64_random_64MiB");
     }
     if (all || only[0] == 'f') {   // footprint sweep: random 8-B loads within the first F bytes
         for (uint64_t f = 16ull << 20; f <= bytes && f <= (4ull << 30); f *= 2) {

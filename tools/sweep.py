@@ -27,7 +27,7 @@ def main():
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--lut", type=int, default=3)
     ap.add_argument("--policies", default="0,1,2,3")
-    ap.add_argument("--widths", default="8,4")
+    ap.add_argument("--formats", default="1,2,3")
     a = ap.parse_args()
     cfg = W.CONFIGS[a.config]
     dev = torch.device("cuda:0")
@@ -44,10 +44,10 @@ def main():
     ref = None
     if cfg.n_updates:
         uk, uv = W.update_batch_torch(cfg, keys_d)
-    for width in [int(x) for x in a.widths.split(",")]:
+    for width in [int(x) for x in a.formats.split(",")]:
         for pol in [int(x) for x in a.policies.split(",")]:
             os.environ["CUART_POLICY"] = str(pol)
-            ix = C.Index.from_layout(lay, device=0, lut_entry_bytes=width)
+            ix = C.Index.from_layout(lay, device=0, lut_format=width)
             ix.lookup(q, out)
             torch.cuda.synchronize()
             chk = int(out[: 1 << 24].sum().item())
@@ -67,9 +67,9 @@ def main():
                 tu.append(e[1].elapsed_time(e[2]))
             lm = float(np.median(ts))
             um = float(np.median(tu))
-            print(json.dumps({"config": a.config, "lut": a.lut, "lut_entry_bytes": width, "policy": pol,
+            print(json.dumps({"config": a.config, "lut": a.lut, "lut_format": width, "policy": pol,
                               "lookup_ms": round(lm, 3), "mlookups_s": round(cfg.n_lookups / lm / 1e3, 1),
-                              "update_ms": round(um, 3),
+                              "lut_exceptions": ix.stats()["lut_exceptions"], "update_ms": round(um, 3),
                               "mupdates_s": round(cfg.n_updates / um / 1e3, 1) if cfg.n_updates else None,
                               "checksum_ok": chk == ref}), flush=True)
             ix.close()
