@@ -273,10 +273,11 @@ int build_host_layout(uint32_t kind, const void* data, const uint8_t* lengths, c
             if (K && gr.pdepth < int32_t(K) && d >= K) L.lut[S.prefix_k(gr.lo, K)] = link;
 
             uint8_t* rec = L.buf[t].data() + idx * kRecordBytes[t];
+            uint8_t* hdr = rec + header_off(t);
             const uint32_t plen = d - gr.depth;
-            rec[0] = uint8_t(plen);
-            rec[1] = uint8_t(c - 1);
-            for (uint32_t b = 0; b < plen && b < kHeaderPrefix; b++) rec[2 + b] = uint8_t(S.byte(gr.lo, gr.depth + b));
+            hdr[0] = uint8_t(plen);
+            hdr[1] = uint8_t(c - 1);
+            for (uint32_t b = 0; b < plen && b < kHeaderPrefix; b++) hdr[2 + b] = uint8_t(S.byte(gr.lo, gr.depth + b));
             if (t == T_N48) memset(rec + kN48Index, kN48Empty, 256);
             uint64_t a = gr.lo, off = noff[g];
             uint32_t j = 0, lastb = 0;
@@ -383,11 +384,12 @@ uint64_t walk_one(const HostLayout& L, const uint8_t* key, uint32_t len, uint32_
         } else {
             const uint32_t nk = t == T_N4 ? 4 : 16;
             const uint8_t* keys = rec + (t == T_N4 ? kN4Keys : kN16Keys);
-            s += t == T_N4 ? sectors(roff + 16, 40) : sectors(roff + kN16Keys, 16);
+            s += t == T_N4 ? sectors(roff, 32) : sectors(roff + kN16Keys, 16);
             uint32_t less = 0, eq = 0;
             for (uint32_t j = 0; j < nk; j++) { less += keys[j] < b; eq |= keys[j] == b; }
             if (!eq) return kMiss;
             if (t == T_N16) s += sectors(roff + kN16Child + 8 * less, 8);
+            if (t == T_N4 && less == 3) s += sectors(roff + kN4Child + 24, 8);
             memcpy(&link, rec + (t == T_N4 ? kN4Child : kN16Child) + 8 * less, 8);
         }
     }

@@ -64,6 +64,7 @@ struct cuart_index {
     uint32_t lut_format = CUART_LUT_LINKS;
     uint64_t lutc_off = 0;             // compact / rank LUT region
     uint64_t lut_exceptions = 0;       // RANK: entries served by the 64-bit table
+    int grid_ctas_per_sm = 0;          // 0 = default grid (8 resident CTAs x 16 waves); else persistent grid
 };
 
 static std::atomic<uint64_t> g_launches{0};
@@ -133,7 +134,10 @@ __global__ void __launch_bounds__(256) k_upd2(DevIndex ix, const uint64_t* __res
 // ============================================================================ helpers
 static int grid_for(const cuart_index* h, uint64_t n) {
     uint64_t blocks = (n + 255) / 256;
-    uint64_t cap = uint64_t(h->num_sms) * 8 * 16;   // 8 resident 256-thread CTAs per SM, 16 waves
+    // Default: one op per thread (measured fastest on c3: CTAs retire and refill
+    // per SM instead of long grid-stride loops).  Tuning knob: a persistent grid.
+    uint64_t cap = (uint64_t(1) << 31) - 1;
+    if (h->grid_ctas_per_sm > 0) cap = uint64_t(h->num_sms) * h->grid_ctas_per_sm;
     if (blocks > cap) blocks = cap;
     return int(blocks < 1 ? 1 : blocks);
 }
@@ -330,50 +334,48 @@ static uint64_t expand_lut32_host(uint32_t e, uint32_t k, uint32_t leaf_len) {
     return make_link(t, k + ((e >> 26) & 7u), e & 0x3FFFFFFu);
 }
 
-// Rank LUT (kernels.cuh expand_lut_rank): 64-entry blocks of 64 B —
-//   u64 plane[3] (type code bits of each entry), u64 exc (entry lives in the 64-bit
-//   link table), u32 base[8] (index of the first entry of each type in the block).
-// An entry is encoded in the block when its target's index is base[type] + (number
-// of earlier entries of that type in the block), its branch depth is k (inner) and
-// its key length is the index's fixed length (leaves).  Everything else is marked
-// as an exception and read from the full 64-bit table.  Integer keys only.
+// Rank LUT (kernels.cuh expand_lut_rank): 32-entry blocks of 32 B —
+//   u32 plane[3] (type code bits of each entry), u32 exc (entry lives in the 64-bit
+//   link table), u32 base[4] (index of the first N4 / N16 / N48 / N256 entry).
+// An inner-node entry is encoded in the block when its branch depth is k and its
+// index is base[type] + (number of earlier entries of that type in the block).
+// Leaves (lexicographically numbered, so not consecutive) and everything else are
+// exceptions read from the full 64-bit table.  Integer keys only.
 static bool rank_lut(const HostLayout& L, std::vector<uint64_t>& blocks, uint64_t& n_exc) {
     if (L.lut.empty() || L.key_kind == CUART_KEY_BYTES) return false;
     const uint32_t k = L.lut_bytes;
-    const uint32_t flen = L.key_kind == CUART_KEY_U64 ? 8 : 4;
-    const uint64_t nb = L.lut.size() / 64;
-    blocks.assign(nb * 8, 0);
+    const uint64_t nb = (L.lut.size() + 31) / 32;
+    blocks.assign(nb * 4, 0);
     n_exc = 0;
     for (uint64_t bi = 0; bi < nb; bi++) {
-        uint64_t plane[3] = {0, 0, 0}, exc = 0;
-        uint32_t base[8] = {0};
-        uint64_t cnt[8] = {0};
-        for (uint32_t j = 0; j < 64; j++) {
-            const uint64_t l = L.lut[bi * 64 + j];
+        uint32_t plane[3] = {0, 0, 0}, exc = 0, base[5] = {0, 0, 0, 0, 0};
+        uint64_t cnt[5] = {0};
+        for (uint32_t j = 0; j < 32 && bi * 32 + j < L.lut.size(); j++) {
+            const uint64_t l = L.lut[bi * 32 + j];
             const uint32_t t = link_type(l);
             if (t == T_NULL) continue;
             const uint64_t idx = link_index(l);
-            bool ok = (t >= T_LEAF8) ? (link_aux(l) == flen) : (link_aux(l) == k);
+            bool ok = t <= T_N256 && link_aux(l) == k;
             if (ok && cnt[t] == 0) {
                 if (idx > 0xFFFFFFFFull) ok = false;
                 else base[t] = uint32_t(idx);
             }
             if (ok && idx != uint64_t(base[t]) + cnt[t]) ok = false;
             if (!ok) {
-                exc |= 1ull << j;
+                exc |= 1u << j;
                 n_exc++;
                 continue;
             }
             cnt[t]++;
             for (int pb = 0; pb < 3; pb++)
-                if (t & (1u << pb)) plane[pb] |= 1ull << j;
+                if (t & (1u << pb)) plane[pb] |= 1u << j;
         }
-        uint64_t* blk = &blocks[bi * 8];
+        uint32_t* blk = reinterpret_cast<uint32_t*>(&blocks[bi * 4]);
         blk[0] = plane[0];
         blk[1] = plane[1];
         blk[2] = plane[2];
         blk[3] = exc;
-        for (int t = 0; t < 8; t += 2) blk[4 + t / 2] = uint64_t(base[t]) | (uint64_t(base[t + 1]) << 32);
+        for (int t = 1; t <= 4; t++) blk[3 + t] = base[t];
     }
     return true;
 }
@@ -421,6 +423,7 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     }
     h->lut_format = fmt;
     if (const char* pe = getenv("CUART_POLICY")) h->policy = atoi(pe);
+    if (const char* pe = getenv("CUART_GRID_CTAS_PER_SM")) h->grid_ctas_per_sm = atoi(pe);   // tuning knob
     // LUT region: 64-bit links (LINKS, and the exception table of RANK) then the compact form
     h->lut_off = off;
     const bool need_links = fmt == CUART_LUT_LINKS || fmt == CUART_LUT_RANK;

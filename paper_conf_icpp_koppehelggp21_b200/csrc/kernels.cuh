@@ -44,6 +44,15 @@ __device__ __forceinline__ uint4 ld_nc_v4(const void* p) {
                  : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
     return v;
 }
+// 256-bit (32 B) load: one request on sm_100 (SASS LDG.E.ENL2.256); p 32-B aligned.
+struct U8x32 { uint32_t w[8]; };
+__device__ __forceinline__ U8x32 ld_nc_v8(const void* p) {
+    U8x32 v;
+    asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(v.w[0]), "=r"(v.w[1]), "=r"(v.w[2]), "=r"(v.w[3]), "=r"(v.w[4]), "=r"(v.w[5]), "=r"(v.w[6]),
+                   "=r"(v.w[7]) : "l"(p));
+    return v;
+}
 // Leaf values are rewritten by the update kernels: read them through L2 (coherent path).
 __device__ __forceinline__ uint64_t ld_cg_u64(const void* p) {
     uint64_t v;
@@ -200,7 +209,15 @@ struct Loader {
         asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(v) : "l"(p));
         return v;
     }
-    __device__ __forceinline__ uint4 lutv4(const void* p) const { return POL ? v4(p, keep) : ld_nc_v4(p); }
+    __device__ __forceinline__ static U8x32 v8(const void* p, uint64_t pol) {
+        U8x32 v;
+        asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                     : "=r"(v.w[0]), "=r"(v.w[1]), "=r"(v.w[2]), "=r"(v.w[3]), "=r"(v.w[4]), "=r"(v.w[5]),
+                       "=r"(v.w[6]), "=r"(v.w[7]) : "l"(p), "l"(pol));
+        return v;
+    }
+    __device__ __forceinline__ U8x32 lutv8(const void* p) const { return POL ? v8(p, keep) : ld_nc_v8(p); }
+    __device__ __forceinline__ U8x32 nodev8(const void* p) const { return POL == 2 ? v8(p, drop) : ld_nc_v8(p); }
     // inner nodes
     __device__ __forceinline__ uint64_t node64(const void* p) const { return POL == 2 ? u64(p, drop) : ld_nc_u64(p); }
     __device__ __forceinline__ uint32_t node8(const void* p) const { return POL == 2 ? u8(p, drop) : ld_nc_u8(p); }
@@ -243,17 +260,18 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Loader<P
             search4(k4.w, bb, l3, e3);
             if ((e0 | e1 | e2 | e3) == 0) return 0;
             link = ld.node64(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
-        } else {  // N4: whole 64-byte record in one round trip
-            const uint4 h = ld.nodev4(rec + 16);          // keys[4] | pad | child[0]
-            const uint4 c12 = ld.nodev4(rec + 32);        // child[1], child[2]
-            const uint64_t c3 = ld.node64(rec + 48);      // child[3]
+        } else {  // N4: keys + child[0..2] in one 256-bit load; child[3] (same line) if taken
+            const U8x32 r = ld.nodev8(rec);
             uint32_t less, eq;
-            search4(h.x, b * 0x01010101u, less, eq);
+            search4(r.w[0], b * 0x01010101u, less, eq);
             if (eq == 0) return 0;
-            const uint64_t c0 = uint64_t(h.z) | (uint64_t(h.w) << 32);
-            const uint64_t c1 = uint64_t(c12.x) | (uint64_t(c12.y) << 32);
-            const uint64_t c2 = uint64_t(c12.z) | (uint64_t(c12.w) << 32);
-            link = less == 0 ? c0 : less == 1 ? c1 : less == 2 ? c2 : c3;
+            if (less == 3) {
+                link = ld.node64(rec + kN4Child + 24);
+            } else {
+                const uint32_t lo = less == 0 ? r.w[2] : less == 1 ? r.w[4] : r.w[6];
+                const uint32_t hi = less == 0 ? r.w[3] : less == 1 ? r.w[5] : r.w[7];
+                link = uint64_t(lo) | (uint64_t(hi) << 32);
+            }
         }
     }
 }
@@ -267,25 +285,21 @@ __device__ __forceinline__ uint64_t expand_lut32(uint32_t e, uint32_t k, uint32_
     return make_link(t, k + ((e >> 26) & 7u), e & 0x3FFFFFFu);
 }
 
-// Rank-form LUT entry p (capi.cu rank_lut): one 64-B block read (one L2 line,
-// sized so the whole table stays L2-resident), type from three bit-planes, index
-// = per-type base + popcount of earlier same-type entries; exceptions go to the
-// 64-bit link table.
+// Rank-form LUT entry p (capi.cu rank_lut): one 256-bit read of a 32-B block per
+// 32 entries (the whole table is 1 B/entry and stays L2-resident).  Type from three
+// bit-planes, index = per-type base + popcount of earlier same-type entries;
+// exceptions (leaves, other depths, non-consecutive indices) go to the link table.
 template <int POL>
 __device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Loader<POL>& ld, uint64_t p) {
-    const uint4* blk = ix.lutr + (p >> 6) * 4;
-    const uint4 a = ld.lutv4(blk), b = ld.lutv4(blk + 1);
-    const uint32_t j = uint32_t(p & 63);
-    const uint64_t p0 = uint64_t(a.x) | (uint64_t(a.y) << 32), p1 = uint64_t(a.z) | (uint64_t(a.w) << 32);
-    const uint64_t p2 = uint64_t(b.x) | (uint64_t(b.y) << 32), ex = uint64_t(b.z) | (uint64_t(b.w) << 32);
-    if ((ex >> j) & 1) return ld.lut64(ix.lut + p);
-    const uint32_t t = uint32_t((p0 >> j) & 1) | (uint32_t((p1 >> j) & 1) << 1) | (uint32_t((p2 >> j) & 1) << 2);
+    const U8x32 blk = ld.lutv8(ix.lutr + (p >> 5) * 2);
+    const uint32_t j = uint32_t(p & 31);
+    if ((blk.w[3] >> j) & 1) return ld.lut64(ix.lut + p);
+    const uint32_t p0 = blk.w[0], p1 = blk.w[1], p2 = blk.w[2];
+    const uint32_t t = ((p0 >> j) & 1) | (((p1 >> j) & 1) << 1) | (((p2 >> j) & 1) << 2);
     if (t == T_NULL) return 0;
-    const uint64_t m = ((t & 1) ? p0 : ~p0) & ((t & 2) ? p1 : ~p1) & ((t & 4) ? p2 : ~p2) & ((1ull << j) - 1);
-    const uint4 c = ld.lutv4(blk + 2 + (t >> 2));      // bases 0..3 | 4..7
-    const uint32_t tt = t & 3;
-    const uint32_t base = tt == 0 ? c.x : tt == 1 ? c.y : tt == 2 ? c.z : c.w;
-    return make_link(t, t >= T_LEAF8 ? ix.fixed_len : ix.lut_bytes, uint64_t(base) + __popcll(m));
+    const uint32_t m = ((t & 1) ? p0 : ~p0) & ((t & 2) ? p1 : ~p1) & ((t & 4) ? p2 : ~p2) & ((1u << j) - 1);
+    const uint32_t base = t == T_N4 ? blk.w[4] : t == T_N16 ? blk.w[5] : t == T_N48 ? blk.w[6] : blk.w[7];
+    return make_link(t, ix.lut_bytes, uint64_t(base) + __popc(m));
 }
 
 template <class Key, int POL>

@@ -11,6 +11,7 @@ import numpy as np
 REC = {1: 64, 2: 160, 3: 672, 4: 2080, 5: 16, 6: 32, 7: 48}
 VALOFF = {5: 8, 6: 16, 7: 32}
 IDX_MASK = (1 << 52) - 1
+HDR = {1: 40, 2: 0, 3: 0, 4: 0}   # header offset inside the record (N4 keeps keys + 3 children first)
 
 
 def split_link(link: int):
@@ -26,8 +27,8 @@ def children(view, t, idx):
     b = view["buf"][t]
     o = idx * REC[t]
     if t == 1 or t == 2:
-        cnt = int(b[o + 1]) + 1
-        ko, co = (16, 24) if t == 1 else (16, 32)
+        cnt = int(b[o + HDR[t] + 1]) + 1
+        ko, co = (0, 8) if t == 1 else (16, 32)
         return [(int(b[o + ko + j]), _u64(b, o + co + 8 * j)) for j in range(cnt)]
     if t == 3:
         out = []
@@ -72,13 +73,14 @@ def to_records(view) -> list[int]:
             return
         b = view["buf"][t]
         o = idx * REC[t]
-        plen = int(b[o])
+        h = o + HDR[t]
+        plen = int(b[h])
         assert aux == depth + plen, "branch depth in the link = depth + prefix length"
         kids = children(view, t, idx)
-        assert int(b[o + 1]) + 1 == len(kids), "header count"
+        assert int(b[h + 1]) + 1 == len(kids), "header count"
         fl = first_leaf(link)
         prefix = fl[depth: depth + plen]
-        stored = bytes(b[o + 2: o + 2 + min(plen, 14)])
+        stored = bytes(b[h + 2: h + 2 + min(plen, 14)])
         assert stored == prefix[:14], "header stores the first 14 prefix bytes"
         out.extend([t, plen, *prefix, len(kids), *[k for k, _ in kids]])
         for _, c in kids:
