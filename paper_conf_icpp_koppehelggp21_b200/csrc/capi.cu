@@ -60,7 +60,7 @@ struct cuart_index {
     uint64_t* stage_val[2] = {nullptr, nullptr};
     size_t stage_cap = 0;
     cudaStream_t streams[2] = {nullptr, nullptr};
-    int policy = 1;                    // cache-policy variant of the kernels (kernels.cuh Loader)
+    int policy = 5;                    // cache-policy variant of the kernels (kernels.cuh Loader)
     uint32_t lut_format = CUART_LUT_LINKS;
     uint64_t lutc_off = 0;             // compact / rank LUT region
     uint64_t lut_exceptions = 0;       // RANK: entries served by the 64-bit table
@@ -160,7 +160,10 @@ static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const voi
     case 0: CUART_LOOKUP(K, 0); break;               \
     case 2: CUART_LOOKUP(K, 2); break;               \
     case 3: CUART_LOOKUP(K, 3); break;               \
-    default: CUART_LOOKUP(K, 1); break;              \
+    case 4: CUART_LOOKUP(K, 4); break;               \
+    case 5: CUART_LOOKUP(K, 5); break;               \
+    case 1: CUART_LOOKUP(K, 1); break;               \
+    default: CUART_LOOKUP(K, 5); break;              \
     }
     switch (kind) {
     case CUART_KEY_U64: CUART_LOOKUP_POL(KeyU64); break;
@@ -204,7 +207,9 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
 #define CUART_UPD1(K, P) k_upd1<K, P><<<grid, 256, 0, s>>>(h->dix, kb, lb, vals + base, m, epoch_hi, h->leafref)
 #define CUART_UPD1_POL(K)                            \
     if (h->policy == 0) CUART_UPD1(K, 0);            \
-    else CUART_UPD1(K, 1);
+    else if (h->policy == 4) CUART_UPD1(K, 4);       \
+    else if (h->policy == 1) CUART_UPD1(K, 1);       \
+    else CUART_UPD1(K, 5);
         switch (kind) {
         case CUART_KEY_U64: CUART_UPD1_POL(KeyU64); break;
         case CUART_KEY_U32: CUART_UPD1_POL(KeyU32); break;

@@ -168,21 +168,32 @@ __device__ __forceinline__ void search4(uint32_t keys, uint32_t bb, uint32_t& le
 }
 
 // Cache policy for the three kinds of dependent loads (B200 L2 is 126 MB; the
-// structure of a large index is not).  POL 0: plain ld.global.nc everywhere.
-// POL 1: LUT evict_last (keep the root table L2-resident), leaves evict_first.
-// POL 2: as 1 and inner nodes evict_first too.  POL 3: LUT evict_last only.
+// structure of a large index is not).
+//   POL 0: plain ld.global.nc everywhere.
+//   POL 1: LUT evict_last (keep the root table L2-resident), leaves evict_first.
+//   POL 2: as 1 and inner nodes evict_first too.
+//   POL 3: LUT evict_last only.
+//   POL 4: as 1, plus the L2::64B fetch-size hint on node and leaf loads (a random
+//          miss fills 64 B instead of a 128-B line: half the DRAM bytes).
+//   POL 5: as 1, L2::64B on leaf loads only.
 template <int POL>
 struct Loader {
-    uint64_t keep, drop;
+    uint64_t keep, drop, norm;
+    static constexpr bool kNode64B = POL == 4;
+    static constexpr bool kLeaf64B = POL == 4 || POL == 5;
+    static constexpr bool kLeafDrop = POL == 1 || POL == 2 || POL == 4 || POL == 5;
     __device__ __forceinline__ Loader() {
         if (POL != 0) {
             asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(keep));
             asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(drop));
         }
+        if (POL == 4) asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(norm));
     }
+    template <bool F64 = false>
     __device__ __forceinline__ static uint64_t u64(const void* p, uint64_t pol) {
         uint64_t v;
-        asm volatile("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+        if (F64) asm volatile("ld.global.nc.L2::cache_hint.L2::64B.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+        else asm volatile("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
         return v;
     }
     __device__ __forceinline__ static uint32_t u32(const void* p, uint64_t pol) {
@@ -190,18 +201,38 @@ struct Loader {
         asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
         return v;
     }
+    template <bool F64 = false>
     __device__ __forceinline__ static uint32_t u8(const void* p, uint64_t pol) {
         uint16_t v;
-        asm volatile("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol));
+        if (F64) asm volatile("ld.global.nc.L2::cache_hint.L2::64B.u8 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol));
+        else asm volatile("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol));
         return v;
     }
+    template <bool F64 = false>
     __device__ __forceinline__ static uint4 v4(const void* p, uint64_t pol) {
         uint4 v;
-        asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
-                     : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol));
+        if (F64)
+            asm volatile("ld.global.nc.L2::cache_hint.L2::64B.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                         : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol));
+        else
+            asm volatile("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                         : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol));
         return v;
     }
-    // LUT entries
+    template <bool F64 = false>
+    __device__ __forceinline__ static U8x32 v8(const void* p, uint64_t pol) {
+        U8x32 v;
+        if (F64)
+            asm volatile("ld.global.nc.L2::cache_hint.L2::64B.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                         : "=r"(v.w[0]), "=r"(v.w[1]), "=r"(v.w[2]), "=r"(v.w[3]), "=r"(v.w[4]), "=r"(v.w[5]),
+                           "=r"(v.w[6]), "=r"(v.w[7]) : "l"(p), "l"(pol));
+        else
+            asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                         : "=r"(v.w[0]), "=r"(v.w[1]), "=r"(v.w[2]), "=r"(v.w[3]), "=r"(v.w[4]), "=r"(v.w[5]),
+                           "=r"(v.w[6]), "=r"(v.w[7]) : "l"(p), "l"(pol));
+        return v;
+    }
+    // LUT entries / blocks
     __device__ __forceinline__ uint64_t lut64(const void* p) const { return POL ? u64(p, keep) : ld_nc_u64(p); }
     __device__ __forceinline__ uint32_t lut32(const void* p) const {
         if (POL) return u32(p, keep);
@@ -209,21 +240,24 @@ struct Loader {
         asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(v) : "l"(p));
         return v;
     }
-    __device__ __forceinline__ static U8x32 v8(const void* p, uint64_t pol) {
-        U8x32 v;
-        asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
-                     : "=r"(v.w[0]), "=r"(v.w[1]), "=r"(v.w[2]), "=r"(v.w[3]), "=r"(v.w[4]), "=r"(v.w[5]),
-                       "=r"(v.w[6]), "=r"(v.w[7]) : "l"(p), "l"(pol));
-        return v;
-    }
     __device__ __forceinline__ U8x32 lutv8(const void* p) const { return POL ? v8(p, keep) : ld_nc_v8(p); }
-    __device__ __forceinline__ U8x32 nodev8(const void* p) const { return POL == 2 ? v8(p, drop) : ld_nc_v8(p); }
     // inner nodes
-    __device__ __forceinline__ uint64_t node64(const void* p) const { return POL == 2 ? u64(p, drop) : ld_nc_u64(p); }
-    __device__ __forceinline__ uint32_t node8(const void* p) const { return POL == 2 ? u8(p, drop) : ld_nc_u8(p); }
-    __device__ __forceinline__ uint4 nodev4(const void* p) const { return POL == 2 ? v4(p, drop) : ld_nc_v4(p); }
+    __device__ __forceinline__ uint64_t node64(const void* p) const {
+        return POL == 2 ? u64(p, drop) : POL == 4 ? u64<true>(p, norm) : ld_nc_u64(p);
+    }
+    __device__ __forceinline__ uint32_t node8(const void* p) const {
+        return POL == 2 ? u8(p, drop) : POL == 4 ? u8<true>(p, norm) : ld_nc_u8(p);
+    }
+    __device__ __forceinline__ uint4 nodev4(const void* p) const {
+        return POL == 2 ? v4(p, drop) : POL == 4 ? v4<true>(p, norm) : ld_nc_v4(p);
+    }
+    __device__ __forceinline__ U8x32 nodev8(const void* p) const {
+        return POL == 2 ? v8(p, drop) : POL == 4 ? v8<true>(p, norm) : ld_nc_v8(p);
+    }
     // leaves
-    __device__ __forceinline__ uint4 leafv4(const void* p) const { return (POL == 1 || POL == 2) ? v4(p, drop) : ld_nc_v4(p); }
+    __device__ __forceinline__ uint4 leafv4(const void* p) const {
+        return kLeaf64B ? v4<true>(p, drop) : kLeafDrop ? v4(p, drop) : ld_nc_v4(p);
+    }
 };
 
 // Walk from `link` to a leaf.  Returns the leaf link on a full-key match (its value
