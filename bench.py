@@ -39,6 +39,11 @@ sys.path.insert(0, ROOT)
 import workloads as W  # noqa: E402
 
 METRIC = "Mlookups/s and Mupdates/s (device-timed)"
+# K-GATHER calibration (tools/kgather*.cu, profiles/r01/): independent random 8-B loads over
+# 8 GiB saturate at ~47.5-48 G requests/s on this B200 (each fills a 128-B L2 line from
+# DRAM by default), whatever the load flavour; L2-resident (<= 32 MiB) random loads ~245 G/s.
+RANDOM_CEILING = {"random_requests_per_s": 47.5e9, "l2_resident_requests_per_s": 245e9,
+                  "source": "profiles/r01/kgather*.json"}
 
 
 def _args():
@@ -52,6 +57,9 @@ def _args():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--e2e-steps", type=int, default=2)
+    p.add_argument("--mode", default="range", choices=["range", "replica"], help="multi-GPU mode (N > 1)")
+    p.add_argument("--traffic", type=float, default=None,
+                   help="ncu dram__bytes_read+write per k_lookup launch (GB), from profiles/, echoed into roofline")
     return p.parse_args()
 
 
@@ -181,6 +189,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_icpp_koppehelggp21_b200 as C
+    from paper_conf_icpp_koppehelggp21_b200.dist import CudaOps, DistIndex
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -189,6 +198,7 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
+    mode = "single" if world == 1 else args.mode
 
     cfg = W.CONFIGS[args.config]
     t0 = time.perf_counter()
@@ -199,30 +209,40 @@ def main():
         keys = np.arange(cfg.n_keys, dtype=np.uint32)
         keys_d = torch.from_numpy(keys.view(np.int32)).to(dev)
     vals = W.values_for(W.SEED_VALUES + W.config_id(cfg), np.arange(cfg.n_keys, dtype=np.uint64))
-    layout = C.Layout(keys, vals, lut_bytes=args.lut)
-    ix = C.Index.from_layout(layout, device=local)
+    ops = CudaOps(dev)
+    if world == 1:
+        layout = C.Layout(keys, vals, lut_bytes=args.lut)
+        ix = C.Index.from_layout(layout, device=local)
+        di = None
+    else:
+        di = DistIndex(keys, vals, mode=mode, ops=ops, lut_bytes=args.lut)
+        ix = di.index
+        layout = None
     build_s = time.perf_counter() - t0
     stats = ix.stats()
 
-    # resident inputs: this rank's shard of the global lookup stream, its update batch
+    # resident inputs: this rank's shard of the global lookup stream and update stream
     nl = cfg.n_lookups
     q = W.lookup_batch_torch(cfg, keys_d, rank * nl, nl, device=dev)
     out = torch.empty(nl, dtype=torch.int64, device=dev)
     nu = cfg.n_updates
+    uk = uv = None
     if nu:
         uk, uv = W.update_batch_torch(cfg, keys_d, rank * nu, nu)
-        if world > 1:   # replica mode: every replica applies all ranks' updates in global order
-            gk = torch.empty(world * nu, dtype=torch.int64, device=dev)
-            gv = torch.empty_like(gk)
-            dist.all_gather_into_tensor(gk, uk)
-            dist.all_gather_into_tensor(gv, uv)
-            uk, uv = gk, gv
     torch.cuda.synchronize()
 
     # algorithmic bytes of the dominant kernel (k_lookup): exact sector count of the
-    # lookup path for a 2^20-query sample (host walker over the same layout) + I/O
+    # lookup path over this rank's layout for a 2^20-query sample + key-in/value-out
+    if layout is None:
+        from paper_conf_icpp_koppehelggp21_b200.dist import owners, prefix8
+        local_keys = keys if mode == "replica" else keys[owners(prefix8(keys), di.splitters_np) == rank]
+        local_vals = np.zeros(local_keys.shape[0], np.uint64)
+        layout = C.Layout(local_keys, local_vals, lut_bytes=args.lut)
     samp = q[: 1 << 20].cpu().numpy()
     samp = samp.view(np.uint64) if cfg.kind == "u64" else samp.view(np.uint32)
+    if mode == "range":   # sample of the queries this rank's index actually serves
+        from paper_conf_icpp_koppehelggp21_b200.dist import owners, prefix8
+        samp = samp[owners(prefix8(samp), di.splitters_np) == rank]
     sec = layout.sectors(samp).astype(np.float64)
     io_bytes = (8 if cfg.kind == "u64" else 4) + 8
     bytes_per_lookup = 32.0 * sec.mean() + io_bytes
@@ -230,14 +250,24 @@ def main():
 
     stream = torch.cuda.current_stream()
 
-    def step(ev=None):
+    def step(ev=None, kev=None):
         if ev is not None:
             ev[0].record(stream)
-        ix.lookup(q, out, stream)
+        if di is None:
+            if kev is not None:
+                kev[0].record(stream)
+            ix.lookup(q, out, stream)
+            if kev is not None:
+                kev[1].record(stream)
+        else:
+            di.lookup(q, events=kev)
         if ev is not None:
             ev[1].record(stream)
         if nu:
-            ix.update(uk, uv, stream)
+            if di is None:
+                ix.update(uk, uv, stream)
+            else:
+                di.update((uk, uv))
         if ev is not None:
             ev[2].record(stream)
 
@@ -247,6 +277,7 @@ def main():
     if world > 1:
         dist.barrier()
     evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    kevs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.3)
@@ -256,7 +287,7 @@ def main():
     t_end = torch.cuda.Event(enable_timing=True)
     t_start.record(stream)
     for s in range(args.steps):
-        step(evs[s])
+        step(evs[s], kevs[s])
     t_end.record(stream)
     torch.cuda.synchronize()
     launches = C.cuart_launch_count() - launches0
@@ -266,25 +297,28 @@ def main():
     total_ms = t_start.elapsed_time(t_end)
     look_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in evs]))
     upd_ms = float(np.mean([e[1].elapsed_time(e[2]) for e in evs])) if nu else 0.0
+    kern_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in kevs]))
+    served = nl if di is None or mode == "replica" else getattr(di, "last_local_lookups", nl)
     tt = torch.tensor([total_ms, look_ms, upd_ms], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
     total_ms, look_ms, upd_ms = tt.tolist()
     ms_step = total_ms / args.steps
-    n_upd_applied = uk.shape[0] if nu else 0
-    # whole job: every rank's lookups + the update ops (each op counted once)
-    ops_per_step = world * nl + (world * nu if nu else 0)
+    # whole job: every rank's lookups + every rank's update ops (each op counted once)
+    ops_per_step = world * nl + world * nu
     value = ops_per_step / (ms_step * 1e-3) / 1e6
 
-    # roofline of the dominant kernel (k_lookup), HBM-bound random gathers
+    # roofline of the dominant kernel (k_lookup on this rank), HBM-bound random gathers
     peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
     if os.path.exists(peaks_path):
         with open(peaks_path) as f:
             peak = float(json.load(f)["hbm_gbs"])
         peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)"
-    achieved = nl * bytes_per_lookup / (look_ms * 1e-3) / 1e9
-    hit = float((out[: 1 << 24] != -1).float().mean().item())
+    achieved = served * bytes_per_lookup / (kern_ms * 1e-3) / 1e9
+    out_now = out if di is None else di.lookup(q)
+    hit = float((out_now[: 1 << 24] != -1).float().mean().item())
+    del out_now
 
     # end-to-end through the public API with HOST buffers (pinned), copies inside the timed region
     e2e = None
@@ -298,18 +332,27 @@ def main():
             uvh = torch.empty_like(ukh)
             ukh.copy_(uk)
             uvh.copy_(uv)
-        qn = qh.numpy()
-        on = oh.numpy()
-        C.cuart_lookup_host(ix.h, qn, on)    # warm-up
+
+        def e2e_step():
+            if di is None:
+                C.cuart_lookup_host(ix.h, qh.numpy(), oh.numpy())
+                if nu:
+                    C.cuart_update_host(ix.h, ukh.numpy(), uvh.numpy())
+            else:
+                qd = qh.to(dev, non_blocking=True)
+                oh.copy_(di.lookup(qd), non_blocking=True)
+                if nu:
+                    di.update((ukh.to(dev, non_blocking=True), uvh.to(dev, non_blocking=True)))
+                torch.cuda.synchronize()
+
+        e2e_step()
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
         ts = []
         for _ in range(args.e2e_steps):
             t0 = time.perf_counter()
-            C.cuart_lookup_host(ix.h, qn, on)
-            if nu:
-                C.cuart_update_host(ix.h, ukh.numpy(), uvh.numpy())
+            e2e_step()
             ts.append(time.perf_counter() - t0)
         et = torch.tensor([float(np.mean(ts))], dtype=torch.float64, device=dev)
         if world > 1:
@@ -317,9 +360,10 @@ def main():
         e_s = et.item()
         ks = q.element_size()
         e2e = {"value": round(ops_per_step / e_s / 1e6, 3), "unit": "Mops/s",
-               "h2d_bytes_per_step": int(nl * ks + (n_upd_applied * 16 if nu else 0)),
-               "d2h_bytes_per_step": int(nl * 8), "ms_per_step": round(e_s * 1e3, 3),
-               "api": "cuart_lookup_host + cuart_update_host (pinned host buffers, chunked H2D/kernel/D2H)"}
+               "h2d_bytes_per_step": int(nl * ks + nu * 16), "d2h_bytes_per_step": int(nl * 8),
+               "ms_per_step": round(e_s * 1e3, 3),
+               "api": ("cuart_lookup_host + cuart_update_host (pinned host buffers, chunked H2D/kernel/D2H)"
+                       if di is None else "pinned H2D + DistIndex.lookup/update + D2H")}
         del qh, oh, ukh, uvh
 
     cpu = None
@@ -340,24 +384,31 @@ def main():
             "data": "synthetic (seeded splitmix64 keys/queries/updates, SURVEY §8(d) recipe)",
             "config": {"workload": f"{args.config}: {cfg.description}", "keys": cfg.n_keys,
                        "lookups_per_rank": nl, "updates_per_rank": nu, "key_kind": cfg.kind,
-                       "lut_bytes": args.lut, "mode": "single" if world == 1 else "replica",
+                       "lut_bytes": args.lut, "lut_format": stats["lut_format"], "mode": mode,
+                       "parallelism": f"{mode}{world}" if world > 1 else "single",
                        "l2": "inputs (8 GiB queries) larger than L2; no flush",
                        "measured_hit_ratio": round(hit, 4), "build_s": round(build_s, 2)},
             "lookup": {"mlookups_per_s": round(world * nl / (look_ms * 1e-3) / 1e6, 3), "ms": round(look_ms, 4)},
             "update": {"mupdates_per_s": round(world * nu / (upd_ms * 1e-3) / 1e6, 3) if nu else None,
-                       "ms": round(upd_ms, 4), "ops_applied_per_rank": n_upd_applied},
+                       "ms": round(upd_ms, 4)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                         "frac": round(achieved / peak, 4), "traffic": None,
+                         "frac": round(achieved / peak, 4), "traffic": args.traffic,
                          "kernel": "k_lookup<KeyU64>" if cfg.kind == "u64" else "k_lookup<KeyU32>",
+                         "kernel_ms": round(kern_ms, 4), "lookups_per_launch": served,
                          "bytes_per_lookup": round(bytes_per_lookup, 3),
-                         "sectors_per_lookup": round(float(sec.mean()), 4), "peak_source": peak_src},
+                         "sectors_per_lookup": round(float(sec.mean()), 4), "peak_source": peak_src,
+                         "random_access_ceiling": RANDOM_CEILING},
             "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": int(launches), "clocks": clk,
-            "index": {k: stats[k] for k in ("n4", "n16", "n48", "n256", "leaf8", "arena_bytes", "max_depth")},
+            "index": {k: stats[k] for k in ("n4", "n16", "n48", "n256", "leaf8", "arena_bytes", "max_depth",
+                                            "lut_exceptions")},
         }
         print(json.dumps(line), flush=True)
+    if di is not None:
+        di.close()
+    else:
+        ix.close()
     if world > 1:
         dist.destroy_process_group()
-    ix.close()
 
 
 if __name__ == "__main__":

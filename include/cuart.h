@@ -178,6 +178,28 @@ cuart_status cuart_layout_sectors(const cuart_layout* l, const cuart_keys* queri
 cuart_status cuart_upload(const cuart_layout* l, const cuart_build_opts* opts, cuart_index** out);
 cuart_status cuart_layout_free(cuart_layout* l);  /* NULL ok */
 
+/* ---- multi-GPU routing (range-partitioned mode) ------------ */
+/* The key space is split by nparts-1 ascending splitters over the first 8 key
+ * bytes read big-endian (U64: the key; U32: key << 32; BYTES: the first 8 bytes,
+ * zero padded): owner(k) = number of splitters <= prefix8(k).  cuart_route
+ * scatters a batch into per-owner contiguous runs, STABLE in op order (so an
+ * owner that receives all sources' runs concatenated by source rank sees the ops
+ * in global rank-major order, which is what the update rule needs), and
+ * writes perm[i] = the slot of op i.  All pointers are DEVICE pointers on one
+ * device; async on `stream`.
+ *   splitters  : uint64_t[nparts-1] (device), nparts in [1, 64]
+ *   values     : uint64_t[n] or NULL (then send_values is not written)
+ *   send_keys  : same element layout as keys->data (8 / 4 / 32 B per key), n slots
+ *   send_lengths: BYTES only, uint8_t[n]
+ *   perm       : uint32_t[n];  counts: uint64_t[nparts] ops per owner
+ *   scratch    : cuart_route_scratch_bytes(n, nparts) bytes
+ * n must be < 2^32.  cuart_unroute gathers out[i] = in[perm[i]]. */
+size_t cuart_route_scratch_bytes(size_t n, uint32_t nparts);
+cuart_status cuart_route(const cuart_keys* keys, size_t n, const uint64_t* splitters, uint32_t nparts,
+                         const uint64_t* values, void* send_keys, uint8_t* send_lengths, uint64_t* send_values,
+                         uint32_t* perm, uint64_t* counts, void* scratch, void* stream);
+cuart_status cuart_unroute(const uint64_t* in, const uint32_t* perm, size_t n, uint64_t* out, void* stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -67,6 +67,12 @@ def lib():
             f.restype = ctypes.c_int
         L.cuart_status_string.argtypes = [ctypes.c_int]
         L.cuart_status_string.restype = ctypes.c_char_p
+        L.cuart_route_scratch_bytes.argtypes = [S, ctypes.c_uint32]
+        L.cuart_route_scratch_bytes.restype = S
+        L.cuart_route.argtypes = [P, S, P, ctypes.c_uint32, P, P, P, P, P, P, P, P]
+        L.cuart_route.restype = ctypes.c_int
+        L.cuart_unroute.argtypes = [P, P, S, P, P]
+        L.cuart_unroute.restype = ctypes.c_int
         L.cuart_launch_count.argtypes = []
         L.cuart_launch_count.restype = ctypes.c_uint64
         _lib = L

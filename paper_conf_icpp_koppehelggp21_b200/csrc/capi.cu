@@ -67,7 +67,7 @@ struct cuart_index {
     int grid_ctas_per_sm = 0;          // 0 = default grid (8 resident CTAs x 16 waves); else persistent grid
 };
 
-static std::atomic<uint64_t> g_launches{0};
+std::atomic<uint64_t> g_cuart_launches{0};   // also counted by route.cu
 
 #define CU_TRY(x)                                   \
     do {                                            \
@@ -172,7 +172,7 @@ static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const voi
     }
 #undef CUART_LOOKUP_POL
 #undef CUART_LOOKUP
-    g_launches++;
+    g_cuart_launches++;
     CU_TRY(cudaGetLastError());
     return CUART_OK;
 }
@@ -217,10 +217,10 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
         }
 #undef CUART_UPD1_POL
 #undef CUART_UPD1
-        g_launches++;
+        g_cuart_launches++;
         CU_TRY(cudaGetLastError());
         k_upd2<<<grid, 256, 0, s>>>(h->dix, vals + base, m, epoch_hi, h->leafref);
-        g_launches++;
+        g_cuart_launches++;
         CU_TRY(cudaGetLastError());
     }
     return CUART_OK;
@@ -246,7 +246,7 @@ const char* cuart_status_string(cuart_status s) {
     return "unknown status";
 }
 
-uint64_t cuart_launch_count(void) { return g_launches.load(); }
+uint64_t cuart_launch_count(void) { return g_cuart_launches.load(); }
 
 cuart_status cuart_layout_build(const cuart_keys* keys, const uint64_t* values, size_t n,
                                 const cuart_build_opts* opts, cuart_layout** out) {

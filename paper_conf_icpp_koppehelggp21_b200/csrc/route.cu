@@ -1,0 +1,223 @@
+// route.cu — K-ROUTE / K-UNROUTE for the range-partitioned multi-GPU layer
+// (SURVEY §8(e)).  The key space is split by P-1 splitters over the first 8 key
+// bytes (big-endian, so numeric order = lexicographic order, reading C2); the
+// owner of a key is the number of splitters <= its 8-byte prefix.  A batch is
+// scattered into per-owner contiguous runs, STABLE in op order, so that an
+// owner receiving the runs of all sources concatenated by source rank sees the
+// ops in global (rank-major) order — the order the update semantics need
+// (the highest op index wins; reading C7).
+//
+//   k_route_hist   : owner of every op (kept in scratch) + per-block histogram
+//   k_route_scan   : exclusive offsets per (owner, block) + per-owner counts
+//   k_route_scatter: stable per-owner placement via warp ballots; perm[i] = slot
+//   k_unroute      : out[i] = results[perm[i]]
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+
+#include "../../include/cuart.h"
+
+namespace {
+
+constexpr int kRouteThreads = 256;
+constexpr int kRouteItems = 16;                 // ops per thread per block
+constexpr int kRouteChunk = kRouteThreads * kRouteItems;
+constexpr uint32_t kMaxParts = 64;
+
+__device__ __forceinline__ uint64_t load_prefix8(uint32_t kind, const void* keys, const uint8_t* lens, uint64_t i) {
+    if (kind == CUART_KEY_U64) return ((const uint64_t*)keys)[i];
+    if (kind == CUART_KEY_U32) return uint64_t(((const uint32_t*)keys)[i]) << 32;
+    const uint8_t* s = (const uint8_t*)keys + i * 32;
+    const uint32_t l = lens[i];
+    uint64_t p = 0;
+#pragma unroll
+    for (int b = 0; b < 8; b++) p = (p << 8) | (uint32_t(b) < l ? s[b] : 0u);
+    return p;
+}
+
+__device__ __forceinline__ uint32_t owner_of(uint64_t prefix, const uint64_t* sp, uint32_t nsp) {
+    uint32_t lo = 0, hi = nsp;                  // number of splitters <= prefix
+    while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (sp[mid] <= prefix) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+__global__ void __launch_bounds__(kRouteThreads) k_route_hist(uint32_t kind, const void* __restrict__ keys,
+                                                              const uint8_t* __restrict__ lens, uint64_t n,
+                                                              const uint64_t* __restrict__ splitters, uint32_t nparts,
+                                                              uint8_t* __restrict__ owner, uint32_t* __restrict__ hist) {
+    __shared__ uint64_t sp[kMaxParts];
+    __shared__ uint32_t h[kMaxParts];
+    for (uint32_t t = threadIdx.x; t < kMaxParts; t += blockDim.x) {
+        if (t + 1 < nparts) sp[t] = splitters[t];
+        h[t] = 0;
+    }
+    __syncthreads();
+    const uint64_t base = uint64_t(blockIdx.x) * kRouteChunk;
+    for (int r = 0; r < kRouteItems; r++) {
+        const uint64_t i = base + uint64_t(r) * kRouteThreads + threadIdx.x;
+        if (i < n) {
+            const uint32_t o = owner_of(load_prefix8(kind, keys, lens, i), sp, nparts - 1);
+            owner[i] = uint8_t(o);
+            atomicAdd(&h[o], 1u);
+        }
+    }
+    __syncthreads();
+    for (uint32_t o = threadIdx.x; o < nparts; o += blockDim.x) hist[uint64_t(o) * gridDim.x + blockIdx.x] = h[o];
+}
+
+// Single CTA: exclusive scan of hist in (owner, block) order -> offsets, counts.
+__global__ void __launch_bounds__(1024) k_route_scan(uint32_t* __restrict__ hist, uint64_t nblocks, uint32_t nparts,
+                                                     uint64_t* __restrict__ counts) {
+    __shared__ uint64_t warp_sums[32];
+    __shared__ uint64_t carry;
+    if (threadIdx.x == 0) carry = 0;
+    __syncthreads();
+    const uint64_t total = nblocks * nparts;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (uint64_t start = 0; start < total; start += blockDim.x) {
+        const uint64_t idx = start + threadIdx.x;
+        const uint64_t v = idx < total ? hist[idx] : 0;
+        uint64_t x = v;                                   // inclusive warp scan
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint64_t y = __shfl_up_sync(0xffffffffu, x, d);
+            if (lane >= d) x += y;
+        }
+        if (lane == 31) warp_sums[warp] = x;
+        __syncthreads();
+        if (warp == 0) {
+            uint64_t w = lane < int(blockDim.x >> 5) ? warp_sums[lane] : 0;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint64_t y = __shfl_up_sync(0xffffffffu, w, d);
+                if (lane >= d) w += y;
+            }
+            warp_sums[lane] = w;
+        }
+        __syncthreads();
+        const uint64_t excl = carry + (warp ? warp_sums[warp - 1] : 0) + x - v;
+        if (idx < total) hist[idx] = uint32_t(excl);      // offsets fit 32 bits (n < 2^32 per call)
+        __syncthreads();
+        if (threadIdx.x == blockDim.x - 1) carry = excl + v;
+        __syncthreads();
+    }
+    // counts[o] = offset of owner o+1 - offset of owner o
+    for (uint32_t o = threadIdx.x; o < nparts; o += blockDim.x) {
+        const uint64_t beg = hist[uint64_t(o) * nblocks];
+        const uint64_t end = (o + 1 < nparts) ? hist[uint64_t(o + 1) * nblocks] : carry;
+        counts[o] = end - beg;
+    }
+}
+
+__global__ void __launch_bounds__(kRouteThreads) k_route_scatter(uint32_t kind, const void* __restrict__ keys,
+                                                                 const uint8_t* __restrict__ lens,
+                                                                 const uint64_t* __restrict__ values, uint64_t n,
+                                                                 uint32_t nparts, const uint8_t* __restrict__ owner,
+                                                                 const uint32_t* __restrict__ offsets,
+                                                                 void* __restrict__ send_keys, uint8_t* __restrict__ send_lens,
+                                                                 uint64_t* __restrict__ send_values,
+                                                                 uint32_t* __restrict__ perm) {
+    constexpr int kWarps = kRouteThreads / 32;
+    __shared__ uint32_t run[kMaxParts];             // placed so far in this block, per owner
+    __shared__ uint32_t wcnt[kWarps][kMaxParts];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (uint32_t o = threadIdx.x; o < nparts; o += blockDim.x) run[o] = offsets[uint64_t(o) * gridDim.x + blockIdx.x];
+    __syncthreads();
+    const uint64_t base = uint64_t(blockIdx.x) * kRouteChunk;
+    const uint32_t lt = (1u << lane) - 1;
+    for (int r = 0; r < kRouteItems; r++) {
+        const uint64_t i = base + uint64_t(r) * kRouteThreads + threadIdx.x;
+        const bool valid = i < n;
+        const uint32_t o = valid ? owner[i] : 0xFFFFFFFFu;
+        // same-owner lanes of this warp and this lane's rank among them (in lane order)
+        const uint32_t peers = __match_any_sync(0xffffffffu, o);
+        const uint32_t rank = __popc(peers & lt);
+        const bool leader = valid && (peers & lt) == 0;
+        for (uint32_t t = threadIdx.x; t < uint32_t(kWarps) * nparts; t += blockDim.x) wcnt[t / nparts][t % nparts] = 0;
+        __syncthreads();
+        if (leader) wcnt[warp][o] = __popc(peers);
+        __syncthreads();
+        if (valid) {
+            uint32_t before = 0;
+            for (int w = 0; w < warp; w++) before += wcnt[w][o];
+            const uint32_t dst = run[o] + before + rank;
+            perm[i] = dst;
+            if (kind == CUART_KEY_U64) ((uint64_t*)send_keys)[dst] = ((const uint64_t*)keys)[i];
+            else if (kind == CUART_KEY_U32) ((uint32_t*)send_keys)[dst] = ((const uint32_t*)keys)[i];
+            else {
+                const uint4* s = (const uint4*)keys + 2 * i;
+                uint4* d = (uint4*)send_keys + 2 * uint64_t(dst);
+                d[0] = s[0];
+                d[1] = s[1];
+                send_lens[dst] = lens[i];
+            }
+            if (values) send_values[dst] = values[i];
+        }
+        __syncthreads();
+        for (uint32_t oo = threadIdx.x; oo < nparts; oo += blockDim.x) {
+            uint32_t tot = 0;
+            for (int w = 0; w < kWarps; w++) tot += wcnt[w][oo];
+            run[oo] += tot;
+        }
+        __syncthreads();
+    }
+}
+
+__global__ void __launch_bounds__(256) k_unroute(const uint64_t* __restrict__ in, const uint32_t* __restrict__ perm,
+                                                 uint64_t n, uint64_t* __restrict__ out) {
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) out[i] = in[perm[i]];
+}
+
+}  // namespace
+
+extern std::atomic<uint64_t> g_cuart_launches;
+
+extern "C" {
+
+size_t cuart_route_scratch_bytes(size_t n, uint32_t nparts) {
+    const uint64_t nblocks = (n + kRouteChunk - 1) / kRouteChunk;
+    return ((n + 255) & ~size_t(255)) + nblocks * nparts * sizeof(uint32_t) + 256;
+}
+
+cuart_status cuart_route(const cuart_keys* keys, size_t n, const uint64_t* splitters, uint32_t nparts,
+                         const uint64_t* values, void* send_keys, uint8_t* send_lengths, uint64_t* send_values,
+                         uint32_t* perm, uint64_t* counts, void* scratch, void* stream) {
+    if (!keys || nparts == 0 || nparts > kMaxParts || (nparts > 1 && !splitters) || !counts) return CUART_ERR_INVALID_ARGUMENT;
+    if (n >= (uint64_t(1) << 32)) return CUART_ERR_INVALID_ARGUMENT;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (n == 0) {
+        if (cudaMemsetAsync(counts, 0, nparts * sizeof(uint64_t), s) != cudaSuccess) return CUART_ERR_CUDA;
+        return CUART_OK;
+    }
+    if (!keys->data || !send_keys || !perm || !scratch) return CUART_ERR_INVALID_ARGUMENT;
+    if (keys->kind == CUART_KEY_BYTES && (!keys->lengths || !send_lengths)) return CUART_ERR_INVALID_ARGUMENT;
+    if (values && !send_values) return CUART_ERR_INVALID_ARGUMENT;
+    const uint64_t nblocks = (n + kRouteChunk - 1) / kRouteChunk;
+    uint8_t* owner = (uint8_t*)scratch;
+    uint32_t* hist = (uint32_t*)((uint8_t*)scratch + ((n + 255) & ~size_t(255)));
+    const uint32_t kind = uint32_t(keys->kind);
+    k_route_hist<<<unsigned(nblocks), kRouteThreads, 0, s>>>(kind, keys->data, keys->lengths, n, splitters, nparts, owner, hist);
+    k_route_scan<<<1, 1024, 0, s>>>(hist, nblocks, nparts, counts);
+    k_route_scatter<<<unsigned(nblocks), kRouteThreads, 0, s>>>(kind, keys->data, keys->lengths, values, n, nparts, owner,
+                                                                hist, send_keys, send_lengths, send_values, perm);
+    g_cuart_launches += 3;
+    return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+}
+
+cuart_status cuart_unroute(const uint64_t* in, const uint32_t* perm, size_t n, uint64_t* out, void* stream) {
+    if (n == 0) return CUART_OK;
+    if (!in || !perm || !out) return CUART_ERR_INVALID_ARGUMENT;
+    uint64_t blocks = (n + 255) / 256;
+    if (blocks > (uint64_t(1) << 31) - 1) blocks = (uint64_t(1) << 31) - 1;
+    k_unroute<<<unsigned(blocks), 256, 0, (cudaStream_t)stream>>>(in, perm, n, out);
+    g_cuart_launches += 1;
+    return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+}
+
+}  // extern "C"

@@ -1,0 +1,234 @@
+"""Multi-GPU layer: one process per GPU, torch.distributed for the
+plumbing (NCCL over NVLink/NVSwitch on the GPU box), CuART kernels for all data
+movement on the device.
+
+Two modes:
+
+* ``replica`` — every rank holds the full index.  Lookups need no exchange: a
+  rank serves its own share of the query stream.  Update batches are
+  all-gathered and applied everywhere in global (rank-major) order, so replicas
+  stay bit-identical.
+* ``range``  — the key space is range-partitioned over the first 8 key bytes
+  (big-endian) with quantile splitters computed from the key distribution, so
+  skewed and dense key sets balance.  Each rank indexes only its range.  A
+  batch is routed to the owners (cuart_route: stable per-owner runs + a
+  permutation), exchanged with all-to-all (counts, then the runs), served by the
+  owner's local index, sent back with the reverse all-to-all and restored to
+  query order (cuart_unroute).  Updates travel with their values; because the
+  runs of all sources arrive concatenated by source rank and are stable in op
+  order, the owner applies them in global rank-major order — the highest global
+  op index wins (reading C7).
+
+The protocol is written once against an ``ops`` object: ``CudaOps`` (product,
+C-ABI kernels, CUDA tensors, NCCL) or an injected test double (CPU tensors and
+the gloo backend) so the exchange logic runs in the CPU test suite.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+from . import _binding as B
+
+
+# ------------------------------------------------------------------ partitioning (host)
+def prefix8(keys) -> np.ndarray:
+    """First 8 key bytes read big-endian, as uint64 (numeric order = key order)."""
+    if isinstance(keys, tuple):
+        slots, lens = keys
+        slots = np.asarray(slots, np.uint8)
+        lens = np.asarray(lens, np.uint8)
+        head = slots[:, :8].copy()
+        head[np.arange(8)[None, :] >= lens[:, None]] = 0
+        return np.ascontiguousarray(head).view(">u8").ravel().astype(np.uint64)
+    keys = np.asarray(keys)
+    if keys.dtype == np.uint32:
+        return keys.astype(np.uint64) << np.uint64(32)
+    return keys.astype(np.uint64)
+
+
+def compute_splitters(sample_prefix: np.ndarray, nparts: int) -> np.ndarray:
+    """nparts-1 quantile splitters; owner(k) = number of splitters <= prefix8(k)."""
+    if nparts <= 1:
+        return np.zeros(0, np.uint64)
+    s = np.sort(np.asarray(sample_prefix, np.uint64))
+    if s.shape[0] == 0:
+        return (np.arange(1, nparts, dtype=np.uint64) * np.uint64((1 << 64) // nparts))
+    idx = (np.arange(1, nparts) * s.shape[0]) // nparts
+    return s[idx].astype(np.uint64)
+
+
+def owners(prefix: np.ndarray, splitters: np.ndarray) -> np.ndarray:
+    return np.searchsorted(splitters, prefix, side="right").astype(np.int64)
+
+
+def select(keys, mask):
+    if isinstance(keys, tuple):
+        return (keys[0][mask], keys[1][mask])
+    return keys[mask]
+
+
+# ------------------------------------------------------------------ device ops (product)
+class CudaOps:
+    """Product ops: CuART C-ABI kernels on CUDA tensors; collectives go over NCCL."""
+
+    def __init__(self, device):
+        self.device = torch.device(device)
+
+    def build(self, keys, values, lut_bytes):
+        return B.Index(keys, values, lut_bytes=lut_bytes, device=self.device.index or 0)
+
+    def tensor(self, a):
+        if isinstance(a, np.ndarray):
+            if a.dtype == np.uint64:
+                a = a.view(np.int64)
+            elif a.dtype == np.uint32:
+                a = a.view(np.int32)
+            return torch.from_numpy(a).to(self.device)
+        return a.to(self.device)
+
+    def route(self, keys, lens, values, splitters, nparts):
+        n = keys.shape[0]
+        send_keys = torch.empty_like(keys)
+        send_lens = torch.empty_like(lens) if lens is not None else None
+        send_vals = torch.empty_like(values) if values is not None else None
+        perm = torch.empty(n, dtype=torch.int32, device=self.device)
+        counts = torch.empty(nparts, dtype=torch.int64, device=self.device)
+        scratch = torch.empty(max(1, B.lib().cuart_route_scratch_bytes(n, nparts)), dtype=torch.uint8, device=self.device)
+        k, _, keep = B.make_keys((keys, lens) if lens is not None else keys)
+        stream = torch.cuda.current_stream(self.device).cuda_stream
+        rc = B.lib().cuart_route(B.ctypes.byref(k), n, splitters.data_ptr() if nparts > 1 else None, nparts,
+                                 values.data_ptr() if values is not None else None, send_keys.data_ptr(),
+                                 send_lens.data_ptr() if send_lens is not None else None,
+                                 send_vals.data_ptr() if send_vals is not None else None,
+                                 perm.data_ptr(), counts.data_ptr(), scratch.data_ptr(), stream)
+        B._check(rc, "cuart_route")
+        return send_keys, send_lens, send_vals, perm, counts
+
+    def unroute(self, res, perm):
+        out = torch.empty_like(res)
+        stream = torch.cuda.current_stream(self.device).cuda_stream
+        B._check(B.lib().cuart_unroute(res.data_ptr(), perm.data_ptr(), res.shape[0], out.data_ptr(), stream),
+                 "cuart_unroute")
+        return out
+
+    def lookup(self, index, keys, lens):
+        out = torch.empty(keys.shape[0], dtype=torch.int64, device=self.device)
+        index.lookup((keys, lens) if lens is not None else keys, out)
+        return out
+
+    def update(self, index, keys, lens, values):
+        index.update((keys, lens) if lens is not None else keys, values)
+
+    def close(self, index):
+        index.close()
+
+
+# ------------------------------------------------------------------ the protocol
+class DistIndex:
+    """A CuART index spread over the ranks of a process group."""
+
+    def __init__(self, keys, values, mode="range", group=None, ops=None, lut_bytes=3, splitters=None):
+        """keys/values: the GLOBAL key set, identical on every rank (host arrays).
+        Range mode keeps this rank's share; replica mode keeps everything."""
+        if mode not in ("range", "replica"):
+            raise ValueError(mode)
+        self.mode = mode
+        self.group = group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.ops = ops
+        values = np.asarray(values, np.uint64)
+        self.kind_bytes = isinstance(keys, tuple)
+        if mode == "range":
+            pre = prefix8(keys)
+            self.splitters_np = compute_splitters(pre, self.world) if splitters is None else np.asarray(splitters, np.uint64)
+            mine = owners(pre, self.splitters_np) == self.rank
+            keys, values = select(keys, mine), values[mine]
+            self.splitters = ops.tensor(self.splitters_np.view(np.int64).copy()) if self.world > 1 else None
+        self.n_local_keys = int(values.shape[0])
+        self.index = ops.build(keys, values, lut_bytes)
+
+    # ---- helpers
+    def _a2a(self, out, inp, out_splits, in_splits):
+        dist.all_to_all_single(out, inp, out_splits, in_splits, group=self.group)
+
+    def _exchange_counts(self, counts):
+        recv = torch.empty_like(counts)
+        dist.all_to_all_single(recv, counts, group=self.group)
+        return recv
+
+    def _split_keys(self, q):
+        return (q[0], q[1]) if isinstance(q, tuple) else (q, None)
+
+    # ---- lookups
+    def lookup(self, queries, events=None):
+        """events: optional (start, end) CUDA events recorded around the local lookup kernel."""
+        keys, lens = self._split_keys(queries)
+        if self.mode == "replica" or self.world == 1:
+            if events:
+                events[0].record()
+            r = self.ops.lookup(self.index, keys, lens)
+            if events:
+                events[1].record()
+            return r
+        sk, sl, _, perm, counts = self.ops.route(keys, lens, None, self.splitters, self.world)
+        rcounts = self._exchange_counts(counts)
+        cs, rs = counts.tolist(), rcounts.tolist()
+        rk = sk.new_empty((sum(rs),) + tuple(sk.shape[1:]))
+        self._a2a(rk, sk, rs, cs)
+        rl = None
+        if sl is not None:
+            rl = sl.new_empty(sum(rs))
+            self._a2a(rl, sl, rs, cs)
+        if events:
+            events[0].record()
+        res = self.ops.lookup(self.index, rk, rl)
+        if events:
+            events[1].record()
+        self.last_local_lookups = int(rk.shape[0])
+        back = res.new_empty(keys.shape[0])
+        self._a2a(back, res, cs, rs)
+        return self.ops.unroute(back, perm)
+
+    # ---- updates (one batch per rank; global order = rank-major)
+    def update(self, keys_vals):
+        (keys, lens), vals = self._split_keys(keys_vals[0]), keys_vals[1]
+        if self.world == 1:
+            self.ops.update(self.index, keys, lens, vals)
+            return
+        if self.mode == "replica":
+            gk, gl, gv = self._all_gather_var(keys), (self._all_gather_var(lens) if lens is not None else None), \
+                self._all_gather_var(vals)
+            self.ops.update(self.index, gk, gl, gv)
+            return
+        sk, sl, sv, _, counts = self.ops.route(keys, lens, vals, self.splitters, self.world)
+        rcounts = self._exchange_counts(counts)
+        cs, rs = counts.tolist(), rcounts.tolist()
+        rk = sk.new_empty((sum(rs),) + tuple(sk.shape[1:]))
+        self._a2a(rk, sk, rs, cs)
+        rv = sv.new_empty(sum(rs))
+        self._a2a(rv, sv, rs, cs)
+        rl = None
+        if sl is not None:
+            rl = sl.new_empty(sum(rs))
+            self._a2a(rl, sl, rs, cs)
+        self.ops.update(self.index, rk, rl, rv)
+
+    def _all_gather_var(self, t):
+        n = torch.tensor([t.shape[0]], dtype=torch.int64, device=t.device)
+        ns = [torch.empty_like(n) for _ in range(self.world)]
+        dist.all_gather(ns, n, group=self.group)
+        sizes = [int(x.item()) for x in ns]
+        m = max(sizes)
+        pad = t.new_zeros((m,) + tuple(t.shape[1:]))
+        pad[: t.shape[0]] = t
+        g = t.new_empty((self.world * m,) + tuple(t.shape[1:]))
+        dist.all_gather_into_tensor(g, pad, group=self.group)
+        return torch.cat([g[r * m: r * m + sizes[r]] for r in range(self.world)])
+
+    def close(self):
+        if self.index is not None:
+            self.ops.close(self.index)
+            self.index = None
