@@ -134,13 +134,13 @@ __global__ void __launch_bounds__(kRouteThreads) k_route_scatter(uint32_t kind, 
         const uint64_t i = base + uint64_t(r) * kRouteThreads + threadIdx.x;
         const bool valid = i < n;
         const uint32_t o = valid ? owner[i] : 0xFFFFFFFFu;
-        // same-owner lanes of this warp and this lane's rank among them (in lane order)
-        const uint32_t peers = __match_any_sync(0xffffffffu, o);
-        const uint32_t rank = __popc(peers & lt);
-        const bool leader = valid && (peers & lt) == 0;
-        for (uint32_t t = threadIdx.x; t < uint32_t(kWarps) * nparts; t += blockDim.x) wcnt[t / nparts][t % nparts] = 0;
-        __syncthreads();
-        if (leader) wcnt[warp][o] = __popc(peers);
+        // per-owner ballots: warp counts, and this lane's rank among same-owner lanes
+        uint32_t rank = 0;
+        for (uint32_t oo = 0; oo < nparts; oo++) {
+            const uint32_t m = __ballot_sync(0xffffffffu, o == oo);
+            if (o == oo) rank = __popc(m & lt);
+            if (lane == 0) wcnt[warp][oo] = __popc(m);
+        }
         __syncthreads();
         if (valid) {
             uint32_t before = 0;
