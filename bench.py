@@ -51,7 +51,7 @@ def _args():
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=10)
     p.add_argument("--warmup", type=int, default=3)
-    p.add_argument("--config", default="c3", choices=["c1", "c2", "c3"])
+    p.add_argument("--config", default="c3", choices=["c1", "c2", "c3", "c4"])
     p.add_argument("--impl", default="cuart", choices=["cuart", "reference"])
     p.add_argument("--lut", type=int, default=3)
     p.add_argument("--no-e2e", action="store_true")
@@ -123,7 +123,7 @@ def oracle_timing(cfg, keys, vals, n_lookup_sample, n_update_sample, reps=1):
     t0 = time.perf_counter()
     o = ArtOracle(keys, vals)
     build_s = time.perf_counter() - t0
-    q = W.lookup_batch(cfg, keys, 0, n_lookup_sample)
+    q = host_lookups(cfg, keys, 0, n_lookup_sample)
     uk, uv = W.update_batch(cfg, keys, 0, n_update_sample) if cfg.n_updates else (None, None)
     times = []
     for _ in range(reps):
@@ -139,6 +139,13 @@ def oracle_timing(cfg, keys, vals, n_lookup_sample, n_update_sample, reps=1):
                             "sample_updates": n_update_sample if uk is not None else 0, "seconds": round(dt, 3)}
 
 
+def host_lookups(cfg, keys, start, m):
+    if isinstance(keys, tuple):
+        idx = W.string_lookup_at(cfg, keys[1].shape[0], np.arange(start, start + m))
+        return (keys[0][idx], keys[1][idx])
+    return W.lookup_batch(cfg, keys, start, m)
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -147,14 +154,18 @@ def run_reference(args):
     keys, vals = W.build_set(cfg)
     from oracle import ArtOracle
     t0 = time.perf_counter()
-    o = ArtOracle(np.sort(keys) if keys.dtype != object else keys, vals[np.argsort(keys)])
+    if isinstance(keys, tuple):
+        o = ArtOracle(keys, vals)
+    else:   # insertion order does not change the tree (pinned); sorted inserts build faster
+        order = np.argsort(keys)
+        o = ArtOracle(keys[order], vals[order])
     build_s = time.perf_counter() - t0
     # bounded sample per step, same lookup:update mix as the workload
     nl = min(cfg.n_lookups, 1 << 20)
     nu = min(cfg.n_updates, max(1, nl * cfg.n_updates // cfg.n_lookups)) if cfg.n_updates else 0
     times = []
     for s in range(args.warmup + args.steps):
-        q = W.lookup_batch(cfg, keys, s * nl, nl)
+        q = host_lookups(cfg, keys, s * nl, nl)
         uk, uv = W.update_batch(cfg, keys, s * nu, nu) if nu else (None, None)
         t0 = time.perf_counter()
         o.lookup(q)
@@ -167,7 +178,7 @@ def run_reference(args):
     val = (nl + nu) / (ms * 1e-3) / 1e6
     line = {"impl": "reference", "metric": METRIC, "value": round(val, 3), "unit": "Mops/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": {"u64": "u64", "u32": "u32", "bytes": "u8[32]"}[cfg.kind],
             "data": "synthetic (seeded splitmix64, SURVEY §8(d) recipe)",
             "config": {"workload": f"{args.config}: {cfg.description}", "sample_per_step":
                        {"lookups": nl, "updates": nu}},
@@ -177,6 +188,28 @@ def run_reference(args):
                                        f"({build_s:.1f} s, untimed)"},
             "e2e": {"value": round(val, 3), "unit": "Mops/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ inputs
+def make_keys(cfg, dev):
+    """(host keys, host values, device keys) of the config's build set."""
+    import torch
+    c = W.config_id(cfg)
+    vals = W.values_for(W.SEED_VALUES + c, np.arange(cfg.n_keys, dtype=np.uint64))
+    if cfg.kind == "u64":
+        keys_d = W.u64_keys_torch(c, cfg.n_keys, dev)
+        return keys_d.cpu().numpy().view(np.uint64), vals, keys_d
+    if cfg.kind == "u32":
+        keys = np.arange(cfg.n_keys, dtype=np.uint32)
+        return keys, vals, torch.from_numpy(keys.view(np.int32)).to(dev)
+    slots, lens = W.string_keys(c, cfg.n_keys)
+    return (slots, lens), vals[: lens.shape[0]], (torch.from_numpy(slots).to(dev), torch.from_numpy(lens).to(dev))
+
+
+def make_lookups(cfg, keys_d, start, m, dev):
+    if cfg.kind == "bytes":
+        return W.string_lookup_torch(cfg, keys_d[0], keys_d[1], start, m)
+    return W.lookup_batch_torch(cfg, keys_d, start, m, device=dev)
 
 
 # ------------------------------------------------------------------ main (GPU)
@@ -202,13 +235,7 @@ def main():
 
     cfg = W.CONFIGS[args.config]
     t0 = time.perf_counter()
-    if cfg.kind == "u64":
-        keys_d = W.u64_keys_torch(W.config_id(cfg), cfg.n_keys, dev)
-        keys = keys_d.cpu().numpy().view(np.uint64)
-    else:
-        keys = np.arange(cfg.n_keys, dtype=np.uint32)
-        keys_d = torch.from_numpy(keys.view(np.int32)).to(dev)
-    vals = W.values_for(W.SEED_VALUES + W.config_id(cfg), np.arange(cfg.n_keys, dtype=np.uint64))
+    keys, vals, keys_d = make_keys(cfg, dev)
     ops = CudaOps(dev)
     if world == 1:
         layout = C.Layout(keys, vals, lut_bytes=args.lut)
@@ -223,7 +250,7 @@ def main():
 
     # resident inputs: this rank's shard of the global lookup stream and update stream
     nl = cfg.n_lookups
-    q = W.lookup_batch_torch(cfg, keys_d, rank * nl, nl, device=dev)
+    q = make_lookups(cfg, keys_d, rank * nl, nl, dev)
     out = torch.empty(nl, dtype=torch.int64, device=dev)
     nu = cfg.n_updates
     uk = uv = None
@@ -233,18 +260,20 @@ def main():
 
     # algorithmic bytes of the dominant kernel (k_lookup): exact sector count of the
     # lookup path over this rank's layout for a 2^20-query sample + key-in/value-out
+    from paper_conf_icpp_koppehelggp21_b200.dist import owners, prefix8, select
     if layout is None:
-        from paper_conf_icpp_koppehelggp21_b200.dist import owners, prefix8
-        local_keys = keys if mode == "replica" else keys[owners(prefix8(keys), di.splitters_np) == rank]
-        local_vals = np.zeros(local_keys.shape[0], np.uint64)
-        layout = C.Layout(local_keys, local_vals, lut_bytes=args.lut)
-    samp = q[: 1 << 20].cpu().numpy()
-    samp = samp.view(np.uint64) if cfg.kind == "u64" else samp.view(np.uint32)
+        local_keys = keys if mode == "replica" else select(keys, owners(prefix8(keys), di.splitters_np) == rank)
+        nloc = local_keys[1].shape[0] if isinstance(local_keys, tuple) else local_keys.shape[0]
+        layout = C.Layout(local_keys, np.zeros(nloc, np.uint64), lut_bytes=args.lut)
+    if isinstance(q, tuple):
+        samp = (q[0][: 1 << 20].cpu().numpy(), q[1][: 1 << 20].cpu().numpy())
+    else:
+        samp = q[: 1 << 20].cpu().numpy()
+        samp = samp.view(np.uint64) if cfg.kind == "u64" else samp.view(np.uint32)
     if mode == "range":   # sample of the queries this rank's index actually serves
-        from paper_conf_icpp_koppehelggp21_b200.dist import owners, prefix8
-        samp = samp[owners(prefix8(samp), di.splitters_np) == rank]
+        samp = select(samp, owners(prefix8(samp), di.splitters_np) == rank)
     sec = layout.sectors(samp).astype(np.float64)
-    io_bytes = (8 if cfg.kind == "u64" else 4) + 8
+    io_bytes = {"u64": 8, "u32": 4, "bytes": 33}[cfg.kind] + 8
     bytes_per_lookup = 32.0 * sec.mean() + io_bytes
     del samp
 
@@ -323,8 +352,14 @@ def main():
     # end-to-end through the public API with HOST buffers (pinned), copies inside the timed region
     e2e = None
     if not args.no_e2e:
-        qh = torch.empty(nl, dtype=q.dtype, pin_memory=True)
-        qh.copy_(q)
+        def pinned(t):
+            h = torch.empty(t.shape, dtype=t.dtype, pin_memory=True)
+            h.copy_(t)
+            return h
+
+        qh = tuple(pinned(t) for t in q) if isinstance(q, tuple) else pinned(q)
+        qn = tuple(t.numpy() for t in qh) if isinstance(qh, tuple) else qh.numpy()
+        qbytes = sum(t.numel() * t.element_size() for t in qh) if isinstance(qh, tuple) else qh.numel() * qh.element_size()
         oh = torch.empty(nl, dtype=torch.int64, pin_memory=True)
         ukh = uvh = None
         if nu:
@@ -335,11 +370,11 @@ def main():
 
         def e2e_step():
             if di is None:
-                C.cuart_lookup_host(ix.h, qh.numpy(), oh.numpy())
+                C.cuart_lookup_host(ix.h, qn, oh.numpy())
                 if nu:
                     C.cuart_update_host(ix.h, ukh.numpy(), uvh.numpy())
             else:
-                qd = qh.to(dev, non_blocking=True)
+                qd = tuple(t.to(dev, non_blocking=True) for t in qh) if isinstance(qh, tuple) else qh.to(dev, non_blocking=True)
                 oh.copy_(di.lookup(qd), non_blocking=True)
                 if nu:
                     di.update((ukh.to(dev, non_blocking=True), uvh.to(dev, non_blocking=True)))
@@ -358,13 +393,12 @@ def main():
         if world > 1:
             dist.all_reduce(et, op=dist.ReduceOp.MAX)
         e_s = et.item()
-        ks = q.element_size()
         e2e = {"value": round(ops_per_step / e_s / 1e6, 3), "unit": "Mops/s",
-               "h2d_bytes_per_step": int(nl * ks + nu * 16), "d2h_bytes_per_step": int(nl * 8),
+               "h2d_bytes_per_step": int(qbytes + nu * 16), "d2h_bytes_per_step": int(nl * 8),
                "ms_per_step": round(e_s * 1e3, 3),
                "api": ("cuart_lookup_host + cuart_update_host (pinned host buffers, chunked H2D/kernel/D2H)"
                        if di is None else "pinned H2D + DistIndex.lookup/update + D2H")}
-        del qh, oh, ukh, uvh
+        del qh, qn, oh, ukh, uvh
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -380,7 +414,8 @@ def main():
         line = {
             "metric": METRIC, "value": round(value, 3), "unit": "Mops/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 4),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": {"u64": "u64", "u32": "u32", "bytes": "u8[32]"}[cfg.kind],
             "data": "synthetic (seeded splitmix64 keys/queries/updates, SURVEY §8(d) recipe)",
             "config": {"workload": f"{args.config}: {cfg.description}", "keys": cfg.n_keys,
                        "lookups_per_rank": nl, "updates_per_rank": nu, "key_kind": cfg.kind,
@@ -393,7 +428,7 @@ def main():
                        "ms": round(upd_ms, 4)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": args.traffic,
-                         "kernel": "k_lookup<KeyU64>" if cfg.kind == "u64" else "k_lookup<KeyU32>",
+                         "kernel": {"u64": "k_lookup<KeyU64>", "u32": "k_lookup<KeyU32>", "bytes": "k_lookup<KeyBytes>"}[cfg.kind],
                          "kernel_ms": round(kern_ms, 4), "lookups_per_launch": served,
                          "bytes_per_lookup": round(bytes_per_lookup, 3),
                          "sectors_per_lookup": round(float(sec.mean()), 4), "peak_source": peak_src,

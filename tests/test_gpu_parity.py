@@ -273,3 +273,63 @@ def test_c3_full_size_sampled():
     mp.update(_u64(uk), _u64(uv))
     assert np.array_equal(_u64(out2), mp.lookup(keys[: 1 << 22]))
     ix.close()
+
+
+def test_c4_strings_scaled():
+    """Config-4 recipe (hierarchical skewed prefixes, 8-32 B keys, Zipf lookups) at
+    2^20 keys / 2^22 lookups, element by element vs the pointer-ART oracle."""
+    cfg = W.CONFIGS["c4"]
+    slots, lens = W.string_keys(4, 1 << 20)
+    vals = W.values_for(W.SEED_VALUES + 4, np.arange(1 << 20, dtype=np.uint64))
+    o = ArtOracle((slots, lens), vals)
+    ix = C.Index((slots, lens), vals)
+    st = ix.stats()
+    os_ = o.stats()
+    assert (st["n4"], st["n16"], st["n48"], st["n256"]) == (os_["n4"], os_["n16"], os_["n48"], os_["n256"])
+    assert st["leaf16"] > 0 and st["leaf32"] > 0
+    sd, ld = torch.from_numpy(slots).to(DEV), torch.from_numpy(lens).to(DEV)
+    qs, ql = W.string_lookup_torch(cfg, sd, ld, 0, 1 << 22)
+    out = torch.empty(1 << 22, dtype=torch.int64, device=DEV)
+    ix.lookup((qs, ql), out)
+    torch.cuda.synchronize()
+    qn = (qs.cpu().numpy(), ql.cpu().numpy())
+    exp = o.lookup(qn)
+    assert np.array_equal(_u64(out), exp)
+    assert not np.any(exp == OART_MISS)                      # 100% hit
+    # perturbed queries: one flipped byte / truncated length -> misses where absent
+    pq = qn[0][:100_000].copy()
+    pq[:, 3] ^= 1
+    pl = qn[1][:100_000].copy()
+    pl[::2] -= 1
+    out2 = torch.empty(100_000, dtype=torch.int64, device=DEV)
+    ix.lookup((torch.from_numpy(pq).to(DEV), torch.from_numpy(pl).to(DEV)), out2)
+    torch.cuda.synchronize()
+    assert np.array_equal(_u64(out2), o.lookup((pq, pl)))
+    # updates with string keys
+    ui = np.random.default_rng(1).integers(0, 1 << 20, 300_000)
+    uv = np.random.default_rng(2).integers(0, 2**63, 300_000, dtype=np.uint64)
+    ix.update((torch.from_numpy(slots[ui]).to(DEV), torch.from_numpy(lens[ui]).to(DEV)), _t(uv))
+    o.update((slots[ui], lens[ui]), uv)
+    assert to_records(ix.dump()) == o.dump_structure().tolist()
+    ix.close()
+
+
+@pytest.mark.slow
+def test_c4_full_size_sampled():
+    """Config 4 at full size (2^25 keys, 2^29 Zipf lookups) in the bench's launch
+    configuration; sampled outputs vs the plain-map oracle; 100% hit everywhere."""
+    cfg = W.CONFIGS["c4"]
+    slots, lens = W.string_keys(4, cfg.n_keys)
+    vals = W.values_for(W.SEED_VALUES + 4, np.arange(cfg.n_keys, dtype=np.uint64))
+    ix = C.Index((slots, lens), vals)
+    sd, ld = torch.from_numpy(slots).to(DEV), torch.from_numpy(lens).to(DEV)
+    qs, ql = W.string_lookup_torch(cfg, sd, ld, 0, cfg.n_lookups)
+    out = torch.empty(cfg.n_lookups, dtype=torch.int64, device=DEV)
+    ix.lookup((qs, ql), out)
+    torch.cuda.synchronize()
+    assert not bool((out == -1).any().item())
+    idx = np.sort(np.random.default_rng(4).choice(cfg.n_lookups, 200_000, replace=False))
+    ti = torch.from_numpy(idx).to(DEV)
+    mp = MapOracle((slots, lens), vals)
+    assert np.array_equal(_u64(out[ti]), mp.lookup((qs[ti].cpu().numpy(), ql[ti].cpu().numpy())))
+    ix.close()

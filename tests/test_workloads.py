@@ -54,3 +54,13 @@ def test_string_keys_prefix_free_and_distinct():
         k = bytes(slots[i, : lens[i]])
         assert k[-1] == 0 and 0 not in k[:-1]
         assert not slots[i, lens[i]:].any()
+
+
+def test_string_lookup_torch_twin():
+    cfg = W.CONFIGS["c4"]
+    slots, lens = W.string_keys(4, 50_000)
+    idx = W.string_lookup_at(cfg, 50_000, np.arange(1000, 6000))
+    qs, ql = W.string_lookup_torch(cfg, torch.from_numpy(slots), torch.from_numpy(lens), 1000, 5000)
+    assert np.array_equal(qs.numpy(), slots[idx]) and np.array_equal(ql.numpy(), lens[idx])
+    # Zipf(0.99) skew: the hottest key takes a large share
+    assert np.bincount(idx).max() > 100

@@ -200,32 +200,60 @@ def string_keys(c: int, n: int, max_len: int = MAX_KEY, min_len: int = 8):
     seed = SEED_KEYS + c
     seg1 = ALPHABET[(splitmix64(seed + 11, np.arange(16 * 6, dtype=np.uint64)) % np.uint64(42)).astype(np.int64)].reshape(16, 6)
     seg2 = ALPHABET[(splitmix64(seed + 12, np.arange(256 * 6, dtype=np.uint64)) % np.uint64(42)).astype(np.int64)].reshape(256, 6)
-    out_slots, out_lens, have = [], [], 0
-    seen = set() if n <= 1 << 16 else None
-    base = 0
+    out_slots, out_lens, out_hash = [], [], []
+    have, base = 0, 0
     while have < n:
-        m = int((n - have) * 1.3) + 1024
+        m = int((n - have) * 1.35) + 1024
         j = np.arange(base, base + m, dtype=np.uint64)
         base += m
         L = (min_len + (splitmix64(seed + 1, j) % np.uint64(max_len - min_len + 1))).astype(np.int64)
         i1 = _zipf_index(_u01(seed + 2, j), 16, 1.2)
         i2 = _zipf_index(_u01(seed + 3, j), 256, 1.0)
-        content = np.empty((m, max_len), dtype=np.uint8)
-        content[:, 0:6] = seg1[i1]
-        content[:, 6:12] = seg2[i2]
-        for col in range(12, max_len):
-            content[:, col] = ALPHABET[(splitmix64(seed + 100 + col, j) % np.uint64(42)).astype(np.int64)]
-        pos = np.arange(max_len)[None, :]
-        slots = np.where(pos < (L - 1)[:, None], content, 0).astype(np.uint8)  # terminator + zero pad
+        slots = np.zeros((m, max_len), dtype=np.uint8)
+        slots[:, 0:6] = seg1[i1]
+        slots[:, 6:12] = seg2[i2]
+        for k, col in enumerate(range(12, max_len, 8)):       # 8 suffix symbols per draw
+            r = splitmix64(seed + 100 + k, j).view(np.uint8).reshape(m, 8)
+            width = min(8, max_len - col)
+            slots[:, col: col + width] = ALPHABET[(r[:, :width].astype(np.uint16) * 42) >> 8]
+        slots[np.arange(max_len)[None, :] >= (L - 1)[:, None]] = 0          # terminator + zero pad
+        # dedupe on a 64-bit digest of the slot (first occurrence wins, draw order kept);
+        # a digest collision between distinct keys only drops a candidate
+        w = slots.view(np.uint64)
+        h = splitmix64(int(w[0, 0]) & 0, w[:, 0])
+        for k in range(1, max_len // 8):
+            h = splitmix64(0, h ^ w[:, k])
         out_slots.append(slots)
         out_lens.append(L.astype(np.uint8))
-        allslots = np.concatenate(out_slots)
-        alllens = np.concatenate(out_lens)
-        _, first = np.unique(allslots.view(np.dtype((np.void, max_len))).ravel(), return_index=True)
+        out_hash.append(h)
+        allh = np.concatenate(out_hash)
+        _, first = np.unique(allh, return_index=True)
         first.sort()
-        out_slots, out_lens = [allslots[first]], [alllens[first]]
+        allslots = np.concatenate(out_slots)[first]
+        out_slots, out_lens, out_hash = [allslots], [np.concatenate(out_lens)[first]], [allh[first]]
         have = first.shape[0]
     return out_slots[0][:n].copy(), out_lens[0][:n].copy()
+
+
+def zipf_ranks(seed: int, counter, n: int, theta: float = 0.99) -> np.ndarray:
+    """Zipf(theta) ranks in [0, n) by inverse CDF of counter-based uniforms."""
+    w = 1.0 / np.arange(1, n + 1, dtype=np.float64) ** theta
+    cdf = np.cumsum(w)
+    cdf /= cdf[-1]
+    return np.minimum(np.searchsorted(cdf, _u01(seed, counter), side="right"), n - 1)
+
+
+def rank_permutation(seed: int, n: int) -> np.ndarray:
+    """Seeded permutation mapping Zipf rank -> key index (hot keys spread over the set)."""
+    return np.argsort(splitmix64(seed, np.arange(n, dtype=np.uint64)), kind="stable")
+
+
+def string_lookup_at(cfg: Config, n_keys: int, j) -> np.ndarray:
+    """Key indices of c4 lookups at stream positions j: Zipf(0.99) over key ranks,
+    ranks mapped to keys by a seeded permutation (100% hit)."""
+    c = config_id(cfg)
+    perm = rank_permutation(SEED_QUERIES + c + 7, n_keys)
+    return perm[zipf_ranks(SEED_QUERIES + c, np.asarray(j, dtype=np.uint64), n_keys)]
 
 
 # ----------------------------------------------------------------------------- torch twins
@@ -311,3 +339,27 @@ def update_batch_torch(cfg: Config, keys, start: int = 0, m: int | None = None):
     vals = splitmix64_torch(SEED_UVALUES + c, j)
     vals = torch.where(vals == -1, torch.zeros_like(vals), vals)
     return out, vals
+
+
+def string_lookup_torch(cfg: Config, slots_d, lens_d, start: int, m: int, cdf_d=None, perm_d=None):
+    """torch twin of string_lookup_at for positions [start, start+m): returns
+    (query slots uint8[m,32], lens uint8[m]) gathered on the keys' device.  The
+    Zipf CDF is built on the host (numpy, exact) and the permutation sorts the
+    same splitmix64 draws as unsigned, so ranks and keys match the numpy twin."""
+    import torch
+    c = config_id(cfg)
+    n = slots_d.shape[0]
+    dev = slots_d.device
+    if cdf_d is None:
+        w = 1.0 / np.arange(1, n + 1, dtype=np.float64) ** 0.99
+        cdf = np.cumsum(w)
+        cdf /= cdf[-1]
+        cdf_d = torch.from_numpy(cdf).to(dev)
+    if perm_d is None:
+        draws = splitmix64_torch(SEED_QUERIES + c + 7, torch.arange(n, dtype=torch.int64, device=dev))
+        perm_d = torch.argsort(draws ^ (-(1 << 63)), stable=True)        # unsigned order
+    j = torch.arange(start, start + m, dtype=torch.int64, device=dev)
+    u = _t_srl(splitmix64_torch(SEED_QUERIES + c, j), 11).to(torch.float64) * (1.0 / (1 << 53))
+    r = torch.clamp(torch.searchsorted(cdf_d, u, right=True), max=n - 1)
+    idx = perm_d[r]
+    return slots_d[idx], lens_d[idx]
