@@ -50,6 +50,10 @@ def _load():
         lib.oart_dump_structure.argtypes = [P, P, SZ]
         lib.oart_dump_structure.restype = SZ
         lib.oart_stats.argtypes = [P, P]
+        lib.oart_erase.argtypes = [P, P, U32]
+        lib.oart_erase.restype = ctypes.c_int
+        lib.oart_apply_batch.argtypes = [P, P, P, U32, SZ, P, P, SZ]
+        lib.oart_apply_batch.restype = ctypes.c_int64
         _lib = lib
     return _lib
 
@@ -137,6 +141,22 @@ class ArtOracle:
             raise ValueError("update value is the reserved miss value")
         return int(hits)
 
+    def erase_one(self, key: bytes) -> int:
+        buf = (ctypes.c_uint8 * max(1, len(key))).from_buffer_copy(key or b"\0")
+        return int(self._lib.oart_erase(self._t, buf, len(key)))
+
+    def apply(self, keys, values, is_delete) -> int:
+        """Batch of updates and deletes (reading C17: keys located on the pre-batch
+        state, the highest op index per key decides: value, or removal)."""
+        slots, lens, flen, stride = canonical_bytes(keys)
+        n = slots.shape[0]
+        vals = np.ascontiguousarray(values if values is not None else np.zeros(n), dtype=np.uint64)
+        dele = np.ascontiguousarray(is_delete, dtype=np.uint8) if is_delete is not None else None
+        hits = self._lib.oart_apply_batch(self._t, _ptr(slots), _ptr(lens), flen, stride, _ptr(vals), _ptr(dele), n)
+        if hits < 0:
+            raise ValueError("update value is the reserved miss value")
+        return int(hits)
+
     def dump_inorder(self):
         n = len(self)
         keys = np.zeros((n, MAX_KEY), dtype=np.uint8)
@@ -180,6 +200,7 @@ class MapOracle:
         last[:-1] = rows_s[1:] != rows_s[:-1]
         self.rows = rows_s[last]
         self.values = vals[order][last].copy()
+        self.present = np.ones(self.rows.shape[0], dtype=bool)
 
     def _rows(self, slots, lens, flen):
         if lens is None:
@@ -199,6 +220,8 @@ class MapOracle:
 
     def lookup(self, queries) -> np.ndarray:
         pos, found = self._find(queries)
+        if found.shape[0]:
+            found &= self.present[pos]
         out = np.full(found.shape[0], OART_MISS, dtype=np.uint64)
         out[found] = self.values[pos[found]]
         return out
@@ -208,6 +231,8 @@ class MapOracle:
         wins.  Absent keys are no-ops (reading C6)."""
         vals = np.ascontiguousarray(values, dtype=np.uint64)
         pos, found = self._find(keys)
+        if found.shape[0]:
+            found &= self.present[pos]
         idx = np.nonzero(found)[0]
         # sequential application == for each key, the value of its LAST op
         p = pos[idx]
@@ -216,6 +241,27 @@ class MapOracle:
         last = np.ones(p_s.shape[0], dtype=bool)
         last[:-1] = p_s[1:] != p_s[:-1]
         self.values[p_s[last]] = vals[i_s[last]]
+        return int(idx.shape[0])
+
+    def apply(self, keys, values, is_delete) -> int:
+        """Reading C17: presence is taken before the batch; per present key the op
+        with the highest index decides (store its value, or remove the key)."""
+        n = len(is_delete)
+        vals = np.ascontiguousarray(values if values is not None else np.zeros(n), dtype=np.uint64)
+        dele = np.asarray(is_delete, dtype=bool)
+        pos, found = self._find(keys)
+        if found.shape[0]:
+            found &= self.present[pos]
+        idx = np.nonzero(found)[0]
+        p = pos[idx]
+        order = np.argsort(p, kind="stable")
+        p_s, i_s = p[order], idx[order]
+        last = np.ones(p_s.shape[0], dtype=bool)
+        last[:-1] = p_s[1:] != p_s[:-1]
+        wp, wi = p_s[last], i_s[last]
+        d = dele[wi]
+        self.values[wp[~d]] = vals[wi[~d]]
+        self.present[wp[d]] = False
         return int(idx.shape[0])
 
     def items(self):

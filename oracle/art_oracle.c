@@ -45,6 +45,7 @@ typedef struct {
     uint32_t len;
     uint8_t key[OART_MAX_KEY];
     uint64_t value;
+    uint64_t pending;               /* batch scratch: 1 + index of the last op on this leaf */
 } oleaf;
 
 typedef struct {
@@ -416,4 +417,124 @@ static void stats_rec(onode* n, uint64_t* out, uint64_t level) {
 void oart_stats(const oart* t, uint64_t out[6]) {
     memset(out, 0, 6 * sizeof(uint64_t));
     stats_rec(t->root, out, 1);
+}
+
+/* ------------------------------------------------------------------ deletes
+ * Non-structural delete (§3.3): the key's leaf is removed and its
+ * reference is dropped from the parent; nodes are NOT collapsed or shrunk. */
+static void remove_child(onode* n, uint8_t b) {
+    switch (n->kind) {
+    case K_N4:
+    case K_N16: {
+        uint8_t* keys = n->kind == K_N4 ? ((onode4*)n)->keys : ((onode16*)n)->keys;
+        onode** child = n->kind == K_N4 ? ((onode4*)n)->child : ((onode16*)n)->child;
+        oinner* h = (oinner*)n;
+        uint32_t pos = 0;
+        while (pos < h->count && keys[pos] != b) pos++;
+        if (pos == h->count) return;
+        memmove(keys + pos, keys + pos + 1, h->count - pos - 1);
+        memmove(child + pos, child + pos + 1, (h->count - pos - 1) * sizeof(onode*));
+        h->count--;
+        return;
+    }
+    case K_N48: {
+        onode48* x = (onode48*)n;
+        if (!x->index[b]) return;
+        uint32_t slot = x->index[b] - 1, last = x->h.count - 1;
+        x->index[b] = 0;
+        if (slot != last) {                         /* keep slots 0..count-1 dense */
+            for (int k = 0; k < 256; k++)
+                if (x->index[k] == last + 1) { x->index[k] = (uint8_t)(slot + 1); break; }
+            x->child[slot] = x->child[last];
+        }
+        x->child[last] = NULL;
+        x->h.count--;
+        return;
+    }
+    case K_N256: {
+        onode256* x = (onode256*)n;
+        if (x->child[b]) { x->child[b] = NULL; x->h.count--; }
+        return;
+    }
+    }
+}
+
+/* Unlink the leaf of key (pessimistic walk); returns the unlinked leaf or NULL.
+ * The leaf is not freed here (the caller may still hold pointers to it). */
+static oleaf* unlink_leaf(oart* t, const uint8_t* key, uint32_t len) {
+    onode* parent = NULL;
+    uint8_t pbyte = 0;
+    onode* n = t->root;
+    uint32_t depth = 0;
+    while (n) {
+        if (n->kind == K_LEAF) {
+            oleaf* l = (oleaf*)n;
+            if (!key_equal(l, key, len)) return NULL;
+            if (parent) remove_child(parent, pbyte);
+            else t->root = NULL;
+            t->n_keys--;
+            return l;
+        }
+        oinner* h = (oinner*)n;
+        if (depth + h->prefix_len >= len) return NULL;
+        if (memcmp(h->prefix, key + depth, h->prefix_len) != 0) return NULL;
+        depth += h->prefix_len;
+        onode** c = find_child(n, key[depth]);
+        if (!c) return NULL;
+        parent = n;
+        pbyte = key[depth];
+        n = *c;
+        depth += 1;
+    }
+    return NULL;
+}
+
+int oart_erase(oart* t, const uint8_t* key, uint32_t len) {
+    oleaf* l = unlink_leaf(t, key, len);
+    if (!l) return 0;
+    free(l);
+    return 1;
+}
+
+/* A batch of updates and deletes (updates replace values; a delete is
+ * the same operation with a "nil" value).  Reading C17: every op
+ * locates its key in the state BEFORE the batch (stage 1 of Fig. 6 is a lookup
+ * over the unmodified tree); for each located key the op with the highest index
+ * decides — its value is stored, or, for a delete, the key is removed.  Ops on
+ * keys absent before the batch are no-ops.  Returns the number of ops that
+ * located their key, -1 for a reserved value on a non-delete op (nothing applied). */
+int64_t oart_apply_batch(oart* t, const uint8_t* keys, const uint8_t* lens, uint32_t fixed_len, size_t stride,
+                         const uint64_t* values, const uint8_t* is_delete, size_t n) {
+    for (size_t i = 0; i < n; i++)
+        if ((!is_delete || !is_delete[i]) && values && values[i] == OART_MISS) return -1;
+    oleaf** at = (oleaf**)calloc(n ? n : 1, sizeof(oleaf*));
+    int64_t hits = 0;
+    for (size_t i = 0; i < n; i++) {                /* stage 1: locate on the pre-batch tree */
+        at[i] = find_leaf(t, keys + i * stride, lens ? lens[i] : fixed_len);
+        if (at[i]) hits++;
+    }
+    /* highest op index per leaf: later ops overwrite the leaf's pending mark */
+    for (size_t i = 0; i < n; i++)
+        if (at[i]) at[i]->pending = (uint64_t)i + 1;
+    uint8_t* win = (uint8_t*)calloc(n ? n : 1, 1);
+    for (size_t i = 0; i < n; i++)
+        if (at[i] && at[i]->pending == (uint64_t)i + 1) win[i] = 1;
+    for (size_t i = 0; i < n; i++)
+        if (at[i]) at[i]->pending = 0;
+    oleaf** dead = (oleaf**)calloc(n ? n : 1, sizeof(oleaf*));
+    size_t nd = 0;
+    for (size_t i = 0; i < n; i++) {                /* stage 2: winners apply */
+        if (!win[i]) continue;
+        if (is_delete && is_delete[i]) {
+            oleaf* l = unlink_leaf(t, keys + i * stride, lens ? lens[i] : fixed_len);
+            if (l) dead[nd++] = l;
+        } else {
+            at[i]->value = values[i];
+        }
+    }
+    for (size_t i = 0; i < nd; i++) free(dead[i]);
+    free(dead);
+    free(win);
+    free(at);
+    return hits;
 }

@@ -292,3 +292,84 @@ def test_map_oracle_strings_length_matters():
     q[1, :2] = [97, 98]
     q[2, :2] = [97, 0]
     assert m.lookup((q, np.array([3, 2, 2], np.uint8))).tolist() == [1, MISS, 2]
+
+
+# ------------------------------------------------------------------ deletes (f1, P:137 / P:143)
+def _k(x):
+    return np.array(x, dtype=np.uint64)
+
+
+def test_delete_hand_pins():
+    keys = _k([1 << 40, 2 << 40, 3 << 40, 3 << 40 | 1])
+    for O in (ArtOracle, MapOracle):
+        o = O(keys, _k([10, 20, 30, 40]))
+        # plain delete; delete of an absent key is a no-op
+        o.apply(_k([keys[0], 12345]), None, [1, 1])
+        assert o.lookup(keys).tolist() == [MISS, 20, 30, 40]
+        # [delete k, update k] -> the higher index (the update) decides (reading C17)
+        o.apply(_k([keys[1], keys[1]]), _k([0, 21]), [1, 0])
+        # [update k, delete k] -> removed
+        o.apply(_k([keys[2], keys[2]]), _k([31, 0]), [0, 1])
+        assert o.lookup(keys).tolist() == [MISS, 21, MISS, 40]
+        # a deleted key stays deleted: later updates are no-ops (no inserts on the device)
+        o.apply(_k([keys[0], keys[2]]), _k([5, 6]), [0, 0])
+        assert o.lookup(keys).tolist() == [MISS, 21, MISS, 40]
+
+
+def test_delete_is_non_structural():
+    """nodes are not collapsed.  Keys {x0, x1} under a 2-child N4 next to a
+    leaf: deleting x1 leaves an N4 with ONE child (no path re-compression)."""
+    keys = _k([0x0100000000000001, 0x0100000000000002, 0x0200000000000000])
+    o = ArtOracle(keys, _k([1, 2, 3]))
+    before = o.dump_structure().tolist()
+    assert before[:5] == [1, 0, 2, 1, 2]
+    assert o.erase_one((0x0100000000000002).to_bytes(8, "big")) == 1
+    rec = o.dump_structure().tolist()
+    # root N4 (2 children) -> child 0x01: N4, prefix 6 zero bytes, now one child
+    assert rec[:5] == [1, 0, 2, 1, 2]
+    assert rec[5:7] == [1, 6] and rec[13:15] == [1, 1]
+    assert o.lookup(keys).tolist() == [1, MISS, 3]
+    assert o.erase_one((0x0100000000000002).to_bytes(8, "big")) == 0
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_delete_batches_vs_bruteforce(seed):
+    rng = random.Random(500 + seed)
+    keys = _random_keyset(rng, 400, ["u64", "u64_shared", "bytes"][seed % 3])
+    ref = {k: rng.getrandbits(62) for k in keys}
+    o = ArtOracle()
+    for k, v in ref.items():
+        o.insert_one(k, v)
+    mp = MapOracle(_as_input("bytes", keys), np.array([ref[k] for k in keys], np.uint64)) if seed % 3 == 2 else \
+        MapOracle(_as_input("u64", keys), np.array([ref[k] for k in keys], np.uint64))
+    for _ in range(4):
+        ops = []
+        for _ in range(600):
+            k = rng.choice(keys) if rng.random() < 0.85 else bytes(rng.getrandbits(8) for _ in range(len(keys[0])))
+            ops.append((k, rng.getrandbits(62), rng.random() < 0.3))
+        # brute force, reading C17: presence before the batch, last op per present key decides
+        present = set(ref)
+        last = {}
+        for k, v, d in ops:
+            if k in present:
+                last[k] = (v, d)
+        for k, (v, d) in last.items():
+            if d:
+                del ref[k]
+            else:
+                ref[k] = v
+        kind = "bytes" if seed % 3 == 2 else "u64"
+        if kind == "u64" and any(len(k) != 8 for k, _, _ in ops):
+            ops = [(k, v, d) for k, v, d in ops if len(k) == 8]
+        inp = _as_input(kind, [k for k, _, _ in ops])
+        vals = np.array([v for _, v, _ in ops], np.uint64)
+        dele = np.array([d for _, _, d in ops], np.uint8)
+        o.apply(inp, vals, dele)
+        mp.apply(inp, vals, dele)
+        q = _as_input(kind, keys)
+        exp = [ref.get(k, MISS) for k in keys]
+        assert o.lookup(q).tolist() == exp
+        assert mp.lookup(q).tolist() == exp
+        assert len(o) == len(ref)
+        ks, ls, vs = o.dump_inorder()
+        assert [(bytes(ks[i, : ls[i]]), int(vs[i])) for i in range(len(ls))] == sorted(ref.items())
