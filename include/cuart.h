@@ -139,6 +139,23 @@ cuart_status cuart_update(cuart_index* h, const cuart_keys* keys, const uint64_t
                           size_t n, void* stream);
 cuart_status cuart_destroy(cuart_index* h);   /* NULL ok */
 
+/* Non-structural device-side deletes (§8(f) f1; §3.3, §3.4: "updates
+ * and nonstructural modifying deletes ... use the same implementation ...
+ * signaling a deletion through a nil pointer").  cuart_update_ex takes a mixed
+ * batch (is_delete[i] != 0 marks op i as a delete; device uint8_t[n]);
+ * cuart_erase deletes every key of the batch.  Semantics (reading C17): every op
+ * locates its key in the state before the batch; per located key the op with the
+ * highest index decides — store its value, or delete.  A delete unlinks the leaf
+ * from its parent's child slot (nodes are not collapsed), overwrites the leaf's
+ * value with the tombstone CUART_MISS (key bytes stay, so the leaf buffer keeps
+ * its lexicographic order) and pushes the leaf id (leaf8 ids, then leaf16, then
+ * leaf32) onto the free-leaf list.  Ops on absent or deleted keys are no-ops. */
+cuart_status cuart_update_ex(cuart_index* h, const cuart_keys* keys, const uint64_t* new_values,
+                             const uint8_t* is_delete, size_t n, void* stream);
+cuart_status cuart_erase(cuart_index* h, const cuart_keys* keys, size_t n, void* stream);
+/* Synchronous read of the free-leaf list: *count entries exist; up to cap copied to ids (host). */
+cuart_status cuart_free_leaves(const cuart_index* h, uint32_t* ids, size_t cap, size_t* count);
+
 /* Host-buffer variants: chunked, stream-pipelined H2D -> kernel -> D2H (P:151
  * §4.1: batches, several command streams).  Synchronous. */
 cuart_status cuart_lookup_host(const cuart_index* h, const cuart_keys* queries, size_t n,

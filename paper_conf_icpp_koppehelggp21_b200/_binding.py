@@ -56,7 +56,8 @@ def lib():
         P, S, I = ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int
         sig = {
             "cuart_build": [P, P, S, P, P], "cuart_lookup": [P, P, S, P, P], "cuart_update": [P, P, P, S, P],
-            "cuart_destroy": [P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
+            "cuart_destroy": [P], "cuart_update_ex": [P, P, P, P, S, P], "cuart_erase": [P, P, S, P],
+            "cuart_free_leaves": [P, P, S, P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
             "cuart_stats": [P, P], "cuart_dump": [P, P], "cuart_get_error": [P],
             "cuart_layout_build": [P, P, S, P, P], "cuart_layout_view_get": [P, P],
             "cuart_layout_lookup": [P, P, S, P, I], "cuart_layout_sectors": [P, P, S, P, I], "cuart_upload": [P, P, P], "cuart_layout_free": [P],
@@ -179,6 +180,26 @@ def cuart_update(h, keys, new_values, stream=None):
     if new_values.shape[0] != n:
         raise ValueError("values length mismatch")
     _check(lib().cuart_update(h, ctypes.byref(k), _ptr(_contig(new_values)), n, _stream_ptr(stream)), "cuart_update")
+
+
+def cuart_update_ex(h, keys, new_values, is_delete, stream=None):
+    """Mixed batch: is_delete (device uint8[n]) marks deletes (reading C17)."""
+    k, n, keep = make_keys(keys)
+    _check(lib().cuart_update_ex(h, ctypes.byref(k), _ptr(_contig(new_values)), _ptr(_contig(is_delete)), n,
+                                 _stream_ptr(stream)), "cuart_update_ex")
+
+
+def cuart_erase(h, keys, stream=None):
+    k, n, keep = make_keys(keys)
+    _check(lib().cuart_erase(h, ctypes.byref(k), n, _stream_ptr(stream)), "cuart_erase")
+
+
+def cuart_free_leaves(h):
+    cnt = ctypes.c_size_t()
+    _check(lib().cuart_free_leaves(h, None, 0, ctypes.byref(cnt)), "cuart_free_leaves")
+    ids = np.zeros(max(1, cnt.value), dtype=np.uint32)
+    _check(lib().cuart_free_leaves(h, _ptr(ids), cnt.value, ctypes.byref(cnt)), "cuart_free_leaves")
+    return ids[: cnt.value]
 
 
 def cuart_lookup_host(h, queries, out=None):
@@ -334,6 +355,15 @@ class Index:
 
     def update(self, keys, new_values, stream=None):
         cuart_update(self.h, keys, new_values, stream)
+
+    def update_ex(self, keys, new_values, is_delete, stream=None):
+        cuart_update_ex(self.h, keys, new_values, is_delete, stream)
+
+    def erase(self, keys, stream=None):
+        cuart_erase(self.h, keys, stream)
+
+    def free_leaves(self):
+        return cuart_free_leaves(self.h)
 
     def lookup_host(self, queries, out=None):
         return cuart_lookup_host(self.h, queries, out)

@@ -53,6 +53,9 @@ struct cuart_index {
     // update scratch (leaf links of the current batch)
     uint64_t* leafref = nullptr;
     size_t leafref_cap = 0;
+    uint64_t* slotref = nullptr;       // parent slot of each located leaf (batches with deletes)
+    size_t slotref_cap = 0;
+    uint64_t free_off = 0;             // free-leaf list (u32 ids) + its counter
     // host-pipeline staging
     void* stage[2] = {nullptr, nullptr};
     uint64_t* stage_out[2] = {nullptr, nullptr};
@@ -99,35 +102,62 @@ __device__ __forceinline__ uint64_t global_leaf_id(const DevIndex& ix, uint64_t 
     return (t == T_LEAF8 ? ix.leaf_base[5] : t == T_LEAF16 ? ix.leaf_base[6] : ix.leaf_base[7]) + link_index(leaf);
 }
 
-template <class Key, int POL>
+// Stage 1 of the two-stage update (Fig. 6).  DEL: the batch may carry
+// deletes ("the same implementation ... signaling a deletion through a
+// nil pointer"): is_delete[i] != 0 (or is_delete == NULL: every op deletes); the
+// parent's child slot of the located leaf is recorded for stage 2 to unlink.
+// A located leaf holding the tombstone (value == CUART_MISS) was deleted earlier
+// and counts as absent (reading C17/C18).
+template <class Key, int POL, bool DEL>
 __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restrict__ q, const uint8_t* __restrict__ lens,
-                                              const uint64_t* __restrict__ vals, uint64_t n, uint64_t epoch_hi,
-                                              uint64_t* __restrict__ leafref) {
+                                              const uint64_t* __restrict__ vals, const uint8_t* __restrict__ is_delete,
+                                              uint64_t n, uint64_t epoch_hi, uint64_t* __restrict__ leafref,
+                                              uint64_t* __restrict__ slotref) {
     const Loader<POL> ld;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
         const Key key = Key::template load<POL != 0>(q, lens, i);
-        uint64_t val;
-        uint64_t leaf = find_leaf(ix, ld, key, start_link(ix, ld, key), val);
-        if (vals[i] == kMiss) {            // reserved value: op rejected, sticky error
+        const bool del = DEL && (is_delete == nullptr || is_delete[i]);
+        uint64_t val, slot = 0;
+        uint64_t leaf = find_leaf<Key, POL, DEL>(ix, ld, key, start_link<Key, POL, DEL>(ix, ld, key, &slot), val, &slot);
+        if (leaf && val == kMiss) leaf = 0;            // tombstone: deleted by an earlier batch
+        if (!del && vals[i] == kMiss) {                // reserved value: op rejected, sticky error
             atomicOr(ix.err, 1u);
             leaf = 0;
         }
         leafref[i] = leaf;
+        if (DEL) slotref[i] = slot;
         if (leaf) atomicMax((unsigned long long*)&ix.winner[global_leaf_id(ix, leaf)], (unsigned long long)(epoch_hi | i));
     }
 }
 
-__global__ void __launch_bounds__(256) k_upd2(DevIndex ix, const uint64_t* __restrict__ vals, uint64_t n,
-                                              uint64_t epoch_hi, const uint64_t* __restrict__ leafref) {
+// Stage 2: after the grid-wide synchronisation (kernel boundary), the op whose
+// index is the registered maximum applies: one aligned 8-byte value store,
+// or, for a delete, unlink the leaf from its parent slot, clear it (value :=
+// tombstone CUART_MISS; key bytes kept so the leaf buffer stays sorted)
+// and push its id on the free-leaf list.
+template <bool DEL>
+__global__ void __launch_bounds__(256) k_upd2(DevIndex ix, const uint64_t* __restrict__ vals,
+                                              const uint8_t* __restrict__ is_delete, uint64_t n, uint64_t epoch_hi,
+                                              const uint64_t* __restrict__ leafref, const uint64_t* __restrict__ slotref) {
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
         const uint64_t leaf = leafref[i];
         if (!leaf) continue;
-        if (__ldcg(&ix.winner[global_leaf_id(ix, leaf)]) != (epoch_hi | i)) continue;
+        const uint64_t gid = global_leaf_id(ix, leaf);
+        if (__ldcg(&ix.winner[gid]) != (epoch_hi | i)) continue;
         const uint32_t t = link_type(leaf);
         uint64_t* dst = (uint64_t*)(ix.base[t] + link_index(leaf) * record_bytes(t) + leaf_value_off(t));
-        *dst = vals[i];                    // one aligned 8-byte store ("atomically replace")
+        if (DEL && (is_delete == nullptr || is_delete[i])) {
+            const uint64_t sl = slotref[i];
+            if (sl & 1) *(uint32_t*)(sl & ~uint64_t(1)) = 0;       // compact 32-bit LUT entry
+            else if (sl) *(uint64_t*)sl = 0;                       // 64-bit link: node child / LUT entry
+            *dst = kMiss;
+            const unsigned long long pos = atomicAdd(ix.free_count, 1ull);
+            ix.free_list[pos] = uint32_t(gid);
+        } else {
+            *dst = vals[i];
+        }
     }
 }
 
@@ -177,23 +207,34 @@ static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const voi
     return CUART_OK;
 }
 
-static cuart_status ensure_leafref(cuart_index* h, size_t n) {
-    if (h->leafref_cap >= n) return CUART_OK;
-    if (h->leafref) cudaFree(h->leafref);
-    h->leafref = nullptr;
-    h->leafref_cap = 0;
-    CU_TRY(cudaMalloc(&h->leafref, n * sizeof(uint64_t)));
-    h->leafref_cap = n;
+static cuart_status ensure_scratch(cuart_index* h, size_t n, bool slots) {
+    if (h->leafref_cap < n) {
+        if (h->leafref) cudaFree(h->leafref);
+        h->leafref = nullptr;
+        h->leafref_cap = 0;
+        CU_TRY(cudaMalloc(&h->leafref, n * sizeof(uint64_t)));
+        h->leafref_cap = n;
+    }
+    if (slots && h->slotref_cap < n) {
+        if (h->slotref) cudaFree(h->slotref);
+        h->slotref = nullptr;
+        h->slotref_cap = 0;
+        CU_TRY(cudaMalloc(&h->slotref, n * sizeof(uint64_t)));
+        h->slotref_cap = n;
+    }
     return CUART_OK;
 }
 
 static constexpr uint64_t kUpdateChunk = uint64_t(1) << 30;   // op index must fit the low 32 bits
 
+// mode: 0 = updates only, 1 = mixed (is_delete[i]), 2 = all deletes (vals unused)
 static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, const uint8_t* lens,
-                                  const uint64_t* vals, uint64_t n, cudaStream_t s) {
+                                  const uint64_t* vals, const uint8_t* is_delete, int mode, uint64_t n,
+                                  cudaStream_t s) {
+    const bool del = mode != 0;
     for (uint64_t base = 0; base < n; base += kUpdateChunk) {
         const uint64_t m = (n - base) < kUpdateChunk ? (n - base) : kUpdateChunk;
-        cuart_status rc = ensure_leafref(h, m);
+        cuart_status rc = ensure_scratch(h, m, del);
         if (rc != CUART_OK) return rc;
         if (++h->epoch == 0xFFFFFFFFu) {        // epoch wrap: clear the conflict words
             CU_TRY(cudaMemsetAsync(h->dix.winner, 0, h->total_leaves * 8, s));
@@ -204,12 +245,15 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
         const size_t kstride = kind == CUART_KEY_U64 ? 8 : kind == CUART_KEY_U32 ? 4 : 32;
         const void* kb = (const uint8_t*)k + base * kstride;
         const uint8_t* lb = lens ? lens + base : nullptr;
-#define CUART_UPD1(K, P) k_upd1<K, P><<<grid, 256, 0, s>>>(h->dix, kb, lb, vals + base, m, epoch_hi, h->leafref)
-#define CUART_UPD1_POL(K)                            \
-    if (h->policy == 0) CUART_UPD1(K, 0);            \
-    else if (h->policy == 4) CUART_UPD1(K, 4);       \
-    else if (h->policy == 1) CUART_UPD1(K, 1);       \
-    else CUART_UPD1(K, 5);
+        const uint64_t* vb = vals ? vals + base : nullptr;
+        const uint8_t* db = (mode == 1) ? is_delete + base : nullptr;
+#define CUART_UPD1(K, P, D) k_upd1<K, P, D><<<grid, 256, 0, s>>>(h->dix, kb, lb, vb, db, m, epoch_hi, h->leafref, h->slotref)
+#define CUART_UPD1_POL(K)                                    \
+    if (h->policy == 0) {                                    \
+        if (del) CUART_UPD1(K, 0, true); else CUART_UPD1(K, 0, false); \
+    } else {                                                 \
+        if (del) CUART_UPD1(K, 5, true); else CUART_UPD1(K, 5, false); \
+    }
         switch (kind) {
         case CUART_KEY_U64: CUART_UPD1_POL(KeyU64); break;
         case CUART_KEY_U32: CUART_UPD1_POL(KeyU32); break;
@@ -219,7 +263,8 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
 #undef CUART_UPD1
         g_cuart_launches++;
         CU_TRY(cudaGetLastError());
-        k_upd2<<<grid, 256, 0, s>>>(h->dix, vals + base, m, epoch_hi, h->leafref);
+        if (del) k_upd2<true><<<grid, 256, 0, s>>>(h->dix, vb, db, m, epoch_hi, h->leafref, h->slotref);
+        else k_upd2<false><<<grid, 256, 0, s>>>(h->dix, vb, nullptr, m, epoch_hi, h->leafref, nullptr);
         g_cuart_launches++;
         CU_TRY(cudaGetLastError());
     }
@@ -415,6 +460,8 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     h->total_leaves = L.count[5] + L.count[6] + L.count[7];
     h->winner_off = off;
     off = align(off + h->total_leaves * 8);
+    h->free_off = off;
+    off = align(off + 8 + h->total_leaves * 4);
     std::vector<uint32_t> lut32;
     std::vector<uint64_t> lutr;
     uint32_t fmt = opts ? opts->lut_format : CUART_LUT_FORMAT_AUTO;
@@ -459,6 +506,7 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     if (rc == CUART_OK && h->total_leaves && cudaMemset(h->arena + h->winner_off, 0, h->total_leaves * 8) != cudaSuccess)
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && cudaMemset(h->arena + h->err_off, 0, 256) != cudaSuccess) rc = CUART_ERR_CUDA;
+    if (rc == CUART_OK && cudaMemset(h->arena + h->free_off, 0, 8) != cudaSuccess) rc = CUART_ERR_CUDA;
     if (rc != CUART_OK) {
         cudaFree(h->arena);
         delete h;
@@ -479,6 +527,8 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     d.leaf_base[6] = L.count[5];
     d.leaf_base[7] = L.count[5] + L.count[6];
     d.err = (uint32_t*)(h->arena + h->err_off);
+    d.free_count = (unsigned long long*)(h->arena + h->free_off);
+    d.free_list = (uint32_t*)(h->arena + h->free_off + 8);
     *out = h;
     return CUART_OK;
 }
@@ -503,6 +553,7 @@ cuart_status cuart_destroy(cuart_index* h) {
     cudaDeviceSynchronize();
     cudaFree(h->arena);
     if (h->leafref) cudaFree(h->leafref);
+    if (h->slotref) cudaFree(h->slotref);
     for (int i = 0; i < 2; i++) {
         if (h->stage[i]) cudaFree(h->stage[i]);
         if (h->stage_out[i]) cudaFree(h->stage_out[i]);
@@ -527,7 +578,37 @@ cuart_status cuart_update(cuart_index* h, const cuart_keys* k, const uint64_t* v
     if (rc != CUART_OK) return rc;
     if (n == 0) return CUART_OK;
     if (!v) return CUART_ERR_INVALID_ARGUMENT;
-    return launch_update(h, h->key_kind, k->data, k->lengths, v, n, (cudaStream_t)stream);
+    return launch_update(h, h->key_kind, k->data, k->lengths, v, nullptr, 0, n, (cudaStream_t)stream);
+}
+
+cuart_status cuart_update_ex(cuart_index* h, const cuart_keys* k, const uint64_t* v, const uint8_t* is_delete, size_t n,
+                             void* stream) {
+    cuart_status rc = check_keys(h, k, n);
+    if (rc != CUART_OK) return rc;
+    if (n == 0) return CUART_OK;
+    if (!v || !is_delete) return CUART_ERR_INVALID_ARGUMENT;
+    return launch_update(h, h->key_kind, k->data, k->lengths, v, is_delete, 1, n, (cudaStream_t)stream);
+}
+
+cuart_status cuart_erase(cuart_index* h, const cuart_keys* k, size_t n, void* stream) {
+    cuart_status rc = check_keys(h, k, n);
+    if (rc != CUART_OK) return rc;
+    if (n == 0) return CUART_OK;
+    return launch_update(h, h->key_kind, k->data, k->lengths, nullptr, nullptr, 2, n, (cudaStream_t)stream);
+}
+
+cuart_status cuart_free_leaves(const cuart_index* h, uint32_t* ids, size_t cap, size_t* count) {
+    if (!h || !count) return CUART_ERR_INVALID_ARGUMENT;
+    CU_TRY(cudaSetDevice(h->device));
+    CU_TRY(cudaDeviceSynchronize());
+    unsigned long long c = 0;
+    CU_TRY(cudaMemcpy(&c, h->dix.free_count, 8, cudaMemcpyDeviceToHost));
+    *count = size_t(c);
+    if (ids && cap) {
+        const size_t m = size_t(c) < cap ? size_t(c) : cap;
+        if (m) CU_TRY(cudaMemcpy(ids, h->dix.free_list, m * 4, cudaMemcpyDeviceToHost));
+    }
+    return CUART_OK;
 }
 
 // ---------------------------------------------------------------- host-buffer pipelines
@@ -590,7 +671,8 @@ cuart_status cuart_update_host(cuart_index* h, const cuart_keys* k, const uint64
         CU_TRY(cudaMemcpyAsync(h->stage[s], (const uint8_t*)k->data + base * ks, m * ks, cudaMemcpyHostToDevice, st));
         if (k->lengths) CU_TRY(cudaMemcpyAsync(h->stage_len[s], k->lengths + base, m, cudaMemcpyHostToDevice, st));
         CU_TRY(cudaMemcpyAsync(h->stage_val[s], v + base, m * 8, cudaMemcpyHostToDevice, st));
-        rc = launch_update(h, h->key_kind, h->stage[s], k->lengths ? h->stage_len[s] : nullptr, h->stage_val[s], m, st);
+        rc = launch_update(h, h->key_kind, h->stage[s], k->lengths ? h->stage_len[s] : nullptr, h->stage_val[s],
+                           nullptr, 0, m, st);
         if (rc != CUART_OK) return rc;
     }
     CU_TRY(cudaStreamSynchronize(st));

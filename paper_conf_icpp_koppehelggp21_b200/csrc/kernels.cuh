@@ -25,6 +25,8 @@ struct DevIndex {
     uint64_t* winner;             // per-leaf conflict word for updates (global leaf id)
     uint64_t leaf_base[8];        // global leaf id = leaf_base[type] + index
     uint32_t* err;                // sticky device error flag
+    uint32_t* free_list;          // freed leaf ids (global leaf id), capacity = #leaves
+    unsigned long long* free_count;  // number of entries in free_list
 };
 
 // ----------------------------------------------------------------------------- loads
@@ -261,10 +263,12 @@ struct Loader {
 };
 
 // Walk from `link` to a leaf.  Returns the leaf link on a full-key match (its value
-// in `val`), 0 otherwise.
-template <class Key, int POL>
+// in `val`), 0 otherwise.  With TRACK, `slot` follows the address of the link last
+// loaded (the parent's child slot of the leaf found — what a delete unlinks,
+// P:137); it starts as the LUT entry address from start_link (0 = root/none).
+template <class Key, int POL, bool TRACK = false>
 __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Loader<POL>& ld, const Key& key, uint64_t link,
-                                              uint64_t& val) {
+                                              uint64_t& val, uint64_t* slot = nullptr) {
     const uint32_t len = key.len();
 #pragma unroll 1
     for (;;) {
@@ -280,10 +284,12 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Loader<P
         const uint8_t* rec = ix.base[t] + idx * record_bytes(t);
         if (t == T_N256) {
             link = ld.node64(rec + kN256Child + 8 * b);
+            if (TRACK) *slot = uint64_t(rec + kN256Child + 8 * b);
         } else if (t == T_N48) {
             const uint32_t s = ld.node8(rec + kN48Index + b);
             if (s == kN48Empty) return 0;
             link = ld.node64(rec + kN48Child + 8 * s);
+            if (TRACK) *slot = uint64_t(rec + kN48Child + 8 * s);
         } else if (t == T_N16) {
             const uint4 k4 = ld.nodev4(rec + kN16Keys);
             const uint32_t bb = b * 0x01010101u;
@@ -294,6 +300,7 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Loader<P
             search4(k4.w, bb, l3, e3);
             if ((e0 | e1 | e2 | e3) == 0) return 0;
             link = ld.node64(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
+            if (TRACK) *slot = uint64_t(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
         } else {  // N4: keys + child[0..2] in one 256-bit load; child[3] (same line) if taken
             const U8x32 r = ld.nodev8(rec);
             uint32_t less, eq;
@@ -306,6 +313,7 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Loader<P
                 const uint32_t hi = less == 0 ? r.w[3] : less == 1 ? r.w[5] : r.w[7];
                 link = uint64_t(lo) | (uint64_t(hi) << 32);
             }
+            if (TRACK) *slot = uint64_t(rec + kN4Child + 8 * less);
         }
     }
 }
@@ -323,11 +331,15 @@ __device__ __forceinline__ uint64_t expand_lut32(uint32_t e, uint32_t k, uint32_
 // 32 entries (the whole table is 1 B/entry and stays L2-resident).  Type from three
 // bit-planes, index = per-type base + popcount of earlier same-type entries;
 // exceptions (leaves, other depths, non-consecutive indices) go to the link table.
-template <int POL>
-__device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Loader<POL>& ld, uint64_t p) {
+template <int POL, bool TRACK = false>
+__device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Loader<POL>& ld, uint64_t p,
+                                                    uint64_t* slot = nullptr) {
     const U8x32 blk = ld.lutv8(ix.lutr + (p >> 5) * 2);
     const uint32_t j = uint32_t(p & 31);
-    if ((blk.w[3] >> j) & 1) return ld.lut64(ix.lut + p);
+    if ((blk.w[3] >> j) & 1) {
+        if (TRACK) *slot = uint64_t(ix.lut + p);
+        return ld.lut64(ix.lut + p);
+    }
     const uint32_t p0 = blk.w[0], p1 = blk.w[1], p2 = blk.w[2];
     const uint32_t t = ((p0 >> j) & 1) | (((p1 >> j) & 1) << 1) | (((p2 >> j) & 1) << 2);
     if (t == T_NULL) return 0;
@@ -336,12 +348,21 @@ __device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Lo
     return make_link(t, ix.lut_bytes, uint64_t(base) + __popc(m));
 }
 
-template <class Key, int POL>
-__device__ __forceinline__ uint64_t start_link(const DevIndex& ix, const Loader<POL>& ld, const Key& key) {
+// Start of a walk: LUT[first k key bytes] or the root.  With TRACK, *slot =
+// address of the LUT entry holding the link (bit 0 set for a 32-bit entry), 0 if
+// the start is the root (a root leaf is never unlinked; its tombstone suffices).
+template <class Key, int POL, bool TRACK = false>
+__device__ __forceinline__ uint64_t start_link(const DevIndex& ix, const Loader<POL>& ld, const Key& key,
+                                               uint64_t* slot = nullptr) {
+    if (TRACK) *slot = 0;
     if (ix.lut_bytes && key.len() >= ix.lut_bytes) {
         const uint64_t p = key.prefix(ix.lut_bytes);
-        if (ix.lutr) return expand_lut_rank(ix, ld, p);
-        if (ix.lut32) return expand_lut32(ld.lut32(ix.lut32 + p), ix.lut_bytes, ix.fixed_len);
+        if (ix.lutr) return expand_lut_rank<POL, TRACK>(ix, ld, p, slot);
+        if (ix.lut32) {
+            if (TRACK) *slot = uint64_t(ix.lut32 + p) | 1u;
+            return expand_lut32(ld.lut32(ix.lut32 + p), ix.lut_bytes, ix.fixed_len);
+        }
+        if (TRACK) *slot = uint64_t(ix.lut + p);
         return ld.lut64(ix.lut + p);
     }
     return ix.root;

@@ -22,19 +22,31 @@ def _u64(buf, off):
     return int(np.frombuffer(bytes(buf[off: off + 8]), dtype="<u8")[0])
 
 
-def children(view, t, idx):
-    """[(byte, child_link)] in byte order."""
+MISS = (1 << 64) - 1
+
+
+def children(view, t, idx, live_only=True):
+    """[(byte, child_link)] in byte order; deleted children (null link, or a leaf
+    holding the tombstone value) are dropped unless live_only is False."""
+    kids = _children_raw(view, t, idx)
+    if not live_only:
+        return kids
+    return [(k, c) for k, c in kids if not (split_link(c)[0] >= 5 and leaf(view, c)[1] == MISS)]
+
+
+def _children_raw(view, t, idx):
     b = view["buf"][t]
     o = idx * REC[t]
     if t == 1 or t == 2:
         cnt = int(b[o + HDR[t] + 1]) + 1
         ko, co = (0, 8) if t == 1 else (16, 32)
-        return [(int(b[o + ko + j]), _u64(b, o + co + 8 * j)) for j in range(cnt)]
+        kids = [(int(b[o + ko + j]), _u64(b, o + co + 8 * j)) for j in range(cnt)]
+        return [(k, c) for k, c in kids if c]
     if t == 3:
         out = []
         for byte in range(256):
             s = int(b[o + 16 + byte])
-            if s != 0xFF:
+            if s != 0xFF and _u64(b, o + 272 + 8 * s):
                 out.append((byte, _u64(b, o + 272 + 8 * s)))
         return out
     out = []
@@ -59,7 +71,10 @@ def to_records(view) -> list[int]:
     def first_leaf(link):
         while split_link(link)[0] < 5:
             t, _, idx = split_link(link)
-            link = children(view, t, idx)[0][1]
+            kids = children(view, t, idx, live_only=False)
+            if not kids:
+                return None
+            link = kids[0][1]
         return leaf(view, link)[0]
 
     def rec(link, depth):
@@ -77,15 +92,20 @@ def to_records(view) -> list[int]:
         plen = int(b[h])
         assert aux == depth + plen, "branch depth in the link = depth + prefix length"
         kids = children(view, t, idx)
-        assert int(b[h + 1]) + 1 == len(kids), "header count"
-        fl = first_leaf(link)
-        prefix = fl[depth: depth + plen]
+        assert int(b[h + 1]) + 1 >= len(kids), "header count (deletes only remove children)"
         stored = bytes(b[h + 2: h + 2 + min(plen, 14)])
+        fl = first_leaf(link)
+        if fl is None:
+            assert plen <= 14
+            prefix = stored
+        else:
+            prefix = fl[depth: depth + plen]
         assert stored == prefix[:14], "header stores the first 14 prefix bytes"
         out.extend([t, plen, *prefix, len(kids), *[k for k, _ in kids]])
         for _, c in kids:
             rec(c, depth + plen + 1)
 
-    if view["root"]:
-        rec(view["root"], 0)
+    root = view["root"]
+    if root and not (split_link(root)[0] >= 5 and leaf(view, root)[1] == MISS):
+        rec(root, 0)
     return out
