@@ -153,6 +153,17 @@ cuart_status cuart_destroy(cuart_index* h);   /* NULL ok */
 cuart_status cuart_update_ex(cuart_index* h, const cuart_keys* keys, const uint64_t* new_values,
                              const uint8_t* is_delete, size_t n, void* stream);
 cuart_status cuart_erase(cuart_index* h, const cuart_keys* keys, size_t n, void* stream);
+/* Range queries (§8(f) f2; §3.2.1: leaves are strictly ordered inside each
+ * leaf buffer, so a range is handed back as start and end indices into the leaf
+ * arrays).  For query i with inclusive bounds [lo[i], hi[i]]:
+ *   bounds[6*i + 2*(c-5)]     = number of class-c leaves with key <  lo[i]
+ *   bounds[6*i + 2*(c-5) + 1] = number of class-c leaves with key <= hi[i]
+ * for c = 5 (leaf8), 6 (leaf16), 7 (leaf32); the matching leaves are the records
+ * [start, end) of that buffer (cuart_dump).  Deleted leaves stay in place with
+ * the tombstone value CUART_MISS.  Integer key kinds only (BYTES returns
+ * CUART_ERR_INVALID_ARGUMENT).  Device pointers, bounds uint64_t[6n]; async. */
+cuart_status cuart_range(const cuart_index* h, const cuart_keys* lo, const cuart_keys* hi, size_t n,
+                         uint64_t* bounds, void* stream);
 /* Synchronous read of the free-leaf list: *count entries exist; up to cap copied to ids (host). */
 cuart_status cuart_free_leaves(const cuart_index* h, uint32_t* ids, size_t cap, size_t* count);
 

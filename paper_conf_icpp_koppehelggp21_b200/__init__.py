@@ -16,5 +16,5 @@ from ._binding import (  # noqa: F401
     cuart_build, cuart_destroy, cuart_dump, cuart_get_error, cuart_launch_count, cuart_layout_build,
     cuart_layout_free, cuart_layout_lookup, cuart_layout_sectors, cuart_layout_view_get, cuart_lookup, cuart_lookup_host,
     cuart_stats, cuart_status_string, cuart_update, cuart_update_host, cuart_upload, lib,
-    cuart_update_ex, cuart_erase, cuart_free_leaves,
+    cuart_update_ex, cuart_erase, cuart_free_leaves, cuart_range,
 )

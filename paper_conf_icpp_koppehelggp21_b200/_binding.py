@@ -57,7 +57,7 @@ def lib():
         sig = {
             "cuart_build": [P, P, S, P, P], "cuart_lookup": [P, P, S, P, P], "cuart_update": [P, P, P, S, P],
             "cuart_destroy": [P], "cuart_update_ex": [P, P, P, P, S, P], "cuart_erase": [P, P, S, P],
-            "cuart_free_leaves": [P, P, S, P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
+            "cuart_free_leaves": [P, P, S, P], "cuart_range": [P, P, P, S, P, P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
             "cuart_stats": [P, P], "cuart_dump": [P, P], "cuart_get_error": [P],
             "cuart_layout_build": [P, P, S, P, P], "cuart_layout_view_get": [P, P],
             "cuart_layout_lookup": [P, P, S, P, I], "cuart_layout_sectors": [P, P, S, P, I], "cuart_upload": [P, P, P], "cuart_layout_free": [P],
@@ -192,6 +192,16 @@ def cuart_update_ex(h, keys, new_values, is_delete, stream=None):
 def cuart_erase(h, keys, stream=None):
     k, n, keep = make_keys(keys)
     _check(lib().cuart_erase(h, ctypes.byref(k), n, _stream_ptr(stream)), "cuart_erase")
+
+
+def cuart_range(h, lo, hi, bounds, stream=None):
+    """bounds: device uint64/int64 tensor [n, 6] (start/end per leaf class)."""
+    kl, n, keep1 = make_keys(lo)
+    kh, n2, keep2 = make_keys(hi)
+    if n2 != n:
+        raise ValueError("lo/hi length mismatch")
+    _check(lib().cuart_range(h, ctypes.byref(kl), ctypes.byref(kh), n, _ptr(bounds), _stream_ptr(stream)), "cuart_range")
+    return bounds
 
 
 def cuart_free_leaves(h):
@@ -364,6 +374,12 @@ class Index:
 
     def free_leaves(self):
         return cuart_free_leaves(self.h)
+
+    def range(self, lo, hi, bounds=None, stream=None):
+        import torch
+        if bounds is None:
+            bounds = torch.empty((lo.shape[0], 6), dtype=torch.int64, device=lo.device)
+        return cuart_range(self.h, lo, hi, bounds, stream)
 
     def lookup_host(self, queries, out=None):
         return cuart_lookup_host(self.h, queries, out)

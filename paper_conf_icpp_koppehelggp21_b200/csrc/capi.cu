@@ -597,6 +597,21 @@ cuart_status cuart_erase(cuart_index* h, const cuart_keys* k, size_t n, void* st
     return launch_update(h, h->key_kind, k->data, k->lengths, nullptr, nullptr, 2, n, (cudaStream_t)stream);
 }
 
+cuart_status cuart_range_leaf8(const uint8_t* leaves, uint64_t nleaves, uint32_t kind, const void* lo, const void* hi,
+                               size_t n, uint64_t* bounds, void* stream);   // route.cu
+
+cuart_status cuart_range(const cuart_index* h, const cuart_keys* lo, const cuart_keys* hi, size_t n, uint64_t* bounds,
+                         void* stream) {
+    cuart_status rc = check_keys(h, lo, n);
+    if (rc == CUART_OK) rc = check_keys(h, hi, n);
+    if (rc != CUART_OK) return rc;
+    if (h->key_kind == CUART_KEY_BYTES) return CUART_ERR_INVALID_ARGUMENT;   // integer keys only
+    if (n == 0) return CUART_OK;
+    if (!bounds) return CUART_ERR_INVALID_ARGUMENT;
+    return cuart_range_leaf8(h->dix.base[T_LEAF8], h->count[T_LEAF8], h->key_kind, lo->data, hi->data, n, bounds,
+                             stream);
+}
+
 cuart_status cuart_free_leaves(const cuart_index* h, uint32_t* ids, size_t cap, size_t* count) {
     if (!h || !count) return CUART_ERR_INVALID_ARGUMENT;
     CU_TRY(cudaSetDevice(h->device));

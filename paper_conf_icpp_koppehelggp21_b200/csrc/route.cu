@@ -221,3 +221,58 @@ cuart_status cuart_unroute(const uint64_t* in, const uint32_t* perm, size_t n, u
 }
 
 }  // extern "C"
+
+// ============================================================================ range queries
+// §8(f) f2 (§3.2.1): leaves are strictly lexicographic inside each leaf
+// buffer, so the answer to a range query [lo, hi] is the pair of leaf indices
+// (start, end) = (#leaves with key < lo, #leaves with key <= hi).  Integer keys
+// live in the leaf8 buffer only; both bounds come from a branch-free binary search
+// over that buffer (the top levels of the implicit search tree stay L2-resident).
+// Deleted leaves keep their key bytes and position (tombstone value).
+namespace {
+
+__device__ __forceinline__ uint64_t bswap64_r(uint64_t x) {
+    uint32_t lo = uint32_t(x), hi = uint32_t(x >> 32);
+    return (uint64_t(__byte_perm(lo, 0, 0x0123)) << 32) | __byte_perm(hi, 0, 0x0123);
+}
+
+// number of leaf8 keys (numeric, fixed length flen) < q (strict) or <= q
+__device__ __forceinline__ uint64_t rank8(const uint8_t* leaves, uint64_t nleaves, uint32_t flen, uint64_t q, bool le) {
+    uint64_t lo = 0, hi = nleaves;
+    while (lo < hi) {
+        const uint64_t mid = (lo + hi) >> 1;
+        uint64_t k = bswap64_r(__ldg((const unsigned long long*)(leaves + mid * 16)));
+        if (flen == 4) k >>= 32;
+        if (k < q || (le && k == q)) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+__global__ void __launch_bounds__(256) k_range(const uint8_t* __restrict__ leaves, uint64_t nleaves, uint32_t kind,
+                                               const void* __restrict__ lo, const void* __restrict__ hi, uint64_t n,
+                                               uint64_t* __restrict__ bounds) {
+    const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const uint32_t flen = kind == CUART_KEY_U64 ? 8 : 4;
+    const uint64_t ql = kind == CUART_KEY_U64 ? ((const uint64_t*)lo)[i] : ((const uint32_t*)lo)[i];
+    const uint64_t qh = kind == CUART_KEY_U64 ? ((const uint64_t*)hi)[i] : ((const uint32_t*)hi)[i];
+    const uint64_t s = rank8(leaves, nleaves, flen, ql, false);
+    uint64_t e = rank8(leaves, nleaves, flen, qh, true);
+    if (e < s) e = s;                               // empty range when hi < lo
+    uint64_t* b = bounds + 6 * i;
+    b[0] = s;
+    b[1] = e;
+    b[2] = b[3] = b[4] = b[5] = 0;                  // leaf16 / leaf32 buffers are unused by integer keys
+}
+
+}  // namespace
+
+extern "C" cuart_status cuart_range_leaf8(const uint8_t* leaves, uint64_t nleaves, uint32_t kind, const void* lo,
+                                          const void* hi, size_t n, uint64_t* bounds, void* stream) {
+    if (n == 0) return CUART_OK;
+    const uint64_t blocks = (n + 255) / 256;
+    k_range<<<unsigned(blocks), 256, 0, (cudaStream_t)stream>>>(leaves, nleaves, kind, lo, hi, n, bounds);
+    g_cuart_launches += 1;
+    return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+}
