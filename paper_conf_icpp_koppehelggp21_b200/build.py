@@ -38,6 +38,7 @@ def build(force: bool = False, verbose_ptxas: bool = False) -> str:
         return OUT
     os.makedirs(BUILD, exist_ok=True)
     inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
+    inc += os.environ.get("CUART_DEFS", "").split()          # e.g. "-DCUART_N16_BYTES=256" (layout experiments)
     objs = []
     for f in sorted(os.listdir(CSRC)):
         src = os.path.join(CSRC, f)

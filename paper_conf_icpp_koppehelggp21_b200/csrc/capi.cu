@@ -34,6 +34,10 @@ struct cuart_layout {
     HostLayout L;
 };
 
+// host-buffer pipelines (cuart_lookup_host / cuart_update_host)
+static constexpr size_t kStageChunk = size_t(1) << 23;   // ops per pipeline chunk
+static constexpr int kStages = 4;                          // chunks in flight (streams / staging sets)
+
 struct cuart_index {
     int device = 0;
     int num_sms = 148;
@@ -57,12 +61,12 @@ struct cuart_index {
     size_t slotref_cap = 0;
     uint64_t free_off = 0;             // free-leaf list (u32 ids) + its counter
     // host-pipeline staging
-    void* stage[2] = {nullptr, nullptr};
-    uint64_t* stage_out[2] = {nullptr, nullptr};
-    uint8_t* stage_len[2] = {nullptr, nullptr};
-    uint64_t* stage_val[2] = {nullptr, nullptr};
+    void* stage[4] = {nullptr, nullptr, nullptr, nullptr};
+    uint64_t* stage_out[4] = {nullptr, nullptr, nullptr, nullptr};
+    uint8_t* stage_len[4] = {nullptr, nullptr, nullptr, nullptr};
+    uint64_t* stage_val[4] = {nullptr, nullptr, nullptr, nullptr};
     size_t stage_cap = 0;
-    cudaStream_t streams[2] = {nullptr, nullptr};
+    cudaStream_t streams[4] = {nullptr, nullptr, nullptr, nullptr};   // host-pipeline streams
     int policy = 5;                    // cache-policy variant of the kernels (kernels.cuh Loader)
     uint32_t lut_format = CUART_LUT_LINKS;
     uint64_t lutc_off = 0;             // compact / rank LUT region
@@ -554,7 +558,7 @@ cuart_status cuart_destroy(cuart_index* h) {
     cudaFree(h->arena);
     if (h->leafref) cudaFree(h->leafref);
     if (h->slotref) cudaFree(h->slotref);
-    for (int i = 0; i < 2; i++) {
+    for (int i = 0; i < kStages; i++) {
         if (h->stage[i]) cudaFree(h->stage[i]);
         if (h->stage_out[i]) cudaFree(h->stage_out[i]);
         if (h->stage_len[i]) cudaFree(h->stage_len[i]);
@@ -627,11 +631,10 @@ cuart_status cuart_free_leaves(const cuart_index* h, uint32_t* ids, size_t cap, 
 }
 
 // ---------------------------------------------------------------- host-buffer pipelines
-static constexpr size_t kStageChunk = size_t(1) << 23;   // ops per pipeline chunk
 
 static cuart_status ensure_stage(cuart_index* h) {
     if (h->stage_cap) return CUART_OK;
-    for (int i = 0; i < 2; i++) {
+    for (int i = 0; i < kStages; i++) {
         CU_TRY(cudaMalloc(&h->stage[i], kStageChunk * 32));
         CU_TRY(cudaMalloc(&h->stage_out[i], kStageChunk * 8));
         CU_TRY(cudaMalloc(&h->stage_len[i], kStageChunk));
@@ -656,7 +659,7 @@ cuart_status cuart_lookup_host(const cuart_index* hc, const cuart_keys* q, size_
     size_t c = 0;
     for (size_t base = 0; base < n; base += kStageChunk, c++) {
         const size_t m = (n - base) < kStageChunk ? (n - base) : kStageChunk;
-        const int s = int(c & 1);
+        const int s = int(c % kStages);
         cudaStream_t st = h->streams[s];
         CU_TRY(cudaMemcpyAsync(h->stage[s], (const uint8_t*)q->data + base * ks, m * ks, cudaMemcpyHostToDevice, st));
         if (q->lengths) CU_TRY(cudaMemcpyAsync(h->stage_len[s], q->lengths + base, m, cudaMemcpyHostToDevice, st));
@@ -664,8 +667,7 @@ cuart_status cuart_lookup_host(const cuart_index* hc, const cuart_keys* q, size_
         if (rc != CUART_OK) return rc;
         CU_TRY(cudaMemcpyAsync(out + base, h->stage_out[s], m * 8, cudaMemcpyDeviceToHost, st));
     }
-    CU_TRY(cudaStreamSynchronize(h->streams[0]));
-    CU_TRY(cudaStreamSynchronize(h->streams[1]));
+    for (int i = 0; i < kStages; i++) CU_TRY(cudaStreamSynchronize(h->streams[i]));
     return CUART_OK;
 }
 
@@ -682,7 +684,7 @@ cuart_status cuart_update_host(cuart_index* h, const cuart_keys* k, const uint64
     size_t c = 0;
     for (size_t base = 0; base < n; base += kStageChunk, c++) {
         const size_t m = (n - base) < kStageChunk ? (n - base) : kStageChunk;
-        const int s = int(c & 1);
+        const int s = int(c % kStages);
         CU_TRY(cudaMemcpyAsync(h->stage[s], (const uint8_t*)k->data + base * ks, m * ks, cudaMemcpyHostToDevice, st));
         if (k->lengths) CU_TRY(cudaMemcpyAsync(h->stage_len[s], k->lengths + base, m, cudaMemcpyHostToDevice, st));
         CU_TRY(cudaMemcpyAsync(h->stage_val[s], v + base, m * 8, cudaMemcpyHostToDevice, st));

@@ -25,6 +25,10 @@ def _u64(buf, off):
 MISS = (1 << 64) - 1
 
 
+def _rec(view, t):
+    return int(view["record_bytes"][t]) if "record_bytes" in view else REC[t]
+
+
 def children(view, t, idx, live_only=True):
     """[(byte, child_link)] in byte order; deleted children (null link, or a leaf
     holding the tombstone value) are dropped unless live_only is False."""
@@ -36,7 +40,7 @@ def children(view, t, idx, live_only=True):
 
 def _children_raw(view, t, idx):
     b = view["buf"][t]
-    o = idx * REC[t]
+    o = idx * _rec(view, t)
     if t == 1 or t == 2:
         cnt = int(b[o + HDR[t] + 1]) + 1
         ko, co = (0, 8) if t == 1 else (16, 32)
@@ -60,7 +64,7 @@ def _children_raw(view, t, idx):
 def leaf(view, link):
     t, ln, idx = split_link(link)
     b = view["buf"][t]
-    o = idx * REC[t]
+    o = idx * _rec(view, t)
     return bytes(b[o: o + ln]), _u64(b, o + VALOFF[t]), bytes(b[o + ln: o + {5: 8, 6: 16, 7: 32}[t]])
 
 
@@ -87,7 +91,7 @@ def to_records(view) -> list[int]:
             out.extend([0, len(k), *k, v - (1 << 64) if v >= 1 << 63 else v])   # oracle dumps int64
             return
         b = view["buf"][t]
-        o = idx * REC[t]
+        o = idx * _rec(view, t)
         h = o + HDR[t]
         plen = int(b[h])
         assert aux == depth + plen, "branch depth in the link = depth + prefix length"
