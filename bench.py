@@ -252,6 +252,7 @@ def main():
     nl = cfg.n_lookups
     q = make_lookups(cfg, keys_d, rank * nl, nl, dev)
     out = torch.empty(nl, dtype=torch.int64, device=dev)
+    q_bytes = sum(t.numel() * t.element_size() for t in q) if isinstance(q, tuple) else q.numel() * q.element_size()
     nu = cfg.n_updates
     uk = uv = None
     if nu:
@@ -421,7 +422,7 @@ def main():
                        "lookups_per_rank": nl, "updates_per_rank": nu, "key_kind": cfg.kind,
                        "lut_bytes": args.lut, "lut_format": stats["lut_format"], "mode": mode,
                        "parallelism": f"{mode}{world}" if world > 1 else "single",
-                       "l2": "inputs (8 GiB queries) larger than L2; no flush",
+                       "l2": f"inputs ({q_bytes / 2**30:.1f} GiB of queries per step) larger than L2; no flush",
                        "measured_hit_ratio": round(hit, 4), "build_s": round(build_s, 2)},
             "lookup": {"mlookups_per_s": round(world * nl / (look_ms * 1e-3) / 1e6, 3), "ms": round(look_ms, 4)},
             "update": {"mupdates_per_s": round(world * nu / (upd_ms * 1e-3) / 1e6, 3) if nu else None,
