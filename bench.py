@@ -51,7 +51,7 @@ def _args():
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=10)
     p.add_argument("--warmup", type=int, default=3)
-    p.add_argument("--config", default="c3", choices=["c1", "c2", "c3", "c4"])
+    p.add_argument("--config", default="c3", choices=["c1", "c2", "c3", "c4", "c5"])
     p.add_argument("--impl", default="cuart", choices=["cuart", "reference"])
     p.add_argument("--lut", type=int, default=3)
     p.add_argument("--no-e2e", action="store_true")
@@ -212,6 +212,104 @@ def make_lookups(cfg, keys_d, start, m, dev):
     return W.lookup_batch_torch(cfg, keys_d, start, m, device=dev)
 
 
+# ------------------------------------------------------------------ config 5 (mixed rounds, partitioned)
+def c5_local_keys(world, rank, dev, chunk=1 << 27):
+    """This rank's share of the 2^30 c5 keys under uniform splitters r*2^64/P (P a
+    power of two: owner = top log2(P) key bits; balanced for uniform random keys)."""
+    import torch
+    c, n = 5, W.C5.n_keys
+    bits = world.bit_length() - 1
+    ks, vs = [], []
+    for s0 in range(0, n, chunk):
+        idx = torch.arange(s0, min(n, s0 + chunk), dtype=torch.int64, device=dev)
+        k = W.splitmix64_torch(W.SEED_KEYS + c, idx)
+        mine = (W._t_srl(k, 64 - bits) == rank) if bits else torch.ones_like(k, dtype=torch.bool)
+        v = W.splitmix64_torch(W.SEED_VALUES + c, idx[mine])
+        v = torch.where(v == -1, torch.zeros_like(v), v)
+        ks.append(k[mine].cpu())
+        vs.append(v.cpu())
+    splitters = np.array([(r << (64 - bits)) for r in range(1, world)], dtype=np.uint64) if bits else np.zeros(0, np.uint64)
+    return torch.cat(ks).numpy().view(np.uint64), torch.cat(vs).numpy().view(np.uint64), splitters
+
+
+def run_c5(args, world, rank, local, dev):
+    """A step = one round of the mixed stream: this rank's 1/P slice of 2^29 global ops
+    (strong scaling: the round is fixed), lookups then updates (reading C7)."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_koppehelggp21_b200 as C
+    from paper_conf_icpp_koppehelggp21_b200.dist import CudaOps, DistIndex
+    if world & (world - 1):
+        raise SystemExit("c5 needs a power-of-two GPU count")
+    t0 = time.perf_counter()
+    keys, vals, sp = c5_local_keys(world, rank, dev)
+    if world == 1 and not dist.is_initialized():
+        dist.init_process_group("gloo", store=dist.HashStore(), rank=0, world_size=1)
+    di = DistIndex(keys, vals, mode="range", ops=CudaOps(dev), lut_bytes=args.lut, splitters=sp, local=True)
+    build_s = time.perf_counter() - t0
+    stats = di.index.stats()
+    R, per = W.C5_ROUND, W.C5_ROUND // world
+    rounds = [W.mixed_ops_torch(5, W.C5.n_keys, r * R + rank * per, per, dev) for r in range(2)]
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+
+    def step(i, ev=None, kev=None):
+        k, u, v = rounds[i % 2]
+        if ev is not None:
+            ev[0].record(stream)
+        di.mixed_round(k, v, u, events=kev)
+        if ev is not None:
+            ev[1].record(stream)
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
+    kevs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    launches0 = C.cuart_launch_count()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    t_start.record(stream)
+    for i in range(args.steps):
+        step(i, evs[i], kevs[i])
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    launches = C.cuart_launch_count() - launches0
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    tt = torch.tensor([t_start.elapsed_time(t_end), float(np.mean([e[0].elapsed_time(e[1]) for e in kevs]))],
+                      dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    total_ms, kern_ms = tt.tolist()
+    ms_step = total_ms / args.steps
+    value = R / (ms_step * 1e-3) / 1e6
+    if rank == 0:
+        print(json.dumps({
+            "metric": METRIC, "value": round(value, 3), "unit": "Mops/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic (seeded splitmix64, SURVEY §8(d) c5 recipe)",
+            "config": {"workload": f"c5: {W.C5.description}", "keys": W.C5.n_keys, "round_ops": R,
+                       "ops_per_rank_per_step": per, "update_fraction": W.C5_UPDATE_P, "mode": "range",
+                       "parallelism": f"range{world}", "local_keys_rank0": int(keys.shape[0]),
+                       "build_s": round(build_s, 2), "lut_format": stats["lut_format"]},
+            "roofline": {"bound": "hbm", "kernel": "k_lookup<KeyU64>", "kernel_ms": round(kern_ms, 4),
+                         "note": "per-rank local lookup kernel of a round; see the c3 line for the roofline fraction"},
+            "e2e": None, "cpu_baseline": None, "gpu_launches": int(launches), "clocks": clk}), flush=True)
+    di.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
 # ------------------------------------------------------------------ main (GPU)
 def main():
     args = _args()
@@ -232,6 +330,9 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     mode = "single" if world == 1 else args.mode
+    if args.config == "c5":
+        run_c5(args, world, rank, local, dev)
+        return
 
     cfg = W.CONFIGS[args.config]
     t0 = time.perf_counter()

@@ -227,6 +227,13 @@ cuart_status cuart_route(const cuart_keys* keys, size_t n, const uint64_t* split
                          const uint64_t* values, void* send_keys, uint8_t* send_lengths, uint64_t* send_values,
                          uint32_t* perm, uint64_t* counts, void* scratch, void* stream);
 cuart_status cuart_unroute(const uint64_t* in, const uint32_t* perm, size_t n, uint64_t* out, void* stream);
+/* Stable two-way split of a batch by a per-op flag (device uint8_t[n]): ops with
+ * flag 0 first, then flag != 0, each in op order; perm/counts/scratch as for
+ * cuart_route with nparts = 2.  Used to split a mixed lookup/update round
+ * (reading C7) into its lookups and its updates. */
+cuart_status cuart_partition_by_flag(const cuart_keys* keys, size_t n, const uint8_t* flags, const uint64_t* values,
+                                     void* out_keys, uint8_t* out_lengths, uint64_t* out_values, uint32_t* perm,
+                                     uint64_t* counts, void* scratch, void* stream);
 
 #ifdef __cplusplus
 }

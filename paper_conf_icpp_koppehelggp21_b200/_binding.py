@@ -72,6 +72,8 @@ def lib():
         L.cuart_route_scratch_bytes.restype = S
         L.cuart_route.argtypes = [P, S, P, ctypes.c_uint32, P, P, P, P, P, P, P, P]
         L.cuart_route.restype = ctypes.c_int
+        L.cuart_partition_by_flag.argtypes = [P, S, P, P, P, P, P, P, P, P, P]
+        L.cuart_partition_by_flag.restype = ctypes.c_int
         L.cuart_unroute.argtypes = [P, P, S, P, P]
         L.cuart_unroute.restype = ctypes.c_int
         L.cuart_launch_count.argtypes = []

@@ -49,11 +49,12 @@ __device__ __forceinline__ uint32_t owner_of(uint64_t prefix, const uint64_t* sp
 __global__ void __launch_bounds__(kRouteThreads) k_route_hist(uint32_t kind, const void* __restrict__ keys,
                                                               const uint8_t* __restrict__ lens, uint64_t n,
                                                               const uint64_t* __restrict__ splitters, uint32_t nparts,
+                                                              const uint8_t* __restrict__ flags,
                                                               uint8_t* __restrict__ owner, uint32_t* __restrict__ hist) {
     __shared__ uint64_t sp[kMaxParts];
     __shared__ uint32_t h[kMaxParts];
     for (uint32_t t = threadIdx.x; t < kMaxParts; t += blockDim.x) {
-        if (t + 1 < nparts) sp[t] = splitters[t];
+        if (splitters && t + 1 < nparts) sp[t] = splitters[t];
         h[t] = 0;
     }
     __syncthreads();
@@ -61,7 +62,7 @@ __global__ void __launch_bounds__(kRouteThreads) k_route_hist(uint32_t kind, con
     for (int r = 0; r < kRouteItems; r++) {
         const uint64_t i = base + uint64_t(r) * kRouteThreads + threadIdx.x;
         if (i < n) {
-            const uint32_t o = owner_of(load_prefix8(kind, keys, lens, i), sp, nparts - 1);
+            const uint32_t o = flags ? (flags[i] ? 1u : 0u) : owner_of(load_prefix8(kind, keys, lens, i), sp, nparts - 1);
             owner[i] = uint8_t(o);
             atomicAdd(&h[o], 1u);
         }
@@ -185,10 +186,30 @@ size_t cuart_route_scratch_bytes(size_t n, uint32_t nparts) {
     return ((n + 255) & ~size_t(255)) + nblocks * nparts * sizeof(uint32_t) + 256;
 }
 
+static cuart_status route_impl(const cuart_keys* keys, size_t n, const uint64_t* splitters, const uint8_t* flags,
+                               uint32_t nparts, const uint64_t* values, void* send_keys, uint8_t* send_lengths,
+                               uint64_t* send_values, uint32_t* perm, uint64_t* counts, void* scratch, void* stream);
+
 cuart_status cuart_route(const cuart_keys* keys, size_t n, const uint64_t* splitters, uint32_t nparts,
                          const uint64_t* values, void* send_keys, uint8_t* send_lengths, uint64_t* send_values,
                          uint32_t* perm, uint64_t* counts, void* scratch, void* stream) {
-    if (!keys || nparts == 0 || nparts > kMaxParts || (nparts > 1 && !splitters) || !counts) return CUART_ERR_INVALID_ARGUMENT;
+    if (nparts > 1 && !splitters) return CUART_ERR_INVALID_ARGUMENT;
+    return route_impl(keys, n, splitters, nullptr, nparts, values, send_keys, send_lengths, send_values, perm, counts,
+                      scratch, stream);
+}
+
+cuart_status cuart_partition_by_flag(const cuart_keys* keys, size_t n, const uint8_t* flags, const uint64_t* values,
+                                     void* out_keys, uint8_t* out_lengths, uint64_t* out_values, uint32_t* perm,
+                                     uint64_t* counts, void* scratch, void* stream) {
+    if (n > 0 && !flags) return CUART_ERR_INVALID_ARGUMENT;
+    return route_impl(keys, n, nullptr, flags, 2, values, out_keys, out_lengths, out_values, perm, counts, scratch,
+                      stream);
+}
+
+static cuart_status route_impl(const cuart_keys* keys, size_t n, const uint64_t* splitters, const uint8_t* flags,
+                               uint32_t nparts, const uint64_t* values, void* send_keys, uint8_t* send_lengths,
+                               uint64_t* send_values, uint32_t* perm, uint64_t* counts, void* scratch, void* stream) {
+    if (!keys || nparts == 0 || nparts > kMaxParts || !counts) return CUART_ERR_INVALID_ARGUMENT;
     if (n >= (uint64_t(1) << 32)) return CUART_ERR_INVALID_ARGUMENT;
     cudaStream_t s = (cudaStream_t)stream;
     if (n == 0) {
@@ -202,7 +223,8 @@ cuart_status cuart_route(const cuart_keys* keys, size_t n, const uint64_t* split
     uint8_t* owner = (uint8_t*)scratch;
     uint32_t* hist = (uint32_t*)((uint8_t*)scratch + ((n + 255) & ~size_t(255)));
     const uint32_t kind = uint32_t(keys->kind);
-    k_route_hist<<<unsigned(nblocks), kRouteThreads, 0, s>>>(kind, keys->data, keys->lengths, n, splitters, nparts, owner, hist);
+    k_route_hist<<<unsigned(nblocks), kRouteThreads, 0, s>>>(kind, keys->data, keys->lengths, n, splitters, nparts,
+                                                             flags, owner, hist);
     k_route_scan<<<1, 1024, 0, s>>>(hist, nblocks, nparts, counts);
     k_route_scatter<<<unsigned(nblocks), kRouteThreads, 0, s>>>(kind, keys->data, keys->lengths, values, n, nparts, owner,
                                                                 hist, send_keys, send_lengths, send_values, perm);

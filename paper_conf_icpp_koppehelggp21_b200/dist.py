@@ -106,6 +106,25 @@ class CudaOps:
         B._check(rc, "cuart_route")
         return send_keys, send_lens, send_vals, perm, counts
 
+    def partition(self, keys, lens, values, flags):
+        """Stable split by flag (0 first): cuart_partition_by_flag."""
+        n = keys.shape[0]
+        ok = torch.empty_like(keys)
+        ol = torch.empty_like(lens) if lens is not None else None
+        ov = torch.empty_like(values) if values is not None else None
+        perm = torch.empty(n, dtype=torch.int32, device=self.device)
+        counts = torch.empty(2, dtype=torch.int64, device=self.device)
+        scratch = torch.empty(max(1, B.lib().cuart_route_scratch_bytes(n, 2)), dtype=torch.uint8, device=self.device)
+        k, _, keep = B.make_keys((keys, lens) if lens is not None else keys)
+        stream = torch.cuda.current_stream(self.device).cuda_stream
+        rc = B.lib().cuart_partition_by_flag(B.ctypes.byref(k), n, flags.data_ptr(),
+                                             values.data_ptr() if values is not None else None, ok.data_ptr(),
+                                             ol.data_ptr() if ol is not None else None,
+                                             ov.data_ptr() if ov is not None else None, perm.data_ptr(),
+                                             counts.data_ptr(), scratch.data_ptr(), stream)
+        B._check(rc, "cuart_partition_by_flag")
+        return ok, ol, ov, perm, counts
+
     def unroute(self, res, perm):
         out = torch.empty_like(res)
         stream = torch.cuda.current_stream(self.device).cuda_stream
@@ -129,9 +148,11 @@ class CudaOps:
 class DistIndex:
     """A CuART index spread over the ranks of a process group."""
 
-    def __init__(self, keys, values, mode="range", group=None, ops=None, lut_bytes=3, splitters=None):
+    def __init__(self, keys, values, mode="range", group=None, ops=None, lut_bytes=3, splitters=None, local=False):
         """keys/values: the GLOBAL key set, identical on every rank (host arrays).
-        Range mode keeps this rank's share; replica mode keeps everything."""
+        Range mode keeps this rank's share; replica mode keeps everything.
+        local=True: keys/values are already this rank's share of a range partition
+        defined by `splitters` (used when the global set is too large to replicate)."""
         if mode not in ("range", "replica"):
             raise ValueError(mode)
         self.mode = mode
@@ -142,10 +163,15 @@ class DistIndex:
         values = np.asarray(values, np.uint64)
         self.kind_bytes = isinstance(keys, tuple)
         if mode == "range":
-            pre = prefix8(keys)
-            self.splitters_np = compute_splitters(pre, self.world) if splitters is None else np.asarray(splitters, np.uint64)
-            mine = owners(pre, self.splitters_np) == self.rank
-            keys, values = select(keys, mine), values[mine]
+            if local:
+                if splitters is None:
+                    raise ValueError("local=True needs the partition's splitters")
+                self.splitters_np = np.asarray(splitters, np.uint64)
+            else:
+                pre = prefix8(keys)
+                self.splitters_np = compute_splitters(pre, self.world) if splitters is None else np.asarray(splitters, np.uint64)
+                mine = owners(pre, self.splitters_np) == self.rank
+                keys, values = select(keys, mine), values[mine]
             self.splitters = ops.tensor(self.splitters_np.view(np.int64).copy()) if self.world > 1 else None
         self.n_local_keys = int(values.shape[0])
         self.index = ops.build(keys, values, lut_bytes)
@@ -215,6 +241,21 @@ class DistIndex:
             rl = sl.new_empty(sum(rs))
             self._a2a(rl, sl, rs, cs)
         self.ops.update(self.index, rk, rl, rv)
+
+    # ---- mixed rounds (config 5, reading C7)
+    def mixed_round(self, keys, values, is_update, lens=None, events=None):
+        """One round of a mixed op stream: this rank's contiguous slice of the round.
+        Every lookup of the round sees the state before the round's updates; the
+        updates then apply in global (rank-major, op) order.  Returns per op the
+        lookup result, CUART_MISS for update ops."""
+        pk, pl, pv, perm, counts = self.ops.partition(keys, lens, values, is_update)
+        n_l, n_u = [int(x) for x in counts.tolist()]
+        q = (pk[:n_l], pl[:n_l]) if pl is not None else pk[:n_l]
+        res = self.lookup(q, events=events)
+        uk = (pk[n_l:], pl[n_l:]) if pl is not None else pk[n_l:]
+        self.update((uk, pv[n_l:]))
+        full = torch.cat([res, res.new_full((n_u,), -1)])
+        return self.ops.unroute(full, perm)
 
     def _all_gather_var(self, t):
         n = torch.tensor([t.shape[0]], dtype=torch.int64, device=t.device)

@@ -178,3 +178,74 @@ def test_splitters_skip_common_prefix():
     lens = np.full(10, 9, np.uint8)
     own = owners(prefix8((slots, lens)), compute_splitters(prefix8((slots, lens)), 4))
     assert len(set(own.tolist())) == 1
+
+
+# ------------------------------------------------------------------ mixed rounds (config 5, reading C7)
+def _np_partition(self, keys, lens, values, flags):
+    f = flags.numpy().astype(bool)
+    order = np.argsort(f, kind="stable")
+    perm = np.empty(order.shape[0], np.int64)
+    perm[order] = np.arange(order.shape[0])
+    counts = np.array([(~f).sum(), f.sum()], np.int64)
+    return (torch.from_numpy(keys.numpy()[order].copy()),
+            torch.from_numpy(lens.numpy()[order].copy()) if lens is not None else None,
+            torch.from_numpy(values.numpy()[order].copy()), torch.from_numpy(perm), torch.from_numpy(counts))
+
+
+NumpyOps.partition = _np_partition
+MIX_KEYS, MIX_ROUND, MIX_ROUNDS = 1 << 14, 1 << 13, 3
+
+
+def _mixed_worker(rank, world, port, mode, outdir):
+    import workloads as W
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_icpp_koppehelggp21_b200.dist import DistIndex
+    keys = W.u64_keys(5, MIX_KEYS)
+    vals = W.values_for(W.SEED_VALUES + 5, np.arange(MIX_KEYS, dtype=np.uint64))
+    di = DistIndex(keys, vals, mode=mode, ops=NumpyOps())
+    per = MIX_ROUND // world
+    outs = []
+    for r in range(MIX_ROUNDS):
+        start = r * MIX_ROUND + rank * per
+        k, u, v = W.mixed_ops(5, MIX_KEYS, np.arange(start, start + per))
+        out = di.mixed_round(torch.from_numpy(k.view(np.int64)), torch.from_numpy(v.view(np.int64)),
+                             torch.from_numpy(u))
+        outs.append(out.numpy())
+    np.save(os.path.join(outdir, f"mix_r{rank}.npy"), np.concatenate(outs))
+    di.close()
+    dist.destroy_process_group()
+
+
+def _replay(world):
+    """Oracle replay of reading C7: per round, all lookups see the pre-round state,
+    then the round's updates apply in global op order."""
+    import workloads as W
+    keys = W.u64_keys(5, MIX_KEYS)
+    o = MapOracle(keys, W.values_for(W.SEED_VALUES + 5, np.arange(MIX_KEYS, dtype=np.uint64)))
+    per = MIX_ROUND // world
+    res = {r: [] for r in range(world)}
+    for rnd in range(MIX_ROUNDS):
+        k, u, v = W.mixed_ops(5, MIX_KEYS, np.arange(rnd * MIX_ROUND, (rnd + 1) * MIX_ROUND))
+        look = o.lookup(k)
+        look[u == 1] = OART_MISS
+        for r in range(world):
+            res[r].append(look[r * per:(r + 1) * per])
+        o.update(k[u == 1], v[u == 1])
+    return {r: np.concatenate(x) for r, x in res.items()}
+
+
+@pytest.mark.parametrize("mode", ["range", "replica"])
+def test_mixed_rounds_world2_p_independent(mode):
+    world = 2
+    with tempfile.TemporaryDirectory() as d:
+        mp.start_processes(_mixed_worker, args=(world, _free_port(), mode, d), nprocs=world, start_method="spawn")
+        exp = _replay(world)
+        for r in range(world):
+            assert np.array_equal(np.load(os.path.join(d, f"mix_r{r}.npy")).view(np.uint64), exp[r])
+        # P-independence: the concatenation equals the single-rank replay
+        one = _replay(1)[0]
+        both = np.concatenate([np.load(os.path.join(d, f"mix_r{r}.npy")).view(np.uint64).reshape(MIX_ROUNDS, -1)
+                               for r in range(world)], axis=1).ravel()
+        assert np.array_equal(both, one)

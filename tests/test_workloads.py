@@ -64,3 +64,15 @@ def test_string_lookup_torch_twin():
     assert np.array_equal(qs.numpy(), slots[idx]) and np.array_equal(ql.numpy(), lens[idx])
     # Zipf(0.99) skew: the hottest key takes a large share
     assert np.bincount(idx).max() > 100
+
+
+def test_mixed_ops_twin_and_mix():
+    k, u, v = W.mixed_ops(5, 1 << 16, np.arange(100, 50_100))
+    tk, tu, tv = W.mixed_ops_torch(5, 1 << 16, 100, 50_000, "cpu")
+    assert np.array_equal(tk.numpy().view(np.uint64), k)
+    assert np.array_equal(tu.numpy(), u) and np.array_equal(tv.numpy().view(np.uint64), v)
+    assert abs(u.mean() - 0.1) < 0.01
+    keys = W.u64_keys(5, 1 << 16)
+    present = np.isin(k, keys)
+    assert present[u == 1].all()                                   # updates target the set
+    assert abs(present[u == 0].mean() - 0.5) < 0.02                # lookups: 50% hit

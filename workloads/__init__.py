@@ -363,3 +363,41 @@ def string_lookup_torch(cfg: Config, slots_d, lens_d, start: int, m: int, cdf_d=
     r = torch.clamp(torch.searchsorted(cdf_d, u, right=True), max=n - 1)
     idx = perm_d[r]
     return slots_d[idx], lens_d[idx]
+
+
+# ----------------------------------------------------------------------------- config 5 (mixed)
+# uniform random u64 keys, one global stream of mixed ops: each op
+# is an update with p = 0.1 (key drawn from the set), else a lookup (50% hit).
+# The stream is cut into rounds of C5_ROUND global ops; rank r of P originates the
+# r-th contiguous 1/P slice of every round (reading C7).
+C5 = Config("c5", "u64", 1 << 30, 4 << 30, 0, 0.5,
+            "1B random 64-bit keys range-partitioned by leading bytes, 4B mixed lookup/update ops (90/10) in rounds")
+C5_ROUND = 1 << 29
+C5_UPDATE_P = 0.1
+
+
+def mixed_ops(c: int, n_keys: int, j):
+    """numpy: (keys u64, is_update u8, values u64) of global ops at positions j."""
+    j = np.asarray(j, dtype=np.uint64)
+    upd = splitmix64(SEED_UPDATES + c, np.uint64(3) * j) < np.uint64(int(C5_UPDATE_P * 2**64))
+    pick = splitmix64(SEED_UPDATES + c, np.uint64(3) * j + np.uint64(1)) % np.uint64(n_keys)
+    hit = splitmix64(SEED_QUERIES + c, np.uint64(2) * j) < np.uint64(1 << 63)
+    present = splitmix64(SEED_KEYS + c, pick)                       # keys are a bijection of their index
+    absent = splitmix64(SEED_KEYS + c, np.uint64(n_keys) + np.uint64(1 << 40) + j)
+    keys = np.where(upd | hit, present, absent)
+    vals = values_for(SEED_UVALUES + c, j)
+    return keys, upd.astype(np.uint8), vals
+
+
+def mixed_ops_torch(c: int, n_keys: int, start: int, m: int, device):
+    import torch
+    j = torch.arange(start, start + m, dtype=torch.int64, device=device)
+    upd = _t_ult(splitmix64_torch(SEED_UPDATES + c, 3 * j), int(C5_UPDATE_P * 2**64))
+    pick = _t_umod(splitmix64_torch(SEED_UPDATES + c, 3 * j + 1), n_keys)
+    hit = _t_ult(splitmix64_torch(SEED_QUERIES + c, 2 * j), 1 << 63)
+    present = splitmix64_torch(SEED_KEYS + c, pick)
+    absent = splitmix64_torch(SEED_KEYS + c, j + (n_keys + (1 << 40)))
+    keys = torch.where(upd | hit, present, absent)
+    vals = splitmix64_torch(SEED_UVALUES + c, j)
+    vals = torch.where(vals == -1, torch.zeros_like(vals), vals)
+    return keys, upd.to(torch.uint8), vals
