@@ -112,6 +112,25 @@ __device__ __forceinline__ uint64_t global_leaf_id(const DevIndex& ix, uint64_t 
 // parent's child slot of the located leaf is recorded for stage 2 to unlink.
 // A located leaf holding the tombstone (value == CUART_MISS) was deleted earlier
 // and counts as absent (reading C17/C18).
+__device__ __forceinline__ uint64_t* winner_word(const DevIndex& ix, uint64_t leaf) {
+#if CUART_COLOCATED_WINNER
+    const uint32_t t = link_type(leaf);
+    return (uint64_t*)(ix.base[t] + link_index(leaf) * record_bytes(t) + leaf_winner_off(t));
+#else
+    return &ix.winner[global_leaf_id(ix, leaf)];
+#endif
+}
+
+// Epoch wrap (every 2^32 - 2 update batches): zero every conflict word.
+__global__ void k_clear_winners(DevIndex ix, uint64_t n8, uint64_t n16, uint64_t n32) {
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n8 + n16 + n32; i += stride) {
+        const uint32_t t = i < n8 ? T_LEAF8 : i < n8 + n16 ? T_LEAF16 : T_LEAF32;
+        const uint64_t idx = i < n8 ? i : i < n8 + n16 ? i - n8 : i - n8 - n16;
+        *winner_word(ix, make_link(t, 0, idx)) = 0;
+    }
+}
+
 template <class Key, int POL, bool DEL>
 __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restrict__ q, const uint8_t* __restrict__ lens,
                                               const uint64_t* __restrict__ vals, const uint8_t* __restrict__ is_delete,
@@ -131,7 +150,7 @@ __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restric
         }
         leafref[i] = leaf;
         if (DEL) slotref[i] = slot;
-        if (leaf) atomicMax((unsigned long long*)&ix.winner[global_leaf_id(ix, leaf)], (unsigned long long)(epoch_hi | i));
+        if (leaf) atomicMax((unsigned long long*)winner_word(ix, leaf), (unsigned long long)(epoch_hi | i));
     }
 }
 
@@ -149,7 +168,7 @@ __global__ void __launch_bounds__(256) k_upd2(DevIndex ix, const uint64_t* __res
         const uint64_t leaf = leafref[i];
         if (!leaf) continue;
         const uint64_t gid = global_leaf_id(ix, leaf);
-        if (__ldcg(&ix.winner[gid]) != (epoch_hi | i)) continue;
+        if (__ldcg(winner_word(ix, leaf)) != (epoch_hi | i)) continue;
         const uint32_t t = link_type(leaf);
         uint64_t* dst = (uint64_t*)(ix.base[t] + link_index(leaf) * record_bytes(t) + leaf_value_off(t));
         if (DEL && (is_delete == nullptr || is_delete[i])) {
@@ -241,7 +260,13 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
         cuart_status rc = ensure_scratch(h, m, del);
         if (rc != CUART_OK) return rc;
         if (++h->epoch == 0xFFFFFFFFu) {        // epoch wrap: clear the conflict words
+#if CUART_COLOCATED_WINNER
+            k_clear_winners<<<h->num_sms * 8, 256, 0, s>>>(h->dix, h->count[5], h->count[6], h->count[7]);
+            g_cuart_launches++;
+            CU_TRY(cudaGetLastError());
+#else
             CU_TRY(cudaMemsetAsync(h->dix.winner, 0, h->total_leaves * 8, s));
+#endif
             h->epoch = 1;
         }
         const uint64_t epoch_hi = uint64_t(h->epoch) << 32;
@@ -463,7 +488,7 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     }
     h->total_leaves = L.count[5] + L.count[6] + L.count[7];
     h->winner_off = off;
-    off = align(off + h->total_leaves * 8);
+    if (!CUART_COLOCATED_WINNER) off = align(off + h->total_leaves * 8);
     h->free_off = off;
     off = align(off + 8 + h->total_leaves * 4);
     std::vector<uint32_t> lut32;
@@ -507,7 +532,8 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     if (rc == CUART_OK && !lutr.empty() &&
         cudaMemcpy(h->arena + h->lutc_off, lutr.data(), lutr.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
         rc = CUART_ERR_CUDA;
-    if (rc == CUART_OK && h->total_leaves && cudaMemset(h->arena + h->winner_off, 0, h->total_leaves * 8) != cudaSuccess)
+    if (rc == CUART_OK && !CUART_COLOCATED_WINNER && h->total_leaves &&
+        cudaMemset(h->arena + h->winner_off, 0, h->total_leaves * 8) != cudaSuccess)
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && cudaMemset(h->arena + h->err_off, 0, 256) != cudaSuccess) rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && cudaMemset(h->arena + h->free_off, 0, 8) != cudaSuccess) rc = CUART_ERR_CUDA;
@@ -526,7 +552,7 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     d.lut_bytes = L.lut_bytes;
     d.fixed_len = L.key_kind == CUART_KEY_U64 ? 8 : L.key_kind == CUART_KEY_U32 ? 4 : 0;
     d.key_kind = L.key_kind;
-    d.winner = (uint64_t*)(h->arena + h->winner_off);
+    d.winner = CUART_COLOCATED_WINNER ? nullptr : (uint64_t*)(h->arena + h->winner_off);
     d.leaf_base[5] = 0;
     d.leaf_base[6] = L.count[5];
     d.leaf_base[7] = L.count[5] + L.count[6];

@@ -17,6 +17,7 @@
 #include <atomic>
 
 #include "../../include/cuart.h"
+#include "layout.h"
 
 namespace {
 
@@ -263,7 +264,7 @@ __device__ __forceinline__ uint64_t rank8(const uint8_t* leaves, uint64_t nleave
     uint64_t lo = 0, hi = nleaves;
     while (lo < hi) {
         const uint64_t mid = (lo + hi) >> 1;
-        uint64_t k = bswap64_r(__ldg((const unsigned long long*)(leaves + mid * 16)));
+        uint64_t k = bswap64_r(__ldg((const unsigned long long*)(leaves + mid * cuart::record_bytes(cuart::T_LEAF8))));
         if (flen == 4) k >>= 32;
         if (k < q || (le && k == q)) lo = mid + 1;
         else hi = mid;

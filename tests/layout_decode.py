@@ -8,7 +8,7 @@ from __future__ import annotations
 
 import numpy as np
 
-REC = {1: 64, 2: 160, 3: 672, 4: 2080, 5: 16, 6: 32, 7: 48}
+REC = {1: 64, 2: 160, 3: 672, 4: 2080, 5: 32, 6: 32, 7: 48}   # fallback; dumps carry record_bytes
 VALOFF = {5: 8, 6: 16, 7: 32}
 IDX_MASK = (1 << 52) - 1
 HDR = {1: 40, 2: 0, 3: 0, 4: 0}   # header offset inside the record (N4 keeps keys + 3 children first)

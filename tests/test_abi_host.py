@@ -161,7 +161,7 @@ def test_builder_matches_oracle_structure_and_lookups(mode, seed):
     view = C.Layout(inp, vals).view()
     for t, ks in cls.items():
         assert view["count"][t] == len(ks)
-        recs = view["buf"][t].reshape(-1, REC[t])
+        recs = view["buf"][t].reshape(-1, view["record_bytes"][t])
         for i, k in enumerate(ks):
             assert bytes(recs[i, : len(k)]) == k
 

@@ -57,7 +57,7 @@ def test_range_bounds(kind):
     assert not b[:, 2:].any()
     # the leaves [start, end) of the leaf8 buffer are exactly the keys in range
     view = ix.dump()
-    leaf_keys = view["buf"][5].reshape(-1, 16)[:, :8].copy()
+    leaf_keys = view["buf"][5].reshape(-1, int(view["record_bytes"][5]))[:, :8].copy()
     if kind == "u64":
         lk = leaf_keys.view(">u8").ravel().astype(np.uint64)
     else:
@@ -73,7 +73,8 @@ def test_range_with_deletes_keeps_positions():
     b = ix.range(_t(np.array([0, 95, 150], np.uint64)), _t(np.array([999, 200, 150], np.uint64)))
     torch.cuda.synchronize()
     assert b.cpu().numpy()[:, :2].tolist() == [[0, 100], [10, 21], [15, 16]]
-    leaves = ix.dump()["buf"][5].reshape(-1, 16)
-    vals = leaves[:, 8:].copy().view(np.uint64).ravel()
+    dv = ix.dump()
+    leaves = dv["buf"][5].reshape(-1, int(dv["record_bytes"][5]))
+    vals = leaves[:, 8:16].copy().view(np.uint64).ravel()
     assert np.all(vals[10:20] == np.uint64(2**64 - 1)) and vals[20] == 201   # tombstones in place
     ix.close()
