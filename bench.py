@@ -408,17 +408,17 @@ def main():
     if world > 1:
         dist.barrier()
     evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
-    kevs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.3)
     launches0 = C.cuart_launch_count()
     torch.cuda.synchronize()
+    C.cuart_kernel_timer(ix.h, True)           # CUDA events around every k_lookup launch
     t_start = torch.cuda.Event(enable_timing=True)
     t_end = torch.cuda.Event(enable_timing=True)
     t_start.record(stream)
     for s in range(args.steps):
-        step(evs[s], kevs[s])
+        step(evs[s])
     t_end.record(stream)
     torch.cuda.synchronize()
     launches = C.cuart_launch_count() - launches0
@@ -428,8 +428,10 @@ def main():
     total_ms = t_start.elapsed_time(t_end)
     look_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in evs]))
     upd_ms = float(np.mean([e[1].elapsed_time(e[2]) for e in evs])) if nu else 0.0
-    kern_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in kevs]))
-    served = nl if di is None or mode == "replica" else getattr(di, "last_local_lookups", nl)
+    ktot, klaunch, kq = C.cuart_kernel_time(ix.h)
+    C.cuart_kernel_timer(ix.h, False)
+    kern_ms = ktot / max(1, klaunch)
+    served = kq / max(1, klaunch)
     tt = torch.tensor([total_ms, look_ms, upd_ms], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -531,7 +533,8 @@ def main():
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": args.traffic,
                          "kernel": {"u64": "k_lookup<KeyU64>", "u32": "k_lookup<KeyU32>", "bytes": "k_lookup<KeyBytes>"}[cfg.kind],
-                         "kernel_ms": round(kern_ms, 4), "lookups_per_launch": served,
+                         "kernel_ms": round(kern_ms, 4), "lookups_per_launch": int(served),
+                         "lookup_call_ms": round(look_ms, 4), "prebucket": "auto (on for batches >= 2^22)",
                          "bytes_per_lookup": round(bytes_per_lookup, 3),
                          "sectors_per_lookup": round(float(sec.mean()), 4), "peak_source": peak_src,
                          "random_access_ceiling": RANDOM_CEILING},

@@ -91,7 +91,15 @@ typedef struct {
                                     blocks per 64 entries: type bit-planes + per-type base
                                     index + rank; 1 B/entry, sized for L2 residency).
                                     COMPACT32 / RANK need integer keys (else LINKS).        */
+    uint32_t prebucket;          /* query pre-bucketing of large lookup batches (§8(a) a5):
+                                    CUART_PREBUCKET_AUTO (on for batches >= 2^22 queries),
+                                    CUART_PREBUCKET_OFF, CUART_PREBUCKET_ON.  Results are
+                                    identical; it reorders the batch so concurrent warps
+                                    share subtrees (stream-ordered scratch ~18 B/query). */
 } cuart_build_opts;
+#define CUART_PREBUCKET_AUTO 0u
+#define CUART_PREBUCKET_OFF 1u
+#define CUART_PREBUCKET_ON 2u
 #define CUART_LUT_FORMAT_AUTO 0u
 #define CUART_LUT_LINKS 1u
 #define CUART_LUT_COMPACT32 2u
@@ -183,6 +191,11 @@ cuart_status cuart_dump(const cuart_index* h, cuart_layout** out);
  * synchronises the index's device and clears the flag. */
 cuart_status cuart_get_error(cuart_index* h);
 const char* cuart_status_string(cuart_status s);
+/* Measurement hooks: while enabled, CUDA events bracket every k_lookup launch of
+ * this index on its stream; cuart_kernel_time sums their elapsed times (and
+ * launch / lookup counts) since the timer was (re)enabled, then resets. */
+cuart_status cuart_kernel_timer(cuart_index* h, int enable);
+cuart_status cuart_kernel_time(cuart_index* h, double* total_ms, uint64_t* launches, uint64_t* lookups);
 /* Kernel launches issued by this library since load (for launch accounting). */
 uint64_t cuart_launch_count(void);
 

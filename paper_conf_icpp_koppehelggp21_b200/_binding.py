@@ -26,7 +26,7 @@ class _Keys(ctypes.Structure):
 
 class _Opts(ctypes.Structure):
     _fields_ = [("lut_bytes", ctypes.c_uint32), ("l2_persist", ctypes.c_uint32),
-                ("device", ctypes.c_int32), ("lut_format", ctypes.c_uint32)]
+                ("device", ctypes.c_int32), ("lut_format", ctypes.c_uint32), ("prebucket", ctypes.c_uint32)]
 
 
 class _Stats(ctypes.Structure):
@@ -57,7 +57,8 @@ def lib():
         sig = {
             "cuart_build": [P, P, S, P, P], "cuart_lookup": [P, P, S, P, P], "cuart_update": [P, P, P, S, P],
             "cuart_destroy": [P], "cuart_update_ex": [P, P, P, P, S, P], "cuart_erase": [P, P, S, P],
-            "cuart_free_leaves": [P, P, S, P], "cuart_range": [P, P, P, S, P, P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
+            "cuart_free_leaves": [P, P, S, P], "cuart_range": [P, P, P, S, P, P],
+            "cuart_kernel_timer": [P, I], "cuart_kernel_time": [P, P, P, P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
             "cuart_stats": [P, P], "cuart_dump": [P, P], "cuart_get_error": [P],
             "cuart_layout_build": [P, P, S, P, P], "cuart_layout_view_get": [P, P],
             "cuart_layout_lookup": [P, P, S, P, I], "cuart_layout_sectors": [P, P, S, P, I], "cuart_upload": [P, P, P], "cuart_layout_free": [P],
@@ -142,8 +143,11 @@ def make_keys(keys, lengths=None):
     return st, n, (keys, lengths)
 
 
-def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0):
-    return _Opts(lut_bytes, l2_persist, device, lut_format)
+PREBUCKET_AUTO, PREBUCKET_OFF, PREBUCKET_ON = 0, 1, 2
+
+
+def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0):
+    return _Opts(lut_bytes, l2_persist, device, lut_format, prebucket)
 
 
 def _stream_ptr(stream):
@@ -156,14 +160,14 @@ def _stream_ptr(stream):
 
 
 # ------------------------------------------------------------------ hot path
-def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0):
+def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0):
     """Build + upload (host buffers).  Returns an opaque handle (int)."""
     k, n, keep = make_keys(keys)
     v = np.ascontiguousarray(values, dtype=np.uint64)
     if v.shape[0] != n:
         raise ValueError("values length mismatch")
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_format)
+    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket)
     _check(lib().cuart_build(ctypes.byref(k), _ptr(v), n, ctypes.byref(o), ctypes.byref(h)), "cuart_build")
     return h.value
 
@@ -204,6 +208,17 @@ def cuart_range(h, lo, hi, bounds, stream=None):
         raise ValueError("lo/hi length mismatch")
     _check(lib().cuart_range(h, ctypes.byref(kl), ctypes.byref(kh), n, _ptr(bounds), _stream_ptr(stream)), "cuart_range")
     return bounds
+
+
+def cuart_kernel_timer(h, enable=True):
+    _check(lib().cuart_kernel_timer(h, 1 if enable else 0), "cuart_kernel_timer")
+
+
+def cuart_kernel_time(h):
+    """(total_ms, launches, lookups) of k_lookup since the timer was enabled; resets."""
+    t, l, q = ctypes.c_double(), ctypes.c_uint64(), ctypes.c_uint64()
+    _check(lib().cuart_kernel_time(h, ctypes.byref(t), ctypes.byref(l), ctypes.byref(q)), "cuart_kernel_time")
+    return t.value, l.value, q.value
 
 
 def cuart_free_leaves(h):
@@ -303,9 +318,9 @@ def cuart_layout_sectors(l, queries, threads=0):
     return out
 
 
-def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_format=0):
+def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_format=0, prebucket=0):
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_format)
+    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket)
     _check(lib().cuart_upload(l, ctypes.byref(o), ctypes.byref(h)), "cuart_upload")
     return h.value
 
@@ -348,14 +363,14 @@ class Layout:
 class Index:
     """Device-resident CuART index on one GPU."""
 
-    def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0):
-        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_format)
+    def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0):
+        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_format, prebucket)
 
     @classmethod
-    def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_format=0):
+    def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_format=0, prebucket=0):
         """Upload an already-built host layout (keeps the host copy usable)."""
         self = cls.__new__(cls)
-        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format)
+        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format, prebucket)
         return self
 
     def lookup(self, queries, out=None, stream=None):

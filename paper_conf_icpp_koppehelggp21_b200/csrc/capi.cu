@@ -21,10 +21,13 @@
 #include <stdlib.h>
 
 #include <atomic>
+#include <mutex>
+#include <utility>
 #include <vector>
 #include <new>
 
 #include "../../include/cuart.h"
+#include "bucket.cuh"
 #include "builder.h"
 #include "kernels.cuh"
 
@@ -71,10 +74,25 @@ struct cuart_index {
     uint32_t lut_format = CUART_LUT_LINKS;
     uint64_t lutc_off = 0;             // compact / rank LUT region
     uint64_t lut_exceptions = 0;       // RANK: entries served by the 64-bit table
-    int grid_ctas_per_sm = 0;          // 0 = default grid (8 resident CTAs x 16 waves); else persistent grid
+    int grid_ctas_per_sm = 0;          // 0 = default grid (one op per thread); else persistent grid
+    bool ktimer = false;               // record CUDA events around every k_lookup launch
+    std::mutex kmu;
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev;
+    uint64_t klookups = 0;
+    uint32_t prebucket = CUART_PREBUCKET_AUTO;   // a5: reorder large lookup batches by bucket (bucket.cuh)
+
 };
 
 std::atomic<uint64_t> g_cuart_launches{0};   // also counted by route.cu
+
+static void drop_kevents(cuart_index* h) {
+    for (auto& e : h->kev) {
+        cudaEventDestroy(e.first);
+        cudaEventDestroy(e.second);
+    }
+    h->kev.clear();
+    h->klookups = 0;
+}   // also counted by route.cu
 
 #define CU_TRY(x)                                   \
     do {                                            \
@@ -203,10 +221,70 @@ static cuart_status check_keys(const cuart_index* h, const cuart_keys* k, size_t
     return CUART_OK;
 }
 
+static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens,
+                                         uint64_t n, uint64_t* out, cudaStream_t s);
+
+// a5 pre-bucketing: bucket -> lookup in bucketed order -> gather (bucket.cuh).
+// Scratch is stream-ordered (cudaMallocAsync from the device pool, whose release
+// threshold is raised at upload so the memory stays mapped between calls), so
+// concurrent lookups on several streams stay independent.
+template <class Key>
+static cuart_status launch_bucketed(const cuart_index* h, const void* q, const uint8_t* lens, uint64_t n, uint64_t* out,
+                                    cudaStream_t s) {
+    const size_t ks = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
+    auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
+    const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
+    const size_t o_hist = 0, o_tot = al(tiles * kBuckets * 4), o_q = o_tot + 1024, o_len = o_q + al(n * ks),
+                 o_pos = o_len + al(Key::kKind == 3 ? n : 0), o_res = o_pos + al(n * 2), total = o_res + al(n * 8);
+    uint8_t* scr = nullptr;
+    CU_TRY(cudaMallocAsync((void**)&scr, total, s));
+    unsigned int* hist = (unsigned int*)(scr + o_hist);
+    unsigned int* tot = (unsigned int*)(scr + o_tot);
+    const uint32_t depth = link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u;
+    k_bhist<Key><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
+    k_bscan_rows<<<kBuckets, 1024, 0, s>>>(hist, tiles, tot);
+    k_bscan<<<1, kBuckets, 0, s>>>(tot);
+    k_bscatter<Key><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key>(), s>>>(
+        q, lens, n, depth, hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, (uint16_t*)(scr + o_pos));
+    g_cuart_launches += 4;
+    CU_TRY(cudaGetLastError());
+    cuart_status rc = launch_lookup_direct(h, Key::kKind, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, n,
+                                           (uint64_t*)(scr + o_res), s);
+    if (rc != CUART_OK) return rc;
+    k_bgather<<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint64_t*)(scr + o_res), (const uint16_t*)(scr + o_pos),
+                                                          n, hist, tot, out);
+    g_cuart_launches++;
+    CU_TRY(cudaGetLastError());
+    CU_TRY(cudaFreeAsync(scr, s));
+    return CUART_OK;
+}
+
+static constexpr uint64_t kBucketMin = uint64_t(1) << 22;   // below this the batch is too small to reorder
+
 static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens, uint64_t n,
                                   uint64_t* out, cudaStream_t s) {
     if (n == 0) return CUART_OK;
+    const bool bucket = h->prebucket == CUART_PREBUCKET_ON ? n >= kBucketTile
+                      : h->prebucket == CUART_PREBUCKET_AUTO && n >= kBucketMin;
+    if (bucket && n < (uint64_t(1) << 32)) {
+        switch (kind) {
+        case CUART_KEY_U64: return launch_bucketed<KeyU64>(h, q, lens, n, out, s);
+        case CUART_KEY_U32: return launch_bucketed<KeyU32>(h, q, lens, n, out, s);
+        default: return launch_bucketed<KeyBytes>(h, q, lens, n, out, s);
+        }
+    }
+    return launch_lookup_direct(h, kind, q, lens, n, out, s);
+}
+
+static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens,
+                                         uint64_t n, uint64_t* out, cudaStream_t s) {
     const int grid = grid_for(h, n);
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    if (h->ktimer) {                                   // per-launch k_lookup timing (cuart_kernel_timer)
+        cudaEventCreate(&ev0);
+        cudaEventCreate(&ev1);
+        cudaEventRecord(ev0, s);
+    }
 #define CUART_LOOKUP(K, P) k_lookup<K, P><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out)
 #define CUART_LOOKUP_POL(K)                          \
     switch (h->policy) {                             \
@@ -226,6 +304,13 @@ static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const voi
 #undef CUART_LOOKUP_POL
 #undef CUART_LOOKUP
     g_cuart_launches++;
+    if (h->ktimer) {
+        cudaEventRecord(ev1, s);
+        cuart_index* hm = const_cast<cuart_index*>(h);
+        std::lock_guard<std::mutex> g(hm->kmu);
+        hm->kev.push_back({ev0, ev1});
+        hm->klookups += n;
+    }
     CU_TRY(cudaGetLastError());
     return CUART_OK;
 }
@@ -505,6 +590,23 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     h->lut_format = fmt;
     if (const char* pe = getenv("CUART_POLICY")) h->policy = atoi(pe);
     if (const char* pe = getenv("CUART_GRID_CTAS_PER_SM")) h->grid_ctas_per_sm = atoi(pe);   // tuning knob
+    h->prebucket = opts ? opts->prebucket : CUART_PREBUCKET_AUTO;
+    if (h->prebucket > CUART_PREBUCKET_ON) {
+        delete h;
+        return CUART_ERR_INVALID_ARGUMENT;
+    }
+    if (const char* pe = getenv("CUART_PREBUCKET")) h->prebucket = atoi(pe) ? CUART_PREBUCKET_ON : CUART_PREBUCKET_OFF;
+    {   // keep stream-ordered scratch mapped between calls (a5 bucketing)
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            uint64_t keep = ~uint64_t(0);
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+        }
+    }
+    cudaFuncSetAttribute(k_bscatter<KeyU64>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bscatter_smem<KeyU64>()));
+    cudaFuncSetAttribute(k_bscatter<KeyU32>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bscatter_smem<KeyU32>()));
+    cudaFuncSetAttribute(k_bscatter<KeyBytes>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         int(bscatter_smem<KeyBytes>()));
     // LUT region: 64-bit links (LINKS, and the exception table of RANK) then the compact form
     h->lut_off = off;
     const bool need_links = fmt == CUART_LUT_LINKS || fmt == CUART_LUT_RANK;
@@ -584,6 +686,7 @@ cuart_status cuart_destroy(cuart_index* h) {
     cudaFree(h->arena);
     if (h->leafref) cudaFree(h->leafref);
     if (h->slotref) cudaFree(h->slotref);
+    drop_kevents(h);
     for (int i = 0; i < kStages; i++) {
         if (h->stage[i]) cudaFree(h->stage[i]);
         if (h->stage_out[i]) cudaFree(h->stage_out[i]);
@@ -640,6 +743,31 @@ cuart_status cuart_range(const cuart_index* h, const cuart_keys* lo, const cuart
     if (!bounds) return CUART_ERR_INVALID_ARGUMENT;
     return cuart_range_leaf8(h->dix.base[T_LEAF8], h->count[T_LEAF8], h->key_kind, lo->data, hi->data, n, bounds,
                              stream);
+}
+
+cuart_status cuart_kernel_timer(cuart_index* h, int enable) {
+    if (!h) return CUART_ERR_INVALID_ARGUMENT;
+    std::lock_guard<std::mutex> g(h->kmu);
+    drop_kevents(h);
+    h->ktimer = enable != 0;
+    return CUART_OK;
+}
+
+cuart_status cuart_kernel_time(cuart_index* h, double* total_ms, uint64_t* launches, uint64_t* lookups) {
+    if (!h || !total_ms || !launches || !lookups) return CUART_ERR_INVALID_ARGUMENT;
+    std::lock_guard<std::mutex> g(h->kmu);
+    double t = 0;
+    for (auto& e : h->kev) {
+        float ms = 0;
+        CU_TRY(cudaEventSynchronize(e.second));
+        CU_TRY(cudaEventElapsedTime(&ms, e.first, e.second));
+        t += ms;
+    }
+    *total_ms = t;
+    *launches = h->kev.size();
+    *lookups = h->klookups;
+    drop_kevents(h);
+    return CUART_OK;
 }
 
 cuart_status cuart_free_leaves(const cuart_index* h, uint32_t* ids, size_t cap, size_t* count) {

@@ -333,3 +333,34 @@ def test_c4_full_size_sampled():
     mp = MapOracle((slots, lens), vals)
     assert np.array_equal(_u64(out[ti]), mp.lookup((qs[ti].cpu().numpy(), ql[ti].cpu().numpy())))
     ix.close()
+
+
+@pytest.mark.parametrize("kind", ["u64", "u32", "bytes"])
+def test_prebucket_equals_direct(kind):
+    """a5 pre-bucketing only reorders the batch: results identical to the direct
+    kernel and to the oracle, for ragged batch sizes across the tile size."""
+    if kind == "u64":
+        cfg = W.CONFIGS["c1"]
+        keys, vals = W.build_set(cfg)
+        mk = lambda m: W.lookup_batch(cfg, keys, 0, m)
+    elif kind == "u32":
+        keys = (np.arange(1 << 18, dtype=np.uint32) * 13) & np.uint32(0xFFFFFF)
+        keys = np.unique(keys)
+        vals = np.arange(keys.shape[0], dtype=np.uint64) + 1
+        rng = np.random.default_rng(0)
+        mk = lambda m: rng.integers(0, 1 << 24, m, dtype=np.uint32)
+    else:
+        keys = W.string_keys(4, 1 << 16)
+        vals = np.arange(1 << 16, dtype=np.uint64) + 5
+        mk = lambda m: (lambda idx: (keys[0][idx].copy(), keys[1][idx].copy()))(
+            W.string_lookup_at(W.CONFIGS["c4"], 1 << 16, np.arange(m)))
+    mp = MapOracle(keys, vals)
+    on = C.Index(keys, vals, prebucket=C.PREBUCKET_ON)
+    off = C.Index(keys, vals, prebucket=C.PREBUCKET_OFF)
+    for m in (4095, 4096, 4097, 100_003, 1 << 20):
+        q = mk(m)
+        a, b = _lookup(on, q), _lookup(off, q)
+        assert np.array_equal(a, b), m
+        assert np.array_equal(a, mp.lookup(q)), m
+    on.close()
+    off.close()
