@@ -117,9 +117,27 @@ __device__ __forceinline__ void copy_key_to_smem(const void* q, const uint8_t* l
     }
 }
 
+// Block-wide exclusive scan of one value per thread (kBucketThreads == kBuckets == 256).
+__device__ __forceinline__ unsigned int block_excl_scan256(unsigned int v, unsigned int* wtot) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    unsigned int x = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const unsigned int y = __shfl_up_sync(0xffffffffu, x, d);
+        if (lane >= d) x += y;
+    }
+    if (lane == 31) wtot[warp] = x;
+    __syncthreads();
+    unsigned int before = 0;
+#pragma unroll
+    for (int w = 0; w < kBucketThreads / 32; w++) before += w < warp ? wtot[w] : 0u;
+    return before + x - v;
+}
+
 // Tile of kBucketTile queries -> per-bucket runs.  Phase 1: bucket + rank in smem,
-// pos[i] written coalesced.  Phase 2: keys staged in smem in bucket order, then
-// written out with consecutive threads on consecutive slots of a run.
+// tile-local position jpos[i] (coalesced).  Phase 2: keys staged in smem in bucket
+// order; phase 3: each warp copies whole bucket runs to the bucketed batch
+// (contiguous source and destination: coalesced reads and writes).
 template <class Key>
 __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restrict__ q, const uint8_t* __restrict__ lens,
                                                              uint64_t n, uint32_t depth,
@@ -127,114 +145,139 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
                                                              const unsigned int* __restrict__ bases,
                                                              void* __restrict__ bq, uint8_t* __restrict__ blens,
                                                              uint16_t* __restrict__ jpos) {
+    static_assert(kBucketThreads == kBuckets, "one thread per bucket in the scans");
     constexpr uint32_t KS = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
     extern __shared__ __align__(16) uint8_t smem[];
     uint8_t* skeys = smem;                                             // kBucketTile * KS
-    uint32_t* sslot = (uint32_t*)(smem + kBucketTile * KS);           // kBucketTile
-    uint8_t* slens = (uint8_t*)(sslot + kBucketTile);                 // kBucketTile (BYTES)
+    uint8_t* slens = smem + kBucketTile * KS;                         // kBucketTile (BYTES)
     __shared__ unsigned int h[kBuckets];
     __shared__ unsigned int loc[kBuckets];
     __shared__ unsigned int glb[kBuckets];
-    for (int b = threadIdx.x; b < kBuckets; b += blockDim.x) h[b] = 0;
+    __shared__ unsigned int wtot[kBucketThreads / 32];
+    h[threadIdx.x] = 0;
     __syncthreads();
     const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
     uint32_t bk[kBucketItems], rk[kBucketItems];
+    uint64_t kv[kBucketItems];                                         // integer keys kept in registers
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {                           // all loads first (16 in flight)
+        const uint64_t i = base + uint64_t(r) * kBucketThreads + threadIdx.x;
+        kv[r] = 0;
+        if (i < n && Key::kKind != 3)
+            kv[r] = Key::kKind == 2 ? uint64_t(__ldcs((const unsigned long long*)q + i))
+                                    : uint64_t(__ldcs((const unsigned int*)q + i));
+    }
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
         const uint64_t i = base + uint64_t(r) * kBucketThreads + threadIdx.x;
         bk[r] = kBuckets;
         if (i < n) {
-            bk[r] = bucket_of(Key::template load<false>(q, lens, i), depth);
+            if (Key::kKind == 2) bk[r] = bucket_of(KeyU64{kv[r]}, depth);
+            else if (Key::kKind == 1) bk[r] = bucket_of(KeyU32{uint32_t(kv[r])}, depth);
+            else bk[r] = bucket_of(Key::template load<false>(q, lens, i), depth);
             rk[r] = atomicAdd(&h[bk[r]], 1u);
         }
     }
     __syncthreads();
-    if (threadIdx.x < kBuckets) {                                      // local exclusive offsets (serial scan, 256)
-        glb[threadIdx.x] = bases[threadIdx.x] + rowoff[uint64_t(threadIdx.x) * gridDim.x + blockIdx.x];
-    }
-    if (threadIdx.x == 0) {
-        unsigned int acc = 0;
-        for (int b = 0; b < kBuckets; b++) {
-            loc[b] = acc;
-            acc += h[b];
-        }
-    }
+    const unsigned int mine = h[threadIdx.x];
+    loc[threadIdx.x] = block_excl_scan256(mine, wtot);
+    glb[threadIdx.x] = bases[threadIdx.x] + rowoff[uint64_t(threadIdx.x) * gridDim.x + blockIdx.x];
     __syncthreads();
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
         const uint64_t i = base + uint64_t(r) * kBucketThreads + threadIdx.x;
         if (bk[r] < uint32_t(kBuckets)) {
             const uint32_t j = loc[bk[r]] + rk[r];                     // position in the staged tile
-            const uint32_t slot = glb[bk[r]] + rk[r];                  // position in the bucketed batch
-            copy_key_to_smem<Key>(q, lens, i, skeys, j);
-            if (Key::kKind == 3) slens[j] = lens[i];
-            sslot[j] = slot;
-            jpos[i] = uint16_t(j);                                     // tile-local position (coalesced)
+            if (Key::kKind == 2) ((uint64_t*)skeys)[j] = kv[r];
+            else if (Key::kKind == 1) ((uint32_t*)skeys)[j] = uint32_t(kv[r]);
+            else {
+                copy_key_to_smem<Key>(q, lens, i, skeys, j);
+                slens[j] = lens[i];
+            }
+            jpos[i] = uint16_t(j);
         }
     }
     __syncthreads();
-    const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
-    for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) {
-        const uint32_t slot = sslot[j];
-        if (KS == 8) ((uint64_t*)bq)[slot] = ((const uint64_t*)skeys)[j];
-        else if (KS == 4) ((uint32_t*)bq)[slot] = ((const uint32_t*)skeys)[j];
-        else {
-            ((uint4*)bq)[2 * uint64_t(slot)] = ((const uint4*)skeys)[2 * j];
-            ((uint4*)bq)[2 * uint64_t(slot) + 1] = ((const uint4*)skeys)[2 * j + 1];
-            blens[slot] = slens[j];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int b = warp; b < kBuckets; b += kBucketThreads / 32) {
+        const uint32_t c = h[b], l0 = loc[b];
+        const uint64_t g0 = glb[b];
+        for (uint32_t k = lane; k < c; k += 32) {
+            if (KS == 8) ((uint64_t*)bq)[g0 + k] = ((const uint64_t*)skeys)[l0 + k];
+            else if (KS == 4) ((uint32_t*)bq)[g0 + k] = ((const uint32_t*)skeys)[l0 + k];
+            else {
+                ((uint4*)bq)[2 * (g0 + k)] = ((const uint4*)skeys)[2 * (l0 + k)];
+                ((uint4*)bq)[2 * (g0 + k) + 1] = ((const uint4*)skeys)[2 * (l0 + k) + 1];
+                blens[g0 + k] = slens[l0 + k];
+            }
         }
     }
 }
 
 template <class Key>
 constexpr size_t bscatter_smem() {
-    return size_t(kBucketTile) * ((Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32) + 4 + (Key::kKind == 3 ? 1 : 0));
+    return size_t(kBucketTile) * ((Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32) + (Key::kKind == 3 ? 1 : 0));
 }
 
 // Per tile: the tile's results sit in 256 contiguous runs of the bucketed result
-// array (one per bucket, located exactly as k_bscatter placed them); load them in
-// tile-local order into shared memory, then out[i] = smem[jpos[i]] (coalesced).
+// array (one per bucket, located exactly as k_bscatter placed them); each warp
+// copies whole runs into shared memory in tile-local order, then
+// out[i] = smem[jpos[i]] (coalesced).
 __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __restrict__ res,
                                                             const uint16_t* __restrict__ jpos, uint64_t n,
                                                             const unsigned int* __restrict__ rowoff,
                                                             const unsigned int* __restrict__ bases,
                                                             uint64_t* __restrict__ out) {
     __shared__ uint64_t sres[kBucketTile];
-    __shared__ unsigned int loc[kBuckets + 1];
+    __shared__ unsigned int cnt_b[kBuckets];
+    __shared__ unsigned int loc[kBuckets];
     __shared__ unsigned int glb[kBuckets];
+    __shared__ unsigned int wtot[kBucketThreads / 32];
     const uint64_t t = blockIdx.x, tiles = gridDim.x;
     const uint64_t base = t * kBucketTile;
     const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
-    if (threadIdx.x < kBuckets) {
+    {
         const int b = threadIdx.x;
         const unsigned int off = rowoff[uint64_t(b) * tiles + t];
         const unsigned int btotal = (b + 1 < kBuckets ? bases[b + 1] : unsigned(n)) - bases[b];
         const unsigned int next = t + 1 < tiles ? rowoff[uint64_t(b) * tiles + t + 1] : btotal;
         glb[b] = bases[b] + off;
-        loc[b + 1] = next - off;                                        // this tile's count in bucket b
+        cnt_b[b] = next - off;
+        loc[b] = block_excl_scan256(next - off, wtot);
     }
     __syncthreads();
-    if (threadIdx.x == 0) {
-        unsigned int acc = 0;
-        loc[0] = 0;
-        for (int b = 0; b < kBuckets; b++) {
-            acc += loc[b + 1];
-            loc[b + 1] = acc;
+    uint64_t v[kBucketItems];
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {                           // 16 independent loads in flight
+        const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
+        v[r] = 0;
+        if (j < cnt) {
+            uint32_t lo = 0, hi = kBuckets;                             // bucket b: loc[b] <= j < loc[b] + cnt_b[b]
+            while (hi - lo > 1) {
+                const uint32_t mid = (lo + hi) >> 1;
+                if (loc[mid] <= j) lo = mid;
+                else hi = mid;
+            }
+            v[r] = __ldcs((const unsigned long long*)res + glb[lo] + (j - loc[lo]));
         }
     }
-    __syncthreads();
-    for (uint32_t j = threadIdx.x; j < cnt; j += blockDim.x) {
-        uint32_t lo = 0, hi = kBuckets;                                 // bucket b with loc[b] <= j < loc[b+1]
-        while (hi - lo > 1) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (loc[mid] <= j) lo = mid;
-            else hi = mid;
-        }
-        sres[j] = __ldcs((const unsigned long long*)res + glb[lo] + (j - loc[lo]));
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
+        if (j < cnt) sres[j] = v[r];
     }
     __syncthreads();
-    for (uint32_t k = threadIdx.x; k < cnt; k += blockDim.x)
-        __stcs((unsigned long long*)out + base + k, (unsigned long long)sres[__ldcs(jpos + base + k)]);
+    uint32_t jp[kBucketItems];
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t k = uint32_t(r) * kBucketThreads + threadIdx.x;
+        jp[r] = k < cnt ? __ldcs(jpos + base + k) : 0u;
+    }
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t k = uint32_t(r) * kBucketThreads + threadIdx.x;
+        if (k < cnt) __stcs((unsigned long long*)out + base + k, (unsigned long long)sres[jp[r]]);
+    }
 }
 
 }  // namespace cuart
