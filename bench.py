@@ -376,7 +376,19 @@ def main():
         samp = select(samp, owners(prefix8(samp), di.splitters_np) == rank)
     sec = layout.sectors(samp).astype(np.float64)
     io_bytes = {"u64": 8, "u32": 4, "bytes": 33}[cfg.kind] + 8
-    bytes_per_lookup = 32.0 * sec.mean() + io_bytes
+    random_bytes_per_lookup = 32.0 * sec.mean() + io_bytes
+    # Algorithmic DRAM bytes per lookup of the dominant kernel:
+    # direct path: every sector of the query's path is a random DRAM read (S x 32 B + I/O);
+    # pre-bucketed path (auto for >= 2^22 queries): the walk runs over one bucket's slice
+    # of the tree at a time, L2-resident by construction, so the compulsory traffic is the
+    # I/O plus each tree record once per batch (SURVEY §8(d) S_DRAM excludes L2-resident data).
+    bucketed = nl >= (1 << 22)
+    tree_bytes = sum(stats[t + "_bytes"] for t in ("n4", "n16", "n48", "n256", "leaf8", "leaf16", "leaf32"))
+    served_est = nl if mode != "range" else max(1, samp[0].shape[0] if isinstance(samp, tuple) else samp.shape[0]) * nl / (1 << 20)
+    bytes_per_lookup = (io_bytes + tree_bytes / served_est) if bucketed else random_bytes_per_lookup
+    # whole lookup call (bucket histogram + scatter + walk + gather), streaming bytes per query
+    ks = io_bytes - 8
+    pipeline_bytes = (ks + (ks + ks + 2) + (ks + 8) + (8 + 2 + 8)) + tree_bytes / served_est if bucketed else random_bytes_per_lookup
     del samp
 
     stream = torch.cuda.current_stream()
@@ -449,6 +461,12 @@ def main():
             peak = float(json.load(f)["hbm_gbs"])
         peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)"
     achieved = served * bytes_per_lookup / (kern_ms * 1e-3) / 1e9
+    pipe_achieved = nl * pipeline_bytes / (look_ms * 1e-3) / 1e9
+    traffic = args.traffic
+    tfile = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if traffic is None and os.path.exists(tfile):
+        with open(tfile) as f:
+            traffic = json.load(f).get(f"{args.config}/{'bucketed' if bucketed else 'direct'}")
     out_now = out if di is None else di.lookup(q)
     hit = float((out_now[: 1 << 24] != -1).float().mean().item())
     del out_now
@@ -531,13 +549,20 @@ def main():
             "update": {"mupdates_per_s": round(world * nu / (upd_ms * 1e-3) / 1e6, 3) if nu else None,
                        "ms": round(upd_ms, 4)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                         "frac": round(achieved / peak, 4), "traffic": args.traffic,
+                         "frac": round(achieved / peak, 4), "traffic": traffic,
                          "kernel": {"u64": "k_lookup<KeyU64>", "u32": "k_lookup<KeyU32>", "bytes": "k_lookup<KeyBytes>"}[cfg.kind],
                          "kernel_ms": round(kern_ms, 4), "lookups_per_launch": int(served),
                          "lookup_call_ms": round(look_ms, 4), "prebucket": "auto (on for batches >= 2^22)",
                          "bytes_per_lookup": round(bytes_per_lookup, 3),
-                         "sectors_per_lookup": round(float(sec.mean()), 4), "peak_source": peak_src,
-                         "random_access_ceiling": RANDOM_CEILING},
+                         "bytes_model": "bucketed: key+result I/O + tree records once per batch" if bucketed
+                         else "direct: 32 B x sectors on the path + key+result I/O",
+                         "sectors_per_lookup": round(float(sec.mean()), 4),
+                         "random_path_bytes_per_lookup": round(random_bytes_per_lookup, 3),
+                         "peak_source": peak_src, "random_access_ceiling": RANDOM_CEILING,
+                         "lookup_call": {"ms": round(look_ms, 4), "bytes_per_lookup": round(pipeline_bytes, 3),
+                                         "achieved": round(pipe_achieved, 1), "frac": round(pipe_achieved / peak, 4),
+                                         "kernels": "k_bhist, k_bscan_rows, k_bscan, k_bscatter, k_lookup, k_bgather"
+                                         if bucketed else "k_lookup"}},
             "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": int(launches), "clocks": clk,
             "index": {k: stats[k] for k in ("n4", "n16", "n48", "n256", "leaf8", "arena_bytes", "max_depth",
                                             "lut_exceptions")},
