@@ -384,7 +384,7 @@ def main():
     # I/O plus each tree record once per batch (SURVEY §8(d) S_DRAM excludes L2-resident data).
     bucketed = nl >= (1 << 22)
     tree_bytes = sum(stats[t + "_bytes"] for t in ("n4", "n16", "n48", "n256", "leaf8", "leaf16", "leaf32"))
-    served_est = nl if mode != "range" else max(1, samp[0].shape[0] if isinstance(samp, tuple) else samp.shape[0]) * nl / (1 << 20)
+    served_est = nl           # range mode: each rank serves ~nl routed lookups (its share of every rank's batch)
     bytes_per_lookup = (io_bytes + tree_bytes / served_est) if bucketed else random_bytes_per_lookup
     # whole lookup call (bucket histogram + scatter + walk + gather), streaming bytes per query
     ks = io_bytes - 8
