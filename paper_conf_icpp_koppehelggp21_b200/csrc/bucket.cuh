@@ -138,13 +138,18 @@ __device__ __forceinline__ unsigned int block_excl_scan256(unsigned int v, unsig
 // tile-local position jpos[i] (coalesced).  Phase 2: keys staged in smem in bucket
 // order; phase 3: each warp copies whole bucket runs to the bucketed batch
 // (contiguous source and destination: coalesced reads and writes).
-template <class Key>
+// OPS (update batches): also carry each op's value and original index (its
+// priority) to the op's slot; no gather follows, so jpos is not written.
+template <class Key, bool OPS = false>
 __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restrict__ q, const uint8_t* __restrict__ lens,
                                                              uint64_t n, uint32_t depth,
                                                              const unsigned int* __restrict__ rowoff,
                                                              const unsigned int* __restrict__ bases,
                                                              void* __restrict__ bq, uint8_t* __restrict__ blens,
-                                                             uint16_t* __restrict__ jpos) {
+                                                             uint16_t* __restrict__ jpos,
+                                                             const uint64_t* __restrict__ vals = nullptr,
+                                                             uint64_t* __restrict__ bvals = nullptr,
+                                                             uint32_t* __restrict__ bidx = nullptr) {
     static_assert(kBucketThreads == kBuckets, "one thread per bucket in the scans");
     constexpr uint32_t KS = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
     extern __shared__ __align__(16) uint8_t smem[];
@@ -194,7 +199,13 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
                 copy_key_to_smem<Key>(q, lens, i, skeys, j);
                 slens[j] = lens[i];
             }
-            jpos[i] = uint16_t(j);
+            if (OPS) {
+                const uint64_t slot = uint64_t(glb[bk[r]]) + rk[r];
+                bvals[slot] = __ldcs((const unsigned long long*)vals + i);
+                bidx[slot] = uint32_t(i);
+            } else {
+                jpos[i] = uint16_t(j);
+            }
         }
     }
     __syncthreads();
@@ -229,7 +240,6 @@ __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __re
                                                             const unsigned int* __restrict__ bases,
                                                             uint64_t* __restrict__ out) {
     __shared__ uint64_t sres[kBucketTile];
-    __shared__ unsigned int cnt_b[kBuckets];
     __shared__ unsigned int loc[kBuckets];
     __shared__ unsigned int glb[kBuckets];
     __shared__ unsigned int wtot[kBucketThreads / 32];
@@ -242,7 +252,6 @@ __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __re
         const unsigned int btotal = (b + 1 < kBuckets ? bases[b + 1] : unsigned(n)) - bases[b];
         const unsigned int next = t + 1 < tiles ? rowoff[uint64_t(b) * tiles + t + 1] : btotal;
         glb[b] = bases[b] + off;
-        cnt_b[b] = next - off;
         loc[b] = block_excl_scan256(next - off, wtot);
     }
     __syncthreads();

@@ -153,7 +153,7 @@ template <class Key, int POL, bool DEL>
 __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restrict__ q, const uint8_t* __restrict__ lens,
                                               const uint64_t* __restrict__ vals, const uint8_t* __restrict__ is_delete,
                                               uint64_t n, uint64_t epoch_hi, uint64_t* __restrict__ leafref,
-                                              uint64_t* __restrict__ slotref) {
+                                              uint64_t* __restrict__ slotref, const uint32_t* __restrict__ opidx) {
     const Loader<POL> ld;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
@@ -168,7 +168,8 @@ __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restric
         }
         leafref[i] = leaf;
         if (DEL) slotref[i] = slot;
-        if (leaf) atomicMax((unsigned long long*)winner_word(ix, leaf), (unsigned long long)(epoch_hi | i));
+        const uint64_t prio = opidx ? uint64_t(opidx[i]) : i;      // priority = original op index
+        if (leaf) atomicMax((unsigned long long*)winner_word(ix, leaf), (unsigned long long)(epoch_hi | prio));
     }
 }
 
@@ -180,13 +181,15 @@ __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restric
 template <bool DEL>
 __global__ void __launch_bounds__(256) k_upd2(DevIndex ix, const uint64_t* __restrict__ vals,
                                               const uint8_t* __restrict__ is_delete, uint64_t n, uint64_t epoch_hi,
-                                              const uint64_t* __restrict__ leafref, const uint64_t* __restrict__ slotref) {
+                                              const uint64_t* __restrict__ leafref, const uint64_t* __restrict__ slotref,
+                                              const uint32_t* __restrict__ opidx) {
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
         const uint64_t leaf = leafref[i];
         if (!leaf) continue;
         const uint64_t gid = global_leaf_id(ix, leaf);
-        if (__ldcg(winner_word(ix, leaf)) != (epoch_hi | i)) continue;
+        const uint64_t prio = opidx ? uint64_t(opidx[i]) : i;
+        if (__ldcg(winner_word(ix, leaf)) != (epoch_hi | prio)) continue;
         const uint32_t t = link_type(leaf);
         uint64_t* dst = (uint64_t*)(ix.base[t] + link_index(leaf) * record_bytes(t) + leaf_value_off(t));
         if (DEL && (is_delete == nullptr || is_delete[i])) {
@@ -335,10 +338,11 @@ static cuart_status ensure_scratch(cuart_index* h, size_t n, bool slots) {
 
 static constexpr uint64_t kUpdateChunk = uint64_t(1) << 30;   // op index must fit the low 32 bits
 
-// mode: 0 = updates only, 1 = mixed (is_delete[i]), 2 = all deletes (vals unused)
+// mode: 0 = updates only, 1 = mixed (is_delete[i]), 2 = all deletes (vals unused).
+// opidx: original op index of each op (pre-bucketed batches), or nullptr (= position).
 static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, const uint8_t* lens,
                                   const uint64_t* vals, const uint8_t* is_delete, int mode, uint64_t n,
-                                  cudaStream_t s) {
+                                  cudaStream_t s, const uint32_t* opidx = nullptr) {
     const bool del = mode != 0;
     for (uint64_t base = 0; base < n; base += kUpdateChunk) {
         const uint64_t m = (n - base) < kUpdateChunk ? (n - base) : kUpdateChunk;
@@ -361,7 +365,8 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
         const uint8_t* lb = lens ? lens + base : nullptr;
         const uint64_t* vb = vals ? vals + base : nullptr;
         const uint8_t* db = (mode == 1) ? is_delete + base : nullptr;
-#define CUART_UPD1(K, P, D) k_upd1<K, P, D><<<grid, 256, 0, s>>>(h->dix, kb, lb, vb, db, m, epoch_hi, h->leafref, h->slotref)
+        const uint32_t* ib = opidx ? opidx + base : nullptr;
+#define CUART_UPD1(K, P, D) k_upd1<K, P, D><<<grid, 256, 0, s>>>(h->dix, kb, lb, vb, db, m, epoch_hi, h->leafref, h->slotref, ib)
 #define CUART_UPD1_POL(K)                                    \
     if (h->policy == 0) {                                    \
         if (del) CUART_UPD1(K, 0, true); else CUART_UPD1(K, 0, false); \
@@ -377,12 +382,58 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
 #undef CUART_UPD1
         g_cuart_launches++;
         CU_TRY(cudaGetLastError());
-        if (del) k_upd2<true><<<grid, 256, 0, s>>>(h->dix, vb, db, m, epoch_hi, h->leafref, h->slotref);
-        else k_upd2<false><<<grid, 256, 0, s>>>(h->dix, vb, nullptr, m, epoch_hi, h->leafref, nullptr);
+        if (del) k_upd2<true><<<grid, 256, 0, s>>>(h->dix, vb, db, m, epoch_hi, h->leafref, h->slotref, ib);
+        else k_upd2<false><<<grid, 256, 0, s>>>(h->dix, vb, nullptr, m, epoch_hi, h->leafref, nullptr, ib);
         g_cuart_launches++;
         CU_TRY(cudaGetLastError());
     }
     return CUART_OK;
+}
+
+// Pre-bucketed update batch (a5 applied to stage 1/2): ops are reordered by bucket
+// together with their values and ORIGINAL op indices, which stay the priorities
+// of the conflict resolution; no inverse permutation is needed because
+// updates return nothing.
+template <class Key>
+static cuart_status launch_update_bucketed(cuart_index* h, const void* k, const uint8_t* lens, const uint64_t* vals,
+                                          uint64_t n, cudaStream_t s) {
+    const size_t ks = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
+    auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
+    const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
+    const size_t o_hist = 0, o_tot = al(tiles * kBuckets * 4), o_q = o_tot + 1024, o_len = o_q + al(n * ks),
+                 o_val = o_len + al(Key::kKind == 3 ? n : 0), o_idx = o_val + al(n * 8), total = o_idx + al(n * 4);
+    uint8_t* scr = nullptr;
+    CU_TRY(cudaMallocAsync((void**)&scr, total, s));
+    unsigned int* hist = (unsigned int*)(scr + o_hist);
+    unsigned int* tot = (unsigned int*)(scr + o_tot);
+    const uint32_t depth = link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u;
+    k_bhist<Key><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
+    k_bscan_rows<<<kBuckets, 1024, 0, s>>>(hist, tiles, tot);
+    k_bscan<<<1, kBuckets, 0, s>>>(tot);
+    k_bscatter<Key, true><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key>(), s>>>(
+        k, lens, n, depth, hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, nullptr, vals,
+        (uint64_t*)(scr + o_val), (uint32_t*)(scr + o_idx));
+    g_cuart_launches += 4;
+    CU_TRY(cudaGetLastError());
+    cuart_status rc = launch_update(h, Key::kKind, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr,
+                                    (const uint64_t*)(scr + o_val), nullptr, 0, n, s, (const uint32_t*)(scr + o_idx));
+    if (rc != CUART_OK) return rc;
+    CU_TRY(cudaFreeAsync(scr, s));
+    return CUART_OK;
+}
+
+static cuart_status dispatch_update(cuart_index* h, const void* k, const uint8_t* lens, const uint64_t* vals, uint64_t n,
+                                    cudaStream_t s) {
+    const bool bucket = h->prebucket == CUART_PREBUCKET_ON ? n >= kBucketTile
+                      : h->prebucket == CUART_PREBUCKET_AUTO && n >= kBucketMin;
+    if (bucket && n < kUpdateChunk) {
+        switch (h->key_kind) {
+        case CUART_KEY_U64: return launch_update_bucketed<KeyU64>(h, k, lens, vals, n, s);
+        case CUART_KEY_U32: return launch_update_bucketed<KeyU32>(h, k, lens, vals, n, s);
+        default: return launch_update_bucketed<KeyBytes>(h, k, lens, vals, n, s);
+        }
+    }
+    return launch_update(h, h->key_kind, k, lens, vals, nullptr, 0, n, s);
 }
 
 // ============================================================================ C ABI
@@ -607,6 +658,12 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     cudaFuncSetAttribute(k_bscatter<KeyU32>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bscatter_smem<KeyU32>()));
     cudaFuncSetAttribute(k_bscatter<KeyBytes>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          int(bscatter_smem<KeyBytes>()));
+    cudaFuncSetAttribute(k_bscatter<KeyU64, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         int(bscatter_smem<KeyU64>()));
+    cudaFuncSetAttribute(k_bscatter<KeyU32, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         int(bscatter_smem<KeyU32>()));
+    cudaFuncSetAttribute(k_bscatter<KeyBytes, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         int(bscatter_smem<KeyBytes>()));
     // LUT region: 64-bit links (LINKS, and the exception table of RANK) then the compact form
     h->lut_off = off;
     const bool need_links = fmt == CUART_LUT_LINKS || fmt == CUART_LUT_RANK;
@@ -711,7 +768,7 @@ cuart_status cuart_update(cuart_index* h, const cuart_keys* k, const uint64_t* v
     if (rc != CUART_OK) return rc;
     if (n == 0) return CUART_OK;
     if (!v) return CUART_ERR_INVALID_ARGUMENT;
-    return launch_update(h, h->key_kind, k->data, k->lengths, v, nullptr, 0, n, (cudaStream_t)stream);
+    return dispatch_update(h, k->data, k->lengths, v, n, (cudaStream_t)stream);
 }
 
 cuart_status cuart_update_ex(cuart_index* h, const cuart_keys* k, const uint64_t* v, const uint8_t* is_delete, size_t n,
@@ -842,8 +899,7 @@ cuart_status cuart_update_host(cuart_index* h, const cuart_keys* k, const uint64
         CU_TRY(cudaMemcpyAsync(h->stage[s], (const uint8_t*)k->data + base * ks, m * ks, cudaMemcpyHostToDevice, st));
         if (k->lengths) CU_TRY(cudaMemcpyAsync(h->stage_len[s], k->lengths + base, m, cudaMemcpyHostToDevice, st));
         CU_TRY(cudaMemcpyAsync(h->stage_val[s], v + base, m * 8, cudaMemcpyHostToDevice, st));
-        rc = launch_update(h, h->key_kind, h->stage[s], k->lengths ? h->stage_len[s] : nullptr, h->stage_val[s],
-                           nullptr, 0, m, st);
+        rc = dispatch_update(h, h->stage[s], k->lengths ? h->stage_len[s] : nullptr, h->stage_val[s], m, st);
         if (rc != CUART_OK) return rc;
     }
     CU_TRY(cudaStreamSynchronize(st));

@@ -364,3 +364,34 @@ def test_prebucket_equals_direct(kind):
         assert np.array_equal(a, mp.lookup(q)), m
     on.close()
     off.close()
+
+
+@pytest.mark.parametrize("kind", ["u64", "u32", "bytes"])
+def test_prebucket_updates_equal_direct(kind):
+    """Pre-bucketed update batches keep the ORIGINAL op index as priority:
+    same final state as the direct kernels and the sequential oracle, with many
+    duplicate keys spread over different tiles and buckets."""
+    rng = np.random.default_rng(9)
+    if kind == "u64":
+        keys, vals = W.build_set(W.CONFIGS["c1"])
+    elif kind == "u32":
+        keys = np.unique((np.arange(1 << 17, dtype=np.uint32) * 29) & np.uint32(0xFFFFFF))
+        vals = np.arange(keys.shape[0], dtype=np.uint64) + 1
+    else:
+        keys = W.string_keys(4, 1 << 15)
+        vals = np.arange(1 << 15, dtype=np.uint64) + 5
+    n = keys[1].shape[0] if isinstance(keys, tuple) else keys.shape[0]
+    on = C.Index(keys, vals, prebucket=C.PREBUCKET_ON)
+    off = C.Index(keys, vals, prebucket=C.PREBUCKET_OFF)
+    mp = MapOracle(keys, vals)
+    for m in (4097, 200_003):
+        pick = rng.integers(0, min(n, 3000), m)                     # heavy duplication
+        uk = (keys[0][pick].copy(), keys[1][pick].copy()) if isinstance(keys, tuple) else keys[pick].copy()
+        uv = rng.integers(0, 2**63, m, dtype=np.uint64)
+        on.update(_t(uk), _t(uv))
+        off.update(_t(uk), _t(uv))
+        mp.update(uk, uv)
+        a, b = _lookup(on, keys), _lookup(off, keys)
+        assert np.array_equal(a, b) and np.array_equal(a, mp.lookup(keys)), m
+    on.close()
+    off.close()
