@@ -382,7 +382,7 @@ def main():
     # pre-bucketed path (auto for >= 2^22 queries): the walk runs over one bucket's slice
     # of the tree at a time, L2-resident by construction, so the compulsory traffic is the
     # I/O plus each tree record once per batch (SURVEY §8(d) S_DRAM excludes L2-resident data).
-    bucketed = nl >= (1 << 22)
+    bucketed = nl >= (1 << 22) and cfg.kind != "bytes"
     tree_bytes = sum(stats[t + "_bytes"] for t in ("n4", "n16", "n48", "n256", "leaf8", "leaf16", "leaf32"))
     served_est = nl           # range mode: each rank serves ~nl routed lookups (its share of every rank's batch)
     bytes_per_lookup = (io_bytes + tree_bytes / served_est) if bucketed else random_bytes_per_lookup
@@ -552,7 +552,7 @@ def main():
                          "frac": round(achieved / peak, 4), "traffic": traffic,
                          "kernel": {"u64": "k_lookup<KeyU64>", "u32": "k_lookup<KeyU32>", "bytes": "k_lookup<KeyBytes>"}[cfg.kind],
                          "kernel_ms": round(kern_ms, 4), "lookups_per_launch": int(served),
-                         "lookup_call_ms": round(look_ms, 4), "prebucket": "auto (on for batches >= 2^22)",
+                         "lookup_call_ms": round(look_ms, 4), "prebucket": "on" if bucketed else "off",
                          "bytes_per_lookup": round(bytes_per_lookup, 3),
                          "bytes_model": "bucketed: key+result I/O + tree records once per batch" if bucketed
                          else "direct: 32 B x sectors on the path + key+result I/O",

@@ -92,7 +92,8 @@ typedef struct {
                                     index + rank; 1 B/entry, sized for L2 residency).
                                     COMPACT32 / RANK need integer keys (else LINKS).        */
     uint32_t prebucket;          /* query pre-bucketing of large lookup batches (§8(a) a5):
-                                    CUART_PREBUCKET_AUTO (on for batches >= 2^22 queries),
+                                    CUART_PREBUCKET_AUTO (on for integer-key batches of
+                                    >= 2^22 ops, lookups and plain updates),
                                     CUART_PREBUCKET_OFF, CUART_PREBUCKET_ON.  Results are
                                     identical; it reorders the batch so concurrent warps
                                     share subtrees (stream-ordered scratch ~18 B/query). */
