@@ -30,6 +30,17 @@ constexpr int kBucketThreads = 256;
 constexpr int kBucketItems = 16;
 constexpr int kBucketTile = kBucketThreads * kBucketItems;
 
+// Histogram layout: [tile group][bucket][tile in group] with groups of kHistGroup
+// tiles, so the per-bucket scan reads 32-B runs and a tile's 256 entries share
+// sectors with the neighbouring tiles that run at the same time.
+constexpr uint64_t kHistGroup = 8;
+__device__ __forceinline__ uint64_t hidx(uint32_t b, uint64_t t) {
+    return ((t / kHistGroup) * kBuckets + b) * kHistGroup + (t % kHistGroup);
+}
+__host__ __device__ constexpr uint64_t hist_entries(uint64_t tiles) {
+    return ((tiles + kHistGroup - 1) / kHistGroup) * kHistGroup * kBuckets;
+}
+
 template <class Key>
 __device__ __forceinline__ uint32_t bucket_of(const Key& k, uint32_t depth) {
     return depth < k.len() ? k.byte(depth) : 0u;
@@ -48,7 +59,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bhist(const void* __restrict
         if (i < n) atomicAdd(&h[bucket_of(Key::template load<true>(q, lens, i), depth)], 1u);
     }
     __syncthreads();
-    for (int b = threadIdx.x; b < kBuckets; b += blockDim.x) hist[uint64_t(b) * gridDim.x + blockIdx.x] = h[b];
+    for (int b = threadIdx.x; b < kBuckets; b += blockDim.x) hist[hidx(b, blockIdx.x)] = h[b];
 }
 
 // One CTA per bucket: exclusive scan of its row over the tiles (in place), row total -> totals[b].
@@ -56,13 +67,12 @@ __global__ void __launch_bounds__(1024) k_bscan_rows(unsigned int* __restrict__ 
                                                      unsigned int* __restrict__ totals) {
     __shared__ unsigned int wsum[32];
     __shared__ unsigned int carry;
-    unsigned int* row = hist + uint64_t(blockIdx.x) * tiles;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     if (threadIdx.x == 0) carry = 0;
     __syncthreads();
     for (uint64_t s0 = 0; s0 < tiles; s0 += blockDim.x) {
         const uint64_t t = s0 + threadIdx.x;
-        const unsigned int v = t < tiles ? row[t] : 0u;
+        const unsigned int v = t < tiles ? hist[hidx(blockIdx.x, t)] : 0u;
         unsigned int x = v;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
@@ -82,7 +92,7 @@ __global__ void __launch_bounds__(1024) k_bscan_rows(unsigned int* __restrict__ 
         }
         __syncthreads();
         const unsigned int excl = carry + (warp ? wsum[warp - 1] : 0u) + x - v;
-        if (t < tiles) row[t] = excl;
+        if (t < tiles) hist[hidx(blockIdx.x, t)] = excl;
         __syncthreads();
         if (threadIdx.x == blockDim.x - 1) carry = excl + v;
         __syncthreads();
@@ -186,7 +196,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
     __syncthreads();
     const unsigned int mine = h[threadIdx.x];
     loc[threadIdx.x] = block_excl_scan256(mine, wtot);
-    glb[threadIdx.x] = bases[threadIdx.x] + rowoff[uint64_t(threadIdx.x) * gridDim.x + blockIdx.x];
+    glb[threadIdx.x] = bases[threadIdx.x] + rowoff[hidx(threadIdx.x, blockIdx.x)];
     __syncthreads();
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
@@ -248,9 +258,9 @@ __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __re
     const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
     {
         const int b = threadIdx.x;
-        const unsigned int off = rowoff[uint64_t(b) * tiles + t];
+        const unsigned int off = rowoff[hidx(b, t)];
         const unsigned int btotal = (b + 1 < kBuckets ? bases[b + 1] : unsigned(n)) - bases[b];
-        const unsigned int next = t + 1 < tiles ? rowoff[uint64_t(b) * tiles + t + 1] : btotal;
+        const unsigned int next = t + 1 < tiles ? rowoff[hidx(b, t + 1)] : btotal;
         glb[b] = bases[b] + off;
         loc[b] = block_excl_scan256(next - off, wtot);
     }
