@@ -177,12 +177,24 @@ class DistIndex:
         self.index = ops.build(keys, values, lut_bytes)
 
     # ---- helpers
+    # Collectives.  NCCL moves CUDA tensors directly (the product path on the GPU
+    # box).  gloo cannot, so CUDA tensors are staged through host memory — this lets
+    # the complete GPU path (CuART kernels + this protocol) run as several processes
+    # sharing one GPU in tests, where NCCL refuses duplicate devices.
+    def _staged(self, t):
+        return t.is_cuda and dist.get_backend(self.group) != "nccl"
+
     def _a2a(self, out, inp, out_splits, in_splits):
+        if self._staged(inp):
+            ho = out.new_empty(out.shape, device="cpu")
+            dist.all_to_all_single(ho, inp.cpu(), out_splits, in_splits, group=self.group)
+            out.copy_(ho)
+            return
         dist.all_to_all_single(out, inp, out_splits, in_splits, group=self.group)
 
     def _exchange_counts(self, counts):
         recv = torch.empty_like(counts)
-        dist.all_to_all_single(recv, counts, group=self.group)
+        self._a2a(recv, counts, None, None)
         return recv
 
     def _split_keys(self, q):
@@ -258,6 +270,8 @@ class DistIndex:
         return self.ops.unroute(full, perm)
 
     def _all_gather_var(self, t):
+        if self._staged(t):
+            return self._all_gather_var(t.cpu()).to(t.device)
         n = torch.tensor([t.shape[0]], dtype=torch.int64, device=t.device)
         ns = [torch.empty_like(n) for _ in range(self.world)]
         dist.all_gather(ns, n, group=self.group)
