@@ -324,11 +324,14 @@ def main():
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        # NCCL over NVLink/NVSwitch; CUART_DIST_BACKEND=gloo only to smoke-test the
+        # multi-rank path with several ranks sharing one GPU (host-staged collectives)
+        backend = os.environ.get("CUART_DIST_BACKEND", "nccl")
+        dist.init_process_group(backend, device_id=dev if backend == "nccl" else None)
     mode = "single" if world == 1 else args.mode
     if args.config == "c5":
         run_c5(args, world, rank, local, dev)
