@@ -172,7 +172,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
     h[threadIdx.x] = 0;
     __syncthreads();
     const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
-    uint32_t bk[kBucketItems], rk[kBucketItems];
+    uint32_t br[kBucketItems];                                         // bucket << 16 | rank (0xFFFFFFFF = none)
     uint64_t kv[kBucketItems];                                         // integer keys kept in registers
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {                           // all loads first (16 in flight)
@@ -185,12 +185,13 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
         const uint64_t i = base + uint64_t(r) * kBucketThreads + threadIdx.x;
-        bk[r] = kBuckets;
+        br[r] = 0xFFFFFFFFu;
         if (i < n) {
-            if (Key::kKind == 2) bk[r] = bucket_of(KeyU64{kv[r]}, depth);
-            else if (Key::kKind == 1) bk[r] = bucket_of(KeyU32{uint32_t(kv[r])}, depth);
-            else bk[r] = bucket_of(Key::template load<false>(q, lens, i), depth);
-            rk[r] = atomicAdd(&h[bk[r]], 1u);
+            uint32_t b;
+            if (Key::kKind == 2) b = bucket_of(KeyU64{kv[r]}, depth);
+            else if (Key::kKind == 1) b = bucket_of(KeyU32{uint32_t(kv[r])}, depth);
+            else b = bucket_of(Key::template load<false>(q, lens, i), depth);
+            br[r] = (b << 16) | atomicAdd(&h[b], 1u);
         }
     }
     __syncthreads();
@@ -201,8 +202,9 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
         const uint64_t i = base + uint64_t(r) * kBucketThreads + threadIdx.x;
-        if (bk[r] < uint32_t(kBuckets)) {
-            const uint32_t j = loc[bk[r]] + rk[r];                     // position in the staged tile
+        if (br[r] != 0xFFFFFFFFu) {
+            const uint32_t b = br[r] >> 16, rk = br[r] & 0xFFFFu;
+            const uint32_t j = loc[b] + rk;                            // position in the staged tile
             if (Key::kKind == 2) ((uint64_t*)skeys)[j] = kv[r];
             else if (Key::kKind == 1) ((uint32_t*)skeys)[j] = uint32_t(kv[r]);
             else {
@@ -210,7 +212,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
                 slens[j] = lens[i];
             }
             if (OPS) {
-                const uint64_t slot = uint64_t(glb[bk[r]]) + rk[r];
+                const uint64_t slot = uint64_t(glb[b]) + rk;
                 bvals[slot] = __ldcs((const unsigned long long*)vals + i);
                 bidx[slot] = uint32_t(i);
             } else {
@@ -250,20 +252,22 @@ __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __re
                                                             const unsigned int* __restrict__ bases,
                                                             uint64_t* __restrict__ out) {
     __shared__ uint64_t sres[kBucketTile];
+    __shared__ uint8_t bof[kBucketTile];                               // bucket of each tile-local position
     __shared__ unsigned int loc[kBuckets];
     __shared__ unsigned int glb[kBuckets];
     __shared__ unsigned int wtot[kBucketThreads / 32];
     const uint64_t t = blockIdx.x, tiles = gridDim.x;
     const uint64_t base = t * kBucketTile;
     const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
-    {
-        const int b = threadIdx.x;
-        const unsigned int off = rowoff[hidx(b, t)];
-        const unsigned int btotal = (b + 1 < kBuckets ? bases[b + 1] : unsigned(n)) - bases[b];
-        const unsigned int next = t + 1 < tiles ? rowoff[hidx(b, t + 1)] : btotal;
-        glb[b] = bases[b] + off;
-        loc[b] = block_excl_scan256(next - off, wtot);
-    }
+    const int b = threadIdx.x;
+    const unsigned int off = rowoff[hidx(b, t)];
+    const unsigned int btotal = (b + 1 < kBuckets ? bases[b + 1] : unsigned(n)) - bases[b];
+    const unsigned int next = t + 1 < tiles ? rowoff[hidx(b, t + 1)] : btotal;
+    const unsigned int c_b = next - off;
+    glb[b] = bases[b] + off;
+    const unsigned int l_b = block_excl_scan256(c_b, wtot);
+    loc[b] = l_b;
+    for (unsigned int k = 0; k < c_b; k++) bof[l_b + k] = uint8_t(b);
     __syncthreads();
     uint64_t v[kBucketItems];
 #pragma unroll
@@ -271,13 +275,8 @@ __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __re
         const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
         v[r] = 0;
         if (j < cnt) {
-            uint32_t lo = 0, hi = kBuckets;                             // bucket b: loc[b] <= j < loc[b] + cnt_b[b]
-            while (hi - lo > 1) {
-                const uint32_t mid = (lo + hi) >> 1;
-                if (loc[mid] <= j) lo = mid;
-                else hi = mid;
-            }
-            v[r] = __ldcs((const unsigned long long*)res + glb[lo] + (j - loc[lo]));
+            const uint32_t bj = bof[j];
+            v[r] = __ldcs((const unsigned long long*)res + glb[bj] + (j - loc[bj]));
         }
     }
 #pragma unroll
