@@ -443,7 +443,7 @@ def main():
     total_ms = t_start.elapsed_time(t_end)
     look_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in evs]))
     upd_ms = float(np.mean([e[1].elapsed_time(e[2]) for e in evs])) if nu else 0.0
-    ktot, klaunch, kq = C.cuart_kernel_time(ix.h)
+    ktot, klaunch, kq, kslice = C.cuart_kernel_time_ex(ix.h)
     C.cuart_kernel_timer(ix.h, False)
     kern_ms = ktot / max(1, klaunch)
     served = kq / max(1, klaunch)
@@ -553,7 +553,8 @@ def main():
                        "ms": round(upd_ms, 4)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
-                         "kernel": {"u64": "k_lookup<KeyU64>", "u32": "k_lookup<KeyU32>", "bytes": "k_lookup<KeyBytes>"}[cfg.kind],
+                         "kernel": ("k_lookup_slice" if kslice else "k_lookup")
+                         + {"u64": "<KeyU64>", "u32": "<KeyU32>", "bytes": "<KeyBytes>"}[cfg.kind],
                          "kernel_ms": round(kern_ms, 4), "lookups_per_launch": int(served),
                          "lookup_call_ms": round(look_ms, 4), "prebucket": "on" if bucketed else "off",
                          "bytes_per_lookup": round(bytes_per_lookup, 3),
@@ -564,7 +565,8 @@ def main():
                          "peak_source": peak_src, "random_access_ceiling": RANDOM_CEILING,
                          "lookup_call": {"ms": round(look_ms, 4), "bytes_per_lookup": round(pipeline_bytes, 3),
                                          "achieved": round(pipe_achieved, 1), "frac": round(pipe_achieved / peak, 4),
-                                         "kernels": "k_bhist, k_bscan_rows, k_bscan, k_bscatter, k_lookup, k_bgather"
+                                         "kernels": "k_bhist, k_bscan_rows, k_bscan, k_bscatter, "
+                                         + ("k_lookup_slice" if kslice else "k_lookup") + ", k_bgather"
                                          if bucketed else "k_lookup"}},
             "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": int(launches), "clocks": clk,
             "index": {k: stats[k] for k in ("n4", "n16", "n48", "n256", "leaf8", "arena_bytes", "max_depth",

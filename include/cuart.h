@@ -97,7 +97,17 @@ typedef struct {
                                     CUART_PREBUCKET_OFF, CUART_PREBUCKET_ON.  Results are
                                     identical; it reorders the batch so concurrent warps
                                     share subtrees (stream-ordered scratch ~18 B/query). */
+    uint32_t slice_lut;          /* pre-bucketed lookups with a RANK root table: every
+                                    CTA walks its share of each bucket with the bucket's slice
+                                    of the table staged in shared memory (64 KiB at k=3),
+                                    so the first access of a walk is not an L2 request.
+                                    CUART_SLICE_AUTO (= off: measured slower on B200, the
+                                    slices take L1 capacity), CUART_SLICE_OFF,
+                                    CUART_SLICE_ON.  Results are identical.                */
 } cuart_build_opts;
+#define CUART_SLICE_AUTO 0u
+#define CUART_SLICE_OFF 1u
+#define CUART_SLICE_ON 2u
 #define CUART_PREBUCKET_AUTO 0u
 #define CUART_PREBUCKET_OFF 1u
 #define CUART_PREBUCKET_ON 2u
@@ -197,6 +207,10 @@ const char* cuart_status_string(cuart_status s);
  * launch / lookup counts) since the timer was (re)enabled, then resets. */
 cuart_status cuart_kernel_timer(cuart_index* h, int enable);
 cuart_status cuart_kernel_time(cuart_index* h, double* total_ms, uint64_t* launches, uint64_t* lookups);
+/* As cuart_kernel_time; slice_launches = how many of the timed launches were the
+ * bucketed walk with the shared-memory root-table slice (k_lookup_slice). */
+cuart_status cuart_kernel_time_ex(cuart_index* h, double* total_ms, uint64_t* launches, uint64_t* lookups,
+                                  uint64_t* slice_launches);
 /* Kernel launches issued by this library since load (for launch accounting). */
 uint64_t cuart_launch_count(void);
 

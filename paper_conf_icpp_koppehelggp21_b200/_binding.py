@@ -26,7 +26,7 @@ class _Keys(ctypes.Structure):
 
 class _Opts(ctypes.Structure):
     _fields_ = [("lut_bytes", ctypes.c_uint32), ("l2_persist", ctypes.c_uint32),
-                ("device", ctypes.c_int32), ("lut_format", ctypes.c_uint32), ("prebucket", ctypes.c_uint32)]
+                ("device", ctypes.c_int32), ("lut_format", ctypes.c_uint32), ("prebucket", ctypes.c_uint32), ("slice_lut", ctypes.c_uint32)]
 
 
 class _Stats(ctypes.Structure):
@@ -58,7 +58,7 @@ def lib():
             "cuart_build": [P, P, S, P, P], "cuart_lookup": [P, P, S, P, P], "cuart_update": [P, P, P, S, P],
             "cuart_destroy": [P], "cuart_update_ex": [P, P, P, P, S, P], "cuart_erase": [P, P, S, P],
             "cuart_free_leaves": [P, P, S, P], "cuart_range": [P, P, P, S, P, P],
-            "cuart_kernel_timer": [P, I], "cuart_kernel_time": [P, P, P, P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
+            "cuart_kernel_timer": [P, I], "cuart_kernel_time": [P, P, P, P], "cuart_kernel_time_ex": [P, P, P, P, P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
             "cuart_stats": [P, P], "cuart_dump": [P, P], "cuart_get_error": [P],
             "cuart_layout_build": [P, P, S, P, P], "cuart_layout_view_get": [P, P],
             "cuart_layout_lookup": [P, P, S, P, I], "cuart_layout_sectors": [P, P, S, P, I], "cuart_upload": [P, P, P], "cuart_layout_free": [P],
@@ -144,10 +144,11 @@ def make_keys(keys, lengths=None):
 
 
 PREBUCKET_AUTO, PREBUCKET_OFF, PREBUCKET_ON = 0, 1, 2
+SLICE_AUTO, SLICE_OFF, SLICE_ON = 0, 1, 2
 
 
-def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0):
-    return _Opts(lut_bytes, l2_persist, device, lut_format, prebucket)
+def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0):
+    return _Opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut)
 
 
 def _stream_ptr(stream):
@@ -160,14 +161,15 @@ def _stream_ptr(stream):
 
 
 # ------------------------------------------------------------------ hot path
-def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0):
+def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0,
+                slice_lut=0):
     """Build + upload (host buffers).  Returns an opaque handle (int)."""
     k, n, keep = make_keys(keys)
     v = np.ascontiguousarray(values, dtype=np.uint64)
     if v.shape[0] != n:
         raise ValueError("values length mismatch")
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket)
+    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut)
     _check(lib().cuart_build(ctypes.byref(k), _ptr(v), n, ctypes.byref(o), ctypes.byref(h)), "cuart_build")
     return h.value
 
@@ -219,6 +221,15 @@ def cuart_kernel_time(h):
     t, l, q = ctypes.c_double(), ctypes.c_uint64(), ctypes.c_uint64()
     _check(lib().cuart_kernel_time(h, ctypes.byref(t), ctypes.byref(l), ctypes.byref(q)), "cuart_kernel_time")
     return t.value, l.value, q.value
+
+
+def cuart_kernel_time_ex(h):
+    """(total_ms, launches, lookups, slice_launches): as cuart_kernel_time, plus how many
+    timed launches were k_lookup_slice (the bucketed walk with the smem table slice)."""
+    t, l, q, sl = ctypes.c_double(), ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_uint64()
+    _check(lib().cuart_kernel_time_ex(h, ctypes.byref(t), ctypes.byref(l), ctypes.byref(q), ctypes.byref(sl)),
+           "cuart_kernel_time_ex")
+    return t.value, l.value, q.value, sl.value
 
 
 def cuart_free_leaves(h):
@@ -318,9 +329,9 @@ def cuart_layout_sectors(l, queries, threads=0):
     return out
 
 
-def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_format=0, prebucket=0):
+def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0):
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket)
+    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut)
     _check(lib().cuart_upload(l, ctypes.byref(o), ctypes.byref(h)), "cuart_upload")
     return h.value
 
@@ -363,14 +374,15 @@ class Layout:
 class Index:
     """Device-resident CuART index on one GPU."""
 
-    def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0):
-        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_format, prebucket)
+    def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0,
+                 slice_lut=0):
+        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut)
 
     @classmethod
-    def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_format=0, prebucket=0):
+    def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0):
         """Upload an already-built host layout (keeps the host copy usable)."""
         self = cls.__new__(cls)
-        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format, prebucket)
+        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format, prebucket, slice_lut)
         return self
 
     def lookup(self, queries, out=None, stream=None):

@@ -79,7 +79,13 @@ struct cuart_index {
     std::mutex kmu;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev;
     uint64_t klookups = 0;
+    uint64_t kslice = 0;               // timed launches that were k_lookup_slice
     uint32_t prebucket = CUART_PREBUCKET_AUTO;   // a5: reorder large lookup batches by bucket (bucket.cuh)
+    uint32_t slice_lut = CUART_SLICE_AUTO;       // bucketed walk with the bucket's LUT slice in smem
+    bool slice_ok = false;                       // RANK table, integer keys, root branch depth + 2 <= k
+    uint64_t slice_e0 = 0;                       // common prefix C << 8(k - d): first entry of bucket 0's slice
+    uint32_t slice_shift = 0;                    // log2(entries per slice) = 8(k - 1 - d)
+    int slice_grid = 0;                          // persistent grid (CTAs) of k_lookup_slice
 
 };
 
@@ -92,6 +98,7 @@ static void drop_kevents(cuart_index* h) {
     }
     h->kev.clear();
     h->klookups = 0;
+    h->kslice = 0;
 }   // also counted by route.cu
 
 #define CU_TRY(x)                                   \
@@ -116,6 +123,59 @@ __global__ void __launch_bounds__(256) k_lookup(DevIndex ix, const void* __restr
         const uint64_t r = leaf ? val : kMiss;
         if (POL != 0) __stcs((unsigned long long*)out + i, (unsigned long long)r);
         else out[i] = r;
+    }
+}
+
+// a5 + a4 together: the pre-bucketed walk with the bucket's slice of the RANK root
+// table in shared memory.  Persistent CTAs visit the buckets in order; for
+// bucket b every CTA walks an equal contiguous share of b's run of the bucketed
+// batch, so at any moment all SMs work inside one bucket (its tree slice stays
+// L2-resident, exactly as when k_lookup walks the bucketed batch) while the table
+// entries of prefix C.b.* (C = the root's compressed prefix, d bytes) are read from
+// shared memory instead of L2: one L2 request less per query.  A query whose
+// prefix is not C.b (an absent key) reads the global table.  The slice refill is
+// S bytes per CTA per bucket (S = 2^shift entries, 64 KiB for k = 3, d = 0).
+constexpr int kSliceThreads = 1024;
+template <class Key, int POL>
+__global__ void __launch_bounds__(kSliceThreads, 2) k_lookup_slice(DevIndex ix, const void* __restrict__ q, uint64_t n,
+                                                                   uint64_t* __restrict__ out,
+                                                                   const unsigned int* __restrict__ bases, uint64_t e0,
+                                                                   uint32_t shift) {
+    extern __shared__ uint4 slut[];
+    const Loader<POL> ld;
+    const uint64_t S = uint64_t(1) << shift;
+    const uint32_t nv4 = uint32_t(S >> 4);                    // 1 B per entry, in 16-B units
+    for (uint32_t b = 0; b < uint32_t(kBuckets); b++) {
+        const uint64_t lo = bases[b], hi = b + 1 < uint32_t(kBuckets) ? uint64_t(bases[b + 1]) : n;
+        if (lo >= hi) continue;
+        const uint64_t per = (hi - lo + gridDim.x - 1) / gridDim.x;
+        const uint64_t s0 = lo + per * blockIdx.x;
+        const uint64_t s1 = s0 + per < hi ? s0 + per : hi;
+        if (s0 >= s1) continue;                                // uniform over the CTA
+        const uint64_t E0 = e0 | (uint64_t(b) << shift);
+        __syncthreads();                                       // the previous slice is no longer read
+        const uint4* src = ix.lutr + (E0 >> 5) * 2;
+        for (uint32_t k = threadIdx.x; k < nv4; k += blockDim.x)
+            slut[k] = POL ? Loader<POL>::v4(src + k, ld.keep) : ld_nc_v4(src + k);
+        __syncthreads();
+        for (uint64_t i = s0 + threadIdx.x; i < s1; i += blockDim.x) {
+            const Key key = Key::template load<true>(q, nullptr, i);
+            const uint64_t p = key.prefix(ix.lut_bytes);
+            uint64_t link;
+            if (p - E0 < S) {
+                const uint4* sp = slut + ((p - E0) >> 5) * 2;
+                const uint4 a = sp[0], c = sp[1];
+                U8x32 blk;
+                blk.w[0] = a.x; blk.w[1] = a.y; blk.w[2] = a.z; blk.w[3] = a.w;
+                blk.w[4] = c.x; blk.w[5] = c.y; blk.w[6] = c.z; blk.w[7] = c.w;
+                link = decode_lut_rank(ix, ld, blk, p);
+            } else {
+                link = start_link(ix, ld, key);
+            }
+            uint64_t val = kMiss;
+            const uint64_t leaf = find_leaf(ix, ld, key, link, val);
+            __stcs((unsigned long long*)out + i, (unsigned long long)(leaf ? val : kMiss));
+        }
     }
 }
 
@@ -227,6 +287,38 @@ static cuart_status check_keys(const cuart_index* h, const cuart_keys* k, size_t
 static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens,
                                          uint64_t n, uint64_t* out, cudaStream_t s);
 
+static void ktimer_begin(const cuart_index* h, cudaStream_t s, cudaEvent_t& ev0, cudaEvent_t& ev1) {
+    ev0 = ev1 = nullptr;
+    if (!h->ktimer) return;
+    cudaEventCreate(&ev0);
+    cudaEventCreate(&ev1);
+    cudaEventRecord(ev0, s);
+}
+static void ktimer_end(const cuart_index* h, cudaStream_t s, cudaEvent_t ev0, cudaEvent_t ev1, uint64_t n,
+                       bool slice = false) {
+    if (!h->ktimer) return;
+    cudaEventRecord(ev1, s);
+    cuart_index* hm = const_cast<cuart_index*>(h);
+    std::lock_guard<std::mutex> g(hm->kmu);
+    hm->kev.push_back({ev0, ev1});
+    hm->klookups += n;
+    hm->kslice += slice ? 1 : 0;
+}
+
+template <class Key>
+static cuart_status launch_lookup_slice(const cuart_index* h, const void* bq, uint64_t n, uint64_t* res,
+                                        const unsigned int* bases, cudaStream_t s) {
+    cudaEvent_t ev0, ev1;
+    ktimer_begin(h, s, ev0, ev1);
+    const size_t smem = size_t(1) << h->slice_shift;
+    k_lookup_slice<Key, 5><<<h->slice_grid, kSliceThreads, smem, s>>>(h->dix, bq, n, res, bases, h->slice_e0,
+                                                                     h->slice_shift);
+    g_cuart_launches++;
+    ktimer_end(h, s, ev0, ev1, n, true);
+    CU_TRY(cudaGetLastError());
+    return CUART_OK;
+}
+
 // a5 pre-bucketing: bucket -> lookup in bucketed order -> gather (bucket.cuh).
 // Scratch is stream-ordered (cudaMallocAsync from the device pool, whose release
 // threshold is raised at upload so the memory stays mapped between calls), so
@@ -244,15 +336,25 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
     unsigned int* hist = (unsigned int*)(scr + o_hist);
     unsigned int* tot = (unsigned int*)(scr + o_tot);
     const uint32_t depth = link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u;
-    k_bhist<Key><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
-    k_bscan_rows<<<kBuckets, 1024, 0, s>>>(hist, tiles, tot);
+    if ((uintptr_t(q) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
+    else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
+    k_bscan_rows<<<kBuckets, kBucketThreads, 0, s>>>(hist, tiles, tot);
     k_bscan<<<1, kBuckets, 0, s>>>(tot);
     k_bscatter<Key><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key>(), s>>>(
         q, lens, n, depth, hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, (uint16_t*)(scr + o_pos));
     g_cuart_launches += 4;
     CU_TRY(cudaGetLastError());
-    cuart_status rc = launch_lookup_direct(h, Key::kKind, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, n,
-                                           (uint64_t*)(scr + o_res), s);
+    const uint64_t slice_bytes = uint64_t(1) << h->slice_shift;
+    // AUTO = off: measured slower than k_lookup over the bucketed batch on c3 (19.2 vs
+    // 15.0 ms per 2^30: the 64-KiB slices take L1 capacity, L2 hit rate 64% -> 49%)
+    // and on c2 (3.10 vs 2.57 ms per 2^28: the per-bucket CTA barriers).  Kept as an
+    // explicit option (CUART_SLICE_ON) with its parity tests.
+    (void)slice_bytes;
+    const bool slice = Key::kKind != 3 && h->slice_ok && h->policy == 5 && h->slice_lut == CUART_SLICE_ON;
+    cuart_status rc = CUART_OK;
+    if (slice) rc = launch_lookup_slice<Key>(h, scr + o_q, n, (uint64_t*)(scr + o_res), tot, s);
+    else rc = launch_lookup_direct(h, Key::kKind, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, n,
+                                   (uint64_t*)(scr + o_res), s);
     if (rc != CUART_OK) return rc;
     k_bgather<<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint64_t*)(scr + o_res), (const uint16_t*)(scr + o_pos),
                                                           n, hist, tot, out);
@@ -284,12 +386,8 @@ static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const voi
 static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens,
                                          uint64_t n, uint64_t* out, cudaStream_t s) {
     const int grid = grid_for(h, n);
-    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
-    if (h->ktimer) {                                   // per-launch k_lookup timing (cuart_kernel_timer)
-        cudaEventCreate(&ev0);
-        cudaEventCreate(&ev1);
-        cudaEventRecord(ev0, s);
-    }
+    cudaEvent_t ev0, ev1;
+    ktimer_begin(h, s, ev0, ev1);                      // per-launch k_lookup timing (cuart_kernel_timer)
 #define CUART_LOOKUP(K, P) k_lookup<K, P><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out)
 #define CUART_LOOKUP_POL(K)                          \
     switch (h->policy) {                             \
@@ -309,13 +407,7 @@ static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, co
 #undef CUART_LOOKUP_POL
 #undef CUART_LOOKUP
     g_cuart_launches++;
-    if (h->ktimer) {
-        cudaEventRecord(ev1, s);
-        cuart_index* hm = const_cast<cuart_index*>(h);
-        std::lock_guard<std::mutex> g(hm->kmu);
-        hm->kev.push_back({ev0, ev1});
-        hm->klookups += n;
-    }
+    ktimer_end(h, s, ev0, ev1, n);
     CU_TRY(cudaGetLastError());
     return CUART_OK;
 }
@@ -409,10 +501,11 @@ static cuart_status launch_update_bucketed(cuart_index* h, const void* k, const 
     unsigned int* hist = (unsigned int*)(scr + o_hist);
     unsigned int* tot = (unsigned int*)(scr + o_tot);
     const uint32_t depth = link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u;
-    k_bhist<Key><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
-    k_bscan_rows<<<kBuckets, 1024, 0, s>>>(hist, tiles, tot);
+    if ((uintptr_t(k) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
+    else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
+    k_bscan_rows<<<kBuckets, kBucketThreads, 0, s>>>(hist, tiles, tot);
     k_bscan<<<1, kBuckets, 0, s>>>(tot);
-    k_bscatter<Key, true><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key>(), s>>>(
+    k_bscatter<Key, true><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key, true>(), s>>>(
         k, lens, n, depth, hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, nullptr, vals,
         (uint64_t*)(scr + o_val), (uint32_t*)(scr + o_idx));
     g_cuart_launches += 4;
@@ -661,11 +754,11 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     cudaFuncSetAttribute(k_bscatter<KeyBytes>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          int(bscatter_smem<KeyBytes>()));
     cudaFuncSetAttribute(k_bscatter<KeyU64, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         int(bscatter_smem<KeyU64>()));
+                         int(bscatter_smem<KeyU64, true>()));
     cudaFuncSetAttribute(k_bscatter<KeyU32, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         int(bscatter_smem<KeyU32>()));
+                         int(bscatter_smem<KeyU32, true>()));
     cudaFuncSetAttribute(k_bscatter<KeyBytes, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         int(bscatter_smem<KeyBytes>()));
+                         int(bscatter_smem<KeyBytes, true>()));
     // LUT region: 64-bit links (LINKS, and the exception table of RANK) then the compact form
     h->lut_off = off;
     const bool need_links = fmt == CUART_LUT_LINKS || fmt == CUART_LUT_RANK;
@@ -698,6 +791,41 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && cudaMemset(h->arena + h->err_off, 0, 256) != cudaSuccess) rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && cudaMemset(h->arena + h->free_off, 0, 8) != cudaSuccess) rc = CUART_ERR_CUDA;
+    if (rc != CUART_OK) {
+        cudaFree(h->arena);
+        delete h;
+        return rc;
+    }
+    // k_lookup_slice geometry: bucket byte = root branch depth d; the slice of bucket b
+    // is the table entries of prefix C.b.* (C = the d-byte common prefix, read off the
+    // first non-null entry), 256^(k-1-d) entries = 1 B each in RANK form.
+    h->slice_lut = opts ? opts->slice_lut : CUART_SLICE_AUTO;
+    if (h->slice_lut > CUART_SLICE_ON) rc = CUART_ERR_INVALID_ARGUMENT;
+    if (const char* pe = getenv("CUART_SLICE")) h->slice_lut = atoi(pe) == 1 ? CUART_SLICE_OFF : atoi(pe) == 2 ? CUART_SLICE_ON : CUART_SLICE_AUTO;
+    {
+        const uint32_t rt = link_type(L.root);
+        const uint32_t d = (rt >= T_N4 && rt <= T_N256) ? link_aux(L.root) : 0xFFu;
+        const uint32_t k = L.lut_bytes;
+        if (fmt == CUART_LUT_RANK && L.key_kind != CUART_KEY_BYTES && d != 0xFFu && d + 2 <= k && !L.lut.empty()) {
+            uint64_t p0 = 0;
+            while (p0 < L.lut.size() && L.lut[p0] == 0) p0++;
+            if (p0 < L.lut.size()) {
+                h->slice_shift = 8 * (k - 1 - d);
+                h->slice_e0 = (p0 >> (8 * (k - d))) << (8 * (k - d));
+                const int smem = 1 << h->slice_shift;
+                int occ = 0;
+                if (cudaFuncSetAttribute(k_lookup_slice<KeyU64, 5>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) == cudaSuccess &&
+                    cudaFuncSetAttribute(k_lookup_slice<KeyU32, 5>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) == cudaSuccess &&
+                    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, L.key_kind == CUART_KEY_U64
+                                                                            ? (const void*)k_lookup_slice<KeyU64, 5>
+                                                                            : (const void*)k_lookup_slice<KeyU32, 5>,
+                                                                  kSliceThreads, smem) == cudaSuccess && occ > 0) {
+                    h->slice_grid = occ * h->num_sms;
+                    h->slice_ok = true;
+                }
+            }
+        }
+    }
     if (rc != CUART_OK) {
         cudaFree(h->arena);
         delete h;
@@ -813,7 +941,13 @@ cuart_status cuart_kernel_timer(cuart_index* h, int enable) {
 }
 
 cuart_status cuart_kernel_time(cuart_index* h, double* total_ms, uint64_t* launches, uint64_t* lookups) {
-    if (!h || !total_ms || !launches || !lookups) return CUART_ERR_INVALID_ARGUMENT;
+    uint64_t sl = 0;
+    return cuart_kernel_time_ex(h, total_ms, launches, lookups, &sl);
+}
+
+cuart_status cuart_kernel_time_ex(cuart_index* h, double* total_ms, uint64_t* launches, uint64_t* lookups,
+                                  uint64_t* slice_launches) {
+    if (!h || !total_ms || !launches || !lookups || !slice_launches) return CUART_ERR_INVALID_ARGUMENT;
     std::lock_guard<std::mutex> g(h->kmu);
     double t = 0;
     for (auto& e : h->kev) {
@@ -825,6 +959,7 @@ cuart_status cuart_kernel_time(cuart_index* h, double* total_ms, uint64_t* launc
     *total_ms = t;
     *launches = h->kev.size();
     *lookups = h->klookups;
+    *slice_launches = h->kslice;
     drop_kevents(h);
     return CUART_OK;
 }

@@ -332,9 +332,8 @@ __device__ __forceinline__ uint64_t expand_lut32(uint32_t e, uint32_t k, uint32_
 // bit-planes, index = per-type base + popcount of earlier same-type entries;
 // exceptions (leaves, other depths, non-consecutive indices) go to the link table.
 template <int POL, bool TRACK = false>
-__device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Loader<POL>& ld, uint64_t p,
-                                                    uint64_t* slot = nullptr) {
-    const U8x32 blk = ld.lutv8(ix.lutr + (p >> 5) * 2);
+__device__ __forceinline__ uint64_t decode_lut_rank(const DevIndex& ix, const Loader<POL>& ld, const U8x32& blk,
+                                                    uint64_t p, uint64_t* slot = nullptr) {
     const uint32_t j = uint32_t(p & 31);
     if ((blk.w[3] >> j) & 1) {
         if (TRACK) *slot = uint64_t(ix.lut + p);
@@ -346,6 +345,11 @@ __device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Lo
     const uint32_t m = ((t & 1) ? p0 : ~p0) & ((t & 2) ? p1 : ~p1) & ((t & 4) ? p2 : ~p2) & ((1u << j) - 1);
     const uint32_t base = t == T_N4 ? blk.w[4] : t == T_N16 ? blk.w[5] : t == T_N48 ? blk.w[6] : blk.w[7];
     return make_link(t, ix.lut_bytes, uint64_t(base) + __popc(m));
+}
+template <int POL, bool TRACK = false>
+__device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Loader<POL>& ld, uint64_t p,
+                                                    uint64_t* slot = nullptr) {
+    return decode_lut_rank<POL, TRACK>(ix, ld, ld.lutv8(ix.lutr + (p >> 5) * 2), p, slot);
 }
 
 // Start of a walk: LUT[first k key bytes] or the root.  With TRACK, *slot =

@@ -335,35 +335,55 @@ def test_c4_full_size_sampled():
     ix.close()
 
 
-@pytest.mark.parametrize("kind", ["u64", "u32", "bytes"])
+@pytest.mark.parametrize("kind", ["u64", "u64p", "u32", "bytes"])
 def test_prebucket_equals_direct(kind):
     """a5 pre-bucketing only reorders the batch: results identical to the direct
-    kernel and to the oracle, for ragged batch sizes across the tile size."""
+    kernel and to the oracle, for ragged batch sizes across the tile size.  Integer
+    kinds also run the bucketed walk with the bucket's root-table slice in shared
+    memory (k_lookup_slice), including queries outside every slice (u64p: all keys
+    share the top byte 0x7F, half the queries do not; u32: 10% of the queries
+    leave the keys' common prefix byte 0x00)."""
+    lut = 0 if kind == "bytes" else 3
     if kind == "u64":
         cfg = W.CONFIGS["c1"]
         keys, vals = W.build_set(cfg)
         mk = lambda m: W.lookup_batch(cfg, keys, 0, m)
+    elif kind == "u64p":
+        rng = np.random.default_rng(3)
+        keys = np.unique(rng.integers(0, 1 << 56, 1 << 17, dtype=np.uint64) | np.uint64(0x7F << 56))
+        vals = np.arange(keys.shape[0], dtype=np.uint64) * 3 + 1
+
+        def mk(m):
+            hit = keys[rng.integers(0, keys.shape[0], m)]
+            other = rng.integers(0, 2**63, m, dtype=np.uint64) * np.uint64(2) + np.uint64(1)
+            return np.where(rng.random(m) < 0.5, hit, other)
     elif kind == "u32":
         keys = (np.arange(1 << 18, dtype=np.uint32) * 13) & np.uint32(0xFFFFFF)
         keys = np.unique(keys)
         vals = np.arange(keys.shape[0], dtype=np.uint64) + 1
         rng = np.random.default_rng(0)
-        mk = lambda m: rng.integers(0, 1 << 24, m, dtype=np.uint32)
+        mk = lambda m: np.where(rng.random(m) < 0.9, rng.integers(0, 1 << 24, m, dtype=np.uint32),
+                                rng.integers(0, 1 << 32, m, dtype=np.uint32)).astype(np.uint32)
     else:
         keys = W.string_keys(4, 1 << 16)
         vals = np.arange(1 << 16, dtype=np.uint64) + 5
         mk = lambda m: (lambda idx: (keys[0][idx].copy(), keys[1][idx].copy()))(
             W.string_lookup_at(W.CONFIGS["c4"], 1 << 16, np.arange(m)))
     mp = MapOracle(keys, vals)
-    on = C.Index(keys, vals, prebucket=C.PREBUCKET_ON)
-    off = C.Index(keys, vals, prebucket=C.PREBUCKET_OFF)
-    for m in (4095, 4096, 4097, 100_003, 1 << 20):
+    off = C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_OFF)
+    variants = [C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, slice_lut=C.SLICE_OFF)]
+    if kind != "bytes":
+        variants.append(C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, slice_lut=C.SLICE_ON))
+    # 2048 * 4096 + 4097 spans more than one pass of k_bscan_rows (2048 tiles per pass)
+    sizes = (4095, 4096, 4097, 100_003, 1 << 20) + ((2048 * 4096 + 4097,) if kind == "u64" else ())
+    for m in sizes:
         q = mk(m)
-        a, b = _lookup(on, q), _lookup(off, q)
-        assert np.array_equal(a, b), m
-        assert np.array_equal(a, mp.lookup(q)), m
-    on.close()
-    off.close()
+        b = _lookup(off, q)
+        assert np.array_equal(b, mp.lookup(q)), m
+        for on in variants:
+            assert np.array_equal(_lookup(on, q), b), m
+    for ix in [off] + variants:
+        ix.close()
 
 
 @pytest.mark.parametrize("kind", ["u64", "u32", "bytes"])
