@@ -58,6 +58,9 @@ def _args():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--e2e-steps", type=int, default=2)
     p.add_argument("--mode", default="range", choices=["range", "replica"], help="multi-GPU mode (N > 1)")
+    p.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
+                   help="range mode exchange: p2p = fused push/return over peer memory (CUDA IPC, NVLink), "
+                        "nccl = route + all-to-all")
     p.add_argument("--traffic", type=float, default=None,
                    help="ncu dram__bytes_read+write per k_lookup launch (GB), from profiles/, echoed into roofline")
     return p.parse_args()
@@ -246,7 +249,8 @@ def run_c5(args, world, rank, local, dev):
     keys, vals, sp = c5_local_keys(world, rank, dev)
     if world == 1 and not dist.is_initialized():
         dist.init_process_group("gloo", store=dist.HashStore(), rank=0, world_size=1)
-    di = DistIndex(keys, vals, mode="range", ops=CudaOps(dev), lut_bytes=args.lut, splitters=sp, local=True)
+    di = DistIndex(keys, vals, mode="range", ops=CudaOps(dev), lut_bytes=args.lut, splitters=sp, local=True,
+                   transport=args.transport)
     build_s = time.perf_counter() - t0
     stats = di.index.stats()
     R, per = W.C5_ROUND, W.C5_ROUND // world
@@ -300,6 +304,7 @@ def run_c5(args, world, rank, local, dev):
             "data": "synthetic (seeded splitmix64, SURVEY §8(d) c5 recipe)",
             "config": {"workload": f"c5: {W.C5.description}", "keys": W.C5.n_keys, "round_ops": R,
                        "ops_per_rank_per_step": per, "update_fraction": W.C5_UPDATE_P, "mode": "range",
+                       "transport": args.transport if world > 1 else None,
                        "parallelism": f"range{world}", "local_keys_rank0": int(keys.shape[0]),
                        "build_s": round(build_s, 2), "lut_format": stats["lut_format"]},
             "roofline": {"bound": "hbm", "kernel": "k_lookup<KeyU64>", "kernel_ms": round(kern_ms, 4),
@@ -346,7 +351,7 @@ def main():
         ix = C.Index.from_layout(layout, device=local)
         di = None
     else:
-        di = DistIndex(keys, vals, mode=mode, ops=ops, lut_bytes=args.lut)
+        di = DistIndex(keys, vals, mode=mode, ops=ops, lut_bytes=args.lut, transport=args.transport)
         ix = di.index
         layout = None
     build_s = time.perf_counter() - t0
@@ -545,6 +550,7 @@ def main():
             "config": {"workload": f"{args.config}: {cfg.description}", "keys": cfg.n_keys,
                        "lookups_per_rank": nl, "updates_per_rank": nu, "key_kind": cfg.kind,
                        "lut_bytes": args.lut, "lut_format": stats["lut_format"], "mode": mode,
+                       "transport": args.transport if world > 1 and mode == "range" else None,
                        "parallelism": f"{mode}{world}" if world > 1 else "single",
                        "l2": f"inputs ({q_bytes / 2**30:.1f} GiB of queries per step) larger than L2; no flush",
                        "measured_hit_ratio": round(hit, 4), "build_s": round(build_s, 2)},

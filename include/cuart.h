@@ -263,6 +263,49 @@ cuart_status cuart_partition_by_flag(const cuart_keys* keys, size_t n, const uin
                                      void* out_keys, uint8_t* out_lengths, uint64_t* out_values, uint32_t* perm,
                                      uint64_t* counts, void* scratch, void* stream);
 
+/* ---- fused multi-GPU exchange over peer memory (transport "p2p", §8(e)) ----
+ * One process per GPU of one box.  Every rank allocates receive windows with
+ * cuart_ipc_alloc, exports them (cuart_ipc_export -> an opaque handle of
+ * CUART_IPC_HANDLE_BYTES bytes, sent to the peers by the caller's collective
+ * library), and maps the peers' windows with cuart_ipc_import (CUDA IPC; peer
+ * access over NVLink/NVSwitch is enabled lazily).  A routed batch then needs no
+ * all-to-all of the data:
+ *   1. cuart_route_count: owner of every op + per-owner counts (device uint64_t
+ *      [nparts]); the P x P count matrix is all-gathered by the caller;
+ *   2. cuart_route_push: the stable per-owner scatter of cuart_route whose stores
+ *      go straight to the owners' windows: op i with owner o lands at
+ *      dst_keys[o][its position in this source's run for o] (and likewise
+ *      dst_lengths / dst_values); dst_*[o] is owner o's window advanced to the
+ *      first slot of this source (sum of the counts of the sources before it), so
+ *      every owner sees the runs of all sources concatenated in rank order (the
+ *      global op order of the update rule, reading C7).  perm[i] = slot of
+ *      op i in this source's owner-major send order (for cuart_unroute);
+ *   3. (all ranks synchronised) the owner serves its window with
+ *      cuart_lookup_segmented, whose last kernel stores result j of source s
+ *      straight into s's result window: seg_dst[s] + (j - seg_start[s]);
+ *   4. (synchronised) each source restores query order with cuart_unroute.
+ * scratch of steps 1-2: cuart_route_scratch_bytes(n, nparts), kept between the
+ * two calls.  nparts <= 16.  All pointers are device pointers (local or mapped
+ * peer memory); calls are async on `stream`. */
+#define CUART_IPC_HANDLE_BYTES 64
+cuart_status cuart_ipc_alloc(size_t bytes, void** dptr);           /* exportable device window        */
+cuart_status cuart_ipc_free(void* dptr);                           /* NULL ok                         */
+cuart_status cuart_ipc_export(void* dptr, void* handle);           /* handle: CUART_IPC_HANDLE_BYTES  */
+cuart_status cuart_ipc_import(const void* handle, void** dptr);    /* another process's window        */
+cuart_status cuart_ipc_close(void* dptr);                          /* unmap an imported window        */
+cuart_status cuart_route_count(const cuart_keys* keys, size_t n, const uint64_t* splitters, uint32_t nparts,
+                               uint64_t* counts, void* scratch, void* stream);
+cuart_status cuart_route_push(const cuart_keys* keys, size_t n, uint32_t nparts, const uint64_t* values,
+                              void* const* dst_keys, uint8_t* const* dst_lengths, uint64_t* const* dst_values,
+                              uint32_t* perm, void* scratch, void* stream);
+/* cuart_lookup whose result i is stored at seg_dst[s] + (i - seg_start[s]) for the
+ * segment s with seg_start[s] <= i < seg_start[s+1] (host arrays: seg_start
+ * [nseg+1] with seg_start[0] = 0 and seg_start[nseg] = n, seg_dst[nseg] device
+ * pointers, local or mapped peer memory); nseg in [1, 16].  The stores are done by
+ * the kernel that produces the results (fused return, Fig. 3 per query). */
+cuart_status cuart_lookup_segmented(const cuart_index* h, const cuart_keys* queries, size_t n, uint32_t nseg,
+                                    const uint64_t* seg_start, uint64_t* const* seg_dst, void* stream);
+
 #ifdef __cplusplus
 }
 #endif

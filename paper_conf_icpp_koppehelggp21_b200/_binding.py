@@ -77,6 +77,15 @@ def lib():
         L.cuart_partition_by_flag.restype = ctypes.c_int
         L.cuart_unroute.argtypes = [P, P, S, P, P]
         L.cuart_unroute.restype = ctypes.c_int
+        U32 = ctypes.c_uint32
+        for name, args in {"cuart_ipc_alloc": [S, P], "cuart_ipc_free": [P], "cuart_ipc_export": [P, P],
+                           "cuart_ipc_import": [P, P], "cuart_ipc_close": [P],
+                           "cuart_route_count": [P, S, P, U32, P, P, P],
+                           "cuart_route_push": [P, S, U32, P, P, P, P, P, P, P],
+                           "cuart_lookup_segmented": [P, P, S, U32, P, P, P]}.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = ctypes.c_int
         L.cuart_launch_count.argtypes = []
         L.cuart_launch_count.restype = ctypes.c_uint64
         _lib = L
@@ -442,3 +451,67 @@ class Index:
             self.close()
         except Exception:
             pass
+
+
+# ------------------------------------------------------------------ fused multi-GPU exchange (p2p)
+IPC_HANDLE_BYTES = 64
+
+
+def raw_keys(kind, data_ptr, lens_ptr=None):
+    """cuart_keys over raw device pointers (windows allocated by cuart_ipc_alloc)."""
+    return _Keys(kind, data_ptr, lens_ptr if kind == KIND_BYTES else None)
+
+
+def ipc_alloc(nbytes):
+    p = ctypes.c_void_p()
+    _check(lib().cuart_ipc_alloc(max(1, int(nbytes)), ctypes.byref(p)), "cuart_ipc_alloc")
+    return p.value
+
+
+def ipc_free(ptr):
+    _check(lib().cuart_ipc_free(ptr), "cuart_ipc_free")
+
+
+def ipc_export(ptr):
+    buf = ctypes.create_string_buffer(IPC_HANDLE_BYTES)
+    _check(lib().cuart_ipc_export(ptr, buf), "cuart_ipc_export")
+    return buf.raw
+
+
+def ipc_import(handle):
+    buf = ctypes.create_string_buffer(bytes(handle), IPC_HANDLE_BYTES)
+    p = ctypes.c_void_p()
+    _check(lib().cuart_ipc_import(buf, ctypes.byref(p)), "cuart_ipc_import")
+    return p.value
+
+
+def ipc_close(ptr):
+    _check(lib().cuart_ipc_close(ptr), "cuart_ipc_close")
+
+
+def route_count(keys_struct, n, splitters_ptr, nparts, counts_ptr, scratch_ptr, stream=None):
+    _check(lib().cuart_route_count(ctypes.byref(keys_struct), n, splitters_ptr, nparts, counts_ptr, scratch_ptr,
+                                   _stream_ptr(stream)), "cuart_route_count")
+
+
+def route_push(keys_struct, n, nparts, values_ptr, dst_keys, dst_lens, dst_vals, perm_ptr, scratch_ptr, stream=None):
+    """dst_* : lists of nparts device addresses (ints) or None."""
+    arr = lambda xs: (ctypes.c_void_p * nparts)(*xs) if xs is not None else None
+    _check(lib().cuart_route_push(ctypes.byref(keys_struct), n, nparts, values_ptr, arr(dst_keys), arr(dst_lens),
+                                  arr(dst_vals), perm_ptr, scratch_ptr, _stream_ptr(stream)), "cuart_route_push")
+
+
+def lookup_segmented(h, keys_struct, n, seg_start, seg_dst, stream=None):
+    nseg = len(seg_dst)
+    st = (ctypes.c_uint64 * (nseg + 1))(*[int(x) for x in seg_start])
+    ds = (ctypes.c_void_p * nseg)(*seg_dst)
+    _check(lib().cuart_lookup_segmented(h, ctypes.byref(keys_struct), n, nseg, st, ds, _stream_ptr(stream)),
+           "cuart_lookup_segmented")
+
+
+def update_raw(h, keys_struct, n, values_ptr, stream=None):
+    _check(lib().cuart_update(h, ctypes.byref(keys_struct), values_ptr, n, _stream_ptr(stream)), "cuart_update")
+
+
+def unroute_raw(in_ptr, perm_ptr, n, out_ptr, stream=None):
+    _check(lib().cuart_unroute(in_ptr, perm_ptr, n, out_ptr, _stream_ptr(stream)), "cuart_unroute")

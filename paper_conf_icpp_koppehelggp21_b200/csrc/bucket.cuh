@@ -333,11 +333,13 @@ __device__ __forceinline__ void cp_async_wait_all() {
 // shared memory with cp.async (no registers held across the DRAM round trip: 3.77
 // ms per 2^30 against 4.19 ms with register staging, tools/bucket_micro.cu), then
 // out[i] = smem[jpos[i]] (coalesced).
+// SEG: out is ignored and result i goes to so.at(i) (fused return to the requesting GPUs).
+template <bool SEG = false>
 __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __restrict__ res,
                                                             const uint16_t* __restrict__ jpos, uint64_t n,
                                                             const unsigned int* __restrict__ rowoff,
                                                             const unsigned int* __restrict__ bases,
-                                                            uint64_t* __restrict__ out) {
+                                                            uint64_t* __restrict__ out, SegOut so = SegOut{}) {
     __shared__ uint64_t sres[kBucketTile];
     __shared__ uint8_t bof[kBucketTile];                               // bucket of each staged position
     __shared__ unsigned int loc[kBuckets];
@@ -376,7 +378,10 @@ __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __re
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
         const uint32_t k = uint32_t(r) * kBucketThreads + threadIdx.x;
-        if (k < cnt) __stcs((unsigned long long*)out + base + k, (unsigned long long)sres[jp[r]]);
+        if (k < cnt) {
+            unsigned long long* dst = SEG ? (unsigned long long*)so.at(base + k) : (unsigned long long*)out + base + k;
+            __stcs(dst, (unsigned long long)sres[jp[r]]);
+        }
     }
 }
 

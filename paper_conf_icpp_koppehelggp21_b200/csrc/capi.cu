@@ -110,10 +110,11 @@ static void drop_kevents(cuart_index* h) {
     } while (0)
 
 // ============================================================================ kernels
-template <class Key, int POL>
+// SEG: out is ignored, result i goes to so.at(i) (fused multi-GPU return, §8(e)).
+template <class Key, int POL, bool SEG = false>
 __global__ void __launch_bounds__(256) k_lookup(DevIndex ix, const void* __restrict__ q,
                                                 const uint8_t* __restrict__ lens, uint64_t n,
-                                                uint64_t* __restrict__ out) {
+                                                uint64_t* __restrict__ out, SegOut so = SegOut{}) {
     const Loader<POL> ld;
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
@@ -121,8 +122,9 @@ __global__ void __launch_bounds__(256) k_lookup(DevIndex ix, const void* __restr
         uint64_t val = kMiss;
         const uint64_t leaf = find_leaf(ix, ld, key, start_link(ix, ld, key), val);
         const uint64_t r = leaf ? val : kMiss;
-        if (POL != 0) __stcs((unsigned long long*)out + i, (unsigned long long)r);
-        else out[i] = r;
+        uint64_t* dst = SEG ? so.at(i) : out + i;
+        if (POL != 0) __stcs((unsigned long long*)dst, (unsigned long long)r);
+        else *dst = r;
     }
 }
 
@@ -285,7 +287,7 @@ static cuart_status check_keys(const cuart_index* h, const cuart_keys* k, size_t
 }
 
 static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens,
-                                         uint64_t n, uint64_t* out, cudaStream_t s);
+                                         uint64_t n, uint64_t* out, cudaStream_t s, const SegOut* so = nullptr);
 
 static void ktimer_begin(const cuart_index* h, cudaStream_t s, cudaEvent_t& ev0, cudaEvent_t& ev1) {
     ev0 = ev1 = nullptr;
@@ -325,7 +327,7 @@ static cuart_status launch_lookup_slice(const cuart_index* h, const void* bq, ui
 // concurrent lookups on several streams stay independent.
 template <class Key>
 static cuart_status launch_bucketed(const cuart_index* h, const void* q, const uint8_t* lens, uint64_t n, uint64_t* out,
-                                    cudaStream_t s) {
+                                    cudaStream_t s, const SegOut* so = nullptr) {
     const size_t ks = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
     auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
     const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
@@ -356,8 +358,11 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
     else rc = launch_lookup_direct(h, Key::kKind, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, n,
                                    (uint64_t*)(scr + o_res), s);
     if (rc != CUART_OK) return rc;
-    k_bgather<<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint64_t*)(scr + o_res), (const uint16_t*)(scr + o_pos),
-                                                          n, hist, tot, out);
+    if (so) k_bgather<true><<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint64_t*)(scr + o_res),
+                                                                        (const uint16_t*)(scr + o_pos), n, hist, tot,
+                                                                        nullptr, *so);
+    else k_bgather<false><<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint64_t*)(scr + o_res),
+                                                                      (const uint16_t*)(scr + o_pos), n, hist, tot, out);
     g_cuart_launches++;
     CU_TRY(cudaGetLastError());
     CU_TRY(cudaFreeAsync(scr, s));
@@ -367,7 +372,7 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
 static constexpr uint64_t kBucketMin = uint64_t(1) << 22;   // below this the batch is too small to reorder
 
 static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens, uint64_t n,
-                                  uint64_t* out, cudaStream_t s) {
+                                  uint64_t* out, cudaStream_t s, const SegOut* so = nullptr) {
     if (n == 0) return CUART_OK;
     // AUTO: integer keys only — for byte strings (c4, Zipf) the 33-B key copies cost
     // more than the locality gains (measured 9.0 vs 10.6 G lookups/s).
@@ -375,17 +380,27 @@ static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const voi
                       : h->prebucket == CUART_PREBUCKET_AUTO && n >= kBucketMin && kind != CUART_KEY_BYTES;
     if (bucket && n < (uint64_t(1) << 32)) {
         switch (kind) {
-        case CUART_KEY_U64: return launch_bucketed<KeyU64>(h, q, lens, n, out, s);
-        case CUART_KEY_U32: return launch_bucketed<KeyU32>(h, q, lens, n, out, s);
-        default: return launch_bucketed<KeyBytes>(h, q, lens, n, out, s);
+        case CUART_KEY_U64: return launch_bucketed<KeyU64>(h, q, lens, n, out, s, so);
+        case CUART_KEY_U32: return launch_bucketed<KeyU32>(h, q, lens, n, out, s, so);
+        default: return launch_bucketed<KeyBytes>(h, q, lens, n, out, s, so);
         }
     }
-    return launch_lookup_direct(h, kind, q, lens, n, out, s);
+    return launch_lookup_direct(h, kind, q, lens, n, out, s, so);
 }
 
 static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens,
-                                         uint64_t n, uint64_t* out, cudaStream_t s) {
+                                         uint64_t n, uint64_t* out, cudaStream_t s, const SegOut* so) {
     const int grid = grid_for(h, n);
+    if (so) {                                          // fused return: the default policy only
+        switch (kind) {
+        case CUART_KEY_U64: k_lookup<KeyU64, 5, true><<<grid, 256, 0, s>>>(h->dix, q, lens, n, nullptr, *so); break;
+        case CUART_KEY_U32: k_lookup<KeyU32, 5, true><<<grid, 256, 0, s>>>(h->dix, q, lens, n, nullptr, *so); break;
+        default: k_lookup<KeyBytes, 5, true><<<grid, 256, 0, s>>>(h->dix, q, lens, n, nullptr, *so); break;
+        }
+        g_cuart_launches++;
+        CU_TRY(cudaGetLastError());
+        return CUART_OK;
+    }
     cudaEvent_t ev0, ev1;
     ktimer_begin(h, s, ev0, ev1);                      // per-launch k_lookup timing (cuart_kernel_timer)
 #define CUART_LOOKUP(K, P) k_lookup<K, P><<<grid, 256, 0, s>>>(h->dix, q, lens, n, out)
@@ -883,6 +898,23 @@ cuart_status cuart_destroy(cuart_index* h) {
     }
     delete h;
     return CUART_OK;
+}
+
+cuart_status cuart_lookup_segmented(const cuart_index* h, const cuart_keys* q, size_t n, uint32_t nseg,
+                                    const uint64_t* seg_start, uint64_t* const* seg_dst, void* stream) {
+    cuart_status rc = check_keys(h, q, n);
+    if (rc != CUART_OK) return rc;
+    if (n == 0) return CUART_OK;
+    if (nseg == 0 || nseg > uint32_t(kMaxSeg) || !seg_start || !seg_dst) return CUART_ERR_INVALID_ARGUMENT;
+    SegOut so{};
+    so.nseg = nseg;
+    for (uint32_t i = 0; i <= nseg; i++) so.start[i] = seg_start[i];
+    for (uint32_t i = 0; i < nseg; i++) {
+        so.dst[i] = seg_dst[i];
+        if (so.start[i] > so.start[i + 1] || (so.start[i + 1] > so.start[i] && !so.dst[i])) return CUART_ERR_INVALID_ARGUMENT;
+    }
+    if (so.start[0] != 0 || so.start[nseg] != n) return CUART_ERR_INVALID_ARGUMENT;
+    return launch_lookup(h, h->key_kind, q->data, q->lengths, n, nullptr, (cudaStream_t)stream, &so);
 }
 
 cuart_status cuart_lookup(const cuart_index* h, const cuart_keys* q, size_t n, uint64_t* out, void* stream) {

@@ -29,6 +29,23 @@ struct DevIndex {
     unsigned long long* free_count;  // number of entries in free_list
 };
 
+// Segmented output (multi-GPU fused return, §8(e)): result i goes to
+// dst[s] + (i - start[s]) for the segment s with start[s] <= i < start[s + 1];
+// dst[s] may be a peer GPU's window (CUDA IPC over NVLink), so the kernel that
+// produces the results also performs the return transfer.
+constexpr int kMaxSeg = 16;
+struct SegOut {
+    uint32_t nseg;
+    uint64_t start[kMaxSeg + 1];
+    uint64_t* dst[kMaxSeg];
+    __device__ __forceinline__ uint64_t* at(uint64_t i) const {
+        uint32_t s = 0;
+#pragma unroll 1
+        while (s + 1 < nseg && i >= start[s + 1]) s++;
+        return dst[s] + (i - start[s]);
+    }
+};
+
 // ----------------------------------------------------------------------------- loads
 __device__ __forceinline__ uint64_t ld_nc_u64(const void* p) {
     uint64_t v;

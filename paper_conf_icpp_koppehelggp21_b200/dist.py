@@ -22,6 +22,17 @@ Two modes:
 The protocol is written once against an ``ops`` object: ``CudaOps`` (product,
 C-ABI kernels, CUDA tensors, NCCL) or an injected test double (CPU tensors and
 the gloo backend) so the exchange logic runs in the CPU test suite.
+
+Range mode has two transports:
+
+* ``nccl`` — route into a local send buffer, then all-to-all of the runs and of
+  the results (the library-collective baseline);
+* ``p2p``  — fused: every rank maps its peers' receive windows (CUDA IPC over
+  NVLink/NVSwitch).  cuart_route_push stores each op straight into its owner's
+  window, and the owner's lookup (cuart_lookup_segmented) stores each result
+  straight into the requester's result window; only the P x P count matrix goes
+  through torch.distributed.  ``p2p_plan`` is the host arithmetic of that
+  exchange (pure, CPU-tested).
 """
 from __future__ import annotations
 
@@ -63,10 +74,79 @@ def owners(prefix: np.ndarray, splitters: np.ndarray) -> np.ndarray:
     return np.searchsorted(splitters, prefix, side="right").astype(np.int64)
 
 
+def ks_bytes(kind):
+    return {B.KIND_U64: 8, B.KIND_U32: 4, B.KIND_BYTES: 32}[kind]
+
+
 def select(keys, mask):
     if isinstance(keys, tuple):
         return (keys[0][mask], keys[1][mask])
     return keys[mask]
+
+
+# ------------------------------------------------------------------ fused p2p exchange: host plan
+def p2p_plan(M, rank):
+    """Offsets of the fused exchange for `rank`, from the P x P count matrix
+    M[s][o] = ops that source s routes to owner o (identical on every rank).
+
+    push_off[o]  : first slot of this rank's run in owner o's receive window
+                   (the runs of all sources are concatenated in rank order there);
+    seg_start    : [P+1] segments of this rank's receive window by source;
+    res_off[s]   : first slot of this rank's results in source s's result window
+                   (s keeps its results in owner-major send order);
+    need_recv / need_res : window capacities every rank must have (max over ranks).
+    """
+    M = np.asarray(M, np.int64)
+    P = M.shape[0]
+    col = M[:, rank]
+    return {
+        "push_off": [int(M[:rank, o].sum()) for o in range(P)],
+        "seg_start": [0] + [int(x) for x in np.cumsum(col)],
+        "recv_total": int(col.sum()),
+        "res_off": [int(M[s, :rank].sum()) for s in range(P)],
+        "need_recv": int(M.sum(axis=0).max()) if P else 0,
+        "need_res": int(M.sum(axis=1).max()) if P else 0,
+    }
+
+
+class P2PWindows:
+    """This rank's receive windows (keys, lengths, values, results), exported to and
+    mapped by every peer (CUDA IPC).  (Re)allocation is collective: every rank calls
+    ensure() with the same capacities (derived from the shared count matrix)."""
+
+    def __init__(self, group, world, rank, key_bytes, strings):
+        self.group, self.world, self.rank = group, world, rank
+        self.kb, self.strings = key_bytes, strings
+        self.cap_recv = self.cap_res = 0
+        self.own = None          # dict name -> local device address
+        self.peer = None         # list over ranks of dict name -> mapped address (own for self)
+
+    def ensure(self, need_recv, need_res):
+        if need_recv <= self.cap_recv and need_res <= self.cap_res and self.own is not None:
+            return
+        self.close()
+        self.cap_recv = max(need_recv, 2 * self.cap_recv, 1)
+        self.cap_res = max(need_res, 2 * self.cap_res, 1)
+        sizes = {"keys": self.cap_recv * self.kb, "vals": self.cap_recv * 8, "res": self.cap_res * 8}
+        if self.strings:
+            sizes["lens"] = self.cap_recv
+        self.own = {k: B.ipc_alloc(v) for k, v in sizes.items()}
+        mine = {k: B.ipc_export(v) for k, v in self.own.items()}
+        allh = [None] * self.world
+        dist.all_gather_object(allh, mine, group=self.group)
+        self.peer = [self.own if r == self.rank else {k: B.ipc_import(h) for k, h in allh[r].items()}
+                     for r in range(self.world)]
+
+    def close(self):
+        if self.peer is not None:
+            for r, m in enumerate(self.peer):
+                if r != self.rank:
+                    for a in m.values():
+                        B.ipc_close(a)
+        if self.own is not None:
+            for a in self.own.values():
+                B.ipc_free(a)
+        self.own = self.peer = None
 
 
 # ------------------------------------------------------------------ device ops (product)
@@ -148,14 +228,21 @@ class CudaOps:
 class DistIndex:
     """A CuART index spread over the ranks of a process group."""
 
-    def __init__(self, keys, values, mode="range", group=None, ops=None, lut_bytes=3, splitters=None, local=False):
+    def __init__(self, keys, values, mode="range", group=None, ops=None, lut_bytes=3, splitters=None, local=False,
+                 transport="nccl"):
         """keys/values: the GLOBAL key set, identical on every rank (host arrays).
         Range mode keeps this rank's share; replica mode keeps everything.
         local=True: keys/values are already this rank's share of a range partition
-        defined by `splitters` (used when the global set is too large to replicate)."""
+        defined by `splitters` (used when the global set is too large to replicate).
+        transport: "nccl" (route + all-to-all) or "p2p" (fused push / return over
+        peer memory; CUDA ops only)."""
         if mode not in ("range", "replica"):
             raise ValueError(mode)
+        if transport not in ("nccl", "p2p"):
+            raise ValueError(transport)
         self.mode = mode
+        self.transport = transport
+        self.windows = None
         self.group = group
         self.world = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
@@ -200,10 +287,76 @@ class DistIndex:
     def _split_keys(self, q):
         return (q[0], q[1]) if isinstance(q, tuple) else (q, None)
 
+    # ---- fused p2p transport (range mode)
+    def _p2p_route(self, keys, lens, vals):
+        """Count, agree on the count matrix, push every op into its owner's window.
+        Returns (plan, perm)."""
+        n = keys.shape[0]
+        kind = B.KIND_BYTES if lens is not None else (B.KIND_U64 if keys.element_size() == 8 else B.KIND_U32)
+        ks = B.raw_keys(kind, keys.data_ptr(), lens.data_ptr() if lens is not None else None)
+        counts = torch.zeros(self.world, dtype=torch.int64, device=keys.device)
+        scratch = torch.empty(max(1, B.lib().cuart_route_scratch_bytes(n, self.world)), dtype=torch.uint8,
+                              device=keys.device)
+        B.route_count(ks, n, self.splitters.data_ptr(), self.world, counts.data_ptr(), scratch.data_ptr())
+        torch.cuda.current_stream(keys.device).synchronize()        # this rank's earlier work on the windows is done
+        allc = [torch.empty_like(counts) for _ in range(self.world)]
+        if self._staged(counts):
+            hc = [torch.empty_like(counts, device="cpu") for _ in range(self.world)]
+            dist.all_gather(hc, counts.cpu(), group=self.group)
+            allc = hc
+        else:
+            dist.all_gather(allc, counts, group=self.group)
+        M = np.stack([c.cpu().numpy() for c in allc])                 # every rank passed its sync point
+        plan = p2p_plan(M, self.rank)
+        if self.windows is None:
+            self.windows = P2PWindows(self.group, self.world, self.rank, ks_bytes(kind), lens is not None)
+        self.windows.ensure(plan["need_recv"], plan["need_res"])
+        W, kb = self.windows.peer, self.windows.kb
+        perm = torch.empty(n, dtype=torch.int32, device=keys.device)
+        B.route_push(ks, n, self.world, vals.data_ptr() if vals is not None else None,
+                     [W[o]["keys"] + plan["push_off"][o] * kb for o in range(self.world)],
+                     [W[o]["lens"] + plan["push_off"][o] for o in range(self.world)] if lens is not None else None,
+                     [W[o]["vals"] + plan["push_off"][o] * 8 for o in range(self.world)] if vals is not None else None,
+                     perm.data_ptr(), scratch.data_ptr())
+        self._p2p_fence(keys.device)
+        return plan, perm, kind
+
+    def _p2p_fence(self, device):
+        """Every rank's pushes / returns have landed (kernel completion + barrier)."""
+        torch.cuda.current_stream(device).synchronize()
+        dist.barrier(group=self.group)
+
+    def _lookup_p2p(self, keys, lens, events=None):
+        plan, perm, kind = self._p2p_route(keys, lens, None)
+        W, me = self.windows.peer, self.rank
+        nr = plan["recv_total"]
+        if events:
+            events[0].record()
+        if nr:
+            rk = B.raw_keys(kind, W[me]["keys"], W[me].get("lens"))
+            B.lookup_segmented(self.index.h, rk, nr, plan["seg_start"],
+                               [W[s]["res"] + plan["res_off"][s] * 8 for s in range(self.world)])
+        if events:
+            events[1].record()
+        self.last_local_lookups = nr
+        self._p2p_fence(keys.device)
+        out = torch.empty(keys.shape[0], dtype=torch.int64, device=keys.device)
+        B.unroute_raw(W[me]["res"], perm.data_ptr(), keys.shape[0], out.data_ptr())
+        return out
+
+    def _update_p2p(self, keys, lens, vals):
+        plan, _, kind = self._p2p_route(keys, lens, vals)
+        W, me = self.windows.peer, self.rank
+        nr = plan["recv_total"]
+        if nr:
+            B.update_raw(self.index.h, B.raw_keys(kind, W[me]["keys"], W[me].get("lens")), nr, W[me]["vals"])
+
     # ---- lookups
     def lookup(self, queries, events=None):
         """events: optional (start, end) CUDA events recorded around the local lookup kernel."""
         keys, lens = self._split_keys(queries)
+        if self.mode == "range" and self.world > 1 and self.transport == "p2p":
+            return self._lookup_p2p(keys, lens, events)
         if self.mode == "replica" or self.world == 1:
             if events:
                 events[0].record()
@@ -240,6 +393,9 @@ class DistIndex:
             gk, gl, gv = self._all_gather_var(keys), (self._all_gather_var(lens) if lens is not None else None), \
                 self._all_gather_var(vals)
             self.ops.update(self.index, gk, gl, gv)
+            return
+        if self.transport == "p2p":
+            self._update_p2p(keys, lens, vals)
             return
         sk, sl, sv, _, counts = self.ops.route(keys, lens, vals, self.splitters, self.world)
         rcounts = self._exchange_counts(counts)
@@ -284,6 +440,11 @@ class DistIndex:
         return torch.cat([g[r * m: r * m + sizes[r]] for r in range(self.world)])
 
     def close(self):
+        if self.windows is not None:
+            torch.cuda.synchronize()
+            dist.barrier(group=self.group)        # no peer still writes into our windows
+            self.windows.close()
+            self.windows = None
         if self.index is not None:
             self.ops.close(self.index)
             self.index = None

@@ -2,7 +2,11 @@
 cuart_unroute, cuart_partition_by_flag, local lookups/updates) + the DistIndex
 protocol — run as 2 processes sharing cuda:0 (gloo, host-staged collectives;
 NCCL refuses duplicate devices).  Range and replica modes, lookups, updates and
-mixed rounds; results equal the single-index oracle."""
+mixed rounds; results equal the single-index oracle.  "range-p2p" runs the fused
+transport: each process maps the other's receive windows through CUDA IPC (same
+device here, NVLink peers on a multi-GPU box), cuart_route_push stores ops into
+the owner's window and cuart_lookup_segmented returns results into the
+requester's window."""
 import os
 import socket
 import tempfile
@@ -28,6 +32,8 @@ def _port():
 
 
 def _worker(rank, world, port, mode, outdir):
+    transport = "p2p" if mode.endswith("-p2p") else "nccl"
+    mode = mode.split("-")[0]
     import workloads as W
     from paper_conf_icpp_koppehelggp21_b200.dist import CudaOps, DistIndex
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -37,7 +43,7 @@ def _worker(rank, world, port, mode, outdir):
     cfg = W.Config("cX", "u64", N_KEYS, N_Q, N_U, 0.5, "")
     keys = W.u64_keys(3, N_KEYS)
     vals = W.values_for(W.SEED_VALUES + 3, np.arange(N_KEYS, dtype=np.uint64))
-    di = DistIndex(keys, vals, mode=mode, ops=CudaOps(dev))
+    di = DistIndex(keys, vals, mode=mode, ops=CudaOps(dev), transport=transport)
     kd = torch.from_numpy(keys.view(np.int64)).to(dev)
     q = W.lookup_batch_torch(W.CONFIGS["c3"], kd, rank * N_Q, N_Q, device=dev)
     r1 = di.lookup(q)
@@ -56,7 +62,7 @@ def _worker(rank, world, port, mode, outdir):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("mode", ["range", "replica"])
+@pytest.mark.parametrize("mode", ["range", "replica", "range-p2p"])
 def test_two_processes_one_gpu(mode):
     import workloads as W
     world = 2

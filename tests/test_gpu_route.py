@@ -106,3 +106,107 @@ def test_loopback_range_partitioned_c1(nparts):
     assert np.array_equal(out.cpu().numpy().view(np.uint64), o.lookup(keys))
     for ix in parts:
         ix.close()
+
+
+@pytest.mark.parametrize("kind", ["u64", "u32", "bytes"])
+@pytest.mark.parametrize("nparts", [2, 4, 8])
+def test_p2p_fused_exchange_loopback(kind, nparts):
+    """The fused p2p exchange with P virtual ranks on one GPU: every 'rank' has its
+    own partition index and windows (plain device buffers stand in for the mapped
+    peer windows), cuart_route_count -> count matrix -> cuart_route_push into the
+    owners' windows -> cuart_lookup_segmented straight into the sources' result
+    windows -> cuart_unroute.  Then a routed update batch (values pushed with the
+    keys, applied in rank-major order).  Results equal the oracle."""
+    from paper_conf_icpp_koppehelggp21_b200 import _binding as B
+    from paper_conf_icpp_koppehelggp21_b200.dist import p2p_plan, ks_bytes
+    rng = np.random.default_rng(nparts * 7 + len(kind))
+    if kind == "u64":
+        keys = np.unique(rng.integers(0, 2**64, 1 << 16, dtype=np.uint64))
+        mkq = lambda m: np.where(rng.random(m) < 0.5, keys[rng.integers(0, keys.shape[0], m)],
+                                 rng.integers(0, 2**64, m, dtype=np.uint64))
+        bk = B.KIND_U64
+    elif kind == "u32":
+        keys = np.unique(rng.integers(0, 1 << 24, 1 << 15, dtype=np.uint32))
+        mkq = lambda m: rng.integers(0, 1 << 24, m, dtype=np.uint32)
+        bk = B.KIND_U32
+    else:
+        keys = W.string_keys(5, 1 << 14)
+        mkq = lambda m: (lambda idx: (keys[0][idx].copy(), keys[1][idx].copy()))(rng.integers(0, 1 << 14, m))
+        bk = B.KIND_BYTES
+    nk = keys[1].shape[0] if isinstance(keys, tuple) else keys.shape[0]
+    vals = rng.integers(0, 2**63, nk, dtype=np.uint64)
+    sp = compute_splitters(prefix8(keys), nparts)
+    own = owners(prefix8(keys), sp)
+    sel = lambda a, m: (a[0][m], a[1][m]) if isinstance(a, tuple) else a[m]
+    idx = [C.Index(sel(keys, own == o), vals[own == o], lut_bytes=0 if kind == "bytes" else 3) for o in range(nparts)]
+    spt = _t(sp)
+    kb = ks_bytes(bk)
+    nq = [5000 + 3001 * s for s in range(nparts)]                   # ragged batch per source
+    qs = [mkq(m) for m in nq]
+    uks = [sel(keys, rng.integers(0, nk, m)) for m in nq]
+    uvs = [rng.integers(0, 2**63, m, dtype=np.uint64) for m in nq]
+
+    def raw(a):
+        t = _t(a)
+        k, l = (t if isinstance(t, tuple) else (t, None))
+        return t, B.raw_keys(bk, k.data_ptr(), l.data_ptr() if l is not None else None)
+
+    def exchange(batches, values):
+        keep = [raw(b) for b in batches]
+        vt = [_t(v) for v in values] if values is not None else None
+        scr = [torch.empty(B.lib().cuart_route_scratch_bytes(n, nparts), dtype=torch.uint8, device=DEV) for n in nq]
+        cnt = [torch.zeros(nparts, dtype=torch.int64, device=DEV) for _ in nq]
+        for s in range(nparts):
+            B.route_count(keep[s][1], nq[s], spt.data_ptr(), nparts, cnt[s].data_ptr(), scr[s].data_ptr())
+        M = np.stack([c.cpu().numpy() for c in cnt])
+        plans = [p2p_plan(M, r) for r in range(nparts)]
+        cap = max(plans[0]["need_recv"], 1)
+        win = [{"keys": torch.empty(cap * kb, dtype=torch.uint8, device=DEV),
+                "lens": torch.empty(cap, dtype=torch.uint8, device=DEV),
+                "vals": torch.empty(cap, dtype=torch.int64, device=DEV),
+                "res": torch.full((max(plans[0]["need_res"], 1),), 7, dtype=torch.int64, device=DEV)} for _ in nq]
+        perms = [torch.empty(n, dtype=torch.int32, device=DEV) for n in nq]
+        for s in range(nparts):
+            B.route_push(keep[s][1], nq[s], nparts, vt[s].data_ptr() if vt else None,
+                         [win[o]["keys"].data_ptr() + plans[s]["push_off"][o] * kb for o in range(nparts)],
+                         [win[o]["lens"].data_ptr() + plans[s]["push_off"][o] for o in range(nparts)]
+                         if kind == "bytes" else None,
+                         [win[o]["vals"].data_ptr() + plans[s]["push_off"][o] * 8 for o in range(nparts)] if vt else None,
+                         perms[s].data_ptr(), scr[s].data_ptr())
+        torch.cuda.synchronize()
+        return plans, win, perms
+
+    plans, win, perms = exchange(qs, None)
+    for o in range(nparts):
+        p = plans[o]
+        if p["recv_total"]:
+            rk = B.raw_keys(bk, win[o]["keys"].data_ptr(), win[o]["lens"].data_ptr())
+            B.lookup_segmented(idx[o].h, rk, p["recv_total"], p["seg_start"],
+                               [win[s]["res"].data_ptr() + p["res_off"][s] * 8 for s in range(nparts)])
+    torch.cuda.synchronize()
+    mp_ = MapOracle(keys, vals)
+    for s in range(nparts):
+        out = torch.empty(nq[s], dtype=torch.int64, device=DEV)
+        B.unroute_raw(win[s]["res"].data_ptr(), perms[s].data_ptr(), nq[s], out.data_ptr())
+        torch.cuda.synchronize()
+        assert np.array_equal(out.cpu().numpy().view(np.uint64), mp_.lookup(qs[s])), s
+    # routed update batch: values travel with the keys, owners apply in rank-major order
+    plans, win, _ = exchange(uks, uvs)
+    for o in range(nparts):
+        p = plans[o]
+        if p["recv_total"]:
+            rk = B.raw_keys(bk, win[o]["keys"].data_ptr(), win[o]["lens"].data_ptr())
+            B.update_raw(idx[o].h, rk, p["recv_total"], win[o]["vals"].data_ptr())
+    torch.cuda.synchronize()
+    for s in range(nparts):
+        mp_.update(uks[s], uvs[s])
+    exp = mp_.lookup(keys)
+    got = np.empty(nk, np.uint64)
+    for o in range(nparts):
+        m = own == o
+        out = torch.empty(int(m.sum()), dtype=torch.int64, device=DEV)
+        idx[o].lookup(_t(sel(keys, m)), out)
+        got[m] = out.cpu().numpy().view(np.uint64)
+    assert np.array_equal(got, exp)
+    for ix in idx:
+        ix.close()

@@ -358,7 +358,7 @@ int main(int argc, char** argv) {
     k_bscan_rows<<<kBuckets, kBucketThreads>>>(hist, tiles, tot);
     k_bscan<<<1, kBuckets>>>(tot);
     timeit("k_bscatter", n * 18.0, [&] { k_bscatter<KeyU64><<<T, 256, smem>>>(q, nullptr, n, 0, hist, tot, bq, nullptr, jpos); });
-    timeit("k_bgather", n * 18.0, [&] { k_bgather<<<T, 256>>>(res, jpos, n, hist, tot, out); });
+    timeit("k_bgather", n * 18.0, [&] { k_bgather<false><<<T, 256>>>(res, jpos, n, hist, tot, out); });
     const unsigned long long c1 = checksum(out, n);
     timeit("g_old", n * 18.0, [&] { g_old<<<T, 256>>>(res, jpos, n, hist, tot, out); });
     const unsigned long long c2 = checksum(out, n);
@@ -377,7 +377,7 @@ int main(int argc, char** argv) {
     g_ca<<<T, 256>>>(bq, jpos, n, hist, tot, out);
     const unsigned long long s2 = checksum(out, n);
     timeit("k_bscatter_again", n * 18.0, [&] { k_bscatter<KeyU64><<<T, 256, smem>>>(q, nullptr, n, 0, hist, tot, bq, nullptr, jpos); });
-    k_bgather<<<T, 256>>>(bq, jpos, n, hist, tot, out);
+    k_bgather<false><<<T, 256>>>(bq, jpos, n, hist, tot, out);
     const unsigned long long s3 = checksum(out, n);
     printf("{\"roundtrip_s_v4\": %s, \"roundtrip_k_bscatter\": %s}\n", s2 == s1b ? "true" : "false", s3 == s1b ? "true" : "false");
     printf("{\"s0\": %llu, \"roundtrip_ok\": %s}\n", s0, s1 == s1b ? "true" : "false");
