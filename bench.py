@@ -54,6 +54,8 @@ def _args():
     p.add_argument("--config", default="c3", choices=["c1", "c2", "c3", "c4", "c5"])
     p.add_argument("--impl", default="cuart", choices=["cuart", "reference"])
     p.add_argument("--lut", type=int, default=3)
+    p.add_argument("--lut-format", default="auto", choices=["auto", "links", "compact32", "rank"],
+                   help="device form of the root table (cuart_build_opts.lut_format)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--e2e-steps", type=int, default=2)
@@ -316,6 +318,9 @@ def run_c5(args, world, rank, local, dev):
 
 
 # ------------------------------------------------------------------ main (GPU)
+LUT_FORMATS = {"auto": 0, "links": 1, "compact32": 2, "rank": 3}
+
+
 def main():
     args = _args()
     if args.impl == "reference":
@@ -348,7 +353,7 @@ def main():
     ops = CudaOps(dev)
     if world == 1:
         layout = C.Layout(keys, vals, lut_bytes=args.lut)
-        ix = C.Index.from_layout(layout, device=local)
+        ix = C.Index.from_layout(layout, device=local, lut_format=LUT_FORMATS[args.lut_format])
         di = None
     else:
         di = DistIndex(keys, vals, mode=mode, ops=ops, lut_bytes=args.lut, transport=args.transport)

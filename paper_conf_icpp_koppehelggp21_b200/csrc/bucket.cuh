@@ -267,8 +267,9 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
     }
     __syncthreads();
     const unsigned int mine = h[threadIdx.x];
-    loc[threadIdx.x] = block_excl_scan256(mine, wtot);
-    glb[threadIdx.x] = gb;
+    const unsigned int lb = block_excl_scan256(mine, wtot);
+    loc[threadIdx.x] = lb;
+    glb[threadIdx.x] = gb - lb;                                        // slot = glb[b] + staged position (mod 2^32)
     __syncthreads();
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
@@ -296,8 +297,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
     for (int r = 0; r < kBucketItems; r++) {
         const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
         if (j < cnt) {
-            const uint32_t b = sb[j];
-            const uint64_t dst = uint64_t(glb[b]) + (j - loc[b]);
+            const uint64_t dst = uint64_t(glb[sb[j]] + j);                // n < 2^32: exact
             if (KS == 8) __stcs((unsigned long long*)bq + dst, (unsigned long long)((const uint64_t*)skeys)[j]);
             else if (KS == 4) __stcs((unsigned int*)bq + dst, ((const uint32_t*)skeys)[j]);
             else {
