@@ -104,7 +104,16 @@ typedef struct {
                                     CUART_SLICE_AUTO (= off: measured slower on B200, the
                                     slices take L1 capacity), CUART_SLICE_OFF,
                                     CUART_SLICE_ON.  Results are identical.                */
+    uint32_t wide_lut;           /* pre-bucketed walks start from a wide root table: 32 B per
+                                    entry = the link + the sorted keys of the N4 / N16 it
+                                    points to ("merged top layers"), so the first
+                                    node's key read is skipped.  CUART_WIDE_AUTO (on when
+                                    most entries lead to an N4/N16), CUART_WIDE_OFF,
+                                    CUART_WIDE_ON.  Results are identical.                 */
 } cuart_build_opts;
+#define CUART_WIDE_AUTO 0u
+#define CUART_WIDE_OFF 1u
+#define CUART_WIDE_ON 2u
 #define CUART_SLICE_AUTO 0u
 #define CUART_SLICE_OFF 1u
 #define CUART_SLICE_ON 2u

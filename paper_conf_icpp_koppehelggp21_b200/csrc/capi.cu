@@ -74,6 +74,8 @@ struct cuart_index {
     int policy = 5;                    // cache-policy variant of the kernels (kernels.cuh Loader)
     uint32_t lut_format = CUART_LUT_LINKS;
     uint64_t lutc_off = 0;             // compact / rank LUT region
+    uint64_t lutw_off = 0;             // wide LUT region (32 B/entry), 0 bytes if absent
+    bool wide = false;
     uint64_t lut_exceptions = 0;       // RANK: entries served by the 64-bit table
     int grid_ctas_per_sm = 0;          // 0 = default grid (one op per thread); else persistent grid
     bool ktimer = false;               // record CUDA events around every k_lookup launch
@@ -259,6 +261,8 @@ __global__ void __launch_bounds__(256) k_upd2(DevIndex ix, const uint64_t* __res
             const uint64_t sl = slotref[i];
             if (sl & 1) *(uint32_t*)(sl & ~uint64_t(1)) = 0;       // compact 32-bit LUT entry
             else if (sl) *(uint64_t*)sl = 0;                       // 64-bit link: node child / LUT entry
+            if (ix.lutw && sl >= uint64_t(ix.lut) && sl < uint64_t(ix.lut + ix.lut_entries))
+                ix.lutw[(sl - uint64_t(ix.lut)) / 8 * 4] = 0;      // the wide table's copy of that entry
             *dst = kMiss;
             const unsigned long long pos = atomicAdd(ix.free_count, 1ull);
             ix.free_list[pos] = uint32_t(gid);
@@ -784,6 +788,41 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     if (need_links) off = align(off + L.lut.size() * 8);
     h->lutc_off = off;
     off = align(off + lut32.size() * 4 + lutr.size() * 8);
+    // wide root table for the pre-bucketed walks (kernels.cuh start_wide)
+    // Worth it when most table entries lead to an N4/N16 (c3: 92%): a 32-B entry costs
+    // the L2 like the N4 block / N16 keys it saves, but more than an 8-B LINKS entry,
+    // so for N48/N256 targets (c2, c5) the walk keeps the LINKS table (measured on c2:
+    // 2.45 ms LINKS vs 2.94 ms wide per 2^28; c3: 14.38 ms LINKS vs 11.12 ms wide per 2^30).
+    h->wide = false;
+    if (need_links && !L.lut.empty()) {
+        uint64_t small = 0, nonnull = 0;
+        for (uint64_t l : L.lut) {
+            nonnull += l != 0;
+            small += link_type(l) == T_N4 || link_type(l) == T_N16;
+        }
+        h->wide = nonnull > 0 && 2 * small >= nonnull;
+    }
+    uint32_t wide_opt = opts ? opts->wide_lut : CUART_WIDE_AUTO;
+    if (const char* pe = getenv("CUART_WIDE")) wide_opt = uint32_t(atoi(pe));
+    if (wide_opt > CUART_WIDE_ON) {
+        delete h;
+        return CUART_ERR_INVALID_ARGUMENT;
+    }
+    if (wide_opt == CUART_WIDE_OFF) h->wide = false;
+    if (wide_opt == CUART_WIDE_ON) h->wide = need_links && !L.lut.empty();
+    std::vector<uint64_t> lutw;
+    if (h->wide) {
+        lutw.assign(L.lut.size() * 4, 0);
+        for (size_t p = 0; p < L.lut.size(); p++) {
+            const uint64_t l = L.lut[p];
+            lutw[4 * p] = l;
+            const uint32_t t = link_type(l);
+            if (t == T_N4) memcpy(&lutw[4 * p + 1], L.buf[t].data() + link_index(l) * record_bytes(t) + kN4Keys, 4);
+            else if (t == T_N16) memcpy(&lutw[4 * p + 1], L.buf[t].data() + link_index(l) * record_bytes(t) + kN16Keys, 16);
+        }
+    }
+    h->lutw_off = off;
+    off = align(off + lutw.size() * 8);
     h->err_off = off;
     off = align(off + 256);
     h->arena_bytes = off;
@@ -804,6 +843,9 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && !lutr.empty() &&
         cudaMemcpy(h->arena + h->lutc_off, lutr.data(), lutr.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
+        rc = CUART_ERR_CUDA;
+    if (rc == CUART_OK && !lutw.empty() &&
+        cudaMemcpy(h->arena + h->lutw_off, lutw.data(), lutw.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && !CUART_COLOCATED_WINNER && h->total_leaves &&
         cudaMemset(h->arena + h->winner_off, 0, h->total_leaves * 8) != cudaSuccess)
@@ -871,10 +913,14 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     // table): with the batch bucketed the bucket's slice of it is L2-resident, and an
     // 8-B request costs the L2 less than the 32-B rank block (K-GATHER: 245 vs 145 G
     // random requests/s); measured -4% walk time on c3 and c2.
+    d.lutw = h->wide ? (uint64_t*)(h->arena + h->lutw_off) : nullptr;
+    d.lut_entries = L.lut.size();
+    d.walk_wide = 0;
     h->dix_links = d;
     if (d.lut) {
         h->dix_links.lutr = nullptr;
         h->dix_links.lut32 = nullptr;
+        h->dix_links.walk_wide = h->wide ? 1u : 0u;
     }
     *out = h;
     return CUART_OK;
@@ -1101,6 +1147,7 @@ cuart_status cuart_stats(const cuart_index* h, cuart_stats_t* s) {
     s->lut_entries = h->lut_bytes ? (uint64_t(1) << (8 * h->lut_bytes)) : 0;
     s->lut_bytes_total = h->lut_format == CUART_LUT_COMPACT32 ? s->lut_entries * 4
                        : h->lut_format == CUART_LUT_RANK ? s->lut_entries * 9 : s->lut_entries * 8;
+    if (h->wide) s->lut_bytes_total += s->lut_entries * 32;       // wide table of the bucketed walks
     s->lut_format = h->lut_format;
     s->lut_exceptions = h->lut_exceptions;
     s->arena_bytes = h->arena_bytes + h->leafref_cap * 8;

@@ -27,6 +27,9 @@ struct DevIndex {
     uint32_t* err;                // sticky device error flag
     uint32_t* free_list;          // freed leaf ids (global leaf id), capacity = #leaves
     unsigned long long* free_count;  // number of entries in free_list
+    uint64_t* lutw;               // wide root table (32 B/entry: link + the target N4/N16's keys), or nullptr
+    uint64_t lut_entries;         // 2^(8 lut_bytes)
+    uint32_t walk_wide;           // 1: lookups start from lutw (pre-bucketed walks, whose lutw slice is L2-resident)
 };
 
 // Segmented output (multi-GPU fused return, §8(e)): result i goes to
@@ -372,12 +375,44 @@ __device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Lo
 // Start of a walk: LUT[first k key bytes] or the root.  With TRACK, *slot =
 // address of the LUT entry holding the link (bit 0 set for a 32-bit entry), 0 if
 // the start is the root (a root leaf is never unlinked; its tombstone suffices).
+// Wide root table ("merged top layers", B200 reading): entry p is 32 B =
+// {link, the 4 / 16 sorted key bytes of the N4 / N16 it points to, pad}.  One
+// 32-B request brings the start link AND the first node's search keys, so the walk
+// skips that node's key read and loads the child link directly: on c3 one L2
+// request less for every query whose LUT target is an N16, a 32-B request
+// replaced by an 8-B one for N4 targets.  Deletes never change a node's keys (they
+// null child links, reading C18), so the embedded keys stay a superset filter.
+template <class Key, int POL>
+__device__ __forceinline__ uint64_t start_wide(const DevIndex& ix, const Loader<POL>& ld, const Key& key, uint64_t p) {
+    const U8x32 e = ld.lutv8(ix.lutw + p * 4);
+    const uint64_t link = uint64_t(e.w[0]) | (uint64_t(e.w[1]) << 32);
+    const uint32_t t = link_type(link);
+    if (t != T_N4 && t != T_N16) return link;
+    const uint32_t aux = link_aux(link);
+    if (aux >= key.len()) return 0;
+    const uint32_t bb = key.byte(aux) * 0x01010101u;
+    const uint8_t* rec = ix.base[t] + link_index(link) * record_bytes(t);
+    uint32_t l0, e0;
+    search4(e.w[2], bb, l0, e0);
+    if (t == T_N4) {
+        if (e0 == 0) return 0;
+        return ld.node64(rec + kN4Child + 8 * l0);
+    }
+    uint32_t l1, l2, l3, e1, e2, e3;
+    search4(e.w[3], bb, l1, e1);
+    search4(e.w[4], bb, l2, e2);
+    search4(e.w[5], bb, l3, e3);
+    if ((e0 | e1 | e2 | e3) == 0) return 0;
+    return ld.node64(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
+}
+
 template <class Key, int POL, bool TRACK = false>
 __device__ __forceinline__ uint64_t start_link(const DevIndex& ix, const Loader<POL>& ld, const Key& key,
                                                uint64_t* slot = nullptr) {
     if (TRACK) *slot = 0;
     if (ix.lut_bytes && key.len() >= ix.lut_bytes) {
         const uint64_t p = key.prefix(ix.lut_bytes);
+        if (!TRACK && ix.walk_wide) return start_wide(ix, ld, key, p);
         if (ix.lutr) return expand_lut_rank<POL, TRACK>(ix, ld, p, slot);
         if (ix.lut32) {
             if (TRACK) *slot = uint64_t(ix.lut32 + p) | 1u;

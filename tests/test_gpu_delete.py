@@ -98,3 +98,34 @@ def test_mixed_batches_vs_oracle(kind, lut, fmt):
     fl = ix.free_leaves()
     assert fl.shape[0] == deleted and np.unique(fl).shape[0] == deleted
     ix.close()
+
+
+@pytest.mark.parametrize("fmt", [1, 3])
+@pytest.mark.parametrize("wide", [0, 2])
+def test_deletes_visible_to_bucketed_wide_walk(fmt, wide):
+    """Pre-bucketed lookups start from the wide root table (LUT link + the target
+    node's keys).  Deletes unlink leaves from node slots AND from LUT entries (at
+    k = 3 most of c1's keys hang directly off a LUT entry); both must be visible to
+    the bucketed walk, and bucketed plain updates after the deletes must skip the
+    deleted keys (reading C18)."""
+    cfg = W.CONFIGS["c1"]
+    keys, vals = W.build_set(cfg)
+    rng = np.random.default_rng(5)
+    # 3-byte prefixes holding 2..16 keys each: LUT entries leading to N4 / N16 nodes
+    dense = (np.repeat(np.arange(1 << 12, dtype=np.uint64), 6) << np.uint64(40)) | \
+        rng.integers(0, 1 << 40, 6 << 12, dtype=np.uint64) | np.uint64(0xAB << 56)
+    keys = np.unique(np.concatenate([keys, dense]))
+    vals = rng.integers(0, 2**63, keys.shape[0], dtype=np.uint64)
+    on = C.Index(keys, vals, lut_bytes=3, lut_format=fmt, prebucket=C.PREBUCKET_ON, wide_lut=wide)
+    mp = MapOracle(keys, vals)
+    dk = keys[rng.random(keys.shape[0]) < 0.4]
+    on.erase(_t(dk))
+    mp.apply(dk, None, np.ones(dk.shape[0], bool))
+    q = np.concatenate([keys, rng.integers(0, 2**64, 1 << 16, dtype=np.uint64)])
+    assert np.array_equal(_lookup(on, q), mp.lookup(q))
+    uk = keys[rng.integers(0, keys.shape[0], 100_000)]
+    uv = rng.integers(0, 2**63, uk.shape[0], dtype=np.uint64)
+    on.update(_t(uk), _t(uv))
+    mp.update(uk, uv)
+    assert np.array_equal(_lookup(on, q), mp.lookup(q))
+    on.close()

@@ -374,6 +374,8 @@ def test_prebucket_equals_direct(kind):
     variants = [C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, slice_lut=C.SLICE_OFF)]
     if kind != "bytes":
         variants.append(C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, slice_lut=C.SLICE_ON))
+        variants.append(C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_ON))
+        variants.append(C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_OFF))
     # 2048 * 4096 + 4097 spans more than one pass of k_bscan_rows (2048 tiles per pass)
     sizes = (4095, 4096, 4097, 100_003, 1 << 20) + ((2048 * 4096 + 4097,) if kind == "u64" else ())
     for m in sizes:
@@ -404,14 +406,18 @@ def test_prebucket_updates_equal_direct(kind):
     on = C.Index(keys, vals, prebucket=C.PREBUCKET_ON)
     off = C.Index(keys, vals, prebucket=C.PREBUCKET_OFF)
     mp = MapOracle(keys, vals)
+    wide = C.Index(keys, vals, prebucket=C.PREBUCKET_ON, lut_bytes=0 if kind == "bytes" else 3, wide_lut=C.WIDE_ON)
     for m in (4097, 200_003):
         pick = rng.integers(0, min(n, 3000), m)                     # heavy duplication
         uk = (keys[0][pick].copy(), keys[1][pick].copy()) if isinstance(keys, tuple) else keys[pick].copy()
         uv = rng.integers(0, 2**63, m, dtype=np.uint64)
         on.update(_t(uk), _t(uv))
         off.update(_t(uk), _t(uv))
+        wide.update(_t(uk), _t(uv))
         mp.update(uk, uv)
         a, b = _lookup(on, keys), _lookup(off, keys)
         assert np.array_equal(a, b) and np.array_equal(a, mp.lookup(keys)), m
+        assert np.array_equal(_lookup(wide, keys), a), m
     on.close()
     off.close()
+    wide.close()
