@@ -387,7 +387,10 @@ def main():
         samp = samp.view(np.uint64) if cfg.kind == "u64" else samp.view(np.uint32)
     if mode == "range":   # sample of the queries this rank's index actually serves
         samp = select(samp, owners(prefix8(samp), di.splitters_np) == rank)
-    sec = layout.sectors(samp).astype(np.float64)
+    bucketed = nl >= (1 << 22) and cfg.kind != "bytes"
+    # sectors of the path the walk kernel takes: the pre-bucketed walk starts from the
+    # wide root table when the index has one (stats["wide_lut"]), else the plain path
+    sec = layout.sectors(samp, wide=bool(bucketed and stats.get("wide_lut", 0))).astype(np.float64)
     io_bytes = {"u64": 8, "u32": 4, "bytes": 33}[cfg.kind] + 8
     random_bytes_per_lookup = 32.0 * sec.mean() + io_bytes
     # Algorithmic DRAM bytes per lookup of the dominant kernel:
@@ -395,7 +398,6 @@ def main():
     # pre-bucketed path (auto for >= 2^22 queries): the walk runs over one bucket's slice
     # of the tree at a time, L2-resident by construction, so the compulsory traffic is the
     # I/O plus each tree record once per batch (SURVEY §8(d) S_DRAM excludes L2-resident data).
-    bucketed = nl >= (1 << 22) and cfg.kind != "bytes"
     tree_bytes = sum(stats[t + "_bytes"] for t in ("n4", "n16", "n48", "n256", "leaf8", "leaf16", "leaf32"))
     served_est = nl           # range mode: each rank serves ~nl routed lookups (its share of every rank's batch)
     bytes_per_lookup = (io_bytes + tree_bytes / served_est) if bucketed else random_bytes_per_lookup
@@ -475,6 +477,9 @@ def main():
         peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)"
     achieved = served * bytes_per_lookup / (kern_ms * 1e-3) / 1e9
     pipe_achieved = nl * pipeline_bytes / (look_ms * 1e-3) / 1e9
+    # BASELINE north_star's definition: 32-B sectors touched per query x queries/s
+    # (the whole lookup call) against peak DRAM bandwidth
+    ns_achieved = nl * random_bytes_per_lookup / (look_ms * 1e-3) / 1e9
     traffic = args.traffic
     tfile = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if traffic is None and os.path.exists(tfile):
@@ -574,6 +579,13 @@ def main():
                          "sectors_per_lookup": round(float(sec.mean()), 4),
                          "random_path_bytes_per_lookup": round(random_bytes_per_lookup, 3),
                          "peak_source": peak_src, "random_access_ceiling": RANDOM_CEILING,
+                         "north_star_random_sector": {
+                             "definition": "BASELINE north_star: 32-B sectors touched per query (host walker over "
+                                           "the kernel's path, 2^20-query sample) x 32 B + key/result I/O, times "
+                                           "lookups/s of the whole lookup call, vs peak DRAM bandwidth",
+                             "sectors_per_lookup": round(float(sec.mean()), 4),
+                             "bytes_per_lookup": round(random_bytes_per_lookup, 3),
+                             "achieved": round(ns_achieved, 1), "frac": round(ns_achieved / peak, 4)},
                          "lookup_call": {"ms": round(look_ms, 4), "bytes_per_lookup": round(pipeline_bytes, 3),
                                          "achieved": round(pipe_achieved, 1), "frac": round(pipe_achieved / peak, 4),
                                          "kernels": "k_bhist, k_bscan_rows, k_bscan, k_bscatter, "

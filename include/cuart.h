@@ -140,6 +140,7 @@ typedef struct {
     uint32_t max_depth;          /* longest root-to-leaf node chain */
     uint32_t lut_format;         /* CUART_LUT_* in use on the device */
     uint64_t lut_exceptions;     /* RANK: entries served by the 64-bit link table */
+    uint32_t wide_lut;           /* 1: pre-bucketed walks start from the wide root table */
 } cuart_stats_t;
 
 typedef struct cuart_index cuart_index;    /* device-resident index (opaque) */
@@ -240,6 +241,11 @@ cuart_status cuart_layout_lookup(const cuart_layout* l, const cuart_keys* querie
  * DESIGN.md "Roofline").  sectors: host uint32_t[n]. */
 cuart_status cuart_layout_sectors(const cuart_layout* l, const cuart_keys* queries, size_t n,
                                   uint32_t* sectors, int threads);
+/* As cuart_layout_sectors for the walk of a given variant: flags CUART_SECTORS_WIDE =
+ * the pre-bucketed walk starting from the wide root table (cuart_build_opts.wide_lut). */
+#define CUART_SECTORS_WIDE 1u
+cuart_status cuart_layout_sectors_ex(const cuart_layout* l, const cuart_keys* queries, size_t n,
+                                     uint32_t* sectors, int threads, uint32_t flags);
 cuart_status cuart_upload(const cuart_layout* l, const cuart_build_opts* opts, cuart_index** out);
 cuart_status cuart_layout_free(cuart_layout* l);  /* NULL ok */
 

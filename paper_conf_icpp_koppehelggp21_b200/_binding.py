@@ -34,7 +34,7 @@ class _Stats(ctypes.Structure):
                 ("lut_entries", ctypes.c_uint64), ("lut_bytes_total", ctypes.c_uint64),
                 ("arena_bytes", ctypes.c_uint64), ("lut_bytes", ctypes.c_uint32), ("key_kind", ctypes.c_uint32),
                 ("root", ctypes.c_uint64), ("max_depth", ctypes.c_uint32), ("lut_format", ctypes.c_uint32),
-                ("lut_exceptions", ctypes.c_uint64)]
+                ("lut_exceptions", ctypes.c_uint64), ("wide_lut", ctypes.c_uint32)]
 
 
 class _View(ctypes.Structure):
@@ -61,7 +61,7 @@ def lib():
             "cuart_kernel_timer": [P, I], "cuart_kernel_time": [P, P, P, P], "cuart_kernel_time_ex": [P, P, P, P, P], "cuart_lookup_host": [P, P, S, P], "cuart_update_host": [P, P, P, S],
             "cuart_stats": [P, P], "cuart_dump": [P, P], "cuart_get_error": [P],
             "cuart_layout_build": [P, P, S, P, P], "cuart_layout_view_get": [P, P],
-            "cuart_layout_lookup": [P, P, S, P, I], "cuart_layout_sectors": [P, P, S, P, I], "cuart_upload": [P, P, P], "cuart_layout_free": [P],
+            "cuart_layout_lookup": [P, P, S, P, I], "cuart_layout_sectors": [P, P, S, P, I], "cuart_layout_sectors_ex": [P, P, S, P, I, ctypes.c_uint32], "cuart_upload": [P, P, P], "cuart_layout_free": [P],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -285,7 +285,7 @@ def _stats_dict(s):
     d.update({f"{names[t]}_bytes": int(s.bytes[t]) for t in names})
     d.update(n_keys=int(s.n_keys), lut_bytes=int(s.lut_bytes), lut_entries=int(s.lut_entries),
              arena_bytes=int(s.arena_bytes), root=int(s.root), max_depth=int(s.max_depth), key_kind=int(s.key_kind),
-             lut_format=int(s.lut_format), lut_exceptions=int(s.lut_exceptions))
+             lut_format=int(s.lut_format), lut_exceptions=int(s.lut_exceptions), wide_lut=int(s.wide_lut))
     return d
 
 
@@ -332,10 +332,11 @@ def cuart_layout_lookup(l, queries, threads=0):
     return out
 
 
-def cuart_layout_sectors(l, queries, threads=0):
+def cuart_layout_sectors(l, queries, threads=0, wide=False):
     q, n, keep = make_keys(queries)
     out = np.empty(n, dtype=np.uint32)
-    _check(lib().cuart_layout_sectors(l, ctypes.byref(q), n, _ptr(out), threads), "cuart_layout_sectors")
+    _check(lib().cuart_layout_sectors_ex(l, ctypes.byref(q), n, _ptr(out), threads, 1 if wide else 0),
+           "cuart_layout_sectors_ex")
     return out
 
 
@@ -366,8 +367,8 @@ class Layout:
     def view(self):
         return cuart_layout_view_get(self.h)
 
-    def sectors(self, queries, threads=0):
-        return cuart_layout_sectors(self.h, queries, threads)
+    def sectors(self, queries, threads=0, wide=False):
+        return cuart_layout_sectors(self.h, queries, threads, wide)
 
     def close(self):
         cuart_layout_free(self.h)

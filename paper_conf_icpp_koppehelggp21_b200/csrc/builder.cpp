@@ -344,17 +344,34 @@ inline uint32_t sectors(uint64_t off, uint32_t bytes) { return uint32_t((off + b
 // (kernels.cuh find_leaf) reads on this path: LUT entry 8 B; N256 child 8 B;
 // N48 index byte + child 8 B; N16 keys 16 B + child 8 B; N4 bytes [16, 56) of its
 // 64-B record; leaves 16 / 32 / 48 B.
-uint64_t walk_one(const HostLayout& L, const uint8_t* key, uint32_t len, uint32_t* sec = nullptr) {
+// wide: the walk starts from the 32-B wide root-table entry (link + the target
+// N4/N16's keys, kernels.cuh start_wide) and reads that node's child link directly.
+uint64_t walk_one(const HostLayout& L, const uint8_t* key, uint32_t len, uint32_t* sec = nullptr, bool wide = false) {
     if (len == 0 || len > kMaxKey) return kMiss;
     uint32_t s = 0;
     uint64_t link = L.root;
+    struct Guard { uint32_t* dst; uint32_t* s; ~Guard() { if (dst) *dst = *s; } } guard{sec, &s};
     if (L.lut_bytes && len >= L.lut_bytes) {
         uint64_t p = 0;
         for (uint32_t b = 0; b < L.lut_bytes; b++) p = (p << 8) | key[b];
         link = L.lut[p];
-        s += sectors(p * 8, 8);
+        s += sectors(p * (wide ? 32 : 8), wide ? 32 : 8);
+        const uint32_t t = link_type(link);
+        if (wide && (t == T_N4 || t == T_N16)) {
+            const uint32_t d = link_aux(link);
+            if (d >= len) return kMiss;
+            const uint64_t roff = link_index(link) * kRecordBytes[t];
+            const uint8_t* rec = L.buf[t].data() + roff;
+            const uint32_t nk = t == T_N4 ? 4 : 16;
+            const uint8_t* keys = rec + (t == T_N4 ? kN4Keys : kN16Keys);
+            uint32_t less = 0, eq = 0;
+            for (uint32_t j = 0; j < nk; j++) { less += keys[j] < key[d]; eq |= keys[j] == key[d]; }
+            if (!eq) return kMiss;
+            const uint64_t co = roff + (t == T_N4 ? kN4Child : kN16Child) + 8 * less;
+            s += sectors(co, 8);
+            memcpy(&link, L.buf[t].data() + co, 8);
+        }
     }
-    struct Guard { uint32_t* dst; uint32_t* s; ~Guard() { if (dst) *dst = *s; } } guard{sec, &s};
     for (;;) {
         const uint32_t t = link_type(link);
         if (t == T_NULL) return kMiss;
@@ -398,7 +415,7 @@ uint64_t walk_one(const HostLayout& L, const uint8_t* key, uint32_t len, uint32_
 }  // namespace
 
 void host_layout_sectors(const HostLayout& L, uint32_t kind, const void* queries, const uint8_t* lengths, uint64_t n,
-                         uint32_t* sec, int threads) {
+                         uint32_t* sec, int threads, bool wide) {
     QView q{kind, queries, lengths};
     if (threads <= 0) threads = omp_get_max_threads();
 #pragma omp parallel for schedule(static) num_threads(threads)
@@ -406,7 +423,7 @@ void host_layout_sectors(const HostLayout& L, uint32_t kind, const void* queries
         uint8_t key[kMaxKey];
         q.bytes(i, key);
         sec[i] = 0;
-        walk_one(L, key, q.len(i), &sec[i]);
+        walk_one(L, key, q.len(i), &sec[i], wide);
     }
 }
 

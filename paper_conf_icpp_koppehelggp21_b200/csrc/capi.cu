@@ -631,6 +631,16 @@ cuart_status cuart_layout_lookup(const cuart_layout* l, const cuart_keys* q, siz
     return CUART_OK;
 }
 
+cuart_status cuart_layout_sectors_ex(const cuart_layout* l, const cuart_keys* q, size_t n, uint32_t* sectors,
+                                     int threads, uint32_t flags) {
+    if (!l || !q || (n > 0 && (!q->data || !sectors))) return CUART_ERR_INVALID_ARGUMENT;
+    if (q->kind == CUART_KEY_BYTES && n > 0 && !q->lengths) return CUART_ERR_INVALID_ARGUMENT;
+    if (uint32_t(q->kind) != l->L.key_kind) return CUART_ERR_INVALID_ARGUMENT;
+    host_layout_sectors(l->L, l->L.key_kind, q->data, q->lengths, n, sectors, threads,
+                        (flags & CUART_SECTORS_WIDE) && !l->L.lut.empty());
+    return CUART_OK;
+}
+
 cuart_status cuart_layout_sectors(const cuart_layout* l, const cuart_keys* q, size_t n, uint32_t* sectors, int threads) {
     if (!l || !q || (n > 0 && (!q->data || !sectors))) return CUART_ERR_INVALID_ARGUMENT;
     if (uint32_t(q->kind) != l->L.key_kind) return CUART_ERR_INVALID_ARGUMENT;
@@ -1150,6 +1160,7 @@ cuart_status cuart_stats(const cuart_index* h, cuart_stats_t* s) {
     if (h->wide) s->lut_bytes_total += s->lut_entries * 32;       // wide table of the bucketed walks
     s->lut_format = h->lut_format;
     s->lut_exceptions = h->lut_exceptions;
+    s->wide_lut = h->wide ? 1u : 0u;
     s->arena_bytes = h->arena_bytes + h->leafref_cap * 8;
     s->key_kind = h->key_kind;
     s->root = h->root;

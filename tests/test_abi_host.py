@@ -218,3 +218,16 @@ def test_dense_u32_shape():
     assert v["count"][4] == 4 + 1024 and v["count"][5] == n
     q = np.array([0, 5, n - 1, n, 1 << 30], np.uint32)
     assert C.Layout(keys, keys.astype(np.uint64) + 1, lut_bytes=3).lookup(q).tolist() == [1, 6, n, MISS, MISS]
+
+
+def test_sector_walker_wide_root_table():
+    """cuart_layout_sectors_ex(WIDE) counts the path of the pre-bucketed walk that
+    starts from the wide root table: the 32-B entry carries the target N16's keys,
+    so the N16 key sector disappears (hand count: LUT + N16 keys + child + leaf = 4
+    sectors plain, LUT + child + leaf = 3 wide; a missing last byte 2 vs 1)."""
+    keys = (np.uint32(0x01020300) + np.arange(10, dtype=np.uint32)).astype(np.uint32)
+    lay = C.Layout(keys, np.arange(10, dtype=np.uint64) + 1, lut_bytes=3)
+    q = np.array([0x01020305, 0x010203F0], np.uint32)
+    assert lay.sectors(q).tolist() == [4, 2]
+    assert lay.sectors(q, wide=True).tolist() == [3, 1]
+    lay.close()
