@@ -68,7 +68,8 @@ typedef enum {
     CUART_ERR_INTERNAL = 10
 } cuart_status;
 
-typedef enum { CUART_KEY_U32 = 1, CUART_KEY_U64 = 2, CUART_KEY_BYTES = 3 } cuart_key_kind;
+typedef enum { CUART_KEY_U32 = 1, CUART_KEY_U64 = 2, CUART_KEY_BYTES = 3,
+               CUART_KEY_LONG = 4 /* f4: 1..255-byte keys, only through the *_long calls */ } cuart_key_kind;
 
 typedef struct {
     cuart_key_kind kind;
@@ -302,6 +303,31 @@ cuart_status cuart_partition_by_flag(const cuart_keys* keys, size_t n, const uin
  * scratch of steps 1-2: cuart_route_scratch_bytes(n, nparts), kept between the
  * two calls.  nparts <= 16.  All pointers are device pointers (local or mapped
  * peer memory); calls are async on `stream`. */
+/* ---- keys longer than 32 bytes (§8(f) f4; §3.2.3, option 2) ----------
+ * An index of kind CUART_KEY_LONG holds prefix-free byte-string keys of 1..255
+ * bytes.  Its inner nodes and the leaves of keys of <= 32 bytes live on the
+ * device as usual; the leaves of longer keys live in a HOST leaf buffer, and the
+ * device node buffers hold links of type 8 (host leaf) to them.  A GPU walk that
+ * reaches such a link signals the host "compare the complete key against host
+ * leaf #idx" ("it sets a specific signal in the return value indicating
+ * that the CPU needs to compare the complete key along with the address of the
+ * actual leaf in main memory"); the library finishes those compares on the host.
+ * Keys and queries are packed: key i = data[offsets[i], offsets[i+1]) (HOST
+ * pointers, offsets uint64_t[n+1]).  All three calls are synchronous.
+ *   cuart_build_long  : as cuart_build (duplicates: last wins; not prefix-free ->
+ *                       CUART_ERR_NOT_PREFIX_FREE; length 0 or > 255 -> KEY_LENGTH)
+ *   cuart_lookup_long : out[i] = value or CUART_MISS (host uint64_t[n])
+ *   cuart_update_long : sequential batch semantics as cuart_update: the
+ *                       device leaves by the two-stage kernels, the host leaves
+ *                       by the host in op order; absent keys are no-ops.
+ * The other calls reject a CUART_KEY_LONG index with CUART_ERR_INVALID_ARGUMENT. */
+cuart_status cuart_build_long(const uint8_t* data, const uint64_t* offsets, const uint64_t* values, size_t n,
+                              const cuart_build_opts* opts, cuart_index** out);
+cuart_status cuart_lookup_long(cuart_index* h, const uint8_t* data, const uint64_t* offsets, size_t n,
+                               uint64_t* out, void* stream);
+cuart_status cuart_update_long(cuart_index* h, const uint8_t* data, const uint64_t* offsets,
+                               const uint64_t* values, size_t n, void* stream);
+
 #define CUART_IPC_HANDLE_BYTES 64
 cuart_status cuart_ipc_alloc(size_t bytes, void** dptr);           /* exportable device window        */
 cuart_status cuart_ipc_free(void* dptr);                           /* NULL ok                         */

@@ -78,6 +78,11 @@ def lib():
         L.cuart_unroute.argtypes = [P, P, S, P, P]
         L.cuart_unroute.restype = ctypes.c_int
         U32 = ctypes.c_uint32
+        for name, args in {"cuart_build_long": [P, P, P, S, P, P], "cuart_lookup_long": [P, P, P, S, P, P],
+                           "cuart_update_long": [P, P, P, P, S, P]}.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = ctypes.c_int
         for name, args in {"cuart_ipc_alloc": [S, P], "cuart_ipc_free": [P], "cuart_ipc_export": [P, P],
                            "cuart_ipc_import": [P, P], "cuart_ipc_close": [P],
                            "cuart_route_count": [P, S, P, U32, P, P, P],
@@ -518,3 +523,46 @@ def update_raw(h, keys_struct, n, values_ptr, stream=None):
 
 def unroute_raw(in_ptr, perm_ptr, n, out_ptr, stream=None):
     _check(lib().cuart_unroute(in_ptr, perm_ptr, n, out_ptr, _stream_ptr(stream)), "cuart_unroute")
+
+
+# ------------------------------------------------------------------ f4: keys longer than 32 bytes
+def pack_long(keys):
+    """list of bytes -> (data uint8[total], offsets uint64[n+1]) (packed form of the *_long calls)."""
+    lens = np.fromiter((len(k) for k in keys), dtype=np.uint64, count=len(keys))
+    offsets = np.zeros(len(keys) + 1, dtype=np.uint64)
+    np.cumsum(lens, out=offsets[1:])
+    data = np.frombuffer(b"".join(keys), dtype=np.uint8) if keys else np.zeros(1, np.uint8)
+    return np.ascontiguousarray(data), offsets
+
+
+class LongIndex:
+    """CUART_KEY_LONG index (§8(f) f4, P:126 option 2): keys of 1..255 bytes; leaves of
+    keys > 32 bytes live in host memory and the host finishes their compares."""
+
+    def __init__(self, keys, values, lut_bytes=0, device=-1):
+        data, off = pack_long(keys)
+        v = np.ascontiguousarray(values, dtype=np.uint64)
+        if v.shape[0] != len(keys):
+            raise ValueError("values length mismatch")
+        h = ctypes.c_void_p()
+        o = _opts(lut_bytes, 0, device, 0, 0, 0, 0)
+        _check(lib().cuart_build_long(_ptr(data), _ptr(off), _ptr(v), len(keys), ctypes.byref(o), ctypes.byref(h)),
+               "cuart_build_long")
+        self.h = h.value
+
+    def lookup(self, queries):
+        data, off = pack_long(queries)
+        out = np.empty(len(queries), dtype=np.uint64)
+        _check(lib().cuart_lookup_long(self.h, _ptr(data), _ptr(off), len(queries), _ptr(out), None),
+               "cuart_lookup_long")
+        return out
+
+    def update(self, keys, values):
+        data, off = pack_long(keys)
+        v = np.ascontiguousarray(values, dtype=np.uint64)
+        _check(lib().cuart_update_long(self.h, _ptr(data), _ptr(off), _ptr(v), len(keys), None), "cuart_update_long")
+
+    def close(self):
+        if self.h:
+            cuart_destroy(self.h)
+            self.h = None

@@ -27,17 +27,23 @@ namespace {
 
 struct SortedKeys {
     uint32_t fixed_len = 0;             // 4 / 8 for integer kinds, 0 for byte strings
+    bool is_long = false;               // CUART_KEY_LONG: variable-length keys in lbytes / loff
     std::vector<uint64_t> ik;           // integer kinds: numeric key (big-endian byte order = numeric order)
     std::vector<uint8_t> slots;         // byte strings: n x 32 zero-padded
     std::vector<uint8_t> lens;
+    std::vector<uint8_t> lbytes;        // long keys: concatenated, sorted
+    std::vector<uint64_t> loff;         // long keys: [n + 1]
     std::vector<uint64_t> vals;
     uint64_t n = 0;
 
+    inline const uint8_t* kptr(uint64_t i) const { return is_long ? &lbytes[loff[i]] : &slots[i * kMaxKey]; }
     inline uint32_t byte(uint64_t i, uint32_t d) const {
         if (fixed_len) return uint32_t(ik[i] >> (8 * (fixed_len - 1 - d))) & 0xFF;
-        return slots[i * kMaxKey + d];
+        return kptr(i)[d];
     }
-    inline uint32_t len(uint64_t i) const { return fixed_len ? fixed_len : lens[i]; }
+    inline uint32_t len(uint64_t i) const {
+        return fixed_len ? fixed_len : is_long ? uint32_t(loff[i + 1] - loff[i]) : lens[i];
+    }
     // Equal bytes of keys i and j from byte `from` on, bounded by the shorter key.
     inline uint32_t lcp(uint64_t i, uint64_t j, uint32_t from) const {
         if (fixed_len) {
@@ -45,9 +51,9 @@ struct SortedKeys {
             uint32_t total = x ? uint32_t(__builtin_clzll(x) - (64 - 8 * fixed_len)) / 8 : fixed_len;
             return total - from;
         }
-        uint32_t m = std::min(lens[i], lens[j]);
-        const uint8_t* a = &slots[i * kMaxKey];
-        const uint8_t* b = &slots[j * kMaxKey];
+        uint32_t m = std::min(len(i), len(j));
+        const uint8_t* a = kptr(i);
+        const uint8_t* b = kptr(j);
         uint32_t p = from;
         while (p < m && a[p] == b[p]) p++;
         return p - from;
@@ -56,7 +62,7 @@ struct SortedKeys {
         if (fixed_len) {
             for (uint32_t b = 0; b < fixed_len; b++) dst[b] = uint8_t(ik[i] >> (8 * (fixed_len - 1 - b)));
         } else {
-            memcpy(dst, &slots[i * kMaxKey], lens[i]);
+            memcpy(dst, kptr(i), len(i));
         }
     }
     inline uint64_t prefix_k(uint64_t i, uint32_t k) const {
@@ -79,10 +85,49 @@ inline uint64_t load_be64(const uint8_t* p) {
     return v;
 }
 
+// f4: variable-length keys (1..255 B): sort the key indices lexicographically
+// (shorter first on a common prefix), keep the LAST occurrence of a duplicate
+// (reading C6), check prefix-freeness (reading C3).
+int canonicalize_long(const uint8_t* data, const uint64_t* off, const uint64_t* values, uint64_t n, SortedKeys& S) {
+    for (uint64_t i = 0; i < n; i++) {
+        if (off[i + 1] < off[i]) return CUART_ERR_INVALID_ARGUMENT;
+        const uint64_t l = off[i + 1] - off[i];
+        if (l == 0 || l > kMaxLongKey) return CUART_ERR_KEY_LENGTH;
+    }
+    std::vector<uint64_t> ord(n);
+    for (uint64_t i = 0; i < n; i++) ord[i] = i;
+    auto cmp3 = [&](uint64_t a, uint64_t b) {
+        const uint64_t la = off[a + 1] - off[a], lb = off[b + 1] - off[b];
+        const int c = memcmp(data + off[a], data + off[b], std::min(la, lb));
+        return c != 0 ? c : (la < lb ? -1 : la > lb ? 1 : 0);
+    };
+    __gnu_parallel::sort(ord.begin(), ord.end(), [&](uint64_t a, uint64_t b) {
+        const int c = cmp3(a, b);
+        return c != 0 ? c < 0 : a < b;
+    });
+    S.is_long = true;
+    S.loff.push_back(0);
+    for (uint64_t i = 0; i < n; i++) {
+        if (i + 1 < n && cmp3(ord[i], ord[i + 1]) == 0) continue;
+        const uint64_t k = ord[i], l = off[k + 1] - off[k];
+        S.lbytes.insert(S.lbytes.end(), data + off[k], data + off[k] + l);
+        S.loff.push_back(S.lbytes.size());
+        S.vals.push_back(values[k]);
+    }
+    S.n = S.vals.size();
+    for (uint64_t j = 0; j + 1 < S.n; j++)
+        if (S.len(j) < S.len(j + 1) && S.lcp(j, j + 1, 0) >= S.len(j)) return CUART_ERR_NOT_PREFIX_FREE;
+    return CUART_OK;
+}
+
 int canonicalize(uint32_t kind, const void* data, const uint8_t* lengths, const uint64_t* values, uint64_t n,
-                 SortedKeys& S) {
+                 SortedKeys& S, const uint64_t* long_offsets) {
     for (uint64_t i = 0; i < n; i++)
         if (values[i] == kMiss) return CUART_ERR_RESERVED_VALUE;
+    if (kind == CUART_KEY_LONG) {
+        if (!long_offsets) return CUART_ERR_INVALID_ARGUMENT;
+        return canonicalize_long((const uint8_t*)data, long_offsets, values, n, S);
+    }
     if (kind == CUART_KEY_U64 || kind == CUART_KEY_U32) {
         S.fixed_len = kind == CUART_KEY_U64 ? 8 : 4;
         std::vector<std::pair<uint64_t, uint64_t>> kv(n);
@@ -175,8 +220,8 @@ inline uint64_t* child_slot(HostLayout& L, uint32_t type, uint64_t idx, uint32_t
 }  // namespace
 
 int build_host_layout(uint32_t kind, const void* data, const uint8_t* lengths, const uint64_t* values, uint64_t n,
-                      uint32_t lut_bytes, HostLayout& L) {
-    if (kind < CUART_KEY_U32 || kind > CUART_KEY_BYTES) return CUART_ERR_INVALID_ARGUMENT;
+                      uint32_t lut_bytes, HostLayout& L, const uint64_t* long_offsets) {
+    if (kind < CUART_KEY_U32 || kind > CUART_KEY_LONG) return CUART_ERR_INVALID_ARGUMENT;
     if (lut_bytes > 3) return CUART_ERR_INVALID_ARGUMENT;
     if (n > 0 && (data == nullptr || values == nullptr)) return CUART_ERR_INVALID_ARGUMENT;
     L = HostLayout();
@@ -184,7 +229,7 @@ int build_host_layout(uint32_t kind, const void* data, const uint8_t* lengths, c
     L.lut_bytes = lut_bytes;
     SortedKeys S;
     if (n > 0) {
-        int rc = canonicalize(kind, data, lengths, values, n, S);
+        int rc = canonicalize(kind, data, lengths, values, n, S, long_offsets);
         if (rc != CUART_OK) return rc;
     }
     L.n_keys = S.n;
@@ -192,19 +237,29 @@ int build_host_layout(uint32_t kind, const void* data, const uint8_t* lengths, c
     const uint32_t K = lut_bytes;
 
     // leaf class ranks: leaves are numbered in lexicographic order per class
+    auto leaf_type = [](uint32_t len) { return len > kMaxKey ? uint32_t(T_LEAF_HOST) : leaf_type_for_len(len); };
     std::vector<uint64_t> leaf_rank(S.n);
     {
-        uint64_t c[8] = {0};
-        for (uint64_t i = 0; i < S.n; i++) leaf_rank[i] = c[leaf_type_for_len(S.len(i))]++;
+        uint64_t c[9] = {0};
+        for (uint64_t i = 0; i < S.n; i++) leaf_rank[i] = c[leaf_type(S.len(i))]++;
         for (uint32_t t = T_LEAF8; t <= T_LEAF32; t++) {
             L.count[t] = c[t];
             if (c[t] > kIndexMask) return CUART_ERR_TOO_LARGE;
             L.buf[t].assign(c[t] * kRecordBytes[t], 0);
         }
+        // f4: host-resident long leaves, in lexicographic order like every leaf class
+        L.long_off.assign(1, 0);
+        for (uint64_t i = 0; i < S.n; i++) {
+            if (leaf_type(S.len(i)) != T_LEAF_HOST) continue;
+            L.long_bytes.insert(L.long_bytes.end(), S.kptr(i), S.kptr(i) + S.len(i));
+            L.long_off.push_back(L.long_bytes.size());
+            L.long_vals.push_back(S.vals[i]);
+        }
     }
     auto write_leaf = [&](uint64_t i) -> uint64_t {
         uint32_t len = S.len(i);
-        uint32_t t = leaf_type_for_len(len);
+        uint32_t t = leaf_type(len);
+        if (t == T_LEAF_HOST) return make_link(t, len, leaf_rank[i]);
         uint8_t* rec = L.buf[t].data() + leaf_rank[i] * kRecordBytes[t];
         S.write_key(i, rec);
         memcpy(rec + kLeafValueOff[t], &S.vals[i], 8);

@@ -17,11 +17,18 @@ struct HostLayout {
     std::vector<uint64_t> lut;             // 2^(8*lut_bytes) links, or empty
     uint64_t n_keys = 0;
     uint32_t max_depth = 0;
+    // f4 (CUART_KEY_LONG): host-resident leaves of keys longer than kMaxKey (P:126
+    // option 2), in lexicographic order; link T_LEAF_HOST, index = position here.
+    std::vector<uint8_t> long_bytes;       // concatenated keys
+    std::vector<uint64_t> long_off;        // [count + 1] offsets into long_bytes
+    std::vector<uint64_t> long_vals;
 };
 
 // Status codes mirror cuart_status (include/cuart.h).
+// kind CUART_KEY_LONG: data = concatenated key bytes, `long_offsets` = uint64_t[n+1]
+// (key i = data[off[i], off[i+1]), length 1..255), `lengths` unused.
 int build_host_layout(uint32_t kind, const void* data, const uint8_t* lengths, const uint64_t* values,
-                      uint64_t n, uint32_t lut_bytes, HostLayout& out);
+                      uint64_t n, uint32_t lut_bytes, HostLayout& out, const uint64_t* long_offsets = nullptr);
 
 // Multi-threaded CPU walk over the flat layout (§4.2, Fig. 7).
 void host_layout_lookup(const HostLayout& L, uint32_t kind, const void* queries, const uint8_t* lengths,

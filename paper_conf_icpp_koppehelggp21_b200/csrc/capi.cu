@@ -83,6 +83,9 @@ struct cuart_index {
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev;
     uint64_t klookups = 0;
     uint64_t kslice = 0;               // timed launches that were k_lookup_slice
+    // f4 (CUART_KEY_LONG): host-resident leaves of the keys longer than 32 bytes
+    std::vector<uint8_t> long_bytes;
+    std::vector<uint64_t> long_off, long_vals;
     uint32_t prebucket = CUART_PREBUCKET_AUTO;   // a5: reorder large lookup batches by bucket (bucket.cuh)
     uint32_t slice_lut = CUART_SLICE_AUTO;       // bucketed walk with the bucket's LUT slice in smem
     bool slice_ok = false;                       // RANK table, integer keys, root branch depth + 2 <= k
@@ -128,6 +131,25 @@ __global__ void __launch_bounds__(256) k_lookup(DevIndex ix, const void* __restr
         uint64_t* dst = SEG ? so.at(i) : out + i;
         if (POL != 0) __stcs((unsigned long long*)dst, (unsigned long long)r);
         else *dst = r;
+    }
+}
+
+// f4 (P:126 option 2): the walk for CUART_KEY_LONG queries.  A query ending at a
+// host-leaf link returns the leaf's host index with sig[i] = 1 ("the CPU needs to
+// compare the complete key"); every other query is final (sig[i] = 0).
+template <int POL>
+__global__ void __launch_bounds__(256) k_lookup_long(DevIndex ix, const uint8_t* __restrict__ q,
+                                                     const uint64_t* __restrict__ off, uint64_t n,
+                                                     uint64_t* __restrict__ out, uint8_t* __restrict__ sig) {
+    const Loader<POL> ld;
+    const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+    for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const KeyLong key = KeyLong::load<true>(q, (const uint8_t*)off, i);
+        uint64_t val = kMiss;
+        const uint64_t leaf = find_leaf(ix, ld, key, start_link(ix, ld, key), val);
+        const bool host = leaf && link_type(leaf) == T_LEAF_HOST;
+        out[i] = host ? link_index(leaf) : (leaf ? val : kMiss);
+        sig[i] = host ? 1 : 0;
     }
 }
 
@@ -234,7 +256,9 @@ __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restric
         leafref[i] = leaf;
         if (DEL) slotref[i] = slot;
         const uint64_t prio = opidx ? uint64_t(opidx[i]) : i;      // priority = original op index
-        if (leaf) atomicMax((unsigned long long*)winner_word(ix, leaf), (unsigned long long)(epoch_hi | prio));
+        // f4: a host leaf (link type 8) is resolved by the host after the kernels
+        if (leaf && (Key::kKind != 4 || link_type(leaf) != T_LEAF_HOST))
+            atomicMax((unsigned long long*)winner_word(ix, leaf), (unsigned long long)(epoch_hi | prio));
     }
 }
 
@@ -251,7 +275,7 @@ __global__ void __launch_bounds__(256) k_upd2(DevIndex ix, const uint64_t* __res
     const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
     for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
         const uint64_t leaf = leafref[i];
-        if (!leaf) continue;
+        if (!leaf || link_type(leaf) == T_LEAF_HOST) continue;   // f4: host leaves are applied by the host
         const uint64_t gid = global_leaf_id(ix, leaf);
         const uint64_t prio = opidx ? uint64_t(opidx[i]) : i;
         if (__ldcg(winner_word(ix, leaf)) != (epoch_hi | prio)) continue;
@@ -285,6 +309,7 @@ static int grid_for(const cuart_index* h, uint64_t n) {
 
 static cuart_status check_keys(const cuart_index* h, const cuart_keys* k, size_t n) {
     if (!h || !k) return CUART_ERR_INVALID_ARGUMENT;
+    if (k->kind == CUART_KEY_LONG || h->key_kind == CUART_KEY_LONG) return CUART_ERR_INVALID_ARGUMENT;   // *_long calls
     if (n > 0 && k->data == nullptr) return CUART_ERR_INVALID_ARGUMENT;
     if (uint32_t(k->kind) != h->key_kind) return CUART_ERR_INVALID_ARGUMENT;
     if (k->kind == CUART_KEY_BYTES && n > 0 && k->lengths == nullptr) return CUART_ERR_INVALID_ARGUMENT;
@@ -493,6 +518,7 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
         switch (kind) {
         case CUART_KEY_U64: CUART_UPD1_POL(KeyU64); break;
         case CUART_KEY_U32: CUART_UPD1_POL(KeyU32); break;
+        case CUART_KEY_LONG: CUART_UPD1_POL(KeyLong); break;
         default: CUART_UPD1_POL(KeyBytes); break;
         }
 #undef CUART_UPD1_POL
@@ -739,6 +765,9 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, dev);
     h->key_kind = L.key_kind;
     h->lut_bytes = L.lut_bytes;
+    h->long_bytes = L.long_bytes;
+    h->long_off = L.long_off;
+    h->long_vals = L.long_vals;
     h->root = L.root;
     h->n_keys = L.n_keys;
     h->max_depth = L.max_depth;
@@ -759,7 +788,8 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     std::vector<uint64_t> lutr;
     uint32_t fmt = opts ? opts->lut_format : CUART_LUT_FORMAT_AUTO;
     if (L.lut.empty()) fmt = CUART_LUT_LINKS;
-    if (fmt == CUART_LUT_FORMAT_AUTO) fmt = (L.key_kind == CUART_KEY_BYTES) ? CUART_LUT_LINKS : CUART_LUT_RANK;
+    if (fmt == CUART_LUT_FORMAT_AUTO) fmt = (L.key_kind >= CUART_KEY_BYTES) ? CUART_LUT_LINKS : CUART_LUT_RANK;
+    if (L.key_kind == CUART_KEY_LONG) fmt = CUART_LUT_LINKS;
     if (fmt == CUART_LUT_RANK && !rank_lut(L, lutr, h->lut_exceptions)) fmt = CUART_LUT_LINKS;
     if (fmt == CUART_LUT_COMPACT32 && !compact_lut(L, lut32)) fmt = CUART_LUT_LINKS;
     if (fmt < CUART_LUT_LINKS || fmt > CUART_LUT_RANK) {
@@ -966,6 +996,125 @@ cuart_status cuart_destroy(cuart_index* h) {
         if (h->streams[i]) cudaStreamDestroy(h->streams[i]);
     }
     delete h;
+    return CUART_OK;
+}
+
+// ---------------------------------------------------------------- f4: long keys
+cuart_status cuart_build_long(const uint8_t* data, const uint64_t* offsets, const uint64_t* values, size_t n,
+                              const cuart_build_opts* opts, cuart_index** out) {
+    if (!out || (n > 0 && (!data || !offsets || !values))) return CUART_ERR_INVALID_ARGUMENT;
+    *out = nullptr;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return CUART_ERR_NO_DEVICE;
+    uint32_t lut = opts ? opts->lut_bytes : 0;
+    if (lut == CUART_LUT_AUTO) lut = 0;
+    cuart_layout* l = new (std::nothrow) cuart_layout();
+    if (!l) return CUART_ERR_OOM;
+    int rc;
+    try {
+        rc = build_host_layout(CUART_KEY_LONG, data, nullptr, values, n, lut, l->L, offsets);
+    } catch (const std::bad_alloc&) {
+        rc = CUART_ERR_OOM;
+    }
+    if (rc == CUART_OK) rc = cuart_upload(l, opts, out);
+    cuart_layout_free(l);
+    return cuart_status(rc);
+}
+
+// Upload a packed host batch (data, offsets) to fresh device buffers on stream s.
+static cuart_status upload_long_batch(const uint8_t* data, const uint64_t* offsets, size_t n, cudaStream_t s,
+                                      uint8_t** dq, uint64_t** doff) {
+    const uint64_t nb = offsets[n];
+    CU_TRY(cudaMallocAsync((void**)dq, nb ? nb : 1, s));
+    CU_TRY(cudaMallocAsync((void**)doff, (n + 1) * 8, s));
+    CU_TRY(cudaMemcpyAsync(*dq, data, nb, cudaMemcpyHostToDevice, s));
+    CU_TRY(cudaMemcpyAsync(*doff, offsets, (n + 1) * 8, cudaMemcpyHostToDevice, s));
+    return CUART_OK;
+}
+
+static bool long_key_equal(const cuart_index* h, uint64_t idx, const uint8_t* key, uint64_t len) {
+    const uint64_t a = h->long_off[idx], b = h->long_off[idx + 1];
+    return b - a == len && memcmp(h->long_bytes.data() + a, key, len) == 0;
+}
+
+static cuart_status check_long_batch(const cuart_index* h, const uint8_t* data, const uint64_t* offsets, size_t n) {
+    if (!h || h->key_kind != CUART_KEY_LONG) return CUART_ERR_INVALID_ARGUMENT;
+    if (n > 0 && (!data || !offsets)) return CUART_ERR_INVALID_ARGUMENT;
+    if (n >= (uint64_t(1) << 30)) return CUART_ERR_INVALID_ARGUMENT;
+    for (size_t i = 0; i < n; i++) {
+        if (offsets[i + 1] < offsets[i]) return CUART_ERR_INVALID_ARGUMENT;
+        const uint64_t l = offsets[i + 1] - offsets[i];
+        if (l == 0 || l > kMaxLongKey) return CUART_ERR_KEY_LENGTH;
+    }
+    return CUART_OK;
+}
+
+cuart_status cuart_lookup_long(cuart_index* h, const uint8_t* data, const uint64_t* offsets, size_t n, uint64_t* out,
+                               void* stream) {
+    cuart_status rc = check_long_batch(h, data, offsets, n);
+    if (rc != CUART_OK) return rc;
+    if (n == 0) return CUART_OK;
+    if (!out) return CUART_ERR_INVALID_ARGUMENT;
+    CU_TRY(cudaSetDevice(h->device));
+    cudaStream_t s = (cudaStream_t)stream;
+    uint8_t* dq = nullptr;
+    uint64_t* doff = nullptr;
+    if ((rc = upload_long_batch(data, offsets, n, s, &dq, &doff)) != CUART_OK) return rc;
+    uint64_t* dout = nullptr;
+    uint8_t* dsig = nullptr;
+    CU_TRY(cudaMallocAsync((void**)&dout, n * 8, s));
+    CU_TRY(cudaMallocAsync((void**)&dsig, n, s));
+    k_lookup_long<5><<<grid_for(h, n), 256, 0, s>>>(h->dix, dq, doff, n, dout, dsig);
+    g_cuart_launches++;
+    CU_TRY(cudaGetLastError());
+    std::vector<uint8_t> sig(n);
+    CU_TRY(cudaMemcpyAsync(out, dout, n * 8, cudaMemcpyDeviceToHost, s));
+    CU_TRY(cudaMemcpyAsync(sig.data(), dsig, n, cudaMemcpyDeviceToHost, s));
+    CU_TRY(cudaFreeAsync(dq, s));
+    CU_TRY(cudaFreeAsync(doff, s));
+    CU_TRY(cudaFreeAsync(dout, s));
+    CU_TRY(cudaFreeAsync(dsig, s));
+    CU_TRY(cudaStreamSynchronize(s));
+    // the host side of P:126 option 2: full-key compare against the host leaf
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < int64_t(n); i++) {
+        if (!sig[i]) continue;
+        const uint64_t idx = out[i];
+        out[i] = long_key_equal(h, idx, data + offsets[i], offsets[i + 1] - offsets[i]) ? h->long_vals[idx] : kMiss;
+    }
+    return CUART_OK;
+}
+
+cuart_status cuart_update_long(cuart_index* h, const uint8_t* data, const uint64_t* offsets, const uint64_t* values,
+                               size_t n, void* stream) {
+    cuart_status rc = check_long_batch(h, data, offsets, n);
+    if (rc != CUART_OK) return rc;
+    if (n == 0) return CUART_OK;
+    if (!values) return CUART_ERR_INVALID_ARGUMENT;
+    CU_TRY(cudaSetDevice(h->device));
+    cudaStream_t s = (cudaStream_t)stream;
+    uint8_t* dq = nullptr;
+    uint64_t* doff = nullptr;
+    if ((rc = upload_long_batch(data, offsets, n, s, &dq, &doff)) != CUART_OK) return rc;
+    uint64_t* dval = nullptr;
+    CU_TRY(cudaMallocAsync((void**)&dval, n * 8, s));
+    CU_TRY(cudaMemcpyAsync(dval, values, n * 8, cudaMemcpyHostToDevice, s));
+    // device leaves: the two-stage kernels; host leaves: stage 1 leaves their links in leafref
+    rc = launch_update(h, CUART_KEY_LONG, dq, (const uint8_t*)doff, dval, nullptr, 0, n, s);
+    if (rc != CUART_OK) return rc;
+    std::vector<uint64_t> ref(n);
+    CU_TRY(cudaMemcpyAsync(ref.data(), h->leafref, n * 8, cudaMemcpyDeviceToHost, s));
+    CU_TRY(cudaFreeAsync(dq, s));
+    CU_TRY(cudaFreeAsync(doff, s));
+    CU_TRY(cudaFreeAsync(dval, s));
+    CU_TRY(cudaStreamSynchronize(s));
+    // host leaves in op order: sequential semantics, the last op on a key wins
+    for (size_t i = 0; i < n; i++) {
+        const uint64_t l = ref[i];
+        if (!l || link_type(l) != T_LEAF_HOST) continue;
+        const uint64_t idx = link_index(l);
+        if (long_key_equal(h, idx, data + offsets[i], offsets[i + 1] - offsets[i])) h->long_vals[idx] = values[i];
+    }
     return CUART_OK;
 }
 

@@ -183,6 +183,36 @@ struct KeyBytes {
     }
 };
 
+// f4 (CUART_KEY_LONG): a 1..255-byte key read in place from the packed query
+// buffer (key i = q[off[i], off[i+1]); `lens` carries the offsets array).
+struct KeyLong {
+    const uint8_t* p;
+    uint32_t l;
+    static constexpr uint32_t kKind = 4;
+    template <bool STREAM>
+    __device__ __forceinline__ static KeyLong load(const void* q, const uint8_t* offs, uint64_t i) {
+        const uint64_t* off = (const uint64_t*)offs;
+        const uint64_t a = off[i], b = off[i + 1];
+        return KeyLong{(const uint8_t*)q + a, uint32_t(b - a)};
+    }
+    __device__ __forceinline__ uint32_t len() const { return l; }
+    __device__ __forceinline__ uint32_t byte(uint32_t d) const { return __ldg(p + d); }
+    __device__ __forceinline__ uint64_t prefix(uint32_t nb) const {
+        uint64_t v = 0;
+        for (uint32_t b = 0; b < nb; b++) v = (v << 8) | byte(b);
+        return v;
+    }
+    // device leaves hold keys of <= 32 bytes: equal length, then byte for byte
+    template <class LD>
+    __device__ __forceinline__ bool leaf_match(const LD&, const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
+        val = ld_cg_u64(rec + leaf_value_off(t));
+        if (aux != l) return false;
+        for (uint32_t b = 0; b < l; b++)
+            if (rec[b] != byte(b)) return false;
+        return true;
+    }
+};
+
 // Count of key bytes < b among 4 packed bytes (sorted keys; padding repeats the last key).
 __device__ __forceinline__ void search4(uint32_t keys, uint32_t bb, uint32_t& less, uint32_t& eq) {
     less = __popc(__vcmpltu4(keys, bb)) >> 3;
@@ -295,6 +325,10 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Loader<P
         const uint32_t t = link_type(link);
         const uint64_t idx = link_index(link);
         const uint32_t aux = link_aux(link);
+        if (Key::kKind == 4 && t == T_LEAF_HOST) {   // f4: host leaf -> signal (the caller finishes on the host)
+            val = idx;
+            return link;
+        }
         if (t >= T_LEAF8) {
             const uint8_t* rec = ix.base[t] + idx * record_bytes(t);
             return key.leaf_match(ld, rec, t, aux, val) ? link : 0;
