@@ -108,9 +108,14 @@ typedef struct {
     uint32_t wide_lut;           /* pre-bucketed walks start from a wide root table: 32 B per
                                     entry = the link + the sorted keys of the N4 / N16 it
                                     points to ("merged top layers"), so the first
-                                    node's key read is skipped.  CUART_WIDE_AUTO (on when
-                                    most entries lead to an N4/N16), CUART_WIDE_OFF,
-                                    CUART_WIDE_ON.  Results are identical.                 */
+                                    node's key read is skipped, + the node's leaf run (when
+                                    all its children are leaves they are consecutive in the
+                                    ordered leaf buffer, so child i = run + i and the
+                                    child-link read is skipped too; for a full N256 of
+                                    leaves child b = run + b).  CUART_WIDE_AUTO (on when
+                                    most entries lead to an N4/N16 or a full N256 of
+                                    leaves), CUART_WIDE_OFF, CUART_WIDE_ON.  Results are
+                                    identical.                                             */
 } cuart_build_opts;
 #define CUART_WIDE_AUTO 0u
 #define CUART_WIDE_OFF 1u

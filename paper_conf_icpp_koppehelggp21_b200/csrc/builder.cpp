@@ -412,7 +412,10 @@ uint64_t walk_one(const HostLayout& L, const uint8_t* key, uint32_t len, uint32_
         link = L.lut[p];
         s += sectors(p * (wide ? 32 : 8), wide ? 32 : 8);
         const uint32_t t = link_type(link);
-        if (wide && (t == T_N4 || t == T_N16)) {
+        if (wide && t == T_N256 && link_aux(link) < len &&
+            leaf_run_link(L.buf[t].data() + link_index(link) * kRecordBytes[t], t)) {   // full N256 of leaves
+            memcpy(&link, L.buf[t].data() + link_index(link) * kRecordBytes[t] + kN256Child + 8 * key[link_aux(link)], 8);
+        } else if (wide && (t == T_N4 || t == T_N16)) {
             const uint32_t d = link_aux(link);
             if (d >= len) return kMiss;
             const uint64_t roff = link_index(link) * kRecordBytes[t];
@@ -423,7 +426,8 @@ uint64_t walk_one(const HostLayout& L, const uint8_t* key, uint32_t len, uint32_
             for (uint32_t j = 0; j < nk; j++) { less += keys[j] < key[d]; eq |= keys[j] == key[d]; }
             if (!eq) return kMiss;
             const uint64_t co = roff + (t == T_N4 ? kN4Child : kN16Child) + 8 * less;
-            s += sectors(co, 8);
+            const uint64_t run = leaf_run_link(rec, t);   // leaf run: no child-link read
+            if (!run) s += sectors(co, 8);
             memcpy(&link, L.buf[t].data() + co, 8);
         }
     }

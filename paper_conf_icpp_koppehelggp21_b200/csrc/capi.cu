@@ -79,6 +79,7 @@ struct cuart_index {
     uint64_t lut_exceptions = 0;       // RANK: entries served by the 64-bit table
     int grid_ctas_per_sm = 0;          // 0 = default grid (one op per thread); else persistent grid
     bool ktimer = false;               // record CUDA events around every k_lookup launch
+    int ilp = 2;                       // queries per thread of the pre-bucketed wide walk (k_lookup_wq)
     std::mutex kmu;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev;
     uint64_t klookups = 0;
@@ -131,6 +132,54 @@ __global__ void __launch_bounds__(256) k_lookup(DevIndex ix, const void* __restr
         uint64_t* dst = SEG ? so.at(i) : out + i;
         if (POL != 0) __stcs((unsigned long long*)dst, (unsigned long long)r);
         else *dst = r;
+    }
+}
+
+// Pre-bucketed walk from the wide root table with Q queries per thread in lockstep
+// phases (integer keys): all Q keys, then all Q wide entries, then all Q leaf
+// records are requested before any of them is used, so a thread keeps Q
+// independent dependent-load chains in flight (the one-query walk is bound by the
+// latency of its chain: 64 warps/SM x 32 queries per ~2 us).  Queries whose path
+// is not "wide entry -> leaf" finish with the generic find_leaf.  Results are
+// identical to k_lookup.
+template <class Key, int POL, int Q, bool SEG = false>
+__global__ void __launch_bounds__(256) k_lookup_wq(DevIndex ix, const void* __restrict__ q,
+                                                   const uint8_t* __restrict__ lens, uint64_t n,
+                                                   uint64_t* __restrict__ out, SegOut so = SegOut{}) {
+    static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
+    const Loader<POL> ld;
+    const uint64_t i0 = uint64_t(blockIdx.x) * (256 * Q) + threadIdx.x;
+    Key k[Q];
+#pragma unroll
+    for (int j = 0; j < Q; j++) {
+        const uint64_t i = i0 + uint64_t(j) * 256;
+        k[j] = i < n ? Key::template load<true>(q, lens, i) : Key{0};
+    }
+    U8x32 e[Q];
+#pragma unroll
+    for (int j = 0; j < Q; j++) e[j] = ld.lutv8(ix.lutw + k[j].prefix(ix.lut_bytes) * 4);
+    uint64_t link[Q];
+#pragma unroll
+    for (int j = 0; j < Q; j++) link[j] = decode_wide(ix, ld, k[j], e[j]);
+    uint4 r[Q];
+#pragma unroll
+    for (int j = 0; j < Q; j++)
+        if (link_type(link[j]) == T_LEAF8) r[j] = ld.leafv4(ix.base[T_LEAF8] + link_index(link[j]) * record_bytes(T_LEAF8));
+#pragma unroll
+    for (int j = 0; j < Q; j++) {
+        const uint64_t i = i0 + uint64_t(j) * 256;
+        if (i >= n) continue;
+        uint64_t res = kMiss;
+        if (link_type(link[j]) == T_LEAF8) {
+            const uint64_t kb = Key::kKind == 2 ? bswap64(uint64_t(k[j].k)) : uint64_t(__byte_perm(uint32_t(k[j].k), 0, 0x0123));
+            if (link_aux(link[j]) == k[j].len() && (uint64_t(r[j].x) | (uint64_t(r[j].y) << 32)) == kb)
+                res = uint64_t(r[j].z) | (uint64_t(r[j].w) << 32);
+        } else if (link[j]) {
+            uint64_t val = kMiss;
+            if (find_leaf(ix, ld, k[j], link[j], val)) res = val;
+        }
+        uint64_t* dst = SEG ? so.at(i) : out + i;
+        __stcs((unsigned long long*)dst, (unsigned long long)res);
     }
 }
 
@@ -435,6 +484,18 @@ static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, co
     }
     cudaEvent_t ev0, ev1;
     ktimer_begin(h, s, ev0, ev1);                      // per-launch k_lookup timing (cuart_kernel_timer)
+    if (bucketed && dx.walk_wide && h->policy == 5 && h->ilp > 1 && (kind == CUART_KEY_U64 || kind == CUART_KEY_U32)) {
+        const unsigned g = unsigned((n + 256 * h->ilp - 1) / (256 * h->ilp));
+#define CUART_WQ(K)                                                                              \
+        if (h->ilp == 2) k_lookup_wq<K, 5, 2><<<g, 256, 0, s>>>(dx, q, lens, n, out);            \
+        else k_lookup_wq<K, 5, 4><<<g, 256, 0, s>>>(dx, q, lens, n, out);
+        if (kind == CUART_KEY_U64) { CUART_WQ(KeyU64) } else { CUART_WQ(KeyU32) }
+#undef CUART_WQ
+        g_cuart_launches++;
+        ktimer_end(h, s, ev0, ev1, n);
+        CU_TRY(cudaGetLastError());
+        return CUART_OK;
+    }
 #define CUART_LOOKUP(K, P) k_lookup<K, P><<<grid, 256, 0, s>>>(dx, q, lens, n, out)
 #define CUART_LOOKUP_POL(K)                          \
     switch (h->policy) {                             \
@@ -799,6 +860,7 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     h->lut_format = fmt;
     if (const char* pe = getenv("CUART_POLICY")) h->policy = atoi(pe);
     if (const char* pe = getenv("CUART_GRID_CTAS_PER_SM")) h->grid_ctas_per_sm = atoi(pe);   // tuning knob
+    if (const char* pe = getenv("CUART_ILP")) h->ilp = atoi(pe);   // queries per thread of the wide walk (1, 2, 4)
     h->prebucket = opts ? opts->prebucket : CUART_PREBUCKET_AUTO;
     if (h->prebucket > CUART_PREBUCKET_ON) {
         delete h;
@@ -838,7 +900,8 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         uint64_t small = 0, nonnull = 0;
         for (uint64_t l : L.lut) {
             nonnull += l != 0;
-            small += link_type(l) == T_N4 || link_type(l) == T_N16;
+            small += link_type(l) == T_N4 || link_type(l) == T_N16 ||
+                     (link_type(l) == T_N256 && leaf_run_link(L.buf[T_N256].data() + link_index(l) * record_bytes(T_N256), T_N256));
         }
         h->wide = nonnull > 0 && 2 * small >= nonnull;
     }
@@ -857,8 +920,14 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
             const uint64_t l = L.lut[p];
             lutw[4 * p] = l;
             const uint32_t t = link_type(l);
-            if (t == T_N4) memcpy(&lutw[4 * p + 1], L.buf[t].data() + link_index(l) * record_bytes(t) + kN4Keys, 4);
-            else if (t == T_N16) memcpy(&lutw[4 * p + 1], L.buf[t].data() + link_index(l) * record_bytes(t) + kN16Keys, 16);
+            if (t != T_N4 && t != T_N16 && t != T_N256) continue;
+            const uint8_t* rec = L.buf[t].data() + link_index(l) * record_bytes(t);
+            if (t == T_N256) {                            // full N256 of leaves: child b = run + b
+                lutw[4 * p + 3] = leaf_run_link(rec, t);
+                continue;
+            }
+            memcpy(&lutw[4 * p + 1], rec + (t == T_N4 ? kN4Keys : kN16Keys), t == T_N4 ? 4 : 16);
+            lutw[4 * p + 3] = leaf_run_link(rec, t);      // child i = run + i when all children are leaves
         }
     }
     h->lutw_off = off;

@@ -163,23 +163,37 @@ struct KeyBytes {
         for (uint32_t b = 0; b < nb; b++) p = (p << 8) | byte(b);
         return p;
     }
+    // leaf8: one 16-B request.  leaf16 (32 B, 32-B aligned): one 256-bit request for
+    // key + value.  leaf32 (48 B; 32-B aligned for even indices, 16 mod 32 for odd
+    // ones): a 32-B and a 16-B request in the order the alignment allows, i.e. 2
+    // requests instead of 3 (random L2 requests are what the walk is bound by, §5).
     template <class LD>
     __device__ __forceinline__ bool leaf_match(const LD& ld, const uint8_t* rec, uint32_t t, uint32_t aux, uint64_t& val) const {
-        const uint4 a = ld.leafv4(rec);
-        const uint64_t a0 = uint64_t(a.x) | (uint64_t(a.y) << 32), a1 = uint64_t(a.z) | (uint64_t(a.w) << 32);
         if (t == T_LEAF8) {
-            val = a1;
-            return aux == l && a0 == w[0];
+            const uint4 a = ld.leafv4(rec);
+            val = uint64_t(a.z) | (uint64_t(a.w) << 32);
+            return aux == l && (uint64_t(a.x) | (uint64_t(a.y) << 32)) == w[0];
         }
-        const uint4 b = ld.leafv4(rec + 16);
-        const uint64_t b0 = uint64_t(b.x) | (uint64_t(b.y) << 32), b1 = uint64_t(b.z) | (uint64_t(b.w) << 32);
         if (t == T_LEAF16) {
-            val = b0;
-            return aux == l && a0 == w[0] && a1 == w[1];
+            const U8x32 r = ld.leafv8(rec);
+            val = uint64_t(r.w[4]) | (uint64_t(r.w[5]) << 32);
+            return aux == l && (uint64_t(r.w[0]) | (uint64_t(r.w[1]) << 32)) == w[0] &&
+                   (uint64_t(r.w[2]) | (uint64_t(r.w[3]) << 32)) == w[1];
         }
-        const uint4 c = ld.leafv4(rec + 32);
-        val = uint64_t(c.x) | (uint64_t(c.y) << 32);
-        return aux == l && a0 == w[0] && a1 == w[1] && b0 == w[2] && b1 == w[3];
+        const bool odd = (uintptr_t(rec) & 16) != 0;              // record index odd: rec = 16 mod 32
+        const uint4 a = ld.leafv4(odd ? rec : rec + 32);           // odd: key[0,16)   even: value | conflict
+        const U8x32 b = ld.leafv8(odd ? rec + 16 : rec);           // odd: key[16,32) | value | conflict   even: key[0,32)
+        uint32_t k[8];
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            k[j] = odd ? (&a.x)[j] : b.w[j];
+            k[4 + j] = odd ? b.w[j] : b.w[4 + j];
+        }
+        val = odd ? (uint64_t(b.w[4]) | (uint64_t(b.w[5]) << 32)) : (uint64_t(a.x) | (uint64_t(a.y) << 32));
+        bool eq = aux == l;
+#pragma unroll
+        for (int j = 0; j < 4; j++) eq &= (uint64_t(k[2 * j]) | (uint64_t(k[2 * j + 1]) << 32)) == w[j];
+        return eq;
     }
 };
 
@@ -310,6 +324,9 @@ struct Loader {
     __device__ __forceinline__ uint4 leafv4(const void* p) const {
         return kLeaf64B ? v4<true>(p, drop) : kLeafDrop ? v4(p, drop) : ld_nc_v4(p);
     }
+    __device__ __forceinline__ U8x32 leafv8(const void* p) const {   // p 32-B aligned
+        return kLeaf64B ? v8<true>(p, drop) : kLeafDrop ? v8(p, drop) : ld_nc_v8(p);
+    }
 };
 
 // Walk from `link` to a leaf.  Returns the leaf link on a full-key match (its value
@@ -410,34 +427,48 @@ __device__ __forceinline__ uint64_t expand_lut_rank(const DevIndex& ix, const Lo
 // address of the LUT entry holding the link (bit 0 set for a 32-bit entry), 0 if
 // the start is the root (a root leaf is never unlinked; its tombstone suffices).
 // Wide root table ("merged top layers", B200 reading): entry p is 32 B =
-// {link, the 4 / 16 sorted key bytes of the N4 / N16 it points to, pad}.  One
+// {link, the 4 / 16 sorted key bytes of the N4 / N16 it points to, leaf run or 0}.  One
 // 32-B request brings the start link AND the first node's search keys, so the walk
 // skips that node's key read and loads the child link directly: on c3 one L2
 // request less for every query whose LUT target is an N16, a 32-B request
 // replaced by an 8-B one for N4 targets.  Deletes never change a node's keys (they
 // null child links, reading C18), so the embedded keys stay a superset filter.
 template <class Key, int POL>
-__device__ __forceinline__ uint64_t start_wide(const DevIndex& ix, const Loader<POL>& ld, const Key& key, uint64_t p) {
-    const U8x32 e = ld.lutv8(ix.lutw + p * 4);
+__device__ __forceinline__ uint64_t decode_wide(const DevIndex& ix, const Loader<POL>& ld, const Key& key, const U8x32& e) {
     const uint64_t link = uint64_t(e.w[0]) | (uint64_t(e.w[1]) << 32);
     const uint32_t t = link_type(link);
+    const uint64_t run = uint64_t(e.w[6]) | (uint64_t(e.w[7]) << 32);
+    if (t == T_N256 && run) {                                  // full N256 of leaves: child b = run + b
+        const uint32_t aux = link_aux(link);
+        return aux >= key.len() ? 0 : run + key.byte(aux);
+    }
     if (t != T_N4 && t != T_N16) return link;
     const uint32_t aux = link_aux(link);
     if (aux >= key.len()) return 0;
     const uint32_t bb = key.byte(aux) * 0x01010101u;
     const uint8_t* rec = ix.base[t] + link_index(link) * record_bytes(t);
+    // Leaf run (layout.h leaf_run_link): when every child of the node is a leaf, the
+    // leaves are consecutive in the lexicographically ordered leaf buffer,
+    // so child i's link is run + i and the child-link request disappears too.  A
+    // child nulled by a delete (C18) leaves a tombstoned leaf (value CUART_MISS)
+    // at run + i, which every caller already reads as absent.
     uint32_t l0, e0;
     search4(e.w[2], bb, l0, e0);
     if (t == T_N4) {
         if (e0 == 0) return 0;
-        return ld.node64(rec + kN4Child + 8 * l0);
+        return run ? run + l0 : ld.node64(rec + kN4Child + 8 * l0);
     }
     uint32_t l1, l2, l3, e1, e2, e3;
     search4(e.w[3], bb, l1, e1);
     search4(e.w[4], bb, l2, e2);
     search4(e.w[5], bb, l3, e3);
     if ((e0 | e1 | e2 | e3) == 0) return 0;
-    return ld.node64(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
+    const uint32_t c = l0 + l1 + l2 + l3;
+    return run ? run + c : ld.node64(rec + kN16Child + 8 * c);
+}
+template <class Key, int POL>
+__device__ __forceinline__ uint64_t start_wide(const DevIndex& ix, const Loader<POL>& ld, const Key& key, uint64_t p) {
+    return decode_wide(ix, ld, key, ld.lutv8(ix.lutw + p * 4));
 }
 
 template <class Key, int POL, bool TRACK = false>

@@ -223,11 +223,33 @@ def test_dense_u32_shape():
 def test_sector_walker_wide_root_table():
     """cuart_layout_sectors_ex(WIDE) counts the path of the pre-bucketed walk that
     starts from the wide root table: the 32-B entry carries the target N16's keys,
-    so the N16 key sector disappears (hand count: LUT + N16 keys + child + leaf = 4
-    sectors plain, LUT + child + leaf = 3 wide; a missing last byte 2 vs 1)."""
+    so the N16 key sector disappears, and when all of the N16's children are leaves
+    (consecutive in the ordered leaf buffer) the entry's leaf run replaces the
+    child-link read too (hand count: LUT + N16 keys + child + leaf = 4 sectors plain,
+    LUT + leaf = 2 wide; a missing last byte 2 vs 1).  With one inner child the run
+    is absent and the wide walk reads the child link: LUT + child + leaf = 3."""
     keys = (np.uint32(0x01020300) + np.arange(10, dtype=np.uint32)).astype(np.uint32)
     lay = C.Layout(keys, np.arange(10, dtype=np.uint64) + 1, lut_bytes=3)
     q = np.array([0x01020305, 0x010203F0], np.uint32)
     assert lay.sectors(q).tolist() == [4, 2]
+    assert lay.sectors(q, wide=True).tolist() == [2, 1]
+    lay.close()
+    base = np.uint64(0x0102030000000000)
+    keys = np.concatenate([base + (np.arange(10, dtype=np.uint64) << np.uint64(32)),
+                           base + np.array([0x0A00000001, 0x0A00000002], np.uint64)])
+    lay = C.Layout(keys, np.arange(12, dtype=np.uint64) + 1, lut_bytes=3)
+    q = np.array([base + np.uint64(5 << 32), base + np.uint64(0xF0 << 32)], np.uint64)
+    assert lay.lookup(q).tolist() == [6, MISS]
+    assert lay.sectors(q).tolist() == [4, 2]
     assert lay.sectors(q, wide=True).tolist() == [3, 1]
+    lay.close()
+    # dense u32 (c2 shape): LUT[3 bytes] -> a full N256 whose 256 children are leaves,
+    # so the wide entry's run gives the leaf directly: LUT + N256 child + leaf = 3
+    # plain, LUT + leaf = 2 wide; an absent 3-byte prefix misses at the LUT (1).
+    keys = np.arange(1 << 16, dtype=np.uint32)
+    lay = C.Layout(keys, keys.astype(np.uint64) + 1, lut_bytes=3)
+    q = np.array([5, 70000, 65535], np.uint32)
+    assert lay.lookup(q).tolist() == [6, MISS, 65536]
+    assert lay.sectors(q).tolist() == [3, 1, 3]
+    assert lay.sectors(q, wide=True).tolist() == [2, 1, 2]
     lay.close()

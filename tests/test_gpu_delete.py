@@ -129,3 +129,28 @@ def test_deletes_visible_to_bucketed_wide_walk(fmt, wide):
     mp.update(uk, uv)
     assert np.array_equal(_lookup(on, q), mp.lookup(q))
     on.close()
+
+
+@pytest.mark.parametrize("wide", [0, 2])
+def test_deletes_visible_through_full_n256_leaf_run(wide):
+    """Dense u32 keys (c2 shape): every 3-byte prefix leads to a full N256 whose 256
+    children are consecutive leaves, so the wide root table's leaf run addresses
+    the leaf without the N256 child link (kernels.cuh start_wide).  A delete nulls
+    that child link; the run still reaches the leaf, whose tombstone (C18) must
+    read as absent to lookups and make later updates skip it."""
+    rng = np.random.default_rng(11)
+    keys = np.arange(1 << 18, dtype=np.uint32)
+    vals = rng.integers(0, 2**63, keys.shape[0], dtype=np.uint64)
+    on = C.Index(keys, vals, lut_bytes=3, prebucket=C.PREBUCKET_ON, wide_lut=wide)
+    mp = MapOracle(keys, vals)
+    dk = keys[rng.random(keys.shape[0]) < 0.4]
+    on.erase(_t(dk))
+    mp.apply(dk, None, np.ones(dk.shape[0], bool))
+    q = np.concatenate([keys, rng.integers(0, 2**32, 1 << 16, dtype=np.uint64).astype(np.uint32)])
+    assert np.array_equal(_lookup(on, q), mp.lookup(q))
+    uk = keys[rng.integers(0, keys.shape[0], 100_000)]
+    uv = rng.integers(0, 2**63, uk.shape[0], dtype=np.uint64)
+    on.update(_t(uk), _t(uv))
+    mp.update(uk, uv)
+    assert np.array_equal(_lookup(on, q), mp.lookup(q))
+    on.close()

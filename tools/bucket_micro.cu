@@ -312,6 +312,204 @@ __global__ void __launch_bounds__(kBucketThreads) s_v4(const uint64_t* __restric
     }
 }
 
+// scatter / gather with more threads per 4096-key tile (THREADS x 4096/THREADS items):
+// more warps per SM to overlap the CTA phases (load -> rank -> scan -> stage -> copy)
+__device__ __forceinline__ unsigned int scan256_wide(unsigned int v, unsigned int* wtot) {
+    // exclusive scan over threads 0..255 (callers pass v for those); all threads sync
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    unsigned int x = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const unsigned int y = __shfl_up_sync(0xffffffffu, x, d);
+        if (lane >= d) x += y;
+    }
+    if (lane == 31 && warp < 8) wtot[warp] = x;
+    __syncthreads();
+    unsigned int before = 0;
+#pragma unroll
+    for (int w = 0; w < 8; w++) before += w < warp ? wtot[w] : 0u;
+    return before + x - v;
+}
+template <int THREADS>
+__global__ void __launch_bounds__(THREADS) s_wide(const uint64_t* __restrict__ q, uint64_t n, uint32_t depth,
+                                                  const unsigned int* __restrict__ rowoff, const unsigned int* __restrict__ bases,
+                                                  uint64_t* __restrict__ bq, uint16_t* __restrict__ jpos) {
+    constexpr int ITEMS = kBucketTile / THREADS;
+    __shared__ uint64_t skeys[kBucketTile];
+    __shared__ uint8_t sb[kBucketTile];
+    __shared__ unsigned int h[kBuckets], loc[kBuckets], glb[kBuckets], wtot[8];
+    const int t = threadIdx.x;
+    unsigned int gb = 0;
+    if (t < kBuckets) { h[t] = 0; gb = bases[t] + rowoff[hidx(t, blockIdx.x)]; }
+    __syncthreads();
+    const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
+    uint64_t kv[ITEMS];
+    uint32_t br[ITEMS];
+#pragma unroll
+    for (int r = 0; r < ITEMS; r++) {
+        const uint32_t j = uint32_t(r) * THREADS + t;
+        kv[r] = j < cnt ? uint64_t(__ldcs((const unsigned long long*)q + base + j)) : 0;
+    }
+#pragma unroll
+    for (int r = 0; r < ITEMS; r++) {
+        const uint32_t j = uint32_t(r) * THREADS + t;
+        br[r] = 0xFFFFFFFFu;
+        if (j < cnt) { const uint32_t b = bucket_of(KeyU64{kv[r]}, depth); br[r] = (b << 16) | atomicAdd(&h[b], 1u); }
+    }
+    __syncthreads();
+    const unsigned int mine = t < kBuckets ? h[t] : 0u;
+    const unsigned int lb = scan256_wide(mine, wtot);
+    if (t < kBuckets) { loc[t] = lb; glb[t] = gb - lb; }
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < ITEMS; r++) {
+        const uint32_t jt = uint32_t(r) * THREADS + t;
+        if (br[r] != 0xFFFFFFFFu) {
+            const uint32_t b = br[r] >> 16, j = loc[b] + (br[r] & 0xFFFFu);
+            sb[j] = uint8_t(b);
+            skeys[j] = kv[r];
+            __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < ITEMS; r++) {
+        const uint32_t j = uint32_t(r) * THREADS + t;
+        if (j < cnt) __stcs((unsigned long long*)bq + uint64_t(glb[sb[j]] + j), (unsigned long long)skeys[j]);
+    }
+}
+template <int THREADS>
+__global__ void __launch_bounds__(THREADS) g_wide(const uint64_t* __restrict__ res, const uint16_t* __restrict__ jpos, uint64_t n,
+                                                  const unsigned int* __restrict__ rowoff, const unsigned int* __restrict__ bases,
+                                                  uint64_t* __restrict__ out) {
+    constexpr int ITEMS = kBucketTile / THREADS;
+    __shared__ uint64_t sres[kBucketTile];
+    __shared__ uint8_t bof[kBucketTile];
+    __shared__ unsigned int loc[kBuckets], glb[kBuckets], wtot[8];
+    const uint64_t tb = blockIdx.x, tiles = gridDim.x;
+    const uint64_t base = tb * kBucketTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
+    const int t = threadIdx.x;
+    uint16_t jp[ITEMS];
+#pragma unroll
+    for (int r = 0; r < ITEMS; r++) {
+        const uint32_t k = uint32_t(r) * THREADS + t;
+        jp[r] = k < cnt ? __ldcs(jpos + base + k) : 0;
+    }
+    unsigned int c_b = 0, off = 0, bb = 0;
+    if (t < kBuckets) {
+        off = rowoff[hidx(t, tb)];
+        bb = bases[t];
+        const unsigned int bnext = t + 1 < kBuckets ? bases[t + 1] : unsigned(n);
+        const unsigned int next = tb + 1 < tiles ? rowoff[hidx(t, tb + 1)] : bnext - bb;
+        c_b = next - off;
+    }
+    const unsigned int l_b = scan256_wide(c_b, wtot);
+    if (t < kBuckets) {
+        glb[t] = bb + off;
+        loc[t] = l_b;
+        for (unsigned int k = 0; k < c_b; k++) bof[l_b + k] = uint8_t(t);
+    }
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < ITEMS; r++) {
+        const uint32_t j = uint32_t(r) * THREADS + t;
+        if (j < cnt) { const uint32_t bj = bof[j]; cp_async8(&sres[j], res + glb[bj] + (j - loc[bj])); }
+    }
+    cp_async_wait_all();
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < ITEMS; r++) {
+        const uint32_t k = uint32_t(r) * THREADS + t;
+        if (k < cnt) __stcs((unsigned long long*)out + base + k, (unsigned long long)sres[jp[r]]);
+    }
+}
+
+// ---- persistent scatter with TMA bulk tile loads (double-buffered, mbarrier-signalled)
+__device__ __forceinline__ uint32_t saddr(const void* p) { return uint32_t(__cvta_generic_to_shared(p)); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(saddr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes, uint64_t* bar) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(saddr(bar)), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(saddr(dst)), "l"(src), "r"(bytes), "r"(saddr(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
+    uint32_t ok = 0;
+    while (!ok)
+        asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
+                     : "=r"(ok) : "r"(saddr(bar)), "r"(parity) : "memory");
+}
+constexpr size_t kTmaScatterSmem = 2 * kBucketTile * 8 + kBucketTile * 8 + kBucketTile + 64;
+__global__ void __launch_bounds__(256) s_tma(const uint64_t* __restrict__ q, uint64_t n, uint32_t depth,
+                                             const unsigned int* __restrict__ rowoff, const unsigned int* __restrict__ bases,
+                                             uint64_t* __restrict__ bq, uint16_t* __restrict__ jpos) {
+    extern __shared__ __align__(128) uint8_t sm[];
+    uint64_t* kin = (uint64_t*)sm;                                   // [2][kBucketTile]
+    uint64_t* skeys = kin + 2 * kBucketTile;                         // staged tile
+    uint8_t* sb = (uint8_t*)(skeys + kBucketTile);
+    uint64_t* bar = (uint64_t*)(sb + kBucketTile);                   // [2]
+    __shared__ unsigned int h[kBuckets], loc[kBuckets], glb[kBuckets], wtot[8];
+    const int t = threadIdx.x;
+    const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
+    const uint64_t full_tiles = n / kBucketTile;                     // tiles loaded by TMA
+    if (t == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    uint64_t tile = blockIdx.x;
+    if (t == 0 && tile < full_tiles) bulk_g2s(kin, q + tile * kBucketTile, kBucketTile * 8, &bar[0]);
+    for (uint32_t it = 0; tile < tiles; it++, tile += gridDim.x) {
+        const uint32_t buf = it & 1;
+        const uint64_t nxt = tile + gridDim.x;
+        if (t == 0 && nxt < full_tiles) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            bulk_g2s(kin + (buf ^ 1) * kBucketTile, q + nxt * kBucketTile, kBucketTile * 8, &bar[buf ^ 1]);
+        }
+        const unsigned int gb = bases[t] + rowoff[hidx(t, tile)];
+        h[t] = 0;
+        const uint64_t base = tile * kBucketTile;
+        const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
+        const uint64_t* kt = kin + buf * kBucketTile;
+        if (tile < full_tiles) mbar_wait(&bar[buf], (it >> 1) & 1);
+        else for (uint32_t j = t; j < cnt; j += 256) ((uint64_t*)kt)[j] = q[base + j];
+        __syncthreads();
+        uint32_t br[kBucketItems];
+#pragma unroll
+        for (int r = 0; r < kBucketItems; r++) {
+            const uint32_t j = uint32_t(r) * 256 + t;
+            br[r] = 0xFFFFFFFFu;
+            if (j < cnt) { const uint32_t b = bucket_of(KeyU64{kt[j]}, depth); br[r] = (b << 16) | atomicAdd(&h[b], 1u); }
+        }
+        __syncthreads();
+        const unsigned int lb = block_excl_scan256(h[t], wtot);
+        loc[t] = lb;
+        glb[t] = gb - lb;
+        __syncthreads();
+#pragma unroll
+        for (int r = 0; r < kBucketItems; r++) {
+            const uint32_t jt = uint32_t(r) * 256 + t;
+            if (br[r] != 0xFFFFFFFFu) {
+                const uint32_t b = br[r] >> 16, j = loc[b] + (br[r] & 0xFFFFu);
+                sb[j] = uint8_t(b);
+                skeys[j] = kt[jt];
+                __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
+            }
+        }
+        __syncthreads();
+#pragma unroll 4
+        for (int r = 0; r < kBucketItems; r++) {
+            const uint32_t j = uint32_t(r) * 256 + t;
+            if (j < cnt) __stcs((unsigned long long*)bq + uint64_t(glb[sb[j]] + j), (unsigned long long)skeys[j]);
+        }
+        __syncthreads();
+    }
+}
+
 __global__ void csum(const uint64_t* a, uint64_t n, unsigned long long* s) {
     uint64_t acc = 0;
     for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x) acc += a[i] * (i | 1);
@@ -379,6 +577,23 @@ int main(int argc, char** argv) {
     timeit("k_bscatter_again", n * 18.0, [&] { k_bscatter<KeyU64><<<T, 256, smem>>>(q, nullptr, n, 0, hist, tot, bq, nullptr, jpos); });
     k_bgather<false><<<T, 256>>>(bq, jpos, n, hist, tot, out);
     const unsigned long long s3 = checksum(out, n);
+    for (int v = 0; v < 2; v++) {
+        const char* sn = v == 0 ? "s_wide512" : "s_wide1024";
+        const char* gn = v == 0 ? "g_wide512" : "g_wide1024";
+        timeit(sn, n * 18.0, [&] { if (v == 0) s_wide<512><<<T, 512>>>(q, n, 0, hist, tot, bq, jpos); else s_wide<1024><<<T, 1024>>>(q, n, 0, hist, tot, bq, jpos); });
+        timeit(gn, n * 18.0, [&] { if (v == 0) g_wide<512><<<T, 512>>>(bq, jpos, n, hist, tot, out); else g_wide<1024><<<T, 1024>>>(bq, jpos, n, hist, tot, out); });
+        printf("{\"roundtrip_%s\": %s}\n", sn, checksum(out, n) == s1b ? "true" : "false");
+    }
+    cudaFuncSetAttribute(s_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kTmaScatterSmem));
+    for (int cps = 1; cps <= 2; cps++) {
+        char nm[32];
+        snprintf(nm, sizeof nm, "s_tma_x%d", cps);
+        int nsm = 0;
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
+        timeit(nm, n * 18.0, [&] { s_tma<<<nsm * cps, 256, kTmaScatterSmem>>>(q, n, 0, hist, tot, bq, jpos); });
+        g_ca<<<T, 256>>>(bq, jpos, n, hist, tot, out);
+        printf("{\"roundtrip_%s\": %s}\n", nm, checksum(out, n) == s1b ? "true" : "false");
+    }
     printf("{\"roundtrip_s_v4\": %s, \"roundtrip_k_bscatter\": %s}\n", s2 == s1b ? "true" : "false", s3 == s1b ? "true" : "false");
     printf("{\"s0\": %llu, \"roundtrip_ok\": %s}\n", s0, s1 == s1b ? "true" : "false");
     return 0;
