@@ -38,7 +38,7 @@ struct cuart_layout {
 };
 
 // host-buffer pipelines (cuart_lookup_host / cuart_update_host)
-static constexpr size_t kStageChunk = size_t(1) << 23;   // ops per pipeline chunk
+static constexpr size_t kStageChunk = size_t(1) << 23;   // ops per pipeline chunk (env CUART_STAGE_CHUNK overrides)
 static constexpr int kStages = 4;                          // chunks in flight (streams / staging sets)
 
 struct cuart_index {
@@ -71,6 +71,9 @@ struct cuart_index {
     uint64_t* stage_val[4] = {nullptr, nullptr, nullptr, nullptr};
     size_t stage_cap = 0;
     cudaStream_t streams[4] = {nullptr, nullptr, nullptr, nullptr};   // host-pipeline streams
+    cudaStream_t ustream = nullptr;                                   // update pipeline: the kernels, in op order
+    cudaEvent_t ev_copied[4] = {nullptr, nullptr, nullptr, nullptr};  // staging set s filled
+    cudaEvent_t ev_free[4] = {nullptr, nullptr, nullptr, nullptr};    // staging set s consumed
     int policy = 5;                    // cache-policy variant of the kernels (kernels.cuh Loader)
     uint32_t lut_format = CUART_LUT_LINKS;
     uint64_t lutc_off = 0;             // compact / rank LUT region
@@ -1063,6 +1066,8 @@ cuart_status cuart_destroy(cuart_index* h) {
         if (h->stage_len[i]) cudaFree(h->stage_len[i]);
         if (h->stage_val[i]) cudaFree(h->stage_val[i]);
         if (h->streams[i]) cudaStreamDestroy(h->streams[i]);
+        if (h->ev_copied[i]) cudaEventDestroy(h->ev_copied[i]);
+        if (h->ev_free[i]) cudaEventDestroy(h->ev_free[i]);
     }
     delete h;
     return CUART_OK;
@@ -1299,20 +1304,33 @@ cuart_status cuart_free_leaves(const cuart_index* h, uint32_t* ids, size_t cap, 
 
 // ---------------------------------------------------------------- host-buffer pipelines
 
+static size_t key_stride(uint32_t kind);
+static size_t stage_chunk();
 static cuart_status ensure_stage(cuart_index* h) {
     if (h->stage_cap) return CUART_OK;
+    const size_t c = stage_chunk(), ks = key_stride(h->key_kind);
     for (int i = 0; i < kStages; i++) {
-        CU_TRY(cudaMalloc(&h->stage[i], kStageChunk * 32));
-        CU_TRY(cudaMalloc(&h->stage_out[i], kStageChunk * 8));
-        CU_TRY(cudaMalloc(&h->stage_len[i], kStageChunk));
-        CU_TRY(cudaMalloc(&h->stage_val[i], kStageChunk * 8));
+        CU_TRY(cudaMalloc(&h->stage[i], c * ks));
+        CU_TRY(cudaMalloc(&h->stage_out[i], c * 8));
+        if (h->key_kind == CUART_KEY_BYTES) CU_TRY(cudaMalloc(&h->stage_len[i], c));
+        CU_TRY(cudaMalloc(&h->stage_val[i], c * 8));
         CU_TRY(cudaStreamCreateWithFlags(&h->streams[i], cudaStreamNonBlocking));
+        CU_TRY(cudaEventCreateWithFlags(&h->ev_copied[i], cudaEventDisableTiming));
+        CU_TRY(cudaEventCreateWithFlags(&h->ev_free[i], cudaEventDisableTiming));
     }
-    h->stage_cap = kStageChunk;
+    CU_TRY(cudaStreamCreateWithFlags(&h->ustream, cudaStreamNonBlocking));
+    h->stage_cap = c;
     return CUART_OK;
 }
 
 static size_t key_stride(uint32_t kind) { return kind == CUART_KEY_U64 ? 8 : kind == CUART_KEY_U32 ? 4 : 32; }
+// ops per host-pipeline chunk: kStageChunk, or CUART_STAGE_CHUNK read when the
+// handle's staging buffers are first allocated (a tuning / test knob)
+static size_t stage_chunk() {
+    size_t v = kStageChunk;
+    if (const char* pe = getenv("CUART_STAGE_CHUNK")) v = size_t(strtoull(pe, nullptr, 0));
+    return v == 0 || v > (size_t(1) << 28) ? kStageChunk : v;
+}
 
 cuart_status cuart_lookup_host(const cuart_index* hc, const cuart_keys* q, size_t n, uint64_t* out) {
     cuart_index* h = const_cast<cuart_index*>(hc);
@@ -1324,13 +1342,14 @@ cuart_status cuart_lookup_host(const cuart_index* hc, const cuart_keys* q, size_
     if ((rc = ensure_stage(h)) != CUART_OK) return rc;
     const size_t ks = key_stride(h->key_kind);
     size_t c = 0;
-    for (size_t base = 0; base < n; base += kStageChunk, c++) {
-        const size_t m = (n - base) < kStageChunk ? (n - base) : kStageChunk;
+    const size_t chunk = h->stage_cap;
+    for (size_t base = 0; base < n; base += chunk, c++) {
+        const size_t m = (n - base) < chunk ? (n - base) : chunk;
         const int s = int(c % kStages);
         cudaStream_t st = h->streams[s];
         CU_TRY(cudaMemcpyAsync(h->stage[s], (const uint8_t*)q->data + base * ks, m * ks, cudaMemcpyHostToDevice, st));
-        if (q->lengths) CU_TRY(cudaMemcpyAsync(h->stage_len[s], q->lengths + base, m, cudaMemcpyHostToDevice, st));
-        rc = launch_lookup(h, h->key_kind, h->stage[s], q->lengths ? h->stage_len[s] : nullptr, m, h->stage_out[s], st);
+        if (h->key_kind == CUART_KEY_BYTES) CU_TRY(cudaMemcpyAsync(h->stage_len[s], q->lengths + base, m, cudaMemcpyHostToDevice, st));
+        rc = launch_lookup(h, h->key_kind, h->stage[s], h->key_kind == CUART_KEY_BYTES ? h->stage_len[s] : nullptr, m, h->stage_out[s], st);
         if (rc != CUART_OK) return rc;
         CU_TRY(cudaMemcpyAsync(out + base, h->stage_out[s], m * 8, cudaMemcpyDeviceToHost, st));
     }
@@ -1346,19 +1365,27 @@ cuart_status cuart_update_host(cuart_index* h, const cuart_keys* k, const uint64
     CU_TRY(cudaSetDevice(h->device));
     if ((rc = ensure_stage(h)) != CUART_OK) return rc;
     const size_t ks = key_stride(h->key_kind);
-    // chunks are applied in op order on ONE stream: sequential semantics across chunks
-    cudaStream_t st = h->streams[0];
+    // The kernels of all chunks run in op order on ONE stream (sequential semantics
+    // across chunks); the H2D copies of the next chunks run on the staging sets' own
+    // streams and overlap them (events: set filled -> kernels; kernels done -> set free).
+    cudaStream_t ust = h->ustream;
     size_t c = 0;
-    for (size_t base = 0; base < n; base += kStageChunk, c++) {
-        const size_t m = (n - base) < kStageChunk ? (n - base) : kStageChunk;
+    const size_t chunk = h->stage_cap;
+    for (size_t base = 0; base < n; base += chunk, c++) {
+        const size_t m = (n - base) < chunk ? (n - base) : chunk;
         const int s = int(c % kStages);
-        CU_TRY(cudaMemcpyAsync(h->stage[s], (const uint8_t*)k->data + base * ks, m * ks, cudaMemcpyHostToDevice, st));
-        if (k->lengths) CU_TRY(cudaMemcpyAsync(h->stage_len[s], k->lengths + base, m, cudaMemcpyHostToDevice, st));
-        CU_TRY(cudaMemcpyAsync(h->stage_val[s], v + base, m * 8, cudaMemcpyHostToDevice, st));
-        rc = dispatch_update(h, h->stage[s], k->lengths ? h->stage_len[s] : nullptr, h->stage_val[s], m, st);
+        cudaStream_t cst = h->streams[s];
+        if (c >= size_t(kStages)) CU_TRY(cudaStreamWaitEvent(cst, h->ev_free[s], 0));
+        CU_TRY(cudaMemcpyAsync(h->stage[s], (const uint8_t*)k->data + base * ks, m * ks, cudaMemcpyHostToDevice, cst));
+        if (h->key_kind == CUART_KEY_BYTES) CU_TRY(cudaMemcpyAsync(h->stage_len[s], k->lengths + base, m, cudaMemcpyHostToDevice, cst));
+        CU_TRY(cudaMemcpyAsync(h->stage_val[s], v + base, m * 8, cudaMemcpyHostToDevice, cst));
+        CU_TRY(cudaEventRecord(h->ev_copied[s], cst));
+        CU_TRY(cudaStreamWaitEvent(ust, h->ev_copied[s], 0));
+        rc = dispatch_update(h, h->stage[s], h->key_kind == CUART_KEY_BYTES ? h->stage_len[s] : nullptr, h->stage_val[s], m, ust);
         if (rc != CUART_OK) return rc;
+        CU_TRY(cudaEventRecord(h->ev_free[s], ust));
     }
-    CU_TRY(cudaStreamSynchronize(st));
+    CU_TRY(cudaStreamSynchronize(ust));
     return CUART_OK;
 }
 

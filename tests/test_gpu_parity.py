@@ -215,6 +215,32 @@ def test_host_buffer_paths_match_device():
     ix.close()
 
 
+@pytest.mark.parametrize("kind", ["u64", "bytes"])
+def test_host_pipeline_many_chunks(kind, monkeypatch):
+    """cuart_lookup_host / cuart_update_host with 4096-op chunks (CUART_STAGE_CHUNK,
+    read when the handle's staging buffers are allocated): lookups spread over the 4
+    staging streams, update chunks whose H2D copies overlap the previous chunks'
+    kernels while the kernels stay in op order — duplicates across chunks must
+    still resolve to the last op, exactly as the plain map."""
+    monkeypatch.setenv("CUART_STAGE_CHUNK", "4096")
+    rng = np.random.default_rng(21)
+    if kind == "u64":
+        keys, vals = W.build_set(W.CONFIGS["c1"])
+    else:
+        keys = W.string_keys(4, 1 << 14)
+        vals = np.arange(1 << 14, dtype=np.uint64) + 3
+    n = keys[1].shape[0] if isinstance(keys, tuple) else keys.shape[0]
+    ix = C.Index(keys, vals, lut_bytes=0 if kind == "bytes" else 3)
+    mp = MapOracle(keys, vals)
+    pick = rng.integers(0, min(n, 500), 60_001)                    # many duplicates, across chunks
+    uk = (keys[0][pick].copy(), keys[1][pick].copy()) if isinstance(keys, tuple) else keys[pick].copy()
+    uv = rng.integers(0, 2**63, pick.shape[0], dtype=np.uint64)
+    ix.update_host(uk, uv)
+    mp.update(uk, uv)
+    assert np.array_equal(ix.lookup_host(keys), mp.lookup(keys))
+    ix.close()
+
+
 def test_c2_full_size_sampled():
     """Config 2 at full size (2^24 dense u32 keys, LUT over the first 3 bytes):
     2^28 lookups in the bench's launch configuration; sampled outputs vs the

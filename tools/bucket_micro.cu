@@ -510,6 +510,113 @@ __global__ void __launch_bounds__(256) s_tma(const uint64_t* __restrict__ q, uin
     }
 }
 
+// scatter without the per-position bucket byte: the copy phase recomputes the bucket
+// from the staged key (one shift) instead of a random smem byte store + a byte load
+__global__ void __launch_bounds__(256, 4) s_nosb(const uint64_t* __restrict__ q, uint64_t n, uint32_t depth,
+                                              const unsigned int* __restrict__ rowoff, const unsigned int* __restrict__ bases,
+                                              uint64_t* __restrict__ bq, uint16_t* __restrict__ jpos) {
+    __shared__ uint64_t skeys[kBucketTile];
+    __shared__ unsigned int h[kBuckets], loc[kBuckets], glb[kBuckets], wtot[8];
+    const int t = threadIdx.x;
+    h[t] = 0;
+    const unsigned int gb = bases[t] + rowoff[hidx(t, blockIdx.x)];
+    __syncthreads();
+    const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
+    uint64_t kv[kBucketItems];
+    uint32_t br[kBucketItems];
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * 256 + t;
+        kv[r] = j < cnt ? uint64_t(__ldcs((const unsigned long long*)q + base + j)) : 0;
+    }
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * 256 + t;
+        br[r] = 0xFFFFFFFFu;
+        if (j < cnt) { const uint32_t b = bucket_of(KeyU64{kv[r]}, depth); br[r] = (b << 16) | atomicAdd(&h[b], 1u); }
+    }
+    __syncthreads();
+    const unsigned int lb = block_excl_scan256(h[t], wtot);
+    loc[t] = lb;
+    glb[t] = gb - lb;
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t jt = uint32_t(r) * 256 + t;
+        if (br[r] != 0xFFFFFFFFu) {
+            const uint32_t b = br[r] >> 16, j = loc[b] + (br[r] & 0xFFFFu);
+            skeys[j] = kv[r];
+            __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
+        }
+    }
+    __syncthreads();
+#pragma unroll 4
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * 256 + t;
+        if (j < cnt) {
+            const uint64_t kk = skeys[j];
+            __stcs((unsigned long long*)bq + uint64_t(glb[bucket_of(KeyU64{kk}, depth)] + j), (unsigned long long)kk);
+        }
+    }
+}
+
+__global__ void __launch_bounds__(256, 4) s_seqw(const uint64_t* __restrict__ q, uint64_t n, uint32_t depth,
+                                              const unsigned int* __restrict__ rowoff, const unsigned int* __restrict__ bases,
+                                              uint64_t* __restrict__ bq, uint16_t* __restrict__ jpos) {
+    __shared__ uint64_t skeys[kBucketTile];
+    __shared__ unsigned int h[kBuckets], loc[kBuckets], glb[kBuckets], wtot[8];
+    const int t = threadIdx.x;
+    h[t] = 0;
+    const unsigned int gb = bases[t] + rowoff[hidx(t, blockIdx.x)];
+    __syncthreads();
+    const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
+    uint64_t kv[kBucketItems];
+    uint32_t br[kBucketItems];
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * 256 + t;
+        kv[r] = j < cnt ? uint64_t(__ldcs((const unsigned long long*)q + base + j)) : 0;
+    }
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * 256 + t;
+        br[r] = 0xFFFFFFFFu;
+        if (j < cnt) { const uint32_t b = bucket_of(KeyU64{kv[r]}, depth); br[r] = (b << 16) | atomicAdd(&h[b], 1u); }
+    }
+    __syncthreads();
+    const unsigned int lb = block_excl_scan256(h[t], wtot);
+    loc[t] = lb;
+    glb[t] = gb - lb;
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t jt = uint32_t(r) * 256 + t;
+        if (br[r] != 0xFFFFFFFFu) {
+            const uint32_t b = br[r] >> 16, j = loc[b] + (br[r] & 0xFFFFu);
+            skeys[j] = kv[r];
+            __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
+        }
+    }
+    __syncthreads();
+#pragma unroll 4
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * 256 + t;
+        if (j < cnt) {
+            const uint64_t kk = skeys[j];
+            __stcs((unsigned long long*)bq + base + j, (unsigned long long)(kk + glb[bucket_of(KeyU64{kk}, depth)]));
+        }
+    }
+}
+
+// diagnostic: one global atomicAdd per (tile, bucket) on 256 counters spread STRIDE words apart
+template <int STRIDE>
+__global__ void __launch_bounds__(256) atom_alloc(unsigned int* fill, unsigned int* sink) {
+    const unsigned int v = atomicAdd(&fill[threadIdx.x * STRIDE], 16u + (blockIdx.x & 3));
+    if (v == 0xFFFFFFFFu) sink[0] = v;
+}
+
 __global__ void csum(const uint64_t* a, uint64_t n, unsigned long long* s) {
     uint64_t acc = 0;
     for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x) acc += a[i] * (i | 1);
@@ -584,6 +691,17 @@ int main(int argc, char** argv) {
         timeit(gn, n * 18.0, [&] { if (v == 0) g_wide<512><<<T, 512>>>(bq, jpos, n, hist, tot, out); else g_wide<1024><<<T, 1024>>>(bq, jpos, n, hist, tot, out); });
         printf("{\"roundtrip_%s\": %s}\n", sn, checksum(out, n) == s1b ? "true" : "false");
     }
+    timeit("s_nosb", n * 18.0, [&] { s_nosb<<<T, 256>>>(q, n, 0, hist, tot, bq, jpos); });
+    g_ca<<<T, 256>>>(bq, jpos, n, hist, tot, out);
+    printf("{\"roundtrip_s_nosb\": %s}\n", checksum(out, n) == s1b ? "true" : "false");
+    {
+        unsigned int* fill; cudaMalloc(&fill, 256 * 1024 * 4); cudaMemset(fill, 0, 256 * 1024 * 4);
+        timeit("atom_alloc_stride1", 0, [&] { atom_alloc<1><<<T, 256>>>(fill, (unsigned int*)sink); });
+        timeit("atom_alloc_stride64", 0, [&] { atom_alloc<64><<<T, 256>>>(fill, (unsigned int*)sink); });
+        timeit("atom_alloc_stride1024", 0, [&] { atom_alloc<1024><<<T, 256>>>(fill, (unsigned int*)sink); });
+        cudaFree(fill);
+    }
+    timeit("s_seqw (diagnostic: sequential writes)", n * 18.0, [&] { s_seqw<<<T, 256>>>(q, n, 0, hist, tot, bq, jpos); });
     cudaFuncSetAttribute(s_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kTmaScatterSmem));
     for (int cps = 1; cps <= 2; cps++) {
         char nm[32];
