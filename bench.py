@@ -388,6 +388,8 @@ def main():
     if mode == "range":   # sample of the queries this rank's index actually serves
         samp = select(samp, owners(prefix8(samp), di.splitters_np) == rank)
     bucketed = nl >= (1 << 22) and cfg.kind != "bytes"
+    # the bucketed wide walk over integer keys runs as k_lookup_wq (2 queries per thread)
+    wq = bucketed and bool(stats.get("wide_lut", 0)) and os.environ.get("CUART_ILP", "2") != "1"
     # sectors of the path the walk kernel takes: the pre-bucketed walk starts from the
     # wide root table when the index has one (stats["wide_lut"]), else the plain path
     sec = layout.sectors(samp, wide=bool(bucketed and stats.get("wide_lut", 0))).astype(np.float64)
@@ -569,7 +571,7 @@ def main():
                        "ms": round(upd_ms, 4)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
-                         "kernel": ("k_lookup_slice" if kslice else "k_lookup")
+                         "kernel": ("k_lookup_slice" if kslice else "k_lookup_wq" if wq else "k_lookup")
                          + {"u64": "<KeyU64>", "u32": "<KeyU32>", "bytes": "<KeyBytes>"}[cfg.kind],
                          "kernel_ms": round(kern_ms, 4), "lookups_per_launch": int(served),
                          "lookup_call_ms": round(look_ms, 4), "prebucket": "on" if bucketed else "off",
@@ -589,7 +591,7 @@ def main():
                          "lookup_call": {"ms": round(look_ms, 4), "bytes_per_lookup": round(pipeline_bytes, 3),
                                          "achieved": round(pipe_achieved, 1), "frac": round(pipe_achieved / peak, 4),
                                          "kernels": "k_bhist, k_bscan_rows, k_bscan, k_bscatter, "
-                                         + ("k_lookup_slice" if kslice else "k_lookup") + ", k_bgather"
+                                         + ("k_lookup_slice" if kslice else "k_lookup_wq" if wq else "k_lookup") + ", k_bgather"
                                          if bucketed else "k_lookup"}},
             "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": int(launches), "clocks": clk,
             "index": {k: stats[k] for k in ("n4", "n16", "n48", "n256", "leaf8", "arena_bytes", "max_depth",

@@ -314,6 +314,62 @@ __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restric
     }
 }
 
+// Stage 1 of a pre-bucketed plain update batch (integer keys, wide root table):
+// k_upd1's work with Q ops per thread in lockstep phases, as k_lookup_wq (keys,
+// values and op indices, then the wide entries, then the leaf records are all
+// requested before use).  Same outputs as k_upd1<Key, 5, false>.
+template <class Key, int Q>
+__global__ void __launch_bounds__(256) k_upd1_wq(DevIndex ix, const void* __restrict__ q, const uint64_t* __restrict__ vals,
+                                                 uint64_t n, uint64_t epoch_hi, uint64_t* __restrict__ leafref,
+                                                 const uint32_t* __restrict__ opidx) {
+    static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
+    const Loader<5> ld;
+    const uint64_t i0 = uint64_t(blockIdx.x) * (256 * Q) + threadIdx.x;
+    Key k[Q];
+    uint64_t v[Q];
+    uint32_t pr[Q];
+#pragma unroll
+    for (int j = 0; j < Q; j++) {
+        const uint64_t i = i0 + uint64_t(j) * 256;
+        const bool ok = i < n;
+        k[j] = ok ? Key::template load<true>(q, nullptr, i) : Key{0};
+        v[j] = ok ? uint64_t(__ldcs((const unsigned long long*)vals + i)) : 0;
+        pr[j] = ok ? (opidx ? __ldcs(opidx + i) : uint32_t(i)) : 0u;
+    }
+    U8x32 e[Q];
+#pragma unroll
+    for (int j = 0; j < Q; j++) e[j] = ld.lutv8(ix.lutw + k[j].prefix(ix.lut_bytes) * 4);
+    uint64_t link[Q];
+#pragma unroll
+    for (int j = 0; j < Q; j++) link[j] = decode_wide(ix, ld, k[j], e[j]);
+    uint4 r[Q];
+#pragma unroll
+    for (int j = 0; j < Q; j++)
+        if (link_type(link[j]) == T_LEAF8) r[j] = ld.leafv4(ix.base[T_LEAF8] + link_index(link[j]) * record_bytes(T_LEAF8));
+#pragma unroll
+    for (int j = 0; j < Q; j++) {
+        const uint64_t i = i0 + uint64_t(j) * 256;
+        if (i >= n) continue;
+        uint64_t leaf = 0, val = kMiss;
+        if (link_type(link[j]) == T_LEAF8) {
+            const uint64_t kb = Key::kKind == 2 ? bswap64(uint64_t(k[j].k)) : uint64_t(__byte_perm(uint32_t(k[j].k), 0, 0x0123));
+            if (link_aux(link[j]) == k[j].len() && (uint64_t(r[j].x) | (uint64_t(r[j].y) << 32)) == kb) {
+                leaf = link[j];
+                val = uint64_t(r[j].z) | (uint64_t(r[j].w) << 32);
+            }
+        } else if (link[j]) {
+            leaf = find_leaf(ix, ld, k[j], link[j], val);
+        }
+        if (leaf && val == kMiss) leaf = 0;            // tombstone: deleted by an earlier batch
+        if (v[j] == kMiss) {                           // reserved value: op rejected, sticky error
+            atomicOr(ix.err, 1u);
+            leaf = 0;
+        }
+        leafref[i] = leaf;
+        if (leaf) atomicMax((unsigned long long*)winner_word(ix, leaf), (unsigned long long)(epoch_hi | pr[j]));
+    }
+}
+
 // Stage 2: after the grid-wide synchronisation (kernel boundary), the op whose
 // index is the registered maximum applies: one aligned 8-byte value store,
 // or, for a delete, unlink the leaf from its parent slot, clear it (value :=
@@ -579,7 +635,12 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
     } else {                                                 \
         if (del) CUART_UPD1(K, 5, true); else CUART_UPD1(K, 5, false); \
     }
-        switch (kind) {
+        const bool wq = !del && bucketed && dx.walk_wide && h->policy == 5 && h->ilp > 1 &&
+                        (kind == CUART_KEY_U64 || kind == CUART_KEY_U32);
+        const unsigned gq = unsigned((m + 512 - 1) / 512);
+        if (wq && kind == CUART_KEY_U64) k_upd1_wq<KeyU64, 2><<<gq, 256, 0, s>>>(dx, kb, vb, m, epoch_hi, h->leafref, ib);
+        else if (wq) k_upd1_wq<KeyU32, 2><<<gq, 256, 0, s>>>(dx, kb, vb, m, epoch_hi, h->leafref, ib);
+        else switch (kind) {
         case CUART_KEY_U64: CUART_UPD1_POL(KeyU64); break;
         case CUART_KEY_U32: CUART_UPD1_POL(KeyU32); break;
         case CUART_KEY_LONG: CUART_UPD1_POL(KeyLong); break;
