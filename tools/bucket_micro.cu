@@ -617,6 +617,124 @@ __global__ void __launch_bounds__(256) atom_alloc(unsigned int* fill, unsigned i
     if (v == 0xFFFFFFFFu) sink[0] = v;
 }
 
+// ---- tile of 8192 keys (512 threads x 16): runs twice as long (avg 32 keys = 256 B per
+// bucket run), half the hist entries
+constexpr int kBigThreads = 512, kBigTile = kBigThreads * kBucketItems;
+__global__ void __launch_bounds__(kBigThreads) h_big(const uint64_t* __restrict__ q, uint64_t n, uint32_t depth, unsigned int* __restrict__ hist) {
+    __shared__ unsigned int h[kBuckets];
+    const int t = threadIdx.x;
+    if (t < kBuckets) h[t] = 0;
+    __syncthreads();
+    const uint64_t base = uint64_t(blockIdx.x) * kBigTile;
+    uint4 v[kBucketItems / 2];
+#pragma unroll
+    for (int r = 0; r < kBucketItems / 2; r++) {
+        const uint64_t i = base + 2 * (uint64_t(r) * kBigThreads + t);
+        v[r] = i + 2 <= n ? __ldcs((const uint4*)(q + i)) : make_uint4(0, 0, 0, 0);
+    }
+#pragma unroll
+    for (int r = 0; r < kBucketItems / 2; r++) {
+        const uint64_t i = base + 2 * (uint64_t(r) * kBigThreads + t);
+        if (i + 2 <= n) {
+            atomicAdd(&h[bucket_of(KeyU64{uint64_t(v[r].x) | (uint64_t(v[r].y) << 32)}, depth)], 1u);
+            atomicAdd(&h[bucket_of(KeyU64{uint64_t(v[r].z) | (uint64_t(v[r].w) << 32)}, depth)], 1u);
+        } else if (i < n) atomicAdd(&h[bucket_of(KeyU64{q[i]}, depth)], 1u);
+    }
+    __syncthreads();
+    if (t < kBuckets) hist[hidx(t, blockIdx.x)] = h[t];
+}
+__global__ void __launch_bounds__(kBigThreads) s_big(const uint64_t* __restrict__ q, uint64_t n, uint32_t depth,
+                                                     const unsigned int* __restrict__ rowoff, const unsigned int* __restrict__ bases,
+                                                     uint64_t* __restrict__ bq, uint16_t* __restrict__ jpos) {
+    extern __shared__ __align__(16) uint64_t skeys[];
+    __shared__ unsigned int h[kBuckets], loc[kBuckets], glb[kBuckets], wtot[8];
+    const int t = threadIdx.x;
+    unsigned int gb = 0;
+    if (t < kBuckets) { h[t] = 0; gb = bases[t] + rowoff[hidx(t, blockIdx.x)]; }
+    __syncthreads();
+    const uint64_t base = uint64_t(blockIdx.x) * kBigTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBigTile) ? n - base : kBigTile);
+    uint64_t kv[kBucketItems];
+    uint32_t br[kBucketItems];
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * kBigThreads + t;
+        kv[r] = j < cnt ? uint64_t(__ldcs((const unsigned long long*)q + base + j)) : 0;
+    }
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * kBigThreads + t;
+        br[r] = 0xFFFFFFFFu;
+        if (j < cnt) { const uint32_t b = bucket_of(KeyU64{kv[r]}, depth); br[r] = (b << 16) | atomicAdd(&h[b], 1u); }
+    }
+    __syncthreads();
+    const unsigned int lb = scan256_wide(t < kBuckets ? h[t] : 0u, wtot);
+    if (t < kBuckets) { loc[t] = lb; glb[t] = gb - lb; }
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t jt = uint32_t(r) * kBigThreads + t;
+        if (br[r] != 0xFFFFFFFFu) {
+            const uint32_t b = br[r] >> 16, j = loc[b] + (br[r] & 0xFFFFu);
+            skeys[j] = kv[r];
+            __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
+        }
+    }
+    __syncthreads();
+#pragma unroll 4
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * kBigThreads + t;
+        if (j < cnt) {
+            const uint64_t kk = skeys[j];
+            __stcs((unsigned long long*)bq + uint64_t(glb[bucket_of(KeyU64{kk}, depth)] + j), (unsigned long long)kk);
+        }
+    }
+}
+__global__ void __launch_bounds__(kBigThreads) g_big(const uint64_t* __restrict__ res, const uint16_t* __restrict__ jpos, uint64_t n,
+                                                     const unsigned int* __restrict__ rowoff, const unsigned int* __restrict__ bases,
+                                                     uint64_t* __restrict__ out) {
+    extern __shared__ __align__(16) uint64_t sres[];
+    uint8_t* bof = (uint8_t*)(sres + kBigTile);
+    __shared__ unsigned int loc[kBuckets], glb[kBuckets], wtot[8];
+    const uint64_t tb = blockIdx.x, tiles = gridDim.x;
+    const uint64_t base = tb * kBigTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBigTile) ? n - base : kBigTile);
+    const int t = threadIdx.x;
+    uint16_t jp[kBucketItems];
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t k = uint32_t(r) * kBigThreads + t;
+        jp[r] = k < cnt ? __ldcs(jpos + base + k) : 0;
+    }
+    unsigned int c_b = 0, off = 0, bb = 0;
+    if (t < kBuckets) {
+        off = rowoff[hidx(t, tb)];
+        bb = bases[t];
+        const unsigned int bnext = t + 1 < kBuckets ? bases[t + 1] : unsigned(n);
+        const unsigned int next = tb + 1 < tiles ? rowoff[hidx(t, tb + 1)] : bnext - bb;
+        c_b = next - off;
+    }
+    const unsigned int l_b = scan256_wide(c_b, wtot);
+    if (t < kBuckets) {
+        glb[t] = bb + off;
+        loc[t] = l_b;
+        for (unsigned int k = 0; k < c_b; k++) bof[l_b + k] = uint8_t(t);
+    }
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * kBigThreads + t;
+        if (j < cnt) { const uint32_t bj = bof[j]; cp_async8(&sres[j], res + glb[bj] + (j - loc[bj])); }
+    }
+    cp_async_wait_all();
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t k = uint32_t(r) * kBigThreads + t;
+        if (k < cnt) __stcs((unsigned long long*)out + base + k, (unsigned long long)sres[jp[r]]);
+    }
+}
+
 __global__ void csum(const uint64_t* a, uint64_t n, unsigned long long* s) {
     uint64_t acc = 0;
     for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x) acc += a[i] * (i | 1);
@@ -711,6 +829,18 @@ int main(int argc, char** argv) {
         timeit(nm, n * 18.0, [&] { s_tma<<<nsm * cps, 256, kTmaScatterSmem>>>(q, n, 0, hist, tot, bq, jpos); });
         g_ca<<<T, 256>>>(bq, jpos, n, hist, tot, out);
         printf("{\"roundtrip_%s\": %s}\n", nm, checksum(out, n) == s1b ? "true" : "false");
+    }
+    {
+        const uint64_t tb = (n + kBigTile - 1) / kBigTile;
+        const size_t ss = size_t(kBigTile) * 8, gs = size_t(kBigTile) * 9;
+        cudaFuncSetAttribute(s_big, cudaFuncAttributeMaxDynamicSharedMemorySize, int(ss));
+        cudaFuncSetAttribute(g_big, cudaFuncAttributeMaxDynamicSharedMemorySize, int(gs));
+        timeit("h_big", n * 8.0, [&] { h_big<<<unsigned(tb), kBigThreads>>>(q, n, 0, hist); });
+        k_bscan_rows<<<kBuckets, kBucketThreads>>>(hist, tb, tot);
+        k_bscan<<<1, kBuckets>>>(tot);
+        timeit("s_big", n * 18.0, [&] { s_big<<<unsigned(tb), kBigThreads, ss>>>(q, n, 0, hist, tot, bq, jpos); });
+        timeit("g_big", n * 18.0, [&] { g_big<<<unsigned(tb), kBigThreads, gs>>>(bq, jpos, n, hist, tot, out); });
+        printf("{\"roundtrip_big\": %s}\n", checksum(out, n) == s1b ? "true" : "false");
     }
     printf("{\"roundtrip_s_v4\": %s, \"roundtrip_k_bscatter\": %s}\n", s2 == s1b ? "true" : "false", s3 == s1b ? "true" : "false");
     printf("{\"s0\": %llu, \"roundtrip_ok\": %s}\n", s0, s1 == s1b ? "true" : "false");
