@@ -387,7 +387,7 @@ def main():
         samp = samp.view(np.uint64) if cfg.kind == "u64" else samp.view(np.uint32)
     if mode == "range":   # sample of the queries this rank's index actually serves
         samp = select(samp, owners(prefix8(samp), di.splitters_np) == rank)
-    bucketed = nl >= (1 << 22) and cfg.kind != "bytes"
+    bucketed = nl >= (1 << 22) and cfg.kind != "bytes" and os.environ.get("CUART_PREBUCKET", "1") != "0"
     # the bucketed wide walk over integer keys runs as k_lookup_wq (2 queries per thread)
     wq = bucketed and bool(stats.get("wide_lut", 0)) and os.environ.get("CUART_ILP", "2") != "1"
     # sectors of the path the walk kernel takes: the pre-bucketed walk starts from the
