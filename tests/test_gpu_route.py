@@ -108,15 +108,19 @@ def test_loopback_range_partitioned_c1(nparts):
         ix.close()
 
 
+@pytest.mark.parametrize("pb", [0, 1])
 @pytest.mark.parametrize("kind", ["u64", "u32", "bytes"])
 @pytest.mark.parametrize("nparts", [2, 4, 8])
-def test_p2p_fused_exchange_loopback(kind, nparts):
+def test_p2p_fused_exchange_loopback(kind, nparts, pb):
     """The fused p2p exchange with P virtual ranks on one GPU: every 'rank' has its
     own partition index and windows (plain device buffers stand in for the mapped
     peer windows), cuart_route_count -> count matrix -> cuart_route_push into the
     owners' windows -> cuart_lookup_segmented straight into the sources' result
     windows -> cuart_unroute.  Then a routed update batch (values pushed with the
-    keys, applied in rank-major order).  Results equal the oracle."""
+    keys, applied in rank-major order).  Results equal the oracle.  pb = 1: the owners'
+    indexes pre-bucket every batch of >= 4096 ops (and walk the wide root table), so
+    the segmented lookup's last kernel is the bucketed gather storing straight into
+    the sources' windows (k_bgather<SEG>)."""
     from paper_conf_icpp_koppehelggp21_b200 import _binding as B
     from paper_conf_icpp_koppehelggp21_b200.dist import p2p_plan, ks_bytes
     rng = np.random.default_rng(nparts * 7 + len(kind))
@@ -138,7 +142,9 @@ def test_p2p_fused_exchange_loopback(kind, nparts):
     sp = compute_splitters(prefix8(keys), nparts)
     own = owners(prefix8(keys), sp)
     sel = lambda a, m: (a[0][m], a[1][m]) if isinstance(a, tuple) else a[m]
-    idx = [C.Index(sel(keys, own == o), vals[own == o], lut_bytes=0 if kind == "bytes" else 3) for o in range(nparts)]
+    opt = dict(prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_ON) if pb else {}
+    idx = [C.Index(sel(keys, own == o), vals[own == o], lut_bytes=0 if kind == "bytes" else 3, **opt)
+           for o in range(nparts)]
     spt = _t(sp)
     kb = ks_bytes(bk)
     nq = [5000 + 3001 * s for s in range(nparts)]                   # ragged batch per source
