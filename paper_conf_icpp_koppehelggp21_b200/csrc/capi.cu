@@ -83,6 +83,8 @@ struct cuart_index {
     int grid_ctas_per_sm = 0;          // 0 = default grid (one op per thread); else persistent grid
     bool ktimer = false;               // record CUDA events around every k_lookup launch
     int ilp = 2;                       // queries per thread of the pre-bucketed wide walk (k_lookup_wq)
+    unsigned wq_tpb = 64;              // k_lookup_wq / k_upd1_wq threads per CTA (CUART_WQ_TPB: 64 / 128 / 256)
+    unsigned lk_tpb = 256;             // k_lookup threads per CTA (CUART_LOOKUP_TPB: 64 / 128 / 256)
     std::mutex kmu;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev;
     uint64_t klookups = 0;
@@ -121,8 +123,8 @@ static void drop_kevents(cuart_index* h) {
 
 // ============================================================================ kernels
 // SEG: out is ignored, result i goes to so.at(i) (fused multi-GPU return, §8(e)).
-template <class Key, int POL, bool SEG = false>
-__global__ void __launch_bounds__(256) k_lookup(DevIndex ix, const void* __restrict__ q,
+template <class Key, int POL, bool SEG = false, int TPB = 256>
+__global__ void __launch_bounds__(TPB) k_lookup(DevIndex ix, const void* __restrict__ q,
                                                 const uint8_t* __restrict__ lens, uint64_t n,
                                                 uint64_t* __restrict__ out, SegOut so = SegOut{}) {
     const Loader<POL> ld;
@@ -145,17 +147,17 @@ __global__ void __launch_bounds__(256) k_lookup(DevIndex ix, const void* __restr
 // latency of its chain: 64 warps/SM x 32 queries per ~2 us).  Queries whose path
 // is not "wide entry -> leaf" finish with the generic find_leaf.  Results are
 // identical to k_lookup.
-template <class Key, int POL, int Q, bool SEG = false>
-__global__ void __launch_bounds__(256) k_lookup_wq(DevIndex ix, const void* __restrict__ q,
+template <class Key, int POL, int Q, int TPB = 256, bool SEG = false>
+__global__ void __launch_bounds__(TPB) k_lookup_wq(DevIndex ix, const void* __restrict__ q,
                                                    const uint8_t* __restrict__ lens, uint64_t n,
                                                    uint64_t* __restrict__ out, SegOut so = SegOut{}) {
     static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
     const Loader<POL> ld;
-    const uint64_t i0 = uint64_t(blockIdx.x) * (256 * Q) + threadIdx.x;
+    const uint64_t i0 = uint64_t(blockIdx.x) * (TPB * Q) + threadIdx.x;
     Key k[Q];
 #pragma unroll
     for (int j = 0; j < Q; j++) {
-        const uint64_t i = i0 + uint64_t(j) * 256;
+        const uint64_t i = i0 + uint64_t(j) * TPB;
         k[j] = i < n ? Key::template load<true>(q, lens, i) : Key{0};
     }
     U8x32 e[Q];
@@ -170,7 +172,7 @@ __global__ void __launch_bounds__(256) k_lookup_wq(DevIndex ix, const void* __re
         if (link_type(link[j]) == T_LEAF8) r[j] = ld.leafv4(ix.base[T_LEAF8] + link_index(link[j]) * record_bytes(T_LEAF8));
 #pragma unroll
     for (int j = 0; j < Q; j++) {
-        const uint64_t i = i0 + uint64_t(j) * 256;
+        const uint64_t i = i0 + uint64_t(j) * TPB;
         if (i >= n) continue;
         uint64_t res = kMiss;
         if (link_type(link[j]) == T_LEAF8) {
@@ -318,19 +320,19 @@ __global__ void __launch_bounds__(256) k_upd1(DevIndex ix, const void* __restric
 // k_upd1's work with Q ops per thread in lockstep phases, as k_lookup_wq (keys,
 // values and op indices, then the wide entries, then the leaf records are all
 // requested before use).  Same outputs as k_upd1<Key, 5, false>.
-template <class Key, int Q>
-__global__ void __launch_bounds__(256) k_upd1_wq(DevIndex ix, const void* __restrict__ q, const uint64_t* __restrict__ vals,
+template <class Key, int Q, int TPB = 64>
+__global__ void __launch_bounds__(TPB) k_upd1_wq(DevIndex ix, const void* __restrict__ q, const uint64_t* __restrict__ vals,
                                                  uint64_t n, uint64_t epoch_hi, uint64_t* __restrict__ leafref,
                                                  const uint32_t* __restrict__ opidx) {
     static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
     const Loader<5> ld;
-    const uint64_t i0 = uint64_t(blockIdx.x) * (256 * Q) + threadIdx.x;
+    const uint64_t i0 = uint64_t(blockIdx.x) * (TPB * Q) + threadIdx.x;
     Key k[Q];
     uint64_t v[Q];
     uint32_t pr[Q];
 #pragma unroll
     for (int j = 0; j < Q; j++) {
-        const uint64_t i = i0 + uint64_t(j) * 256;
+        const uint64_t i = i0 + uint64_t(j) * TPB;
         const bool ok = i < n;
         k[j] = ok ? Key::template load<true>(q, nullptr, i) : Key{0};
         v[j] = ok ? uint64_t(__ldcs((const unsigned long long*)vals + i)) : 0;
@@ -348,7 +350,7 @@ __global__ void __launch_bounds__(256) k_upd1_wq(DevIndex ix, const void* __rest
         if (link_type(link[j]) == T_LEAF8) r[j] = ld.leafv4(ix.base[T_LEAF8] + link_index(link[j]) * record_bytes(T_LEAF8));
 #pragma unroll
     for (int j = 0; j < Q; j++) {
-        const uint64_t i = i0 + uint64_t(j) * 256;
+        const uint64_t i = i0 + uint64_t(j) * TPB;
         if (i >= n) continue;
         uint64_t leaf = 0, val = kMiss;
         if (link_type(link[j]) == T_LEAF8) {
@@ -544,9 +546,12 @@ static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, co
     cudaEvent_t ev0, ev1;
     ktimer_begin(h, s, ev0, ev1);                      // per-launch k_lookup timing (cuart_kernel_timer)
     if (bucketed && dx.walk_wide && h->policy == 5 && h->ilp > 1 && (kind == CUART_KEY_U64 || kind == CUART_KEY_U32)) {
-        const unsigned g = unsigned((n + 256 * h->ilp - 1) / (256 * h->ilp));
+        const unsigned tpb = h->wq_tpb;
+        const unsigned g = unsigned((n + tpb * h->ilp - 1) / (tpb * h->ilp));
 #define CUART_WQ(K)                                                                              \
-        if (h->ilp == 2) k_lookup_wq<K, 5, 2><<<g, 256, 0, s>>>(dx, q, lens, n, out);            \
+        if (h->ilp == 2 && tpb == 128) k_lookup_wq<K, 5, 2, 128><<<g, 128, 0, s>>>(dx, q, lens, n, out); \
+        else if (h->ilp == 2 && tpb == 64) k_lookup_wq<K, 5, 2, 64><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
+        else if (h->ilp == 2) k_lookup_wq<K, 5, 2><<<g, 256, 0, s>>>(dx, q, lens, n, out);       \
         else k_lookup_wq<K, 5, 4><<<g, 256, 0, s>>>(dx, q, lens, n, out);
         if (kind == CUART_KEY_U64) { CUART_WQ(KeyU64) } else { CUART_WQ(KeyU32) }
 #undef CUART_WQ
@@ -555,7 +560,12 @@ static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, co
         CU_TRY(cudaGetLastError());
         return CUART_OK;
     }
-#define CUART_LOOKUP(K, P) k_lookup<K, P><<<grid, 256, 0, s>>>(dx, q, lens, n, out)
+    const unsigned ltpb = h->lk_tpb == 64 || h->lk_tpb == 128 ? h->lk_tpb : 256u;
+    const unsigned lgrid = ltpb == 256 ? unsigned(grid) : unsigned((n + ltpb - 1) / ltpb);
+#define CUART_LOOKUP(K, P)                                                                      \
+    if (ltpb == 64) k_lookup<K, P, false, 64><<<lgrid, 64, 0, s>>>(dx, q, lens, n, out);        \
+    else if (ltpb == 128) k_lookup<K, P, false, 128><<<lgrid, 128, 0, s>>>(dx, q, lens, n, out); \
+    else k_lookup<K, P><<<grid, 256, 0, s>>>(dx, q, lens, n, out)
 #define CUART_LOOKUP_POL(K)                          \
     switch (h->policy) {                             \
     case 0: CUART_LOOKUP(K, 0); break;               \
@@ -637,9 +647,9 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
     }
         const bool wq = !del && bucketed && dx.walk_wide && h->policy == 5 && h->ilp > 1 &&
                         (kind == CUART_KEY_U64 || kind == CUART_KEY_U32);
-        const unsigned gq = unsigned((m + 512 - 1) / 512);
-        if (wq && kind == CUART_KEY_U64) k_upd1_wq<KeyU64, 2><<<gq, 256, 0, s>>>(dx, kb, vb, m, epoch_hi, h->leafref, ib);
-        else if (wq) k_upd1_wq<KeyU32, 2><<<gq, 256, 0, s>>>(dx, kb, vb, m, epoch_hi, h->leafref, ib);
+        const unsigned gq = unsigned((m + 128 - 1) / 128);         // 64 threads x 2 ops per CTA
+        if (wq && kind == CUART_KEY_U64) k_upd1_wq<KeyU64, 2><<<gq, 64, 0, s>>>(dx, kb, vb, m, epoch_hi, h->leafref, ib);
+        else if (wq) k_upd1_wq<KeyU32, 2><<<gq, 64, 0, s>>>(dx, kb, vb, m, epoch_hi, h->leafref, ib);
         else switch (kind) {
         case CUART_KEY_U64: CUART_UPD1_POL(KeyU64); break;
         case CUART_KEY_U32: CUART_UPD1_POL(KeyU32); break;
@@ -924,7 +934,9 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     h->lut_format = fmt;
     if (const char* pe = getenv("CUART_POLICY")) h->policy = atoi(pe);
     if (const char* pe = getenv("CUART_GRID_CTAS_PER_SM")) h->grid_ctas_per_sm = atoi(pe);   // tuning knob
-    if (const char* pe = getenv("CUART_ILP")) h->ilp = atoi(pe);   // queries per thread of the wide walk (1, 2, 4)
+    if (const char* pe = getenv("CUART_ILP")) h->ilp = atoi(pe);
+    if (const char* pe = getenv("CUART_WQ_TPB")) h->wq_tpb = unsigned(atoi(pe));
+    if (const char* pe = getenv("CUART_LOOKUP_TPB")) h->lk_tpb = unsigned(atoi(pe));   // queries per thread of the wide walk (1, 2, 4)
     h->prebucket = opts ? opts->prebucket : CUART_PREBUCKET_AUTO;
     if (h->prebucket > CUART_PREBUCKET_ON) {
         delete h;
