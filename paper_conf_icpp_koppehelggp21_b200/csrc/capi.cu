@@ -85,6 +85,7 @@ struct cuart_index {
     int ilp = 2;                       // queries per thread of the pre-bucketed wide walk (k_lookup_wq)
     unsigned wq_tpb = 64;              // k_lookup_wq / k_upd1_wq threads per CTA (CUART_WQ_TPB: 64 / 128 / 256)
     unsigned lk_tpb = 256;             // k_lookup threads per CTA (CUART_LOOKUP_TPB: 64 / 128 / 256)
+    unsigned upd2_tpb = 256;           // k_upd2 threads per CTA (CUART_UPD2_TPB: 64 / 256)
     std::mutex kmu;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev;
     uint64_t klookups = 0;
@@ -377,8 +378,8 @@ __global__ void __launch_bounds__(TPB) k_upd1_wq(DevIndex ix, const void* __rest
 // or, for a delete, unlink the leaf from its parent slot, clear it (value :=
 // tombstone CUART_MISS; key bytes kept so the leaf buffer stays sorted)
 // and push its id on the free-leaf list.
-template <bool DEL>
-__global__ void __launch_bounds__(256) k_upd2(DevIndex ix, const uint64_t* __restrict__ vals,
+template <bool DEL, int TPB = 256>
+__global__ void __launch_bounds__(TPB) k_upd2(DevIndex ix, const uint64_t* __restrict__ vals,
                                               const uint8_t* __restrict__ is_delete, uint64_t n, uint64_t epoch_hi,
                                               const uint64_t* __restrict__ leafref, const uint64_t* __restrict__ slotref,
                                               const uint32_t* __restrict__ opidx) {
@@ -546,15 +547,18 @@ static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, co
     cudaEvent_t ev0, ev1;
     ktimer_begin(h, s, ev0, ev1);                      // per-launch k_lookup timing (cuart_kernel_timer)
     if (bucketed && dx.walk_wide && h->policy == 5 && h->ilp > 1 && (kind == CUART_KEY_U64 || kind == CUART_KEY_U32)) {
-        const unsigned tpb = h->wq_tpb;
-        const unsigned g = unsigned((n + tpb * h->ilp - 1) / (tpb * h->ilp));
-#define CUART_WQ(K)                                                                              \
-        if (h->ilp == 2 && tpb == 128) k_lookup_wq<K, 5, 2, 128><<<g, 128, 0, s>>>(dx, q, lens, n, out); \
-        else if (h->ilp == 2 && tpb == 64) k_lookup_wq<K, 5, 2, 64><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
-        else if (h->ilp == 2) k_lookup_wq<K, 5, 2><<<g, 256, 0, s>>>(dx, q, lens, n, out);       \
-        else k_lookup_wq<K, 5, 4><<<g, 256, 0, s>>>(dx, q, lens, n, out);
+        const unsigned tpb = h->wq_tpb == 128 || h->wq_tpb == 256 ? h->wq_tpb : 64u;
+        const unsigned qpt = h->ilp == 4 ? 4u : 2u;                   // queries per thread (template Q)
+        const unsigned g = unsigned((n + tpb * qpt - 1) / (tpb * qpt));
+#define CUART_WQ_Q(K, Q)                                                                          \
+        if (tpb == 64) k_lookup_wq<K, 5, Q, 64><<<g, 64, 0, s>>>(dx, q, lens, n, out);            \
+        else if (tpb == 128) k_lookup_wq<K, 5, Q, 128><<<g, 128, 0, s>>>(dx, q, lens, n, out);    \
+        else k_lookup_wq<K, 5, Q, 256><<<g, 256, 0, s>>>(dx, q, lens, n, out);
+#define CUART_WQ(K)                                                                               \
+        if (qpt == 4) { CUART_WQ_Q(K, 4) } else { CUART_WQ_Q(K, 2) }
         if (kind == CUART_KEY_U64) { CUART_WQ(KeyU64) } else { CUART_WQ(KeyU32) }
 #undef CUART_WQ
+#undef CUART_WQ_Q
         g_cuart_launches++;
         ktimer_end(h, s, ev0, ev1, n);
         CU_TRY(cudaGetLastError());
@@ -661,6 +665,7 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
         g_cuart_launches++;
         CU_TRY(cudaGetLastError());
         if (del) k_upd2<true><<<grid, 256, 0, s>>>(dx, vb, db, m, epoch_hi, h->leafref, h->slotref, ib);
+        else if (h->upd2_tpb == 64) k_upd2<false, 64><<<unsigned((m + 63) / 64), 64, 0, s>>>(dx, vb, nullptr, m, epoch_hi, h->leafref, nullptr, ib);
         else k_upd2<false><<<grid, 256, 0, s>>>(dx, vb, nullptr, m, epoch_hi, h->leafref, nullptr, ib);
         g_cuart_launches++;
         CU_TRY(cudaGetLastError());
@@ -936,7 +941,8 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     if (const char* pe = getenv("CUART_GRID_CTAS_PER_SM")) h->grid_ctas_per_sm = atoi(pe);   // tuning knob
     if (const char* pe = getenv("CUART_ILP")) h->ilp = atoi(pe);
     if (const char* pe = getenv("CUART_WQ_TPB")) h->wq_tpb = unsigned(atoi(pe));
-    if (const char* pe = getenv("CUART_LOOKUP_TPB")) h->lk_tpb = unsigned(atoi(pe));   // queries per thread of the wide walk (1, 2, 4)
+    if (const char* pe = getenv("CUART_LOOKUP_TPB")) h->lk_tpb = unsigned(atoi(pe));
+    if (const char* pe = getenv("CUART_UPD2_TPB")) h->upd2_tpb = unsigned(atoi(pe));   // queries per thread of the wide walk (1, 2, 4)
     h->prebucket = opts ? opts->prebucket : CUART_PREBUCKET_AUTO;
     if (h->prebucket > CUART_PREBUCKET_ON) {
         delete h;
