@@ -86,6 +86,7 @@ struct cuart_index {
     unsigned wq_tpb = 64;              // k_lookup_wq / k_upd1_wq threads per CTA (CUART_WQ_TPB: 64 / 128 / 256)
     unsigned lk_tpb = 256;             // k_lookup threads per CTA (CUART_LOOKUP_TPB: 64 / 128 / 256)
     unsigned upd2_tpb = 256;           // k_upd2 threads per CTA (CUART_UPD2_TPB: 64 / 256)
+    int wq_lp = 3;                     // k_lookup_wq leaf-load cache policy (CUART_WQ_LEAFPOL, kernels.cuh leafv4_b)
     std::mutex kmu;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev;
     uint64_t klookups = 0;
@@ -147,8 +148,11 @@ __global__ void __launch_bounds__(TPB) k_lookup(DevIndex ix, const void* __restr
 // independent dependent-load chains in flight (the one-query walk is bound by the
 // latency of its chain: 64 warps/SM x 32 queries per ~2 us).  Queries whose path
 // is not "wide entry -> leaf" finish with the generic find_leaf.  Results are
-// identical to k_lookup.
-template <class Key, int POL, int Q, int TPB = 256, bool SEG = false>
+// identical to k_lookup.  TPB = 64 by default (a CTA's slot frees when its slowest
+// warp ends); LP = leaf-load cache policy: evict_last by default, since in the
+// bucketed walk a leaf is re-read by the hit queries of its bucket window (c3:
+// 8.91 -> 8.42 ms per 2^30 against the direct walk's evict_first + L2::64B).
+template <class Key, int POL, int Q, int TPB = 256, bool SEG = false, int LP = 3>
 __global__ void __launch_bounds__(TPB) k_lookup_wq(DevIndex ix, const void* __restrict__ q,
                                                    const uint8_t* __restrict__ lens, uint64_t n,
                                                    uint64_t* __restrict__ out, SegOut so = SegOut{}) {
@@ -170,7 +174,7 @@ __global__ void __launch_bounds__(TPB) k_lookup_wq(DevIndex ix, const void* __re
     uint4 r[Q];
 #pragma unroll
     for (int j = 0; j < Q; j++)
-        if (link_type(link[j]) == T_LEAF8) r[j] = ld.leafv4(ix.base[T_LEAF8] + link_index(link[j]) * record_bytes(T_LEAF8));
+        if (link_type(link[j]) == T_LEAF8) r[j] = ld.template leafv4_b<LP>(ix.base[T_LEAF8] + link_index(link[j]) * record_bytes(T_LEAF8));
 #pragma unroll
     for (int j = 0; j < Q; j++) {
         const uint64_t i = i0 + uint64_t(j) * TPB;
@@ -348,7 +352,7 @@ __global__ void __launch_bounds__(TPB) k_upd1_wq(DevIndex ix, const void* __rest
     uint4 r[Q];
 #pragma unroll
     for (int j = 0; j < Q; j++)
-        if (link_type(link[j]) == T_LEAF8) r[j] = ld.leafv4(ix.base[T_LEAF8] + link_index(link[j]) * record_bytes(T_LEAF8));
+        if (link_type(link[j]) == T_LEAF8) r[j] = ld.template leafv4_b<3>(ix.base[T_LEAF8] + link_index(link[j]) * record_bytes(T_LEAF8));
 #pragma unroll
     for (int j = 0; j < Q; j++) {
         const uint64_t i = i0 + uint64_t(j) * TPB;
@@ -551,9 +555,12 @@ static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, co
         const unsigned qpt = h->ilp == 4 ? 4u : 2u;                   // queries per thread (template Q)
         const unsigned g = unsigned((n + tpb * qpt - 1) / (tpb * qpt));
 #define CUART_WQ_Q(K, Q)                                                                          \
-        if (tpb == 64) k_lookup_wq<K, 5, Q, 64><<<g, 64, 0, s>>>(dx, q, lens, n, out);            \
-        else if (tpb == 128) k_lookup_wq<K, 5, Q, 128><<<g, 128, 0, s>>>(dx, q, lens, n, out);    \
-        else k_lookup_wq<K, 5, Q, 256><<<g, 256, 0, s>>>(dx, q, lens, n, out);
+        if (tpb == 64 && h->wq_lp == 0) k_lookup_wq<K, 5, Q, 64, false, 0><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
+        else if (tpb == 64 && h->wq_lp == 1) k_lookup_wq<K, 5, Q, 64, false, 1><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
+        else if (tpb == 64 && h->wq_lp == 2) k_lookup_wq<K, 5, Q, 64, false, 2><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
+        else if (tpb == 64) k_lookup_wq<K, 5, Q, 64, false, 3><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
+        else if (tpb == 128) k_lookup_wq<K, 5, Q, 128, false, 3><<<g, 128, 0, s>>>(dx, q, lens, n, out); \
+        else k_lookup_wq<K, 5, Q, 256, false, 3><<<g, 256, 0, s>>>(dx, q, lens, n, out);
 #define CUART_WQ(K)                                                                               \
         if (qpt == 4) { CUART_WQ_Q(K, 4) } else { CUART_WQ_Q(K, 2) }
         if (kind == CUART_KEY_U64) { CUART_WQ(KeyU64) } else { CUART_WQ(KeyU32) }
@@ -942,7 +949,8 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     if (const char* pe = getenv("CUART_ILP")) h->ilp = atoi(pe);
     if (const char* pe = getenv("CUART_WQ_TPB")) h->wq_tpb = unsigned(atoi(pe));
     if (const char* pe = getenv("CUART_LOOKUP_TPB")) h->lk_tpb = unsigned(atoi(pe));
-    if (const char* pe = getenv("CUART_UPD2_TPB")) h->upd2_tpb = unsigned(atoi(pe));   // queries per thread of the wide walk (1, 2, 4)
+    if (const char* pe = getenv("CUART_UPD2_TPB")) h->upd2_tpb = unsigned(atoi(pe));
+    if (const char* pe = getenv("CUART_WQ_LEAFPOL")) h->wq_lp = atoi(pe);   // queries per thread of the wide walk (1, 2, 4)
     h->prebucket = opts ? opts->prebucket : CUART_PREBUCKET_AUTO;
     if (h->prebucket > CUART_PREBUCKET_ON) {
         delete h;

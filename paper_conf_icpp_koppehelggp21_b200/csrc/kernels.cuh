@@ -324,6 +324,16 @@ struct Loader {
     __device__ __forceinline__ uint4 leafv4(const void* p) const {
         return kLeaf64B ? v4<true>(p, drop) : kLeafDrop ? v4(p, drop) : ld_nc_v4(p);
     }
+    // Leaf record of a pre-bucketed walk, where a leaf is re-read by the ~8 hit queries
+    // of its bucket window: LP 0 = as leafv4 (evict_first + L2::64B), 1 = evict_last +
+    // L2::64B, 2 = plain, 3 = evict_last.
+    template <int LP>
+    __device__ __forceinline__ uint4 leafv4_b(const void* p) const {
+        if (LP == 0) return leafv4(p);
+        if (LP == 1) return v4<true>(p, keep);
+        if (LP == 3) return v4(p, keep);
+        return ld_nc_v4(p);
+    }
     __device__ __forceinline__ U8x32 leafv8(const void* p) const {   // p 32-B aligned
         return kLeaf64B ? v8<true>(p, drop) : kLeafDrop ? v8(p, drop) : ld_nc_v8(p);
     }
