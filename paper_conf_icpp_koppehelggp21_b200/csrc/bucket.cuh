@@ -45,9 +45,13 @@ __host__ __device__ constexpr uint64_t hist_entries(uint64_t tiles) {
     return ((tiles + kHistGroup - 1) / kHistGroup) * kHistGroup * kBuckets;
 }
 
+// `depth` packs the key byte the buckets are taken from (bits 7..0: the root's
+// branch depth) and a right shift of that byte (bits 15..8): shift s gives 256 >> s
+// buckets (the upper bucket ids stay empty; every kernel below is unchanged).
 template <class Key>
 __device__ __forceinline__ uint32_t bucket_of(const Key& k, uint32_t depth) {
-    return depth < k.len() ? k.byte(depth) : 0u;
+    const uint32_t d = depth & 0xFFu;
+    return d < k.len() ? k.byte(d) >> (depth >> 8) : 0u;
 }
 
 // Bucket of query i straight from the batch: integer keys from their word, byte
@@ -56,8 +60,8 @@ template <class Key>
 __device__ __forceinline__ uint32_t bucket_at(const void* q, const uint8_t* lens, uint64_t i, uint32_t depth) {
     if (Key::kKind == 2) return bucket_of(KeyU64{uint64_t(__ldcs((const unsigned long long*)q + i))}, depth);
     if (Key::kKind == 1) return bucket_of(KeyU32{uint32_t(__ldcs((const unsigned int*)q + i))}, depth);
-    const uint32_t l = __ldcs(lens + i);
-    return depth < l ? uint32_t(__ldcs((const uint8_t*)q + 32 * i + depth)) : 0u;
+    const uint32_t l = __ldcs(lens + i), d = depth & 0xFFu;
+    return d < l ? uint32_t(__ldcs((const uint8_t*)q + 32 * i + d)) >> (depth >> 8) : 0u;
 }
 
 // Block-wide exclusive scan of one value per thread (kBucketThreads == kBuckets == 256).

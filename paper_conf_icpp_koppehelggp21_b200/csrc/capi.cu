@@ -87,6 +87,11 @@ struct cuart_index {
     unsigned lk_tpb = 256;             // k_lookup threads per CTA (CUART_LOOKUP_TPB: 64 / 128 / 256)
     unsigned upd2_tpb = 256;           // k_upd2 threads per CTA (CUART_UPD2_TPB: 64 / 256)
     int wq_lp = 3;                     // k_lookup_wq leaf-load cache policy (CUART_WQ_LEAFPOL, kernels.cuh leafv4_b)
+    // K-BUCKET on the root byte >> shift: 256 >> shift buckets (CUART_BUCKET_SHIFT).  Set
+    // at upload: 64 buckets when a bucket's slice of the walked records stays within
+    // 64 MB (c2, c3: runs of ~64 keys per tile cut the run-scattered traffic of scatter
+    // and gather while the slice stays L2-resident), else 256 (c5 at N = 1: 60 GB).
+    uint32_t bucket_shift = 0;
     std::mutex kmu;
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev;
     uint64_t klookups = 0;
@@ -483,7 +488,8 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
     CU_TRY(cudaMallocAsync((void**)&scr, total, s));
     unsigned int* hist = (unsigned int*)(scr + o_hist);
     unsigned int* tot = (unsigned int*)(scr + o_tot);
-    const uint32_t depth = link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u;
+    const uint32_t depth = (link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u) |
+                           (h->bucket_shift << 8);
     if ((uintptr_t(q) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
     else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
     k_bscan_rows<<<kBuckets, kBucketThreads, 0, s>>>(hist, tiles, tot);
@@ -498,7 +504,8 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
     // and on c2 (3.10 vs 2.57 ms per 2^28: the per-bucket CTA barriers).  Kept as an
     // explicit option (CUART_SLICE_ON) with its parity tests.
     (void)slice_bytes;
-    const bool slice = Key::kKind != 3 && h->slice_ok && h->policy == 5 && h->slice_lut == CUART_SLICE_ON;
+    const bool slice = Key::kKind != 3 && h->slice_ok && h->policy == 5 && h->slice_lut == CUART_SLICE_ON &&
+                       h->bucket_shift == 0;
     cuart_status rc = CUART_OK;
     if (slice) rc = launch_lookup_slice<Key>(h, scr + o_q, n, (uint64_t*)(scr + o_res), tot, s);
     else rc = launch_lookup_direct(h, Key::kKind, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, n,
@@ -696,7 +703,8 @@ static cuart_status launch_update_bucketed(cuart_index* h, const void* k, const 
     CU_TRY(cudaMallocAsync((void**)&scr, total, s));
     unsigned int* hist = (unsigned int*)(scr + o_hist);
     unsigned int* tot = (unsigned int*)(scr + o_tot);
-    const uint32_t depth = link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u;
+    const uint32_t depth = (link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u) |
+                           (h->bucket_shift << 8);
     if ((uintptr_t(k) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
     else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
     k_bscan_rows<<<kBuckets, kBucketThreads, 0, s>>>(hist, tiles, tot);
@@ -945,12 +953,13 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     }
     h->lut_format = fmt;
     if (const char* pe = getenv("CUART_POLICY")) h->policy = atoi(pe);
-    if (const char* pe = getenv("CUART_GRID_CTAS_PER_SM")) h->grid_ctas_per_sm = atoi(pe);   // tuning knob
+    // tuning knobs (environment; the defaults are the measured best)
+    if (const char* pe = getenv("CUART_GRID_CTAS_PER_SM")) h->grid_ctas_per_sm = atoi(pe);
     if (const char* pe = getenv("CUART_ILP")) h->ilp = atoi(pe);
     if (const char* pe = getenv("CUART_WQ_TPB")) h->wq_tpb = unsigned(atoi(pe));
     if (const char* pe = getenv("CUART_LOOKUP_TPB")) h->lk_tpb = unsigned(atoi(pe));
     if (const char* pe = getenv("CUART_UPD2_TPB")) h->upd2_tpb = unsigned(atoi(pe));
-    if (const char* pe = getenv("CUART_WQ_LEAFPOL")) h->wq_lp = atoi(pe);   // queries per thread of the wide walk (1, 2, 4)
+    if (const char* pe = getenv("CUART_WQ_LEAFPOL")) h->wq_lp = atoi(pe);
     h->prebucket = opts ? opts->prebucket : CUART_PREBUCKET_AUTO;
     if (h->prebucket > CUART_PREBUCKET_ON) {
         delete h;
@@ -1025,6 +1034,12 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     h->err_off = off;
     off = align(off + 256);
     h->arena_bytes = off;
+    {
+        uint64_t walked = lutw.size() * 8;                // records a bucketed walk reads
+        for (int t = 1; t < 8; t++) walked += L.buf[t].size();
+        h->bucket_shift = walked <= (uint64_t(64) << 26) ? 2u : 0u;   // slice <= 64 MB at 64 buckets
+        if (const char* pe = getenv("CUART_BUCKET_SHIFT")) h->bucket_shift = uint32_t(atoi(pe)) & 7u;
+    }
     cudaError_t e = cudaMalloc(&h->arena, off);
     if (e != cudaSuccess) {
         delete h;
@@ -1062,6 +1077,7 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     h->slice_lut = opts ? opts->slice_lut : CUART_SLICE_AUTO;
     if (h->slice_lut > CUART_SLICE_ON) rc = CUART_ERR_INVALID_ARGUMENT;
     if (const char* pe = getenv("CUART_SLICE")) h->slice_lut = atoi(pe) == 1 ? CUART_SLICE_OFF : atoi(pe) == 2 ? CUART_SLICE_ON : CUART_SLICE_AUTO;
+    if (h->slice_lut == CUART_SLICE_ON) h->bucket_shift = 0;    // the slice walk needs one bucket per root byte
     {
         const uint32_t rt = link_type(L.root);
         const uint32_t d = (rt >= T_N4 && rt <= T_N256) ? link_aux(L.root) : 0xFFu;
