@@ -182,10 +182,13 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscan_rows(unsigned int* __r
 }
 
 // totals -> exclusive bucket bases (in place), one CTA of kBuckets threads
-__global__ void __launch_bounds__(kBuckets) k_bscan(unsigned int* __restrict__ counts) {
+// Only the first nb buckets are in use (256 >> shift): the others count 0 (their
+// totals were never written) and get base = n.
+__global__ void __launch_bounds__(kBuckets) k_bscan(unsigned int* __restrict__ counts, uint32_t nb) {
     __shared__ unsigned int s[kBuckets];
     const int t = threadIdx.x;
-    s[t] = counts[t];
+    const unsigned int own = uint32_t(t) < nb ? counts[t] : 0u;
+    s[t] = own;
     __syncthreads();
     for (int d = 1; d < kBuckets; d <<= 1) {
         const unsigned int v = t >= d ? s[t - d] : 0u;
@@ -193,7 +196,7 @@ __global__ void __launch_bounds__(kBuckets) k_bscan(unsigned int* __restrict__ c
         s[t] += v;
         __syncthreads();
     }
-    counts[t] = s[t] - counts[t];   // exclusive
+    counts[t] = s[t] - own;   // exclusive
 }
 
 template <class Key>

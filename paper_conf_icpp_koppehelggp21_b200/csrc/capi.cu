@@ -492,8 +492,8 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
                            (h->bucket_shift << 8);
     if ((uintptr_t(q) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
     else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
-    k_bscan_rows<<<kBuckets, kBucketThreads, 0, s>>>(hist, tiles, tot);
-    k_bscan<<<1, kBuckets, 0, s>>>(tot);
+    k_bscan_rows<<<kBuckets >> h->bucket_shift, kBucketThreads, 0, s>>>(hist, tiles, tot);   // rows in use only
+    k_bscan<<<1, kBuckets, 0, s>>>(tot, kBuckets >> h->bucket_shift);
     k_bscatter<Key><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key>(), s>>>(
         q, lens, n, depth, hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, (uint16_t*)(scr + o_pos));
     g_cuart_launches += 4;
@@ -707,8 +707,8 @@ static cuart_status launch_update_bucketed(cuart_index* h, const void* k, const 
                            (h->bucket_shift << 8);
     if ((uintptr_t(k) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
     else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
-    k_bscan_rows<<<kBuckets, kBucketThreads, 0, s>>>(hist, tiles, tot);
-    k_bscan<<<1, kBuckets, 0, s>>>(tot);
+    k_bscan_rows<<<kBuckets >> h->bucket_shift, kBucketThreads, 0, s>>>(hist, tiles, tot);   // rows in use only
+    k_bscan<<<1, kBuckets, 0, s>>>(tot, kBuckets >> h->bucket_shift);
     k_bscatter<Key, true><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key, true>(), s>>>(
         k, lens, n, depth, hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, nullptr, vals,
         (uint64_t*)(scr + o_val), (uint32_t*)(scr + o_idx));

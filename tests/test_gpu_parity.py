@@ -241,6 +241,34 @@ def test_host_pipeline_many_chunks(kind, monkeypatch):
     ix.close()
 
 
+@pytest.mark.parametrize("shift", ["0", "2", "3"])
+def test_prebucket_bucket_counts_and_skew(shift, monkeypatch):
+    """K-BUCKET with 256 / 64 / 32 buckets (CUART_BUCKET_SHIFT, read at upload) on
+    skewed batches: every query in one bucket, queries in two buckets, and a ragged
+    uniform batch; lookups and a bucketed update batch must equal the plain map."""
+    monkeypatch.setenv("CUART_BUCKET_SHIFT", shift)
+    rng = np.random.default_rng(int(shift) + 40)
+    keys, vals = W.build_set(W.CONFIGS["c1"])
+    ix = C.Index(keys, vals, lut_bytes=3, prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_ON)
+    mp = MapOracle(keys, vals)
+    top = keys >> np.uint64(56)
+    one = keys[top == top[0]]
+    two = keys[(top == top[0]) | (top == top[1])]
+    batches = [one[rng.integers(0, one.shape[0], 20_000)],
+               np.concatenate([two[rng.integers(0, two.shape[0], 9_000)],
+                               (rng.integers(0, 2**56, 3_000, dtype=np.uint64) | (top[0] << np.uint64(56)))]),
+               np.where(rng.random(70_001) < 0.5, keys[rng.integers(0, keys.shape[0], 70_001)],
+                        rng.integers(0, 2**64, 70_001, dtype=np.uint64))]
+    for q in batches:
+        assert np.array_equal(_lookup(ix, q), mp.lookup(q))
+    uk = one[rng.integers(0, one.shape[0], 30_000)]
+    uv = rng.integers(0, 2**63, uk.shape[0], dtype=np.uint64)
+    ix.update(_t(uk), _t(uv))
+    mp.update(uk, uv)
+    assert np.array_equal(_lookup(ix, keys), mp.lookup(keys))
+    ix.close()
+
+
 def test_c2_full_size_sampled():
     """Config 2 at full size (2^24 dense u32 keys, LUT over the first 3 bytes):
     2^28 lookups in the bench's launch configuration; sampled outputs vs the

@@ -779,7 +779,7 @@ int main(int argc, char** argv) {
     timeit("k_bscan_rows", hist_entries(tiles) * 8.0, [&] { k_bhist<KeyU64, true><<<T, 256>>>(q, nullptr, n, 0, hist); k_bscan_rows<<<kBuckets, kBucketThreads>>>(hist, tiles, tot); });
     k_bhist<KeyU64, true><<<T, 256>>>(q, nullptr, n, 0, hist);
     k_bscan_rows<<<kBuckets, kBucketThreads>>>(hist, tiles, tot);
-    k_bscan<<<1, kBuckets>>>(tot);
+    k_bscan<<<1, kBuckets>>>(tot, kBuckets);
     timeit("k_bscatter", n * 18.0, [&] { k_bscatter<KeyU64><<<T, 256, smem>>>(q, nullptr, n, 0, hist, tot, bq, nullptr, jpos); });
     timeit("k_bgather", n * 18.0, [&] { k_bgather<false><<<T, 256>>>(res, jpos, n, hist, tot, out); });
     const unsigned long long c1 = checksum(out, n);
@@ -837,7 +837,7 @@ int main(int argc, char** argv) {
         cudaFuncSetAttribute(g_big, cudaFuncAttributeMaxDynamicSharedMemorySize, int(gs));
         timeit("h_big", n * 8.0, [&] { h_big<<<unsigned(tb), kBigThreads>>>(q, n, 0, hist); });
         k_bscan_rows<<<kBuckets, kBucketThreads>>>(hist, tb, tot);
-        k_bscan<<<1, kBuckets>>>(tot);
+        k_bscan<<<1, kBuckets>>>(tot, kBuckets);
         timeit("s_big", n * 18.0, [&] { s_big<<<unsigned(tb), kBigThreads, ss>>>(q, n, 0, hist, tot, bq, jpos); });
         timeit("g_big", n * 18.0, [&] { g_big<<<unsigned(tb), kBigThreads, gs>>>(bq, jpos, n, hist, tot, out); });
         printf("{\"roundtrip_big\": %s}\n", checksum(out, n) == s1b ? "true" : "false");
