@@ -561,6 +561,62 @@ __global__ void __launch_bounds__(256, 4) s_nosb(const uint64_t* __restrict__ q,
     }
 }
 
+__global__ void __launch_bounds__(256, 4) s_match(const uint64_t* __restrict__ q, uint64_t n, uint32_t depth,
+                                              const unsigned int* __restrict__ rowoff, const unsigned int* __restrict__ bases,
+                                              uint64_t* __restrict__ bq, uint16_t* __restrict__ jpos) {
+    __shared__ uint64_t skeys[kBucketTile];
+    __shared__ unsigned int h[kBuckets], loc[kBuckets], glb[kBuckets], wtot[8];
+    const int t = threadIdx.x;
+    h[t] = 0;
+    const unsigned int gb = bases[t] + rowoff[hidx(t, blockIdx.x)];
+    __syncthreads();
+    const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
+    uint64_t kv[kBucketItems];
+    uint32_t br[kBucketItems];
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * 256 + t;
+        kv[r] = j < cnt ? uint64_t(__ldcs((const unsigned long long*)q + base + j)) : 0;
+    }
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * 256 + t;
+        br[r] = 0xFFFFFFFFu;
+        const uint32_t b = j < cnt ? bucket_of(KeyU64{kv[r]}, depth) : 0xFFFFu;   // inactive lanes: own group
+        const unsigned peers = __match_any_sync(0xffffffffu, b);
+        const unsigned lane = threadIdx.x & 31u;
+        const int leader = __ffs(peers) - 1;
+        unsigned basev = 0;
+        if (int(lane) == leader && b != 0xFFFFu) basev = atomicAdd(&h[b], unsigned(__popc(peers)));
+        basev = __shfl_sync(0xffffffffu, basev, leader);
+        if (j < cnt) br[r] = (b << 16) | (basev + __popc(peers & ((1u << lane) - 1u)));
+    }
+    __syncthreads();
+    const unsigned int lb = block_excl_scan256(h[t], wtot);
+    loc[t] = lb;
+    glb[t] = gb - lb;
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t jt = uint32_t(r) * 256 + t;
+        if (br[r] != 0xFFFFFFFFu) {
+            const uint32_t b = br[r] >> 16, j = loc[b] + (br[r] & 0xFFFFu);
+            skeys[j] = kv[r];
+            __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
+        }
+    }
+    __syncthreads();
+#pragma unroll 4
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * 256 + t;
+        if (j < cnt) {
+            const uint64_t kk = skeys[j];
+            __stcs((unsigned long long*)bq + uint64_t(glb[bucket_of(KeyU64{kk}, depth)] + j), (unsigned long long)kk);
+        }
+    }
+}
+
 __global__ void __launch_bounds__(256, 4) s_seqw(const uint64_t* __restrict__ q, uint64_t n, uint32_t depth,
                                               const unsigned int* __restrict__ rowoff, const unsigned int* __restrict__ bases,
                                               uint64_t* __restrict__ bq, uint16_t* __restrict__ jpos) {
@@ -812,6 +868,24 @@ int main(int argc, char** argv) {
     timeit("s_nosb", n * 18.0, [&] { s_nosb<<<T, 256>>>(q, n, 0, hist, tot, bq, jpos); });
     g_ca<<<T, 256>>>(bq, jpos, n, hist, tot, out);
     printf("{\"roundtrip_s_nosb\": %s}\n", checksum(out, n) == s1b ? "true" : "false");
+    timeit("s_match (match_any ranking, 256 buckets)", n * 18.0, [&] { s_match<<<T, 256>>>(q, n, 0, hist, tot, bq, jpos); });
+    g_ca<<<T, 256>>>(bq, jpos, n, hist, tot, out);
+    printf("{\"roundtrip_s_match\": %s}\n", checksum(out, n) == s1b ? "true" : "false");
+    {   // 64 buckets (root byte >> 2), as the product default for c3
+        const uint32_t d64 = 2u << 8;
+        k_bhist<KeyU64, true><<<T, 256>>>(q, nullptr, n, d64, hist);
+        k_bscan_rows<<<kBuckets, kBucketThreads>>>(hist, tiles, tot);
+        k_bscan<<<1, kBuckets>>>(tot, kBuckets);
+        timeit("k_bscatter_64", n * 18.0, [&] { k_bscatter<KeyU64><<<T, 256, smem>>>(q, nullptr, n, d64, hist, tot, bq, nullptr, jpos); });
+        timeit("k_bgather_64", n * 18.0, [&] { k_bgather<false><<<T, 256>>>(bq, jpos, n, hist, tot, out); });
+        printf("{\"roundtrip_64\": %s}\n", checksum(out, n) == s1b ? "true" : "false");
+        timeit("s_match_64", n * 18.0, [&] { s_match<<<T, 256>>>(q, n, d64, hist, tot, bq, jpos); });
+        k_bgather<false><<<T, 256>>>(bq, jpos, n, hist, tot, out);
+        printf("{\"roundtrip_s_match_64\": %s}\n", checksum(out, n) == s1b ? "true" : "false");
+        k_bhist<KeyU64, true><<<T, 256>>>(q, nullptr, n, 0, hist);
+        k_bscan_rows<<<kBuckets, kBucketThreads>>>(hist, tiles, tot);
+        k_bscan<<<1, kBuckets>>>(tot, kBuckets);
+    }
     {
         unsigned int* fill; cudaMalloc(&fill, 256 * 1024 * 4); cudaMemset(fill, 0, 256 * 1024 * 4);
         timeit("atom_alloc_stride1", 0, [&] { atom_alloc<1><<<T, 256>>>(fill, (unsigned int*)sink); });
