@@ -16,6 +16,10 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "lts__t_sectors_op_atom.sum", "lts__t_sectors_op_red.sum", "lts__t_sectors_op_write.sum"]
 
 
+STALL_PREFIX = "smsp__average_warps_issue_stalled_"
+STALL_SUFFIX = "_per_issue_active.ratio"
+
+
 def main(path):
     raw = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(raw.splitlines()))
@@ -25,6 +29,19 @@ def main(path):
         for w in WANT:
             if w in hdr:
                 print(f"    {w:75s} {r[hdr.index(w)]:>22s} {units[hdr.index(w)]}")
+        # stall breakdown: cycles between issues by reason (the dependent-load chain
+        # shows up as long_scoreboard), largest first
+        stalls = []
+        for i, h in enumerate(hdr):
+            if h.startswith(STALL_PREFIX) and h.endswith(STALL_SUFFIX):
+                try:
+                    stalls.append((float(r[i].replace(",", "")), h[len(STALL_PREFIX):-len(STALL_SUFFIX)]))
+                except ValueError:
+                    pass
+        tot = sum(v for v, _ in stalls) or 1.0
+        print("    stall cycles per issued instruction (share):")
+        for v, name in sorted(stalls, reverse=True)[:6]:
+            print(f"        {name:30s} {v:8.2f}  ({100 * v / tot:4.1f}%)")
 
 
 if __name__ == "__main__":
