@@ -136,8 +136,8 @@ __global__ void __launch_bounds__(kBucketThreads) k_bhist(const void* __restrict
 }
 
 // One CTA per bucket: exclusive scan of its row over the tiles (in place), row
-// total -> totals[b].  A thread owns one hist group (kHistGroup = 8 consecutive
-// tiles of this bucket = one 32-B sector), so one pass covers 2048 tiles.
+// total -> totals[b].  A hist group is kHistGroup = 8 consecutive tiles of this
+// bucket = one 32-B sector.
 __global__ void __launch_bounds__(kBucketThreads) k_bscan_rows(unsigned int* __restrict__ hist, uint64_t tiles,
                                                                unsigned int* __restrict__ totals) {
     static_assert(kHistGroup == 8, "one 32-B sector per thread");
@@ -145,33 +145,48 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscan_rows(unsigned int* __r
     __shared__ unsigned int pass_total;
     const uint32_t b = blockIdx.x;
     const uint64_t groups = (tiles + kHistGroup - 1) / kHistGroup;
+    // a thread owns GPT consecutive hist groups per pass (GPT x 32 B in flight), so
+    // one pass covers 256 x GPT x 8 tiles
+    constexpr int GPT = 4;
     unsigned int carry = 0;
-    for (uint64_t g0 = 0; g0 < groups; g0 += kBucketThreads) {
-        const uint64_t g = g0 + threadIdx.x;
-        uint4* p = (uint4*)(hist + (g * kBuckets + b) * kHistGroup);
-        unsigned int v[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-        if (g < groups) {
-            const uint4 a = p[0], c = p[1];
-            v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w;
-            v[4] = c.x; v[5] = c.y; v[6] = c.z; v[7] = c.w;
+    for (uint64_t g0 = 0; g0 < groups; g0 += uint64_t(kBucketThreads) * GPT) {
+        unsigned int v[GPT][8];
 #pragma unroll
-            for (int k = 0; k < 8; k++)
-                if (g * kHistGroup + k >= tiles) v[k] = 0;      // padding entries are never written by k_bhist
+        for (int u = 0; u < GPT; u++) {
+            const uint64_t g = g0 + uint64_t(threadIdx.x) * GPT + u;
+#pragma unroll
+            for (int k = 0; k < 8; k++) v[u][k] = 0;
+            if (g < groups) {
+                const uint4* p = (const uint4*)(hist + (g * kBuckets + b) * kHistGroup);
+                const uint4 a = p[0], c = p[1];
+                v[u][0] = a.x; v[u][1] = a.y; v[u][2] = a.z; v[u][3] = a.w;
+                v[u][4] = c.x; v[u][5] = c.y; v[u][6] = c.z; v[u][7] = c.w;
+#pragma unroll
+                for (int k = 0; k < 8; k++)
+                    if (g * kHistGroup + k >= tiles) v[u][k] = 0;   // padding entries are never written by k_bhist
+            }
         }
         unsigned int s = 0;
 #pragma unroll
-        for (int k = 0; k < 8; k++) s += v[k];
+        for (int u = 0; u < GPT; u++)
+#pragma unroll
+            for (int k = 0; k < 8; k++) s += v[u][k];
         const unsigned int ex = block_excl_scan256(s, wtot);
         unsigned int run = carry + ex;
-        unsigned int o[8];
 #pragma unroll
-        for (int k = 0; k < 8; k++) {
-            o[k] = run;
-            run += v[k];
-        }
-        if (g < groups) {
-            p[0] = make_uint4(o[0], o[1], o[2], o[3]);
-            p[1] = make_uint4(o[4], o[5], o[6], o[7]);
+        for (int u = 0; u < GPT; u++) {
+            const uint64_t g = g0 + uint64_t(threadIdx.x) * GPT + u;
+            unsigned int o[8];
+#pragma unroll
+            for (int k = 0; k < 8; k++) {
+                o[k] = run;
+                run += v[u][k];
+            }
+            if (g < groups) {
+                uint4* p = (uint4*)(hist + (g * kBuckets + b) * kHistGroup);
+                p[0] = make_uint4(o[0], o[1], o[2], o[3]);
+                p[1] = make_uint4(o[4], o[5], o[6], o[7]);
+            }
         }
         if (threadIdx.x == kBucketThreads - 1) pass_total = ex + s;
         __syncthreads();

@@ -1025,7 +1025,14 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
                 lutw[4 * p + 3] = leaf_run_link(rec, t);
                 continue;
             }
-            memcpy(&lutw[4 * p + 1], rec + (t == T_N4 ? kN4Keys : kN16Keys), t == T_N4 ? 4 : 16);
+            uint8_t keys16[16];
+            if (t == T_N4) {                              // padded to 16 with the last key, like an N16,
+                memcpy(keys16, rec + kN4Keys, 4);         // so the walk searches both the same way
+                memset(keys16 + 4, rec[kN4Keys + 3], 12);
+            } else {
+                memcpy(keys16, rec + kN16Keys, 16);
+            }
+            memcpy(&lutw[4 * p + 1], keys16, 16);
             lutw[4 * p + 3] = leaf_run_link(rec, t);      // child i = run + i when all children are leaves
         }
     }

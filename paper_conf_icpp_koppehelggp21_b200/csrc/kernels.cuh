@@ -448,33 +448,30 @@ __device__ __forceinline__ uint64_t decode_wide(const DevIndex& ix, const Loader
     const uint64_t link = uint64_t(e.w[0]) | (uint64_t(e.w[1]) << 32);
     const uint32_t t = link_type(link);
     const uint64_t run = uint64_t(e.w[6]) | (uint64_t(e.w[7]) << 32);
-    if (t == T_N256 && run) {                                  // full N256 of leaves: child b = run + b
-        const uint32_t aux = link_aux(link);
-        return aux >= key.len() ? 0 : run + key.byte(aux);
-    }
-    if (t != T_N4 && t != T_N16) return link;
     const uint32_t aux = link_aux(link);
+    if (t == T_N256 && run)                                    // full N256 of leaves: child b = run + b
+        return aux >= key.len() ? 0 : run + key.byte(aux);
+    if (t != T_N4 && t != T_N16) return link;
     if (aux >= key.len()) return 0;
+    // The entry's 16 key bytes are the N16's keys, or the N4's padded with its last
+    // key (capi.cu), so both take the same branch-free search: "count of keys < b"
+    // is the child slot whenever some key equals b.
     const uint32_t bb = key.byte(aux) * 0x01010101u;
-    const uint8_t* rec = ix.base[t] + link_index(link) * record_bytes(t);
-    // Leaf run (layout.h leaf_run_link): when every child of the node is a leaf, the
-    // leaves are consecutive in the lexicographically ordered leaf buffer (P:110),
-    // so child i's link is run + i and the child-link request disappears too.  A
-    // child nulled by a delete (C18) leaves a tombstoned leaf (value CUART_MISS)
-    // at run + i, which every caller already reads as absent.
-    uint32_t l0, e0;
+    uint32_t l0, l1, l2, l3, e0, e1, e2, e3;
     search4(e.w[2], bb, l0, e0);
-    if (t == T_N4) {
-        if (e0 == 0) return 0;
-        return run ? run + l0 : ld.node64(rec + kN4Child + 8 * l0);
-    }
-    uint32_t l1, l2, l3, e1, e2, e3;
     search4(e.w[3], bb, l1, e1);
     search4(e.w[4], bb, l2, e2);
     search4(e.w[5], bb, l3, e3);
     if ((e0 | e1 | e2 | e3) == 0) return 0;
     const uint32_t c = l0 + l1 + l2 + l3;
-    return run ? run + c : ld.node64(rec + kN16Child + 8 * c);
+    // Leaf run (layout.h leaf_run_link): when every child of the node is a leaf, the
+    // leaves are consecutive in the lexicographically ordered leaf buffer (P:110),
+    // so child c's link is run + c and the child-link request disappears too.  A
+    // child nulled by a delete (C18) leaves a tombstoned leaf (value CUART_MISS)
+    // at run + c, which every caller already reads as absent.
+    if (run) return run + c;
+    const uint8_t* rec = ix.base[t] + link_index(link) * record_bytes(t);
+    return ld.node64(rec + (t == T_N4 ? kN4Child : kN16Child) + 8 * c);
 }
 template <class Key, int POL>
 __device__ __forceinline__ uint64_t start_wide(const DevIndex& ix, const Loader<POL>& ld, const Key& key, uint64_t p) {

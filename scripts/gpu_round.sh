@@ -9,4 +9,4 @@ timeout 900 python bench.py --impl reference --steps 2 --warmup 3 > gpurun_out/b
 for c in c2 c4; do timeout 900 python bench.py --config $c --steps 5 --no-cpu-baseline > gpurun_out/bench_$c.log 2>&1; done
 timeout 1500 python bench.py --config c5 --steps 3 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/bench_c5.log 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -k regex:'k_' --csv --log-file gpurun_out/launches_c3.csv python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu-baseline > gpurun_out/ncu_launch.log 2>&1
-timeout 1200 ncu --set full --import-source on --clock-control none -k regex:'k_lookup_wq|k_bscatter|k_bgather|k_upd1_wq|k_upd2' -c 5 -o gpurun_out/c3_full python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > gpurun_out/ncu_full.log 2>&1
+timeout 1200 ncu --set full --import-source on --clock-control none -k regex:'k_lookup_wq|k_bscatter|k_bgather|k_upd1_wq|k_upd2|k_bhist' -c 6 -o gpurun_out/c3_full python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > gpurun_out/ncu_full.log 2>&1
