@@ -227,10 +227,26 @@ struct KeyLong {
     }
 };
 
-// Count of key bytes < b among 4 packed bytes (sorted keys; padding repeats the last key).
-__device__ __forceinline__ void search4(uint32_t keys, uint32_t bb, uint32_t& less, uint32_t& eq) {
-    less = __popc(__vcmpltu4(keys, bb)) >> 3;
-    eq = __vcmpeq4(keys, bb);
+// Child slot of key byte b among a node's sorted keys (little-endian packed words;
+// unused slots repeat the last key), or -1.  The keys are unique, so the slot is the
+// position of the FIRST byte equal to b (= the count of keys < b).  Zero-byte test
+// on x = word ^ b...b: (x - 0x01..) & ~x & 0x80.. flags every zero byte, and may also
+// flag bytes ABOVE a zero byte (borrow) but never below one, so the lowest flag is
+// exact.  3 instructions per word instead of the emulated __vcmpltu4/__vcmpeq4 pair.
+__device__ __forceinline__ uint32_t zero_bytes(uint32_t w, uint32_t bb) {
+    const uint32_t x = w ^ bb;
+    return (x - 0x01010101u) & ~x & 0x80808080u;
+}
+__device__ __forceinline__ int find_key4(uint32_t w0, uint32_t b) {
+    const uint32_t z = zero_bytes(w0, b * 0x01010101u);
+    return z ? int(__ffs(z) - 1) >> 3 : -1;
+}
+__device__ __forceinline__ int find_key16(uint32_t w0, uint32_t w1, uint32_t w2, uint32_t w3, uint32_t b) {
+    const uint32_t bb = b * 0x01010101u;
+    const uint32_t z0 = zero_bytes(w0, bb), z1 = zero_bytes(w1, bb), z2 = zero_bytes(w2, bb), z3 = zero_bytes(w3, bb);
+    const uint32_t z = z0 ? z0 : z1 ? z1 : z2 ? z2 : z3;
+    const int base = z0 ? 0 : z1 ? 4 : z2 ? 8 : 12;
+    return z ? base + (int(__ffs(z) - 1) >> 3) : -1;
 }
 
 // Cache policy for the three kinds of dependent loads (B200 L2 is 126 MB; the
@@ -373,20 +389,15 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Loader<P
             if (TRACK) *slot = uint64_t(rec + kN48Child + 8 * s);
         } else if (t == T_N16) {
             const uint4 k4 = ld.nodev4(rec + kN16Keys);
-            const uint32_t bb = b * 0x01010101u;
-            uint32_t l0, l1, l2, l3, e0, e1, e2, e3;
-            search4(k4.x, bb, l0, e0);
-            search4(k4.y, bb, l1, e1);
-            search4(k4.z, bb, l2, e2);
-            search4(k4.w, bb, l3, e3);
-            if ((e0 | e1 | e2 | e3) == 0) return 0;
-            link = ld.node64(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
-            if (TRACK) *slot = uint64_t(rec + kN16Child + 8 * (l0 + l1 + l2 + l3));
+            const int c = find_key16(k4.x, k4.y, k4.z, k4.w, b);
+            if (c < 0) return 0;
+            link = ld.node64(rec + kN16Child + 8 * c);
+            if (TRACK) *slot = uint64_t(rec + kN16Child + 8 * c);
         } else {  // N4: keys + child[0..2] in one 256-bit load; child[3] (same line) if taken
             const U8x32 r = ld.nodev8(rec);
-            uint32_t less, eq;
-            search4(r.w[0], b * 0x01010101u, less, eq);
-            if (eq == 0) return 0;
+            const int c = find_key4(r.w[0], b);
+            if (c < 0) return 0;
+            const uint32_t less = uint32_t(c);
             if (less == 3) {
                 link = ld.node64(rec + kN4Child + 24);
             } else {
@@ -454,16 +465,9 @@ __device__ __forceinline__ uint64_t decode_wide(const DevIndex& ix, const Loader
     if (t != T_N4 && t != T_N16) return link;
     if (aux >= key.len()) return 0;
     // The entry's 16 key bytes are the N16's keys, or the N4's padded with its last
-    // key (capi.cu), so both take the same branch-free search: "count of keys < b"
-    // is the child slot whenever some key equals b.
-    const uint32_t bb = key.byte(aux) * 0x01010101u;
-    uint32_t l0, l1, l2, l3, e0, e1, e2, e3;
-    search4(e.w[2], bb, l0, e0);
-    search4(e.w[3], bb, l1, e1);
-    search4(e.w[4], bb, l2, e2);
-    search4(e.w[5], bb, l3, e3);
-    if ((e0 | e1 | e2 | e3) == 0) return 0;
-    const uint32_t c = l0 + l1 + l2 + l3;
+    // key (capi.cu), so both take the same branch-free search.
+    const int c = find_key16(e.w[2], e.w[3], e.w[4], e.w[5], key.byte(aux));
+    if (c < 0) return 0;
     // Leaf run (layout.h leaf_run_link): when every child of the node is a leaf, the
     // leaves are consecutive in the lexicographically ordered leaf buffer,
     // so child c's link is run + c and the child-link request disappears too.  A
