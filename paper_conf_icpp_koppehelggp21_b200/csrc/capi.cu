@@ -176,6 +176,24 @@ __global__ void __launch_bounds__(TPB) k_lookup_wq(DevIndex ix, const void* __re
     uint64_t link[Q];
 #pragma unroll
     for (int j = 0; j < Q; j++) link[j] = decode_wide(ix, ld, k[j], e[j]);
+    // one inline N4 step (the wide entry's node had an inner child: on c3 a depth-4
+    // N4), so only deeper paths take the generic find_leaf loop
+#pragma unroll
+    for (int j = 0; j < Q; j++)
+        if (link_type(link[j]) == T_N4) e[j] = ld.nodev8(ix.base[T_N4] + link_index(link[j]) * record_bytes(T_N4));
+#pragma unroll
+    for (int j = 0; j < Q; j++) {
+        if (link_type(link[j]) != T_N4) continue;
+        const uint32_t aux = link_aux(link[j]);
+        const int c = aux < k[j].len() ? find_key4(e[j].w[0], k[j].byte(aux)) : -1;
+        if (c < 0) link[j] = 0;
+        else if (c == 3) link[j] = ld.node64(ix.base[T_N4] + link_index(link[j]) * record_bytes(T_N4) + kN4Child + 24);
+        else {
+            const uint32_t lo = c == 0 ? e[j].w[2] : c == 1 ? e[j].w[4] : e[j].w[6];
+            const uint32_t hi = c == 0 ? e[j].w[3] : c == 1 ? e[j].w[5] : e[j].w[7];
+            link[j] = uint64_t(lo) | (uint64_t(hi) << 32);
+        }
+    }
     uint4 r[Q];
 #pragma unroll
     for (int j = 0; j < Q; j++)
