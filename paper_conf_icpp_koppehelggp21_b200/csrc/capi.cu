@@ -83,7 +83,7 @@ struct cuart_index {
     int grid_ctas_per_sm = 0;          // 0 = default grid (one op per thread); else persistent grid
     bool ktimer = false;               // record CUDA events around every k_lookup launch
     int ilp = 2;                       // queries per thread of the pre-bucketed wide walk (k_lookup_wq)
-    unsigned wq_tpb = 64;              // k_lookup_wq / k_upd1_wq threads per CTA (CUART_WQ_TPB: 64 / 128 / 256)
+    unsigned wq_tpb = 64;              // k_lookup_wq threads per CTA (CUART_WQ_TPB: 32 / 64 / 128 / 256)
     unsigned lk_tpb = 256;             // k_lookup threads per CTA (CUART_LOOKUP_TPB: 64 / 128 / 256)
     unsigned upd2_tpb = 256;           // k_upd2 threads per CTA (CUART_UPD2_TPB: 64 / 256)
     int wq_lp = 3;                     // k_lookup_wq leaf-load cache policy (CUART_WQ_LEAFPOL, kernels.cuh leafv4_b)
@@ -576,18 +576,19 @@ static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, co
     cudaEvent_t ev0, ev1;
     ktimer_begin(h, s, ev0, ev1);                      // per-launch k_lookup timing (cuart_kernel_timer)
     if (bucketed && dx.walk_wide && h->policy == 5 && h->ilp > 1 && (kind == CUART_KEY_U64 || kind == CUART_KEY_U32)) {
-        const unsigned tpb = h->wq_tpb == 128 || h->wq_tpb == 256 ? h->wq_tpb : 64u;
-        const unsigned qpt = h->ilp == 4 ? 4u : 2u;                   // queries per thread (template Q)
+        const unsigned tpb = h->wq_tpb == 32 || h->wq_tpb == 128 || h->wq_tpb == 256 ? h->wq_tpb : 64u;
+        const unsigned qpt = h->ilp == 4 ? 4u : h->ilp == 3 ? 3u : 2u;   // queries per thread (template Q)
         const unsigned g = unsigned((n + tpb * qpt - 1) / (tpb * qpt));
 #define CUART_WQ_Q(K, Q)                                                                          \
         if (tpb == 64 && h->wq_lp == 0) k_lookup_wq<K, 5, Q, 64, false, 0><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
         else if (tpb == 64 && h->wq_lp == 1) k_lookup_wq<K, 5, Q, 64, false, 1><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
         else if (tpb == 64 && h->wq_lp == 2) k_lookup_wq<K, 5, Q, 64, false, 2><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
         else if (tpb == 64) k_lookup_wq<K, 5, Q, 64, false, 3><<<g, 64, 0, s>>>(dx, q, lens, n, out); \
+        else if (tpb == 32) k_lookup_wq<K, 5, Q, 32, false, 3><<<g, 32, 0, s>>>(dx, q, lens, n, out); \
         else if (tpb == 128) k_lookup_wq<K, 5, Q, 128, false, 3><<<g, 128, 0, s>>>(dx, q, lens, n, out); \
         else k_lookup_wq<K, 5, Q, 256, false, 3><<<g, 256, 0, s>>>(dx, q, lens, n, out);
 #define CUART_WQ(K)                                                                               \
-        if (qpt == 4) { CUART_WQ_Q(K, 4) } else { CUART_WQ_Q(K, 2) }
+        if (qpt == 4) { CUART_WQ_Q(K, 4) } else if (qpt == 3) { CUART_WQ_Q(K, 3) } else { CUART_WQ_Q(K, 2) }
         if (kind == CUART_KEY_U64) { CUART_WQ(KeyU64) } else { CUART_WQ(KeyU32) }
 #undef CUART_WQ
 #undef CUART_WQ_Q
