@@ -237,6 +237,18 @@ def c5_local_keys(world, rank, dev, chunk=1 << 27):
     return torch.cat(ks).numpy().view(np.uint64), torch.cat(vs).numpy().view(np.uint64), splitters
 
 
+def hbm_peak():
+    """(GB/s, source): MEASURED_PEAKS.json hbm_gbs, else the profiling guide's fallback."""
+    peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(peaks_path):
+        with open(peaks_path) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+C5_STREAM_BYTES = 8 + (8 + 8 + 2) + (8 + 8) + (8 + 2 + 8)   # bhist, bscatter, walk I/O, bgather (u64)
+
+
 def run_c5(args, world, rank, local, dev):
     """A step = one round of the mixed stream: this rank's 1/P slice of 2^29 global ops
     (strong scaling: the round is fixed), lookups then updates (reading C7)."""
@@ -298,6 +310,9 @@ def run_c5(args, world, rank, local, dev):
     total_ms, kern_ms = tt.tolist()
     ms_step = total_ms / args.steps
     value = R / (ms_step * 1e-3) / 1e6
+    n_look = int(sum(int((r[1] == 0).sum().item()) for r in rounds) // len(rounds))
+    peak, peak_src = hbm_peak()
+    c5_achieved = C5_STREAM_BYTES * n_look / (kern_ms * 1e-3) / 1e9
     if rank == 0:
         print(json.dumps({
             "metric": METRIC, "value": round(value, 3), "unit": "Mops/s", "n_gpus": world, "steps": args.steps,
@@ -309,8 +324,15 @@ def run_c5(args, world, rank, local, dev):
                        "transport": args.transport if world > 1 else None,
                        "parallelism": f"range{world}", "local_keys_rank0": int(keys.shape[0]),
                        "build_s": round(build_s, 2), "lut_format": stats["lut_format"]},
-            "roofline": {"bound": "hbm", "kernel": "k_lookup<KeyU64>", "kernel_ms": round(kern_ms, 4),
-                         "note": "per-rank local lookup kernel of a round; see the c3 line for the roofline fraction"},
+            "roofline": {"bound": "hbm", "achieved": round(c5_achieved, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(c5_achieved / peak, 4), "traffic": None,
+                         "kernel": "cuart_lookup (local, pre-bucketed: k_bhist .. k_lookup .. k_bgather)",
+                         "kernel_ms": round(kern_ms, 4), "lookups_per_launch": n_look,
+                         "bytes_per_lookup": C5_STREAM_BYTES,
+                         "bytes_model": "lower bound: the bucketed call's streaming key/result/permutation bytes "
+                                        "(8+18+16+18 B per u64 lookup); tree reads not counted",
+                         "peak_source": peak_src,
+                         "note": "per-rank local lookup call of a round; the c3 line carries the walk kernel's roofline"},
             "e2e": None, "cpu_baseline": None, "gpu_launches": int(launches), "clocks": clk}), flush=True)
     di.close()
     if world > 1:
@@ -471,12 +493,7 @@ def main():
     value = ops_per_step / (ms_step * 1e-3) / 1e6
 
     # roofline of the dominant kernel (k_lookup on this rank), HBM-bound random gathers
-    peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
-    peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
-    if os.path.exists(peaks_path):
-        with open(peaks_path) as f:
-            peak = float(json.load(f)["hbm_gbs"])
-        peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)"
+    peak, peak_src = hbm_peak()
     achieved = served * bytes_per_lookup / (kern_ms * 1e-3) / 1e9
     pipe_achieved = nl * pipeline_bytes / (look_ms * 1e-3) / 1e9
     # BASELINE north_star's definition: 32-B sectors touched per query x queries/s
