@@ -269,6 +269,30 @@ def test_prebucket_bucket_counts_and_skew(shift, monkeypatch):
     ix.close()
 
 
+@pytest.mark.parametrize("n", [4096, 70_001, 3 * 4096 + 1])
+def test_prebucket_gather_misaligned_out(n):
+    """The pre-bucketed lookup's final gather writes a caller-owned `out` of any
+    8-B alignment: an `out` view 8 B into its buffer, and an aligned one, both
+    equal the plain map (ragged and odd tile tails included) and nothing outside
+    the view is written."""
+    rng = np.random.default_rng(n)
+    keys, vals = W.build_set(W.CONFIGS["c1"])
+    ix = C.Index(keys, vals, lut_bytes=3, prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_ON)
+    mp = MapOracle(keys, vals)
+    q = np.where(rng.random(n) < 0.5, keys[rng.integers(0, keys.shape[0], n)],
+                 rng.integers(0, 2**64, n, dtype=np.uint64))
+    want = mp.lookup(q)
+    for off in (0, 1):
+        buf = torch.full((n + 2,), 7, dtype=torch.int64, device=DEV)
+        out = buf[off:off + n]
+        ix.lookup(_t(q), out)
+        torch.cuda.synchronize()
+        got = buf.cpu().numpy().view(np.uint64)
+        assert np.array_equal(got[off:off + n], want)
+        assert got[off + n] == 7 and (off == 0 or got[0] == 7)
+    ix.close()
+
+
 def test_c2_full_size_sampled():
     """Config 2 at full size (2^24 dense u32 keys, LUT over the first 3 bytes):
     2^28 lookups in the bench's launch configuration; sampled outputs vs the
