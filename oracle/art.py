@@ -22,7 +22,7 @@ def build_oracle_lib(force: bool = False) -> str:
     """Compile art_oracle.c with plain gcc (no OpenMP, no vectorisation tricks)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-o", tmp, _SRC])
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-pthread", "-o", tmp, _SRC])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -43,7 +43,9 @@ def _load():
         lib.oart_lookup.argtypes = [P, P, U32]
         lib.oart_lookup.restype = U64
         lib.oart_lookup_batch.argtypes = [P, P, P, U32, SZ, SZ, P]
-        lib.oart_update_batch.argtypes = [P, P, P, U32, SZ, P, SZ]
+        lib.oart_lookup_batch_mt.argtypes = [P, P, P, U32, SZ, SZ, P, ctypes.c_int]
+        lib.oart_lookup_batch_mt.restype = ctypes.c_int
+        lib.oart_update_batch.argtypes = [P, P, P, U32, SZ, P, SZ, P]
         lib.oart_update_batch.restype = ctypes.c_int64
         lib.oart_dump_inorder.argtypes = [P, P, P, P, SZ]
         lib.oart_dump_inorder.restype = SZ
@@ -52,7 +54,7 @@ def _load():
         lib.oart_stats.argtypes = [P, P]
         lib.oart_erase.argtypes = [P, P, U32]
         lib.oart_erase.restype = ctypes.c_int
-        lib.oart_apply_batch.argtypes = [P, P, P, U32, SZ, P, P, SZ]
+        lib.oart_apply_batch.argtypes = [P, P, P, U32, SZ, P, P, SZ, P]
         lib.oart_apply_batch.restype = ctypes.c_int64
         _lib = lib
     return _lib
@@ -133,12 +135,24 @@ class ArtOracle:
         self._lib.oart_lookup_batch(self._t, _ptr(slots), _ptr(lens), flen, stride, slots.shape[0], _ptr(out))
         return out
 
+    def lookup_mt(self, queries, threads: int) -> np.ndarray:
+        """oart_lookup_batch split over `threads` POSIX threads (read-only)."""
+        slots, lens, flen, stride = canonical_bytes(queries)
+        out = np.empty(slots.shape[0], dtype=np.uint64)
+        self._lib.oart_lookup_batch_mt(self._t, _ptr(slots), _ptr(lens), flen, stride, slots.shape[0], _ptr(out),
+                                       int(threads))
+        return out
+
     def update(self, keys, values) -> int:
+        """Sequential batch update; ops carrying the reserved value are dropped
+        (reading C5) and counted in ``self.last_rejected``.  Returns the number of
+        applied ops that hit a stored key."""
         slots, lens, flen, stride = canonical_bytes(keys)
         vals = np.ascontiguousarray(values, dtype=np.uint64)
-        hits = self._lib.oart_update_batch(self._t, _ptr(slots), _ptr(lens), flen, stride, _ptr(vals), slots.shape[0])
-        if hits < 0:
-            raise ValueError("update value is the reserved miss value")
+        rej = ctypes.c_uint64()
+        hits = self._lib.oart_update_batch(self._t, _ptr(slots), _ptr(lens), flen, stride, _ptr(vals), slots.shape[0],
+                                           ctypes.byref(rej))
+        self.last_rejected = int(rej.value)
         return int(hits)
 
     def erase_one(self, key: bytes) -> int:
@@ -152,9 +166,10 @@ class ArtOracle:
         n = slots.shape[0]
         vals = np.ascontiguousarray(values if values is not None else np.zeros(n), dtype=np.uint64)
         dele = np.ascontiguousarray(is_delete, dtype=np.uint8) if is_delete is not None else None
-        hits = self._lib.oart_apply_batch(self._t, _ptr(slots), _ptr(lens), flen, stride, _ptr(vals), _ptr(dele), n)
-        if hits < 0:
-            raise ValueError("update value is the reserved miss value")
+        rej = ctypes.c_uint64()
+        hits = self._lib.oart_apply_batch(self._t, _ptr(slots), _ptr(lens), flen, stride, _ptr(vals), _ptr(dele), n,
+                                          ctypes.byref(rej))
+        self.last_rejected = int(rej.value)
         return int(hits)
 
     def dump_inorder(self):
@@ -228,11 +243,14 @@ class MapOracle:
 
     def update(self, keys, values) -> int:
         """Ops applied in index order; equivalently the highest op index per key
-        wins.  Absent keys are no-ops (reading C6)."""
+        wins.  Absent keys are no-ops (reading C6); ops carrying the
+        reserved value are dropped (reading C5) and counted in last_rejected."""
         vals = np.ascontiguousarray(values, dtype=np.uint64)
         pos, found = self._find(keys)
+        reserved = vals == OART_MISS
+        self.last_rejected = int(reserved.sum())
         if found.shape[0]:
-            found &= self.present[pos]
+            found &= self.present[pos] & ~reserved
         idx = np.nonzero(found)[0]
         # sequential application == for each key, the value of its LAST op
         p = pos[idx]
@@ -250,8 +268,10 @@ class MapOracle:
         vals = np.ascontiguousarray(values if values is not None else np.zeros(n), dtype=np.uint64)
         dele = np.asarray(is_delete, dtype=bool)
         pos, found = self._find(keys)
+        reserved = ~dele & (vals == OART_MISS)          # reading C5: dropped
+        self.last_rejected = int(reserved.sum())
         if found.shape[0]:
-            found &= self.present[pos]
+            found &= self.present[pos] & ~reserved
         idx = np.nonzero(found)[0]
         p = pos[idx]
         order = np.argsort(p, kind="stable")

@@ -27,6 +27,7 @@
  * expansion: a key is stored in a leaf hung at the shallowest node where it is
  * unique.  Insert-only: no shrinking (structural delete is out of scope).
  */
+#include <pthread.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -293,6 +294,39 @@ void oart_lookup_batch(const oart* t, const uint8_t* keys, const uint8_t* lens, 
         out[i] = oart_lookup(t, keys + i * stride, lens ? lens[i] : fixed_len);
 }
 
+/* The same read-only loop split into `threads` contiguous slices, one POSIX thread
+ * each (the all-core CPU baseline of SURVEY §8(d); lookups never write the tree,
+ * so the slices are independent and the result equals oart_lookup_batch's). */
+typedef struct {
+    const oart* t; const uint8_t* keys; const uint8_t* lens; uint32_t fixed_len; size_t stride;
+    size_t lo, hi; uint64_t* out;
+} lookup_slice;
+
+static void* lookup_slice_run(void* arg) {
+    const lookup_slice* a = (const lookup_slice*)arg;
+    for (size_t i = a->lo; i < a->hi; i++)
+        a->out[i] = oart_lookup(a->t, a->keys + i * a->stride, a->lens ? a->lens[i] : a->fixed_len);
+    return NULL;
+}
+
+int oart_lookup_batch_mt(const oart* t, const uint8_t* keys, const uint8_t* lens, uint32_t fixed_len,
+                         size_t stride, size_t n, uint64_t* out, int threads) {
+    if (threads < 1) threads = 1;
+    if (threads > 1024) threads = 1024;
+    pthread_t tid[1024];
+    int created[1024];
+    lookup_slice sl[1024];
+    for (int k = 0; k < threads; k++) {
+        sl[k] = (lookup_slice){t, keys, lens, fixed_len, stride, n * (size_t)k / (size_t)threads,
+                               n * (size_t)(k + 1) / (size_t)threads, out};
+        created[k] = k < threads - 1 && pthread_create(&tid[k], NULL, lookup_slice_run, &sl[k]) == 0;
+        if (!created[k]) lookup_slice_run(&sl[k]);   /* the caller's thread takes the last slice */
+    }
+    for (int k = 0; k < threads; k++)
+        if (created[k]) pthread_join(tid[k], NULL);
+    return threads;
+}
+
 static oleaf* find_leaf(const oart* t, const uint8_t* key, uint32_t len) {
     onode* n = t->root;
     uint32_t depth = 0;
@@ -315,16 +349,20 @@ static oleaf* find_leaf(const oart* t, const uint8_t* key, uint32_t len) {
 
 /* Sequential batch update: ops applied in index order, so the op
  * with the highest index wins per key; absent keys are a no-op (reading C6).
- * Returns the number of ops that hit a stored key.  A reserved value is
- * rejected (returns -1 and applies nothing from that op on). */
+ * Reading C5: CUART_MISS is reserved (it is the lookup's "absent" answer, so it
+ * can never be stored); an op carrying it is DROPPED -- a no-op, as if its key
+ * were absent -- and counted in *rejected; the other ops of the batch apply.
+ * Returns the number of applied ops that hit a stored key. */
 int64_t oart_update_batch(oart* t, const uint8_t* keys, const uint8_t* lens, uint32_t fixed_len,
-                          size_t stride, const uint64_t* values, size_t n) {
+                          size_t stride, const uint64_t* values, size_t n, uint64_t* rejected) {
     int64_t hits = 0;
+    uint64_t rej = 0;
     for (size_t i = 0; i < n; i++) {
-        if (values[i] == OART_MISS) return -1;
+        if (values[i] == OART_MISS) { rej++; continue; }
         oleaf* l = find_leaf(t, keys + i * stride, lens ? lens[i] : fixed_len);
         if (l) { l->value = values[i]; hits++; }
     }
+    if (rejected) *rejected = rej;
     return hits;
 }
 
@@ -500,19 +538,25 @@ int oart_erase(oart* t, const uint8_t* key, uint32_t len) {
  * the same operation with a "nil" value).  Reading C17: every op
  * locates its key in the state BEFORE the batch (stage 1 of Fig. 6 is a lookup
  * over the unmodified tree); for each located key the op with the highest index
- * decides — its value is stored, or, for a delete, the key is removed.  Ops on
- * keys absent before the batch are no-ops.  Returns the number of ops that
- * located their key, -1 for a reserved value on a non-delete op (nothing applied). */
+ * decides -- its value is stored, or, for a delete, the key is removed.  Ops on
+ * keys absent before the batch are no-ops.  Reading C5: a non-delete op carrying
+ * the reserved value CUART_MISS is dropped (it locates nothing, so it never wins)
+ * and counted in *rejected.  Returns the number of ops that located their key. */
 int64_t oart_apply_batch(oart* t, const uint8_t* keys, const uint8_t* lens, uint32_t fixed_len, size_t stride,
-                         const uint64_t* values, const uint8_t* is_delete, size_t n) {
-    for (size_t i = 0; i < n; i++)
-        if ((!is_delete || !is_delete[i]) && values && values[i] == OART_MISS) return -1;
+                         const uint64_t* values, const uint8_t* is_delete, size_t n, uint64_t* rejected) {
+    uint64_t rej = 0;
     oleaf** at = (oleaf**)calloc(n ? n : 1, sizeof(oleaf*));
     int64_t hits = 0;
     for (size_t i = 0; i < n; i++) {                /* stage 1: locate on the pre-batch tree */
+        if ((!is_delete || !is_delete[i]) && values && values[i] == OART_MISS) {
+            at[i] = NULL;                           /* reading C5: dropped */
+            rej++;
+            continue;
+        }
         at[i] = find_leaf(t, keys + i * stride, lens ? lens[i] : fixed_len);
         if (at[i]) hits++;
     }
+    if (rejected) *rejected = rej;
     /* highest op index per leaf: later ops overwrite the leaf's pending mark */
     for (size_t i = 0; i < n; i++)
         if (at[i]) at[i]->pending = (uint64_t)i + 1;

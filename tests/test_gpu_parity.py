@@ -190,14 +190,36 @@ def test_edge_cases():
     ix.close()
 
 
-def test_reserved_value_update_sets_sticky_error():
+@pytest.mark.parametrize("prebucket", [1, 2])
+def test_reserved_value_update_sets_sticky_error(prebucket):
+    """Reading C5: an op carrying CUART_MISS is dropped and sets the sticky flag;
+    the post-batch state equals the oracle's (which drops the same ops)."""
     keys = np.array([1, 2, 3], np.uint64)
-    ix = C.Index(keys, np.array([10, 20, 30], np.uint64))
-    ix.update(_t(np.array([1, 2], np.uint64)), _t(np.array([MISS, 5], np.uint64)))
+    ix = C.Index(keys, np.array([10, 20, 30], np.uint64), prebucket=prebucket)
+    o = ArtOracle(keys, np.array([10, 20, 30], np.uint64))
+    for uk, uv in ((np.array([1, 2], np.uint64), np.array([MISS, 5], np.uint64)),
+                   (np.array([3, 3, 2], np.uint64), np.array([7, MISS, MISS], np.uint64))):
+        ix.update(_t(uk), _t(uv))
+        torch.cuda.synchronize()
+        o.update(uk, uv)
+        assert o.last_rejected > 0
+        assert ix.get_error() == 4
+        assert ix.get_error() == 0                       # cleared on read
+        assert _lookup(ix, keys).tolist() == o.lookup(keys).tolist()
+    ix.close()
+    # a large batch with reserved values sprinkled in, through the bucketed path
+    cfg = W.CONFIGS["c1"]
+    keys, vals = W.build_set(cfg)
+    ix = C.Index(keys, vals, lut_bytes=3, prebucket=prebucket)
+    o = MapOracle(keys, vals)
+    uk, uv = W.update_batch(cfg, keys)
+    uv = uv.copy()
+    uv[::97] = OART_MISS
+    ix.update(_t(uk), _t(uv))
     torch.cuda.synchronize()
+    o.update(uk, uv)
     assert ix.get_error() == 4
-    assert ix.get_error() == 0                       # cleared on read
-    assert _lookup(ix, keys).tolist() == [10, 5, 30]  # the rejected op is a no-op
+    assert np.array_equal(_lookup(ix, keys), o.lookup(keys))
     ix.close()
 
 

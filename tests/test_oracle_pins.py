@@ -213,12 +213,14 @@ def test_update_vs_sequential_dict(seed):
         o.insert_one(k, v)
     ops = []
     for _ in range(2000):
-        if rng.random() < 0.8:
+        if rng.random() < 0.02:            # reserved value: the op is dropped (reading C5)
+            ops.append((rng.choice(keys), MISS))
+        elif rng.random() < 0.8:
             ops.append((rng.choice(keys), rng.getrandbits(62)))
         else:
             ops.append((rng.getrandbits(64).to_bytes(8, "big") if rng.random() < 0.5 else b"nope\x00", rng.getrandbits(62)))
     for k, v in ops:                   # brute force: apply in order, present keys only
-        if k in ref:
+        if k in ref and v != MISS:
             ref[k] = v
     if all(len(k) == 8 for k, _ in ops) and all(len(k) == 8 for k in keys):
         o.update(np.array([int.from_bytes(k, "big") for k, _ in ops], dtype=np.uint64),
@@ -232,6 +234,36 @@ def test_update_vs_sequential_dict(seed):
         o.update((slots, lens), np.array([v for _, v in ops], dtype=np.uint64))
     for k in keys:
         assert o.lookup_one(k) == ref[k]
+
+
+def test_reserved_value_ops_are_dropped():
+    """Reading C5 (CUART_MISS is the lookup's absent answer, so it cannot be
+    stored): an op carrying it is a no-op -- it neither writes nor wins over an
+    earlier op on the same key -- and the rest of the batch applies."""
+    k = np.array([1, 2, 3], np.uint64)
+    for mk in (ArtOracle, MapOracle):
+        x = mk(k, np.array([10, 20, 30], np.uint64))
+        x.update(np.array([1, 2], np.uint64), np.array([MISS, 5], np.uint64))
+        assert x.lookup(k).tolist() == [10, 5, 30] and x.last_rejected == 1
+        x.update(np.array([3, 3, 2], np.uint64), np.array([7, MISS, MISS], np.uint64))
+        assert x.lookup(k).tolist() == [10, 5, 7] and x.last_rejected == 2
+        # mixed batch (reading C17): a dropped op does not locate, so an earlier op wins;
+        # a delete carries no value, so the reserved value does not drop it
+        x.apply(np.array([1, 1, 2, 3], np.uint64), np.array([11, MISS, MISS, MISS], np.uint64),
+                np.array([0, 0, 1, 0], np.uint8))
+        assert x.lookup(k).tolist() == [11, MISS, 7] and x.last_rejected == 2
+
+
+def test_lookup_mt_equals_single_thread():
+    import workloads as W
+    cfg = W.CONFIGS["c1"]
+    keys, vals = W.build_set(cfg)
+    o = ArtOracle(keys, vals)
+    q = W.lookup_batch(cfg, keys, 0, 100_003)
+    ref = o.lookup(q)
+    for t in (1, 3, 8):
+        assert np.array_equal(o.lookup_mt(q, t), ref)
+    assert np.array_equal(ref, MapOracle(keys, vals).lookup(q))
 
 
 # ------------------------------------------------------------------ errors
