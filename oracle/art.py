@@ -219,6 +219,12 @@ class MapOracle:
 
     def _rows(self, slots, lens, flen):
         if lens is None:
+            # fixed-length keys: the big-endian bytes read as one unsigned integer
+            # compare exactly like the byte strings (lexicographic = numeric order),
+            # and numpy sorts / searches integers much faster than void rows
+            if slots.shape[1] in (4, 8):
+                be = ">u8" if slots.shape[1] == 8 else ">u4"
+                return np.ascontiguousarray(slots).view(be).ravel().astype(be[1:])
             return np.ascontiguousarray(slots).view(np.dtype((np.void, slots.shape[1]))).ravel()
         # append the length byte AFTER the zero-padded content so "ab"(2) != "ab\0"(3);
         # for a prefix-free set this keeps lexicographic order of the true keys.

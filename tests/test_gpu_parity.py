@@ -342,36 +342,72 @@ def test_c2_full_size_sampled():
 
 
 @pytest.mark.slow
-def test_c3_full_size_sampled():
-    """Config 3 at full size: 2^26 random u64 keys, 2^30 lookups at 50% hit and
-    the 2^26-op update batch, in the bench's launch configuration; sampled
-    outputs vs the plain-map oracle (the generator recomputes any element)."""
+def test_c3_full_size_every_lookup_and_post_update_state():
+    """Config 3 at full size in the bench's launch configuration (2^26 random u64
+    keys, one 2^30-query lookup call, one 2^26-op update call):
+
+    * EVERY lookup against its closed form from the generator (plain definition
+      M[q]: a hit query is key #pick of the set, whose value is vals[pick]; a miss
+      query is a guaranteed-absent key -> CUART_MISS), cross-checked against the
+      plain-map oracle on a 300K sample (pins the closed form to the oracle);
+    * the FULL post-update tree state: every one of the 2^26 keys looked
+      up against the plain-map oracle's sequential replay of the batch, and the
+      device dump compared with the pre-update dump -- inner-node buffers and root
+      table byte-identical (updates are non-structural), leaf keys unchanged and
+      leaf values equal to the oracle's values in key order (leaves are stored in
+      lexicographic order)."""
     cfg = W.CONFIGS["c3"]
-    keys_d = W.u64_keys_torch(3, cfg.n_keys, DEV)
+    n = cfg.n_keys
+    keys_d = W.u64_keys_torch(3, n, DEV)
     keys = _u64(keys_d)
-    _, vals = W.build_set(W.Config("c3", "u64", cfg.n_keys, 0, 0, 0.5, ""))
+    vals = W.values_for(W.SEED_VALUES + 3, np.arange(n, dtype=np.uint64))
     ix = C.Index(keys, vals, lut_bytes=3)
-    n = cfg.n_lookups
-    out = torch.empty(n, dtype=torch.int64, device=DEV)
-    qd = W.lookup_batch_torch(cfg, keys_d, 0, n)
+    pre = ix.dump()
+    nl = cfg.n_lookups
+    out = torch.empty(nl, dtype=torch.int64, device=DEV)
+    qd = W.lookup_batch_torch(cfg, keys_d, 0, nl)
     ix.lookup(qd, out)
+    torch.cuda.synchronize()
+    # sampled cross-check of the generator's queries and of the closed form vs the oracle
+    mp = MapOracle(keys, vals)
+    idx = np.sort(np.random.default_rng(3).choice(nl, 300_000, replace=False))
+    ti = torch.from_numpy(idx).to(DEV)
+    qs = W.lookup_at(cfg, keys, idx)
+    assert np.array_equal(_u64(qd[ti]), qs)
+    assert np.array_equal(_u64(out[ti]), mp.lookup(qs))
+    del qd
+    vals_d = torch.from_numpy(vals.view(np.int64)).to(DEV)
+    hits = 0
+    for s0 in range(0, nl, 1 << 27):
+        j = torch.arange(s0, s0 + (1 << 27), dtype=torch.int64, device=DEV)
+        hit = W._t_ult(W.splitmix64_torch(W.SEED_QUERIES + 3, 2 * j), 1 << 63)
+        pick = W._t_umod(W.splitmix64_torch(W.SEED_QUERIES + 3, 2 * j + 1), n)
+        exp = torch.where(hit, vals_d[pick], torch.full_like(j, -1))
+        assert torch.equal(out[s0: s0 + (1 << 27)], exp), f"lookup mismatch in [{s0}, {s0 + (1 << 27)})"
+        hits += int(hit.sum().item())
+    assert abs(hits / nl - 0.5) < 0.001
+    del out
+    # the update batch, then the full post-update state
     uk, uv = W.update_batch_torch(cfg, keys_d)
     ix.update(uk, uv)
-    out2 = torch.empty(1 << 22, dtype=torch.int64, device=DEV)
-    ix.lookup(keys_d[: 1 << 22], out2)
+    out2 = torch.empty(n, dtype=torch.int64, device=DEV)
+    ix.lookup(keys_d, out2)
     torch.cuda.synchronize()
     assert ix.get_error() == 0
-    mp = MapOracle(keys, vals)
-    idx = np.sort(np.random.default_rng(3).choice(n, 300_000, replace=False))
-    qs = W.lookup_at(cfg, keys, idx)
-    ti = torch.from_numpy(idx).to(DEV)
-    assert np.array_equal(_u64(qd[ti]), qs)
-    got = _u64(out[ti])
-    assert np.array_equal(got, mp.lookup(qs))
-    hit = (out != -1).float().mean().item()
-    assert abs(hit - 0.5) < 0.001
     mp.update(_u64(uk), _u64(uv))
-    assert np.array_equal(_u64(out2), mp.lookup(keys[: 1 << 22]))
+    assert mp.last_rejected == 0
+    assert np.array_equal(_u64(out2), mp.lookup(keys))
+    post = ix.dump()
+    for t in (1, 2, 3, 4):
+        assert np.array_equal(post["buf"][t], pre["buf"][t]), f"inner buffer {t} changed"
+    assert np.array_equal(post["lut"], pre["lut"])
+    assert post["root"] == pre["root"]
+    leaf = post["buf"][5].reshape(-1, 16)
+    assert np.array_equal(leaf[:, :8], pre["buf"][5].reshape(-1, 16)[:, :8])
+    assert np.array_equal(np.ascontiguousarray(leaf[:, :8]).view(">u8").ravel().astype(np.uint64), mp.rows)
+    assert np.array_equal(np.ascontiguousarray(leaf[:, 8:]).view(np.uint64).ravel(), mp.values)
+    pre_v = np.ascontiguousarray(pre["buf"][5].reshape(-1, 16)[:, 8:]).view(np.uint64).ravel()
+    assert int((pre_v != mp.values).sum()) > n // 2        # the batch rewrote ~60% of the leaves
     ix.close()
 
 
@@ -415,21 +451,28 @@ def test_c4_strings_scaled():
 
 
 @pytest.mark.slow
-def test_c4_full_size_sampled():
-    """Config 4 at full size (2^25 keys, 2^29 Zipf lookups) in the bench's launch
-    configuration; sampled outputs vs the plain-map oracle; 100% hit everywhere."""
+def test_c4_full_size_every_lookup():
+    """Config 4 at full size (2^25 Zipf-prefixed strings, one 2^29-query lookup call
+    as the bench times it): EVERY lookup against its closed form from the generator
+    (query j is key #idx_j of the set, 100% hit, so its value is vals[idx_j]), and a
+    200K sample against the plain-map oracle (pins the closed form to the oracle)."""
     cfg = W.CONFIGS["c4"]
-    slots, lens = W.string_keys(4, cfg.n_keys)
-    vals = W.values_for(W.SEED_VALUES + 4, np.arange(cfg.n_keys, dtype=np.uint64))
+    n = cfg.n_keys
+    slots, lens = W.string_keys(4, n)
+    vals = W.values_for(W.SEED_VALUES + 4, np.arange(n, dtype=np.uint64))
     ix = C.Index((slots, lens), vals)
     sd, ld = torch.from_numpy(slots).to(DEV), torch.from_numpy(lens).to(DEV)
-    qs, ql = W.string_lookup_torch(cfg, sd, ld, 0, cfg.n_lookups)
-    out = torch.empty(cfg.n_lookups, dtype=torch.int64, device=DEV)
+    nl = cfg.n_lookups
+    qidx = W.string_lookup_index_torch(cfg, n, 0, nl, DEV, W.zipf_cdf_torch(n, DEV), W.rank_permutation_torch(cfg, n, DEV))
+    qs, ql = sd[qidx], ld[qidx]
+    out = torch.empty(nl, dtype=torch.int64, device=DEV)
     ix.lookup((qs, ql), out)
     torch.cuda.synchronize()
-    assert not bool((out == -1).any().item())
-    idx = np.sort(np.random.default_rng(4).choice(cfg.n_lookups, 200_000, replace=False))
+    vals_d = torch.from_numpy(vals.view(np.int64)).to(DEV)
+    assert torch.equal(out, vals_d[qidx])
+    idx = np.sort(np.random.default_rng(4).choice(nl, 200_000, replace=False))
     ti = torch.from_numpy(idx).to(DEV)
+    assert np.array_equal(qidx[ti].cpu().numpy(), W.string_lookup_at(cfg, n, idx))
     mp = MapOracle((slots, lens), vals)
     assert np.array_equal(_u64(out[ti]), mp.lookup((qs[ti].cpu().numpy(), ql[ti].cpu().numpy())))
     ix.close()

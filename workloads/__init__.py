@@ -341,28 +341,54 @@ def update_batch_torch(cfg: Config, keys, start: int = 0, m: int | None = None):
     return out, vals
 
 
-def string_lookup_torch(cfg: Config, slots_d, lens_d, start: int, m: int, cdf_d=None, perm_d=None):
-    """torch twin of string_lookup_at for positions [start, start+m): returns
-    (query slots uint8[m,32], lens uint8[m]) gathered on the keys' device.  The
-    Zipf CDF is built on the host (numpy, exact) and the permutation sorts the
-    same splitmix64 draws as unsigned, so ranks and keys match the numpy twin."""
+def string_lookup_index_torch(cfg: Config, n: int, start: int, m: int, device, cdf_d=None, perm_d=None):
+    """torch twin of string_lookup_at for positions [start, start+m): the KEY INDICES
+    (int64[m]) the Zipf draws select.  The Zipf CDF is built on the host (numpy,
+    exact) and the permutation sorts the same splitmix64 draws as unsigned, so ranks
+    and keys match the numpy twin."""
     import torch
     c = config_id(cfg)
-    n = slots_d.shape[0]
-    dev = slots_d.device
     if cdf_d is None:
         w = 1.0 / np.arange(1, n + 1, dtype=np.float64) ** 0.99
         cdf = np.cumsum(w)
         cdf /= cdf[-1]
-        cdf_d = torch.from_numpy(cdf).to(dev)
+        cdf_d = torch.from_numpy(cdf).to(device)
     if perm_d is None:
-        draws = splitmix64_torch(SEED_QUERIES + c + 7, torch.arange(n, dtype=torch.int64, device=dev))
+        draws = splitmix64_torch(SEED_QUERIES + c + 7, torch.arange(n, dtype=torch.int64, device=device))
         perm_d = torch.argsort(draws ^ (-(1 << 63)), stable=True)        # unsigned order
-    j = torch.arange(start, start + m, dtype=torch.int64, device=dev)
+    j = torch.arange(start, start + m, dtype=torch.int64, device=device)
     u = _t_srl(splitmix64_torch(SEED_QUERIES + c, j), 11).to(torch.float64) * (1.0 / (1 << 53))
     r = torch.clamp(torch.searchsorted(cdf_d, u, right=True), max=n - 1)
-    idx = perm_d[r]
+    return perm_d[r]
+
+
+def string_lookup_torch(cfg: Config, slots_d, lens_d, start: int, m: int, cdf_d=None, perm_d=None):
+    """torch twin of string_lookup_at for positions [start, start+m): returns
+    (query slots uint8[m,32], lens uint8[m]) gathered on the keys' device."""
+    idx = string_lookup_index_torch(cfg, slots_d.shape[0], start, m, slots_d.device, cdf_d, perm_d)
     return slots_d[idx], lens_d[idx]
+
+
+def zipf_cdf_torch(n: int, device, theta: float = 0.99):
+    """The Zipf(theta) CDF over [0, n) (numpy, exact) on `device`, for reuse across chunks."""
+    import torch
+    w = 1.0 / np.arange(1, n + 1, dtype=np.float64) ** theta
+    cdf = np.cumsum(w)
+    cdf /= cdf[-1]
+    return torch.from_numpy(cdf).to(device)
+
+
+def rank_permutation_torch(cfg: Config, n: int, device):
+    import torch
+    draws = splitmix64_torch(SEED_QUERIES + config_id(cfg) + 7, torch.arange(n, dtype=torch.int64, device=device))
+    return torch.argsort(draws ^ (-(1 << 63)), stable=True)
+
+
+def values_torch(seed: int, start: int, m: int, device):
+    """torch twin of values_for over counters [start, start+m)."""
+    import torch
+    v = splitmix64_torch(seed, torch.arange(start, start + m, dtype=torch.int64, device=device))
+    return torch.where(v == -1, torch.zeros_like(v), v)
 
 
 # ----------------------------------------------------------------------------- config 5 (mixed)
