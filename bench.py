@@ -256,15 +256,13 @@ def run_c5(args, world, rank, local, dev):
     import torch.distributed as dist
 
     import paper_conf_icpp_koppehelggp21_b200 as C
-    from paper_conf_icpp_koppehelggp21_b200.dist import CudaOps, DistIndex
+    from paper_conf_icpp_koppehelggp21_b200.dist import DistIndex
     if world & (world - 1):
         raise SystemExit("c5 needs a power-of-two GPU count")
     t0 = time.perf_counter()
     keys, vals, sp = c5_local_keys(world, rank, dev)
-    if world == 1 and not dist.is_initialized():
-        dist.init_process_group("gloo", store=dist.HashStore(), rank=0, world_size=1)
-    di = DistIndex(keys, vals, mode="range", ops=CudaOps(dev), lut_bytes=args.lut, splitters=sp, local=True,
-                   transport=args.transport)
+    di = DistIndex(keys, vals, mode="range", transport=args.transport, lut_bytes=args.lut, splitters=sp,
+                   keys_local=True, rank=rank, world=world)
     build_s = time.perf_counter() - t0
     stats = di.index.stats()
     R, per = W.C5_ROUND, W.C5_ROUND // world
@@ -272,11 +270,11 @@ def run_c5(args, world, rank, local, dev):
     torch.cuda.synchronize()
     stream = torch.cuda.current_stream()
 
-    def step(i, ev=None, kev=None):
+    def step(i, ev=None):
         k, u, v = rounds[i % 2]
         if ev is not None:
             ev[0].record(stream)
-        di.mixed_round(k, v, u, events=kev)
+        di.mixed_round(k, v, u)
         if ev is not None:
             ev[1].record(stream)
 
@@ -286,7 +284,6 @@ def run_c5(args, world, rank, local, dev):
     if world > 1:
         dist.barrier()
     evs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
-    kevs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.3)
@@ -294,17 +291,19 @@ def run_c5(args, world, rank, local, dev):
     t_start = torch.cuda.Event(enable_timing=True)
     t_end = torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
+    C.cuart_kernel_timer(di.h, True)           # CUDA events around every owner walk launch
     t_start.record(stream)
     for i in range(args.steps):
-        step(i, evs[i], kevs[i])
+        step(i, evs[i])
     t_end.record(stream)
     torch.cuda.synchronize()
     launches = C.cuart_launch_count() - launches0
+    ktot, klaunch, kq, _ = C.cuart_kernel_time_ex(di.h)
+    C.cuart_kernel_timer(di.h, False)
     if world > 1:
         dist.barrier()
     clk = clocks.stop()
-    tt = torch.tensor([t_start.elapsed_time(t_end), float(np.mean([e[0].elapsed_time(e[1]) for e in kevs]))],
-                      dtype=torch.float64, device=dev)
+    tt = torch.tensor([t_start.elapsed_time(t_end), ktot / args.steps], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
     total_ms, kern_ms = tt.tolist()
@@ -352,7 +351,7 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_icpp_koppehelggp21_b200 as C
-    from paper_conf_icpp_koppehelggp21_b200.dist import CudaOps, DistIndex
+    from paper_conf_icpp_koppehelggp21_b200.dist import DistIndex
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -372,13 +371,12 @@ def main():
     cfg = W.CONFIGS[args.config]
     t0 = time.perf_counter()
     keys, vals, keys_d = make_keys(cfg, dev)
-    ops = CudaOps(dev)
     if world == 1:
         layout = C.Layout(keys, vals, lut_bytes=args.lut)
         ix = C.Index.from_layout(layout, device=local, lut_format=LUT_FORMATS[args.lut_format])
         di = None
     else:
-        di = DistIndex(keys, vals, mode=mode, ops=ops, lut_bytes=args.lut, transport=args.transport)
+        di = DistIndex(keys, vals, mode=mode, transport=args.transport, lut_bytes=args.lut)
         ix = di.index
         layout = None
     build_s = time.perf_counter() - t0
@@ -399,7 +397,7 @@ def main():
     # lookup path over this rank's layout for a 2^20-query sample + key-in/value-out
     from paper_conf_icpp_koppehelggp21_b200.dist import owners, prefix8, select
     if layout is None:
-        local_keys = keys if mode == "replica" else select(keys, owners(prefix8(keys), di.splitters_np) == rank)
+        local_keys = keys if mode == "replica" else select(keys, owners(prefix8(keys), di.splitters) == rank)
         nloc = local_keys[1].shape[0] if isinstance(local_keys, tuple) else local_keys.shape[0]
         layout = C.Layout(local_keys, np.zeros(nloc, np.uint64), lut_bytes=args.lut)
     if isinstance(q, tuple):
@@ -408,7 +406,7 @@ def main():
         samp = q[: 1 << 20].cpu().numpy()
         samp = samp.view(np.uint64) if cfg.kind == "u64" else samp.view(np.uint32)
     if mode == "range":   # sample of the queries this rank's index actually serves
-        samp = select(samp, owners(prefix8(samp), di.splitters_np) == rank)
+        samp = select(samp, owners(prefix8(samp), di.splitters) == rank)
     bucketed = nl >= (1 << 22) and cfg.kind != "bytes" and os.environ.get("CUART_PREBUCKET", "1") != "0"
     # the bucketed wide walk over integer keys runs as k_lookup_wq (2 queries per thread)
     wq = bucketed and bool(stats.get("wide_lut", 0)) and os.environ.get("CUART_ILP", "2") != "1"
@@ -442,14 +440,14 @@ def main():
             if kev is not None:
                 kev[1].record(stream)
         else:
-            di.lookup(q, events=kev)
+            di.lookup(q, out)
         if ev is not None:
             ev[1].record(stream)
         if nu:
             if di is None:
                 ix.update(uk, uv, stream)
             else:
-                di.update((uk, uv))
+                di.update(uk, uv)
         if ev is not None:
             ev[2].record(stream)
 
@@ -504,7 +502,7 @@ def main():
     if traffic is None and os.path.exists(tfile):
         with open(tfile) as f:
             traffic = json.load(f).get(f"{args.config}/{'bucketed' if bucketed else 'direct'}")
-    out_now = out if di is None else di.lookup(q)
+    out_now = out if di is None else di.lookup(q, out)
     hit = float((out_now[: 1 << 24] != -1).float().mean().item())
     del out_now
 
@@ -534,9 +532,9 @@ def main():
                     C.cuart_update_host(ix.h, ukh.numpy(), uvh.numpy())
             else:
                 qd = tuple(t.to(dev, non_blocking=True) for t in qh) if isinstance(qh, tuple) else qh.to(dev, non_blocking=True)
-                oh.copy_(di.lookup(qd), non_blocking=True)
+                oh.copy_(di.lookup(qd, out), non_blocking=True)
                 if nu:
-                    di.update((ukh.to(dev, non_blocking=True), uvh.to(dev, non_blocking=True)))
+                    di.update(ukh.to(dev, non_blocking=True), uvh.to(dev, non_blocking=True))
                 torch.cuda.synchronize()
 
         e2e_step()

@@ -83,13 +83,16 @@ typedef struct {
     uint32_t lut_bytes;          /* 0..3: dense root lookup table over the first k key bytes
                                     (§3.2.2, 2^(8k) links; k=3 -> 128 MiB).
                                     CUART_LUT_AUTO (0xFFFFFFFF) = library choice.          */
-    uint32_t l2_persist;         /* 1: request a persisting L2 access-policy window over the
-                                    LUT / top levels (cudaAccessPolicyWindow).               */
+    uint32_t l2_persist;         /* 1: a persisting L2 access-policy window (cudaAccessPolicyWindow,
+                                    hitRatio 1) over the root lookup table the walks start from
+                                    (§3.2.2: the merged upper layers are what the cache
+                                    should keep), set on the caller's stream of every call.  It
+                                    changes performance only.                                 */
     int32_t device;              /* CUDA device ordinal; -1 = current device                */
     uint32_t lut_format;         /* device form of the root table ("compacted pointers"):
                                     CUART_LUT_FORMAT_AUTO, CUART_LUT_LINKS (8-B links),
-                                    CUART_LUT_COMPACT32 (4-B entries), CUART_LUT_RANK (64-B
-                                    blocks per 64 entries: type bit-planes + per-type base
+                                    CUART_LUT_COMPACT32 (4-B entries), CUART_LUT_RANK (32-B
+                                    blocks per 32 entries: type bit-planes + per-type base
                                     index + rank; 1 B/entry, sized for L2 residency).
                                     COMPACT32 / RANK need integer keys (else LINKS).        */
     uint32_t prebucket;          /* query pre-bucketing of large lookup batches (§8(a) a5):
@@ -284,30 +287,6 @@ cuart_status cuart_partition_by_flag(const cuart_keys* keys, size_t n, const uin
                                      void* out_keys, uint8_t* out_lengths, uint64_t* out_values, uint32_t* perm,
                                      uint64_t* counts, void* scratch, void* stream);
 
-/* ---- fused multi-GPU exchange over peer memory (transport "p2p", §8(e)) ----
- * One process per GPU of one box.  Every rank allocates receive windows with
- * cuart_ipc_alloc, exports them (cuart_ipc_export -> an opaque handle of
- * CUART_IPC_HANDLE_BYTES bytes, sent to the peers by the caller's collective
- * library), and maps the peers' windows with cuart_ipc_import (CUDA IPC; peer
- * access over NVLink/NVSwitch is enabled lazily).  A routed batch then needs no
- * all-to-all of the data:
- *   1. cuart_route_count: owner of every op + per-owner counts (device uint64_t
- *      [nparts]); the P x P count matrix is all-gathered by the caller;
- *   2. cuart_route_push: the stable per-owner scatter of cuart_route whose stores
- *      go straight to the owners' windows: op i with owner o lands at
- *      dst_keys[o][its position in this source's run for o] (and likewise
- *      dst_lengths / dst_values); dst_*[o] is owner o's window advanced to the
- *      first slot of this source (sum of the counts of the sources before it), so
- *      every owner sees the runs of all sources concatenated in rank order (the
- *      global op order of the update rule, reading C7).  perm[i] = slot of
- *      op i in this source's owner-major send order (for cuart_unroute);
- *   3. (all ranks synchronised) the owner serves its window with
- *      cuart_lookup_segmented, whose last kernel stores result j of source s
- *      straight into s's result window: seg_dst[s] + (j - seg_start[s]);
- *   4. (synchronised) each source restores query order with cuart_unroute.
- * scratch of steps 1-2: cuart_route_scratch_bytes(n, nparts), kept between the
- * two calls.  nparts <= 16.  All pointers are device pointers (local or mapped
- * peer memory); calls are async on `stream`. */
 /* ---- keys longer than 32 bytes (§8(f) f4; §3.2.3, option 2) ----------
  * An index of kind CUART_KEY_LONG holds prefix-free byte-string keys of 1..255
  * bytes.  Its inner nodes and the leaves of keys of <= 32 bytes live on the
@@ -333,24 +312,111 @@ cuart_status cuart_lookup_long(cuart_index* h, const uint8_t* data, const uint64
 cuart_status cuart_update_long(cuart_index* h, const uint8_t* data, const uint64_t* offsets,
                                const uint64_t* values, size_t n, void* stream);
 
-#define CUART_IPC_HANDLE_BYTES 64
-cuart_status cuart_ipc_alloc(size_t bytes, void** dptr);           /* exportable device window        */
-cuart_status cuart_ipc_free(void* dptr);                           /* NULL ok                         */
-cuart_status cuart_ipc_export(void* dptr, void* handle);           /* handle: CUART_IPC_HANDLE_BYTES  */
-cuart_status cuart_ipc_import(const void* handle, void** dptr);    /* another process's window        */
-cuart_status cuart_ipc_close(void* dptr);                          /* unmap an imported window        */
-cuart_status cuart_route_count(const cuart_keys* keys, size_t n, const uint64_t* splitters, uint32_t nparts,
-                               uint64_t* counts, void* scratch, void* stream);
-cuart_status cuart_route_push(const cuart_keys* keys, size_t n, uint32_t nparts, const uint64_t* values,
-                              void* const* dst_keys, uint8_t* const* dst_lengths, uint64_t* const* dst_values,
-                              uint32_t* perm, void* scratch, void* stream);
-/* cuart_lookup whose result i is stored at seg_dst[s] + (i - seg_start[s]) for the
- * segment s with seg_start[s] <= i < seg_start[s+1] (host arrays: seg_start
- * [nseg+1] with seg_start[0] = 0 and seg_start[nseg] = n, seg_dst[nseg] device
- * pointers, local or mapped peer memory); nseg in [1, 16].  The stores are done by
- * the kernel that produces the results (fused return, Fig. 3 per query). */
-cuart_status cuart_lookup_segmented(const cuart_index* h, const cuart_keys* queries, size_t n, uint32_t nseg,
-                                    const uint64_t* seg_start, uint64_t* const* seg_dst, void* stream);
+/* out[i] = CUART_MISS for i < n (device pointer; async): the result slots of ops that
+ * return no lookup value (the update ops of a mixed round, reading C7). */
+cuart_status cuart_fill_miss(uint64_t* out, size_t n, void* stream);
+
+/* ---- multi-GPU index: one process per GPU of one box --------
+ * The paper runs one GPU (§4.1 mentions a 2-GPU server only as hardware);
+ * the multi-GPU layer is the north star's scaling of its batched lookups and
+ * updates (§4.1: batches, several command streams) over NVLink/NVSwitch.
+ *
+ * Modes:
+ *   CUART_DIST_RANGE   : the key space is range-partitioned over the first 8 key
+ *                        bytes read big-endian (nranks-1 ascending splitters; owner(k)
+ *                        = number of splitters <= prefix8(k)).  Every rank indexes its
+ *                        range; a batch is routed to the owners, served there and the
+ *                        results routed back (K-ROUTE fused with K-BUCKET: the source's
+ *                        pre-bucketing partitions by (owner, owner's bucket), so every
+ *                        owner receives runs that are already bucketed for its walk).
+ *   CUART_DIST_REPLICA : every rank holds the full index; lookups are served locally
+ *                        with no exchange; update batches are exchanged and applied by
+ *                        every rank, so the replicas stay bit-identical.
+ * Transports:
+ *   CUART_TRANSPORT_P2P  : receive windows in device memory exported with CUDA IPC and
+ *                        mapped by every peer (NVLink / NVSwitch).  The source's scatter
+ *                        kernel stores every op straight into its owner's window, the
+ *                        owner's walk stores every result straight into the source's
+ *                        result window; cross-rank ordering uses device-side release /
+ *                        acquire flags (no host barrier, no stream synchronisation); the
+ *                        host only reads the per-chunk count matrix from mapped pinned
+ *                        memory to size the owner's launches.  Batches are cut into
+ *                        chunks with two window slots in flight, so the routing of chunk
+ *                        c+1 overlaps the walk of chunk c.
+ *   CUART_TRANSPORT_NCCL : route into a local send buffer, then grouped ncclSend /
+ *                        ncclRecv of the runs (and of the results), counts via
+ *                        ncclAllGather (the library-collective baseline).
+ * Semantics (reading C7): the ops of one cuart_dist_update call are ordered rank-major
+ * (all of rank 0's batch, then rank 1's, ...), each rank's batch in its own order; the
+ * highest op in that global order wins per key.  Lookups of a call see the
+ * state before any later update call.  Results are independent of nranks, mode and
+ * transport, and equal a single index updated with the concatenated batches.
+ * All dist calls are COLLECTIVE: every rank of the group calls them in the same order
+ * (n may differ per rank, including 0).
+ */
+#define CUART_DIST_REPLICA 1u
+#define CUART_DIST_RANGE 2u
+#define CUART_TRANSPORT_NCCL 1u
+#define CUART_TRANSPORT_P2P 2u
+#define CUART_DIST_MAX_RANKS 16
+#define CUART_NCCL_ID_BYTES 128
+/* Host bootstrap collective: gather `bytes` bytes from every rank into recv
+ * (nranks * bytes, rank order).  Returns 0 on success.  Called only inside
+ * cuart_dist_build / cuart_destroy / cuart_dist_partition (setup and teardown). */
+typedef int (*cuart_allgather_fn)(void* ctx, const void* send, void* recv, size_t bytes);
+typedef struct {
+    int32_t rank;                 /* this process's rank in [0, nranks)                        */
+    int32_t nranks;               /* 1 .. CUART_DIST_MAX_RANKS, one GPU per rank               */
+    uint32_t mode;                /* CUART_DIST_RANGE | CUART_DIST_REPLICA                     */
+    uint32_t transport;           /* CUART_TRANSPORT_P2P | CUART_TRANSPORT_NCCL                */
+    uint8_t nccl_id[CUART_NCCL_ID_BYTES];  /* ncclUniqueId (cuart_dist_unique_id on rank 0, the
+                                     same bytes on every rank); unused when transport is P2P and
+                                     allgather is set                                          */
+    cuart_allgather_fn allgather; /* optional host bootstrap; NULL = ncclAllGather on the comm */
+    void* allgather_ctx;
+    const uint64_t* splitters;    /* RANGE: nranks-1 ascending host splitters, or NULL = quantiles
+                                     of the key set's 8-byte prefixes (identical on every rank)  */
+    uint32_t keys_local;          /* RANGE: 1 = keys/values passed to cuart_dist_build are already
+                                     this rank's share (splitters required)                    */
+    uint32_t reserved0;
+    uint64_t chunk;               /* ops per pipeline chunk per rank; 0 = library default       */
+    cuart_build_opts opts;        /* the local index (opts.device = this rank's GPU)           */
+} cuart_dist_cfg;
+/* Writes a fresh ncclUniqueId (CUART_NCCL_ID_BYTES) to id.  Host only. */
+cuart_status cuart_dist_unique_id(void* id);
+/* Collective build.  keys/values: HOST buffers; RANGE with keys_local = 0 and REPLICA:
+ * the global key set, identical on every rank; RANGE with keys_local = 1: this rank's
+ * share.  Returns a cuart_index of the local part; cuart_lookup / cuart_update on it act
+ * on the local part only; cuart_destroy on it is collective.  Errors as cuart_build,
+ * plus CUART_ERR_NCCL (bootstrap / NCCL failure) and CUART_ERR_INVALID_ARGUMENT (bad
+ * cfg: rank / nranks / mode / transport, splitters not ascending, ranks disagreeing on
+ * the splitters, key kind, window sizes). */
+cuart_status cuart_dist_build(const cuart_dist_cfg* cfg, const cuart_keys* keys, const uint64_t* values, size_t n,
+                              cuart_index** out);
+/* Collective lookup of this rank's batch (DEVICE pointers on this rank's GPU, n may be 0):
+ * out[i] = value of queries[i] in the distributed index, else CUART_MISS.  Enqueued on
+ * `stream` (internal streams join it); returns after the last chunk's launches are
+ * enqueued; n <= 2^32 / nranks. */
+cuart_status cuart_dist_lookup(cuart_index* h, const cuart_keys* queries, size_t n, uint64_t* out, void* stream);
+/* Collective update: this rank's batch (DEVICE pointers) joins the call's global batch
+ * at position rank (reading C7).  Values equal to CUART_MISS are dropped and set the
+ * sticky error flag of the owner's index (reading C5).  n <= 2^32 / nranks. */
+cuart_status cuart_dist_update(cuart_index* h, const cuart_keys* keys, const uint64_t* new_values, size_t n,
+                               void* stream);
+/* Host-only planning (no GPU): the splitters the build uses (RANGE; nranks-1 entries)
+ * and the owner of each key (owner[i], may be NULL).  With a bootstrap in cfg the
+ * splitters are all-gathered and compared across ranks (INVALID_ARGUMENT on mismatch). */
+cuart_status cuart_dist_partition(const cuart_dist_cfg* cfg, const cuart_keys* keys, size_t n, uint64_t* splitters,
+                                  uint8_t* owner);
+/* Host-only: the exchange plan of one chunk for rank `me` from the nranks x nranks count
+ * matrix M (row-major, M[s*P + o] = ops source s routes to owner o), as the library uses
+ * it: seg_start[P+1] (source segments of me's receive window), res_off[P] (first slot of
+ * me's results in source s's send order), push_off[P] (first slot of me's run in owner
+ * o's window). */
+cuart_status cuart_dist_chunk_plan(uint32_t nranks, uint32_t me, const uint64_t* M, uint64_t* seg_start,
+                                   uint64_t* res_off, uint64_t* push_off);
+/* Statistics of the last dist call on this rank: ops received as owner, chunks. */
+cuart_status cuart_dist_last(const cuart_index* h, uint64_t* recv_ops, uint64_t* chunks);
 
 #ifdef __cplusplus
 }

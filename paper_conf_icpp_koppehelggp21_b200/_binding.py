@@ -83,14 +83,8 @@ def lib():
             f = getattr(L, name)
             f.argtypes = args
             f.restype = ctypes.c_int
-        for name, args in {"cuart_ipc_alloc": [S, P], "cuart_ipc_free": [P], "cuart_ipc_export": [P, P],
-                           "cuart_ipc_import": [P, P], "cuart_ipc_close": [P],
-                           "cuart_route_count": [P, S, P, U32, P, P, P],
-                           "cuart_route_push": [P, S, U32, P, P, P, P, P, P, P],
-                           "cuart_lookup_segmented": [P, P, S, U32, P, P, P]}.items():
-            f = getattr(L, name)
-            f.argtypes = args
-            f.restype = ctypes.c_int
+        L.cuart_fill_miss.argtypes = [P, S, P]
+        L.cuart_fill_miss.restype = ctypes.c_int
         L.cuart_launch_count.argtypes = []
         L.cuart_launch_count.restype = ctypes.c_uint64
         _lib = L
@@ -138,6 +132,25 @@ def _contig(x):
     if _is_torch(x):
         return x.contiguous()
     return np.ascontiguousarray(x)
+
+
+def _check_dev(t, device=None, what="tensor"):
+    """A device-pointer argument: a contiguous CUDA tensor (on `device` if given)."""
+    if not _is_torch(t) or not t.is_cuda:
+        raise ValueError(f"{what} must be a CUDA tensor (device pointer)")
+    if not t.is_contiguous():
+        raise ValueError(f"{what} must be contiguous")
+    if device is not None and t.device != device:
+        raise ValueError(f"{what} is on {t.device}, the index on {device}")
+
+
+def _check_out(out, n, device=None, width=8):
+    """The result buffer the kernels write n x `width` bytes into, in a row."""
+    _check_dev(out, device, "out")
+    if out.element_size() != width or out.dim() < 1:
+        raise ValueError(f"out must have {width}-byte elements")
+    if out.numel() < n * (out.shape[-1] if out.dim() == 2 else 1) or out.shape[0] < n:
+        raise ValueError("out too small")
 
 
 def make_keys(keys, lengths=None):
@@ -189,40 +202,58 @@ def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1,
     return h.value
 
 
-def cuart_lookup(h, queries, out, stream=None):
+def _dev_keys(keys, device=None):
+    """make_keys for a device batch: the key (and length) tensors are checked to be
+    contiguous CUDA tensors on the index's device."""
+    k, n, keep = make_keys(keys)
+    _check_dev(keep[0], device, "keys")
+    if keep[1] is not None:
+        _check_dev(keep[1], device, "lengths")
+    return k, n, keep
+
+
+def cuart_lookup(h, queries, out, stream=None, device=None):
     """Device buffers (torch CUDA tensors); async on `stream` (default: current)."""
-    q, n, keep = make_keys(queries)
-    if out.shape[0] < n:
-        raise ValueError("out too small")
+    q, n, keep = _dev_keys(queries, device)
+    _check_out(out, n, device)
     _check(lib().cuart_lookup(h, ctypes.byref(q), n, _ptr(out), _stream_ptr(stream)), "cuart_lookup")
     return out
 
 
-def cuart_update(h, keys, new_values, stream=None):
-    k, n, keep = make_keys(keys)
-    if new_values.shape[0] != n:
-        raise ValueError("values length mismatch")
-    _check(lib().cuart_update(h, ctypes.byref(k), _ptr(_contig(new_values)), n, _stream_ptr(stream)), "cuart_update")
+def cuart_update(h, keys, new_values, stream=None, device=None):
+    k, n, keep = _dev_keys(keys, device)
+    _check_dev(new_values, device, "new_values")
+    if new_values.shape[0] != n or new_values.element_size() != 8:
+        raise ValueError("new_values must be n 8-byte values")
+    _check(lib().cuart_update(h, ctypes.byref(k), _ptr(new_values), n, _stream_ptr(stream)), "cuart_update")
 
 
-def cuart_update_ex(h, keys, new_values, is_delete, stream=None):
+def cuart_update_ex(h, keys, new_values, is_delete, stream=None, device=None):
     """Mixed batch: is_delete (device uint8[n]) marks deletes (reading C17)."""
-    k, n, keep = make_keys(keys)
-    _check(lib().cuart_update_ex(h, ctypes.byref(k), _ptr(_contig(new_values)), _ptr(_contig(is_delete)), n,
+    k, n, keep = _dev_keys(keys, device)
+    _check_dev(new_values, device, "new_values")
+    _check_dev(is_delete, device, "is_delete")
+    if new_values.shape[0] != n or new_values.element_size() != 8 or is_delete.shape[0] != n or \
+            is_delete.element_size() != 1:
+        raise ValueError("new_values / is_delete must be n 8-byte / 1-byte elements")
+    _check(lib().cuart_update_ex(h, ctypes.byref(k), _ptr(new_values), _ptr(is_delete), n,
                                  _stream_ptr(stream)), "cuart_update_ex")
 
 
-def cuart_erase(h, keys, stream=None):
-    k, n, keep = make_keys(keys)
+def cuart_erase(h, keys, stream=None, device=None):
+    k, n, keep = _dev_keys(keys, device)
     _check(lib().cuart_erase(h, ctypes.byref(k), n, _stream_ptr(stream)), "cuart_erase")
 
 
-def cuart_range(h, lo, hi, bounds, stream=None):
+def cuart_range(h, lo, hi, bounds, stream=None, device=None):
     """bounds: device uint64/int64 tensor [n, 6] (start/end per leaf class)."""
-    kl, n, keep1 = make_keys(lo)
-    kh, n2, keep2 = make_keys(hi)
+    kl, n, keep1 = _dev_keys(lo, device)
+    kh, n2, keep2 = _dev_keys(hi, device)
     if n2 != n:
         raise ValueError("lo/hi length mismatch")
+    _check_dev(bounds, device, "bounds")
+    if bounds.element_size() != 8 or bounds.numel() < 6 * n:
+        raise ValueError("bounds must hold 6 x n 8-byte entries")
     _check(lib().cuart_range(h, ctypes.byref(kl), ctypes.byref(kh), n, _ptr(bounds), _stream_ptr(stream)), "cuart_range")
     return bounds
 
@@ -387,12 +418,24 @@ class Layout:
             pass
 
 
+def _torch_device(device):
+    """The CUDA device the library put the index on (-1 = the current device)."""
+    try:
+        import torch
+        if not torch.cuda.is_available():
+            return None
+        return torch.device("cuda", torch.cuda.current_device() if device is None or device < 0 else device)
+    except Exception:        # noqa: BLE001 -- no torch / no CUDA: the C library reports NO_DEVICE itself
+        return None
+
+
 class Index:
     """Device-resident CuART index on one GPU."""
 
     def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0,
                  slice_lut=0, wide_lut=0):
         self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut)
+        self.device = _torch_device(device)
 
     @classmethod
     def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0,
@@ -400,6 +443,7 @@ class Index:
         """Upload an already-built host layout (keeps the host copy usable)."""
         self = cls.__new__(cls)
         self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut)
+        self.device = _torch_device(device)
         return self
 
     def lookup(self, queries, out=None, stream=None):
@@ -407,16 +451,16 @@ class Index:
         if out is None:
             q = queries[0] if isinstance(queries, tuple) else queries
             out = torch.empty(q.shape[0], dtype=torch.uint64, device=q.device)
-        return cuart_lookup(self.h, queries, out, stream)
+        return cuart_lookup(self.h, queries, out, stream, getattr(self, "device", None))
 
     def update(self, keys, new_values, stream=None):
-        cuart_update(self.h, keys, new_values, stream)
+        cuart_update(self.h, keys, new_values, stream, getattr(self, "device", None))
 
     def update_ex(self, keys, new_values, is_delete, stream=None):
-        cuart_update_ex(self.h, keys, new_values, is_delete, stream)
+        cuart_update_ex(self.h, keys, new_values, is_delete, stream, getattr(self, "device", None))
 
     def erase(self, keys, stream=None):
-        cuart_erase(self.h, keys, stream)
+        cuart_erase(self.h, keys, stream, getattr(self, "device", None))
 
     def free_leaves(self):
         return cuart_free_leaves(self.h)
@@ -425,7 +469,7 @@ class Index:
         import torch
         if bounds is None:
             bounds = torch.empty((lo.shape[0], 6), dtype=torch.int64, device=lo.device)
-        return cuart_range(self.h, lo, hi, bounds, stream)
+        return cuart_range(self.h, lo, hi, bounds, stream, getattr(self, "device", None))
 
     def lookup_host(self, queries, out=None):
         return cuart_lookup_host(self.h, queries, out)
@@ -459,70 +503,6 @@ class Index:
             self.close()
         except Exception:
             pass
-
-
-# ------------------------------------------------------------------ fused multi-GPU exchange (p2p)
-IPC_HANDLE_BYTES = 64
-
-
-def raw_keys(kind, data_ptr, lens_ptr=None):
-    """cuart_keys over raw device pointers (windows allocated by cuart_ipc_alloc)."""
-    return _Keys(kind, data_ptr, lens_ptr if kind == KIND_BYTES else None)
-
-
-def ipc_alloc(nbytes):
-    p = ctypes.c_void_p()
-    _check(lib().cuart_ipc_alloc(max(1, int(nbytes)), ctypes.byref(p)), "cuart_ipc_alloc")
-    return p.value
-
-
-def ipc_free(ptr):
-    _check(lib().cuart_ipc_free(ptr), "cuart_ipc_free")
-
-
-def ipc_export(ptr):
-    buf = ctypes.create_string_buffer(IPC_HANDLE_BYTES)
-    _check(lib().cuart_ipc_export(ptr, buf), "cuart_ipc_export")
-    return buf.raw
-
-
-def ipc_import(handle):
-    buf = ctypes.create_string_buffer(bytes(handle), IPC_HANDLE_BYTES)
-    p = ctypes.c_void_p()
-    _check(lib().cuart_ipc_import(buf, ctypes.byref(p)), "cuart_ipc_import")
-    return p.value
-
-
-def ipc_close(ptr):
-    _check(lib().cuart_ipc_close(ptr), "cuart_ipc_close")
-
-
-def route_count(keys_struct, n, splitters_ptr, nparts, counts_ptr, scratch_ptr, stream=None):
-    _check(lib().cuart_route_count(ctypes.byref(keys_struct), n, splitters_ptr, nparts, counts_ptr, scratch_ptr,
-                                   _stream_ptr(stream)), "cuart_route_count")
-
-
-def route_push(keys_struct, n, nparts, values_ptr, dst_keys, dst_lens, dst_vals, perm_ptr, scratch_ptr, stream=None):
-    """dst_* : lists of nparts device addresses (ints) or None."""
-    arr = lambda xs: (ctypes.c_void_p * nparts)(*xs) if xs is not None else None
-    _check(lib().cuart_route_push(ctypes.byref(keys_struct), n, nparts, values_ptr, arr(dst_keys), arr(dst_lens),
-                                  arr(dst_vals), perm_ptr, scratch_ptr, _stream_ptr(stream)), "cuart_route_push")
-
-
-def lookup_segmented(h, keys_struct, n, seg_start, seg_dst, stream=None):
-    nseg = len(seg_dst)
-    st = (ctypes.c_uint64 * (nseg + 1))(*[int(x) for x in seg_start])
-    ds = (ctypes.c_void_p * nseg)(*seg_dst)
-    _check(lib().cuart_lookup_segmented(h, ctypes.byref(keys_struct), n, nseg, st, ds, _stream_ptr(stream)),
-           "cuart_lookup_segmented")
-
-
-def update_raw(h, keys_struct, n, values_ptr, stream=None):
-    _check(lib().cuart_update(h, ctypes.byref(keys_struct), values_ptr, n, _stream_ptr(stream)), "cuart_update")
-
-
-def unroute_raw(in_ptr, perm_ptr, n, out_ptr, stream=None):
-    _check(lib().cuart_unroute(in_ptr, perm_ptr, n, out_ptr, _stream_ptr(stream)), "cuart_unroute")
 
 
 # ------------------------------------------------------------------ f4: keys longer than 32 bytes

@@ -22,6 +22,17 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
+def _nccl_root():
+    """NCCL 2.28 shipped with the PyTorch wheels (headers + libnccl.so.2); the multi-GPU
+    layer (csrc/dist.cu) links it for its NCCL transport and bootstrap."""
+    import nvidia.nccl
+    return list(nvidia.nccl.__path__)[0]
+
+
+NCCL_ROOT = _nccl_root()
+NCCL_LIB = os.path.join(NCCL_ROOT, "lib")
+
+
 def _sources():
     return [os.path.join(CSRC, f) for f in sorted(os.listdir(CSRC))
             if f.endswith((".cu", ".cpp", ".h", ".cuh"))] + [os.path.join(ROOT, "include", "cuart.h")]
@@ -37,7 +48,7 @@ def build(force: bool = False, verbose_ptxas: bool = False) -> str:
     if not force and os.path.exists(OUT) and os.path.getmtime(OUT) >= max(os.path.getmtime(s) for s in srcs):
         return OUT
     os.makedirs(BUILD, exist_ok=True)
-    inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
+    inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", os.path.join(NCCL_ROOT, "include")]
     inc += os.environ.get("CUART_DEFS", "").split()          # e.g. "-DCUART_N16_BYTES=256" (layout experiments)
     objs = []
     for f in sorted(os.listdir(CSRC)):
@@ -55,7 +66,8 @@ def build(force: bool = False, verbose_ptxas: bool = False) -> str:
             continue
         objs.append(obj)
     tmp = OUT + f".tmp{os.getpid()}"
-    _run([NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs, "-Xcompiler", "-fopenmp", "-lgomp"])
+    _run([NVCC, *ARCH, "-shared", "-cudart", "static", "-o", tmp, *objs, "-Xcompiler", "-fopenmp", "-lgomp",
+          "-L", NCCL_LIB, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + NCCL_LIB])
     os.replace(tmp, OUT)
     return OUT
 

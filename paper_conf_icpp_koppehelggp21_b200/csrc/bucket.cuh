@@ -64,6 +64,72 @@ __device__ __forceinline__ uint32_t bucket_at(const void* q, const uint8_t* lens
     return d < l ? uint32_t(__ldcs((const uint8_t*)q + 32 * i + d)) >> (depth >> 8) : 0u;
 }
 
+// Part functions of the K-BUCKET kernels.  ByteBucket: the single-GPU bucket (root
+// branch byte >> shift, packed in `depth` as above).  OwnerPart (multi-GPU, §8(e)):
+// K-ROUTE fused with K-BUCKET -- part = owner << lbpo | (the owner's root branch
+// byte >> (8 - lbpo)), owner = number of splitters <= the key's first 8 bytes read
+// big-endian.  Parts are numbered owner-major, so the bucketed batch is also the
+// routed batch: owner o's ops are one contiguous run of the send order, already
+// bucketed for o's walk.
+struct ByteBucket {
+    uint32_t depth;
+    __host__ __device__ ByteBucket(uint32_t d = 0) : depth(d) {}
+    template <class Key>
+    __device__ __forceinline__ uint32_t of(const Key& k) const { return bucket_of(k, depth); }
+    template <class Key>
+    __device__ __forceinline__ uint32_t at(const void* q, const uint8_t* lens, uint64_t i) const {
+        return bucket_at<Key>(q, lens, i, depth);
+    }
+};
+
+template <class Key>
+__device__ __forceinline__ uint64_t key_prefix8(const Key& k) {
+    if (Key::kKind == 2) return uint64_t(((const KeyU64&)k).k);
+    if (Key::kKind == 1) return uint64_t(((const KeyU32&)k).k) << 32;
+    return bswap64(((const KeyBytes&)k).w[0]);                 // zero-padded past the length
+}
+
+struct OwnerPart {
+    uint32_t nsp;                      // number of splitters (ranks - 1)
+    uint32_t lbpo;                     // bucket bits per owner
+    uint64_t sp[kMaxSeg - 1];          // ascending splitters over the 8-byte prefix
+    uint8_t depth[kMaxSeg];            // every owner's root branch depth
+    template <class Key>
+    __device__ __forceinline__ uint32_t owner(const Key& k) const {
+        const uint64_t p = key_prefix8(k);
+        uint32_t o = 0;
+#pragma unroll 1
+        for (uint32_t j = 0; j < nsp; j++) o += sp[j] <= p ? 1u : 0u;
+        return o;
+    }
+    template <class Key>
+    __device__ __forceinline__ uint32_t of(const Key& k) const {
+        const uint32_t o = owner(k);
+        const uint32_t d = depth[o];
+        const uint32_t b = d < k.len() ? k.byte(d) : 0u;
+        return (o << lbpo) | (b >> (8 - lbpo));
+    }
+    template <class Key>
+    __device__ __forceinline__ uint32_t at(const void* q, const uint8_t* lens, uint64_t i) const {
+        return of(Key::template load<true>(q, lens, i));
+    }
+};
+
+// Fused push of the multi-GPU exchange (transport p2p): the staged runs of k_bscatter
+// are stored straight into the receive windows of their owners (peer memory mapped
+// over NVLink / NVSwitch): send-order slot d of a part of owner o lands at
+// keys[o] + d + adj[o] (adj = this source's first slot in o's window minus o's first
+// send-order slot).  nrep > 0 (replica mode): every op goes to all nrep windows.
+struct PushDst {
+    void* keys[kMaxSeg];
+    uint8_t* lens[kMaxSeg];
+    uint64_t* vals[kMaxSeg];
+    uint32_t* prio[kMaxSeg];
+    const long long* adj;              // device, per owner (written by the count exchange)
+    uint32_t lbpo;
+    uint32_t nrep;
+};
+
 // Block-wide exclusive scan of one value per thread (kBucketThreads == kBuckets == 256).
 // Contains one __syncthreads; the caller syncs before reusing wtot.
 __device__ __forceinline__ unsigned int block_excl_scan256(unsigned int v, unsigned int* wtot) {
@@ -86,9 +152,9 @@ __device__ __forceinline__ unsigned int block_excl_scan256(unsigned int v, unsig
 // is loaded before the first shared-memory atomic; with VEC (queries 16-B aligned)
 // integer keys arrive in 16-B loads (2 u64 / 4 u32 keys per load): 1.27 ms per
 // 2^30 u64 keys (6.8 TB/s) against 2.08 ms with 8-B loads (tools/bucket_micro.cu).
-template <class Key, bool VEC>
+template <class Key, bool VEC, class PF = ByteBucket>
 __global__ void __launch_bounds__(kBucketThreads) k_bhist(const void* __restrict__ q, const uint8_t* __restrict__ lens,
-                                                          uint64_t n, uint32_t depth, unsigned int* __restrict__ hist) {
+                                                          uint64_t n, PF pf, unsigned int* __restrict__ hist) {
     __shared__ unsigned int h[kBuckets];
     h[threadIdx.x] = 0;
     __syncthreads();
@@ -108,16 +174,16 @@ __global__ void __launch_bounds__(kBucketThreads) k_bhist(const void* __restrict
             const uint64_t i = base + uint64_t(PER) * (uint64_t(r) * kBucketThreads + threadIdx.x);
             if (i + PER <= n) {
                 if (Key::kKind == 2) {
-                    atomicAdd(&h[bucket_of(KeyU64{uint64_t(v[r].x) | (uint64_t(v[r].y) << 32)}, depth)], 1u);
-                    atomicAdd(&h[bucket_of(KeyU64{uint64_t(v[r].z) | (uint64_t(v[r].w) << 32)}, depth)], 1u);
+                    atomicAdd(&h[pf.of(KeyU64{uint64_t(v[r].x) | (uint64_t(v[r].y) << 32)})], 1u);
+                    atomicAdd(&h[pf.of(KeyU64{uint64_t(v[r].z) | (uint64_t(v[r].w) << 32)})], 1u);
                 } else {
-                    atomicAdd(&h[bucket_of(KeyU32{v[r].x}, depth)], 1u);
-                    atomicAdd(&h[bucket_of(KeyU32{v[r].y}, depth)], 1u);
-                    atomicAdd(&h[bucket_of(KeyU32{v[r].z}, depth)], 1u);
-                    atomicAdd(&h[bucket_of(KeyU32{v[r].w}, depth)], 1u);
+                    atomicAdd(&h[pf.of(KeyU32{v[r].x})], 1u);
+                    atomicAdd(&h[pf.of(KeyU32{v[r].y})], 1u);
+                    atomicAdd(&h[pf.of(KeyU32{v[r].z})], 1u);
+                    atomicAdd(&h[pf.of(KeyU32{v[r].w})], 1u);
                 }
             } else {
-                for (uint64_t e = i; e < n && e < i + PER; e++) atomicAdd(&h[bucket_at<Key>(q, lens, e, depth)], 1u);
+                for (uint64_t e = i; e < n && e < i + PER; e++) atomicAdd(&h[pf.template at<Key>(q, lens, e)], 1u);
             }
         }
     } else {
@@ -125,7 +191,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bhist(const void* __restrict
 #pragma unroll
         for (int r = 0; r < kBucketItems; r++) {
             const uint64_t i = base + uint64_t(r) * kBucketThreads + threadIdx.x;
-            bk[r] = i < n ? bucket_at<Key>(q, lens, i, depth) : 0xFFFFFFFFu;
+            bk[r] = i < n ? pf.template at<Key>(q, lens, i) : 0xFFFFFFFFu;
         }
 #pragma unroll
         for (int r = 0; r < kBucketItems; r++)
@@ -138,7 +204,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bhist(const void* __restrict
 // One CTA per bucket: exclusive scan of its row over the tiles (in place), row
 // total -> totals[b].  A hist group is kHistGroup = 8 consecutive tiles of this
 // bucket = one 32-B sector.
-__global__ void __launch_bounds__(kBucketThreads) k_bscan_rows(unsigned int* __restrict__ hist, uint64_t tiles,
+static __global__ void __launch_bounds__(kBucketThreads) k_bscan_rows(unsigned int* __restrict__ hist, uint64_t tiles,
                                                                unsigned int* __restrict__ totals) {
     static_assert(kHistGroup == 8, "one 32-B sector per thread");
     __shared__ unsigned int wtot[kBucketThreads / 32];
@@ -199,7 +265,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscan_rows(unsigned int* __r
 // totals -> exclusive bucket bases (in place), one CTA of kBuckets threads
 // Only the first nb buckets are in use (256 >> shift): the others count 0 (their
 // totals were never written) and get base = n.
-__global__ void __launch_bounds__(kBuckets) k_bscan(unsigned int* __restrict__ counts, uint32_t nb) {
+static __global__ void __launch_bounds__(kBuckets) k_bscan(unsigned int* __restrict__ counts, uint32_t nb) {
     __shared__ unsigned int s[kBuckets];
     const int t = threadIdx.x;
     const unsigned int own = uint32_t(t) < nb ? counts[t] : 0u;
@@ -236,16 +302,20 @@ __device__ __forceinline__ void copy_key_to_smem(const void* q, uint64_t i, uint
 // has 16 independent stores.
 // OPS (update batches): each op's value and original index (its priority)
 // travel with it; no gather follows, so jpos is not written.
-template <class Key, bool OPS = false>
+// prio_base (OPS): the priority written with an op is prio_base + its index in the
+// batch (the multi-GPU layer numbers ops globally, rank-major, reading C7).
+// PUSH: the runs go to the owners' receive windows (PushDst), not to bq/blens/bvals/bidx.
+template <class Key, bool OPS = false, class PF = ByteBucket, bool PUSH = false>
 __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restrict__ q, const uint8_t* __restrict__ lens,
-                                                             uint64_t n, uint32_t depth,
+                                                             uint64_t n, PF pf,
                                                              const unsigned int* __restrict__ rowoff,
                                                              const unsigned int* __restrict__ bases,
                                                              void* __restrict__ bq, uint8_t* __restrict__ blens,
                                                              uint16_t* __restrict__ jpos,
                                                              const uint64_t* __restrict__ vals = nullptr,
                                                              uint64_t* __restrict__ bvals = nullptr,
-                                                             uint32_t* __restrict__ bidx = nullptr) {
+                                                             uint32_t* __restrict__ bidx = nullptr,
+                                                             uint32_t prio_base = 0, PushDst pd = PushDst{}) {
     static_assert(kBucketThreads == kBuckets, "one thread per bucket in the scans");
     constexpr uint32_t KS = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
     extern __shared__ __align__(16) uint8_t smem[];
@@ -258,8 +328,20 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
     __shared__ unsigned int loc[kBuckets];
     __shared__ unsigned int glb[kBuckets];
     __shared__ unsigned int wtot[kBucketThreads / 32];
+    __shared__ long long padj[PUSH ? kBuckets : 1];                   // PUSH: per-part window adjustment
+    __shared__ void* swin[PUSH ? 4 * kMaxSeg : 1];                     // PUSH: keys / lens / vals / prio windows
     h[threadIdx.x] = 0;
     const unsigned int gb = bases[threadIdx.x] + rowoff[hidx(threadIdx.x, blockIdx.x)];   // issued first
+    if (PUSH) {
+        if (pd.nrep == 0) padj[threadIdx.x] = pd.adj[threadIdx.x >> pd.lbpo < kMaxSeg ? threadIdx.x >> pd.lbpo : 0];
+        if (threadIdx.x < kMaxSeg) {
+            swin[threadIdx.x] = pd.keys[threadIdx.x];
+            swin[kMaxSeg + threadIdx.x] = pd.lens[threadIdx.x];
+            swin[2 * kMaxSeg + threadIdx.x] = pd.vals[threadIdx.x];
+            swin[3 * kMaxSeg + threadIdx.x] = pd.prio[threadIdx.x];
+            if (pd.nrep) padj[threadIdx.x] = threadIdx.x < pd.nrep ? pd.adj[threadIdx.x] : 0;
+        }
+    }
     __syncthreads();
     const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
     const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
@@ -281,9 +363,9 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
         br[r] = 0xFFFFFFFFu;
         if (j < cnt) {
             uint32_t b;
-            if (Key::kKind == 2) b = bucket_of(KeyU64{kv[r]}, depth);
-            else if (Key::kKind == 1) b = bucket_of(KeyU32{uint32_t(kv[r])}, depth);
-            else b = bucket_at<Key>(q, lens, base + j, depth);
+            if (Key::kKind == 2) b = pf.of(KeyU64{kv[r]});
+            else if (Key::kKind == 1) b = pf.of(KeyU32{uint32_t(kv[r])});
+            else b = pf.template at<Key>(q, lens, base + j);
             br[r] = (b << 16) | atomicAdd(&h[b], 1u);
         }
     }
@@ -315,6 +397,32 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
         }
     }
     __syncthreads();
+    if (PUSH) {                                                        // fused route: runs -> owner windows
+#pragma unroll 4
+        for (int r = 0; r < kBucketItems; r++) {
+            const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
+            if (j >= cnt) continue;
+            const uint32_t b = sb[j];
+            const uint64_t dsend = uint64_t(glb[b] + j);                  // send-order slot
+            const uint32_t w0 = pd.nrep ? 0u : (b >> pd.lbpo), w1 = pd.nrep ? pd.nrep : w0 + 1;
+            for (uint32_t w = w0; w < w1; w++) {
+                const uint64_t dst = dsend + uint64_t(padj[pd.nrep ? w : b]);
+                void* kw = swin[w];
+                if (KS == 8) __stcs((unsigned long long*)kw + dst, (unsigned long long)((const uint64_t*)skeys)[j]);
+                else if (KS == 4) __stcs((unsigned int*)kw + dst, ((const uint32_t*)skeys)[j]);
+                else {
+                    __stcs((uint4*)kw + 2 * dst, ((const uint4*)skeys)[2 * j]);
+                    __stcs((uint4*)kw + 2 * dst + 1, ((const uint4*)skeys)[2 * j + 1]);
+                    ((uint8_t*)swin[kMaxSeg + w])[dst] = slens[j];
+                }
+                if (OPS) {
+                    __stcs((unsigned long long*)swin[2 * kMaxSeg + w] + dst, (unsigned long long)svals[j]);
+                    __stcs((unsigned int*)swin[3 * kMaxSeg + w] + dst, unsigned(prio_base + base + sidx[j]));
+                }
+            }
+        }
+        return;
+    }
 #pragma unroll 4
     for (int r = 0; r < kBucketItems; r++) {
         const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
@@ -329,7 +437,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
             }
             if (OPS) {
                 __stcs((unsigned long long*)bvals + dst, (unsigned long long)svals[j]);
-                __stcs((unsigned int*)bidx + dst, unsigned(base + sidx[j]));
+                __stcs((unsigned int*)bidx + dst, unsigned(prio_base + base + sidx[j]));
             }
         }
     }

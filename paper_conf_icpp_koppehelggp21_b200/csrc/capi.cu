@@ -33,80 +33,7 @@
 
 using namespace cuart;
 
-struct cuart_layout {
-    HostLayout L;
-};
-
-// host-buffer pipelines (cuart_lookup_host / cuart_update_host)
-static constexpr size_t kStageChunk = size_t(1) << 23;   // ops per pipeline chunk (env CUART_STAGE_CHUNK overrides)
-static constexpr int kStages = 4;                          // chunks in flight (streams / staging sets)
-
-struct cuart_index {
-    int device = 0;
-    int num_sms = 148;
-    uint32_t key_kind = 0;
-    uint32_t lut_bytes = 0;
-    uint64_t root = 0;
-    uint64_t count[8] = {0};
-    uint64_t n_keys = 0;
-    uint32_t max_depth = 0;
-    uint8_t* arena = nullptr;          // all record buffers + winner words + LUT + error flag
-    size_t arena_bytes = 0;
-    uint64_t off[8] = {0};
-    uint64_t lut_off = 0, winner_off = 0, err_off = 0;
-    uint64_t total_leaves = 0;
-    DevIndex dix{};
-    DevIndex dix_links{};              // dix reading the 8-B LINKS root table (bucketed walks; §5)
-    uint32_t epoch = 0;                // update batch epoch (high half of winner words)
-    // update scratch (leaf links of the current batch)
-    uint64_t* leafref = nullptr;
-    size_t leafref_cap = 0;
-    uint64_t* slotref = nullptr;       // parent slot of each located leaf (batches with deletes)
-    size_t slotref_cap = 0;
-    uint64_t free_off = 0;             // free-leaf list (u32 ids) + its counter
-    // host-pipeline staging
-    void* stage[4] = {nullptr, nullptr, nullptr, nullptr};
-    uint64_t* stage_out[4] = {nullptr, nullptr, nullptr, nullptr};
-    uint8_t* stage_len[4] = {nullptr, nullptr, nullptr, nullptr};
-    uint64_t* stage_val[4] = {nullptr, nullptr, nullptr, nullptr};
-    size_t stage_cap = 0;
-    cudaStream_t streams[4] = {nullptr, nullptr, nullptr, nullptr};   // host-pipeline streams
-    cudaStream_t ustream = nullptr;                                   // update pipeline: the kernels, in op order
-    cudaEvent_t ev_copied[4] = {nullptr, nullptr, nullptr, nullptr};  // staging set s filled
-    cudaEvent_t ev_free[4] = {nullptr, nullptr, nullptr, nullptr};    // staging set s consumed
-    int policy = 5;                    // cache-policy variant of the kernels (kernels.cuh Loader)
-    uint32_t lut_format = CUART_LUT_LINKS;
-    uint64_t lutc_off = 0;             // compact / rank LUT region
-    uint64_t lutw_off = 0;             // wide LUT region (32 B/entry), 0 bytes if absent
-    bool wide = false;
-    uint64_t lut_exceptions = 0;       // RANK: entries served by the 64-bit table
-    int grid_ctas_per_sm = 0;          // 0 = default grid (one op per thread); else persistent grid
-    bool ktimer = false;               // record CUDA events around every k_lookup launch
-    int ilp = 2;                       // queries per thread of the pre-bucketed wide walk (k_lookup_wq)
-    unsigned wq_tpb = 64;              // k_lookup_wq threads per CTA (CUART_WQ_TPB: 32 / 64 / 128 / 256)
-    unsigned lk_tpb = 256;             // k_lookup threads per CTA (CUART_LOOKUP_TPB: 64 / 128 / 256)
-    unsigned upd2_tpb = 256;           // k_upd2 threads per CTA (CUART_UPD2_TPB: 64 / 256)
-    int wq_lp = 3;                     // k_lookup_wq leaf-load cache policy (CUART_WQ_LEAFPOL, kernels.cuh leafv4_b)
-    // K-BUCKET on the root byte >> shift: 256 >> shift buckets (CUART_BUCKET_SHIFT).  Set
-    // at upload: 64 buckets when a bucket's slice of the walked records stays within
-    // 64 MB (c2, c3: runs of ~64 keys per tile cut the run-scattered traffic of scatter
-    // and gather while the slice stays L2-resident), else 256 (c5 at N = 1: 60 GB).
-    uint32_t bucket_shift = 0;
-    std::mutex kmu;
-    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> kev;
-    uint64_t klookups = 0;
-    uint64_t kslice = 0;               // timed launches that were k_lookup_slice
-    // f4 (CUART_KEY_LONG): host-resident leaves of the keys longer than 32 bytes
-    std::vector<uint8_t> long_bytes;
-    std::vector<uint64_t> long_off, long_vals;
-    uint32_t prebucket = CUART_PREBUCKET_AUTO;   // a5: reorder large lookup batches by bucket (bucket.cuh)
-    uint32_t slice_lut = CUART_SLICE_AUTO;       // bucketed walk with the bucket's LUT slice in smem
-    bool slice_ok = false;                       // RANK table, integer keys, root branch depth + 2 <= k
-    uint64_t slice_e0 = 0;                       // common prefix C << 8(k - d): first entry of bucket 0's slice
-    uint32_t slice_shift = 0;                    // log2(entries per slice) = 8(k - 1 - d)
-    int slice_grid = 0;                          // persistent grid (CTAs) of k_lookup_slice
-
-};
+#include "index.h"
 
 std::atomic<uint64_t> g_cuart_launches{0};   // also counted by route.cu
 
@@ -454,9 +381,6 @@ static cuart_status check_keys(const cuart_index* h, const cuart_keys* k, size_t
     return CUART_OK;
 }
 
-static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens,
-                                         uint64_t n, uint64_t* out, cudaStream_t s, const SegOut* so = nullptr,
-                                         bool bucketed = false);
 
 static void ktimer_begin(const cuart_index* h, cudaStream_t s, cudaEvent_t& ev0, cudaEvent_t& ev1) {
     ev0 = ev1 = nullptr;
@@ -503,19 +427,23 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
     const size_t o_hist = 0, o_tot = al(hist_entries(tiles) * 4), o_q = o_tot + 1024, o_len = o_q + al(n * ks),
                  o_pos = o_len + al(Key::kKind == 3 ? n : 0), o_res = o_pos + al(n * 2), total = o_res + al(n * 8);
     uint8_t* scr = nullptr;
-    CU_TRY(cudaMallocAsync((void**)&scr, total, s));
+    cuart_status rc = scratch_alloc(h, (void**)&scr, total, s);
+    if (rc != CUART_OK) return rc;
     unsigned int* hist = (unsigned int*)(scr + o_hist);
     unsigned int* tot = (unsigned int*)(scr + o_tot);
     const uint32_t depth = (link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u) |
                            (h->bucket_shift << 8);
-    if ((uintptr_t(q) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
-    else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, depth, hist);
+    if ((uintptr_t(q) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, ByteBucket(depth), hist);
+    else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, ByteBucket(depth), hist);
     k_bscan_rows<<<kBuckets >> h->bucket_shift, kBucketThreads, 0, s>>>(hist, tiles, tot);   // rows in use only
     k_bscan<<<1, kBuckets, 0, s>>>(tot, kBuckets >> h->bucket_shift);
     k_bscatter<Key><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key>(), s>>>(
-        q, lens, n, depth, hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, (uint16_t*)(scr + o_pos));
+        q, lens, n, ByteBucket(depth), hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, (uint16_t*)(scr + o_pos));
     g_cuart_launches += 4;
-    CU_TRY(cudaGetLastError());
+    if (cudaGetLastError() != cudaSuccess) {
+        scratch_free(h, scr, s);
+        return CUART_ERR_CUDA;
+    }
     const uint64_t slice_bytes = uint64_t(1) << h->slice_shift;
     // AUTO = off: measured slower than k_lookup over the bucketed batch on c3 (19.2 vs
     // 15.0 ms per 2^30: the 64-KiB slices take L1 capacity, L2 hit rate 64% -> 49%)
@@ -524,26 +452,28 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
     (void)slice_bytes;
     const bool slice = Key::kKind != 3 && h->slice_ok && h->policy == 5 && h->slice_lut == CUART_SLICE_ON &&
                        h->bucket_shift == 0;
-    cuart_status rc = CUART_OK;
     if (slice) rc = launch_lookup_slice<Key>(h, scr + o_q, n, (uint64_t*)(scr + o_res), tot, s);
     else rc = launch_lookup_direct(h, Key::kKind, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, n,
                                    (uint64_t*)(scr + o_res), s, nullptr, true);
-    if (rc != CUART_OK) return rc;
+    if (rc != CUART_OK) {
+        scratch_free(h, scr, s);
+        return rc;
+    }
     if (so) k_bgather<true><<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint64_t*)(scr + o_res),
                                                                         (const uint16_t*)(scr + o_pos), n, hist, tot,
                                                                         nullptr, *so);
     else k_bgather<false><<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint64_t*)(scr + o_res),
                                                                       (const uint16_t*)(scr + o_pos), n, hist, tot, out);
     g_cuart_launches++;
-    CU_TRY(cudaGetLastError());
-    CU_TRY(cudaFreeAsync(scr, s));
-    return CUART_OK;
+    rc = cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+    scratch_free(h, scr, s);
+    return rc;
 }
 
 static constexpr uint64_t kBucketMin = uint64_t(1) << 22;   // below this the batch is too small to reorder
 
-static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens, uint64_t n,
-                                  uint64_t* out, cudaStream_t s, const SegOut* so = nullptr) {
+cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens, uint64_t n,
+                                  uint64_t* out, cudaStream_t s, const SegOut* so) {
     if (n == 0) return CUART_OK;
     // AUTO: integer keys only — for byte strings (c4, Zipf) the 33-B key copies cost
     // more than the locality gains (measured 9.0 vs 10.6 G lookups/s).
@@ -559,10 +489,22 @@ static cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const voi
     return launch_lookup_direct(h, kind, q, lens, n, out, s, so);
 }
 
-static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens,
-                                         uint64_t n, uint64_t* out, cudaStream_t s, const SegOut* so, bool bucketed) {
+cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens,
+                                  uint64_t n, uint64_t* out, cudaStream_t s, const SegOut* so, bool bucketed) {
     const int grid = grid_for(h, n);
     const DevIndex& dx = bucketed ? h->dix_links : h->dix;
+    if (so && bucketed && dx.walk_wide && h->policy == 5 && h->ilp > 1 &&
+        (kind == CUART_KEY_U64 || kind == CUART_KEY_U32)) {   // fused return from the wide walk (multi-GPU owner)
+        cudaEvent_t ev0, ev1;
+        ktimer_begin(h, s, ev0, ev1);
+        const unsigned g = unsigned((n + 127) / 128);
+        if (kind == CUART_KEY_U64) k_lookup_wq<KeyU64, 5, 2, 64, true, 3><<<g, 64, 0, s>>>(dx, q, lens, n, nullptr, *so);
+        else k_lookup_wq<KeyU32, 5, 2, 64, true, 3><<<g, 64, 0, s>>>(dx, q, lens, n, nullptr, *so);
+        g_cuart_launches++;
+        ktimer_end(h, s, ev0, ev1, n);
+        CU_TRY(cudaGetLastError());
+        return CUART_OK;
+    }
     if (so) {                                          // fused return: the default policy only
         switch (kind) {
         case CUART_KEY_U64: k_lookup<KeyU64, 5, true><<<grid, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
@@ -626,47 +568,44 @@ static cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, co
     return CUART_OK;
 }
 
-static cuart_status ensure_scratch(cuart_index* h, size_t n, bool slots) {
-    if (h->leafref_cap < n) {
-        if (h->leafref) cudaFree(h->leafref);
-        h->leafref = nullptr;
-        h->leafref_cap = 0;
-        CU_TRY(cudaMalloc(&h->leafref, n * sizeof(uint64_t)));
-        h->leafref_cap = n;
+cuart_status scratch_alloc(const cuart_index* h, void** p, size_t bytes, cudaStream_t s) {
+    *p = nullptr;
+    if (bytes == 0) bytes = 256;
+    const cudaError_t e = h->pool ? cudaMallocFromPoolAsync(p, bytes, h->pool, s) : cudaMallocAsync(p, bytes, s);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        *p = nullptr;
+        return e == cudaErrorMemoryAllocation ? CUART_ERR_OOM : CUART_ERR_CUDA;
     }
-    if (slots && h->slotref_cap < n) {
-        if (h->slotref) cudaFree(h->slotref);
-        h->slotref = nullptr;
-        h->slotref_cap = 0;
-        CU_TRY(cudaMalloc(&h->slotref, n * sizeof(uint64_t)));
-        h->slotref_cap = n;
+    return CUART_OK;
+}
+
+void scratch_free(const cuart_index*, void* p, cudaStream_t s) {
+    if (p) cudaFreeAsync(p, s);
+}
+
+cuart_status next_epoch(cuart_index* h, cudaStream_t s) {
+    if (++h->epoch == 0xFFFFFFFFu) {        // epoch wrap: clear the conflict words
+#if CUART_COLOCATED_WINNER
+        k_clear_winners<<<h->num_sms * 8, 256, 0, s>>>(h->dix, h->count[5], h->count[6], h->count[7]);
+        g_cuart_launches++;
+        CU_TRY(cudaGetLastError());
+#else
+        if (h->total_leaves) CU_TRY(cudaMemsetAsync(h->dix.winner, 0, h->total_leaves * 8, s));
+#endif
+        h->epoch = 1;
     }
     return CUART_OK;
 }
 
 static constexpr uint64_t kUpdateChunk = uint64_t(1) << 30;   // op index must fit the low 32 bits
 
-// mode: 0 = updates only, 1 = mixed (is_delete[i]), 2 = all deletes (vals unused).
-// opidx: original op index of each op (pre-bucketed batches), or nullptr (= position).
-static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, const uint8_t* lens,
-                                  const uint64_t* vals, const uint8_t* is_delete, int mode, uint64_t n,
-                                  cudaStream_t s, const uint32_t* opidx = nullptr, bool bucketed = false) {
+static cuart_status update_chunk(cuart_index* h, const DevIndex& dx, uint32_t kind, const void* k, const uint8_t* lens,
+                                 const uint64_t* vals, const uint8_t* is_delete, int mode, uint64_t base, uint64_t m,
+                                 cudaStream_t s, const uint32_t* opidx, bool bucketed, uint64_t* leafref,
+                                 uint64_t* slotref) {
     const bool del = mode != 0;
-    const DevIndex& dx = bucketed ? h->dix_links : h->dix;
-    for (uint64_t base = 0; base < n; base += kUpdateChunk) {
-        const uint64_t m = (n - base) < kUpdateChunk ? (n - base) : kUpdateChunk;
-        cuart_status rc = ensure_scratch(h, m, del);
-        if (rc != CUART_OK) return rc;
-        if (++h->epoch == 0xFFFFFFFFu) {        // epoch wrap: clear the conflict words
-#if CUART_COLOCATED_WINNER
-            k_clear_winners<<<h->num_sms * 8, 256, 0, s>>>(h->dix, h->count[5], h->count[6], h->count[7]);
-            g_cuart_launches++;
-            CU_TRY(cudaGetLastError());
-#else
-            CU_TRY(cudaMemsetAsync(h->dix.winner, 0, h->total_leaves * 8, s));
-#endif
-            h->epoch = 1;
-        }
+    {
         const uint64_t epoch_hi = uint64_t(h->epoch) << 32;
         const int grid = grid_for(h, m);
         const size_t kstride = kind == CUART_KEY_U64 ? 8 : kind == CUART_KEY_U32 ? 4 : 32;
@@ -675,7 +614,7 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
         const uint64_t* vb = vals ? vals + base : nullptr;
         const uint8_t* db = (mode == 1) ? is_delete + base : nullptr;
         const uint32_t* ib = opidx ? opidx + base : nullptr;
-#define CUART_UPD1(K, P, D) k_upd1<K, P, D><<<grid, 256, 0, s>>>(dx, kb, lb, vb, db, m, epoch_hi, h->leafref, h->slotref, ib)
+#define CUART_UPD1(K, P, D) k_upd1<K, P, D><<<grid, 256, 0, s>>>(dx, kb, lb, vb, db, m, epoch_hi, leafref, slotref, ib)
 #define CUART_UPD1_POL(K)                                    \
     if (h->policy == 0) {                                    \
         if (del) CUART_UPD1(K, 0, true); else CUART_UPD1(K, 0, false); \
@@ -685,8 +624,8 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
         const bool wq = !del && bucketed && dx.walk_wide && h->policy == 5 && h->ilp > 1 &&
                         (kind == CUART_KEY_U64 || kind == CUART_KEY_U32);
         const unsigned gq = unsigned((m + 128 - 1) / 128);         // 64 threads x 2 ops per CTA
-        if (wq && kind == CUART_KEY_U64) k_upd1_wq<KeyU64, 2><<<gq, 64, 0, s>>>(dx, kb, vb, m, epoch_hi, h->leafref, ib);
-        else if (wq) k_upd1_wq<KeyU32, 2><<<gq, 64, 0, s>>>(dx, kb, vb, m, epoch_hi, h->leafref, ib);
+        if (wq && kind == CUART_KEY_U64) k_upd1_wq<KeyU64, 2><<<gq, 64, 0, s>>>(dx, kb, vb, m, epoch_hi, leafref, ib);
+        else if (wq) k_upd1_wq<KeyU32, 2><<<gq, 64, 0, s>>>(dx, kb, vb, m, epoch_hi, leafref, ib);
         else switch (kind) {
         case CUART_KEY_U64: CUART_UPD1_POL(KeyU64); break;
         case CUART_KEY_U32: CUART_UPD1_POL(KeyU32); break;
@@ -697,13 +636,37 @@ static cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, 
 #undef CUART_UPD1
         g_cuart_launches++;
         CU_TRY(cudaGetLastError());
-        if (del) k_upd2<true><<<grid, 256, 0, s>>>(dx, vb, db, m, epoch_hi, h->leafref, h->slotref, ib);
-        else if (h->upd2_tpb == 64) k_upd2<false, 64><<<unsigned((m + 63) / 64), 64, 0, s>>>(dx, vb, nullptr, m, epoch_hi, h->leafref, nullptr, ib);
-        else k_upd2<false><<<grid, 256, 0, s>>>(dx, vb, nullptr, m, epoch_hi, h->leafref, nullptr, ib);
+        if (del) k_upd2<true><<<grid, 256, 0, s>>>(dx, vb, db, m, epoch_hi, leafref, slotref, ib);
+        else if (h->upd2_tpb == 64) k_upd2<false, 64><<<unsigned((m + 63) / 64), 64, 0, s>>>(dx, vb, nullptr, m, epoch_hi, leafref, nullptr, ib);
+        else k_upd2<false><<<grid, 256, 0, s>>>(dx, vb, nullptr, m, epoch_hi, leafref, nullptr, ib);
         g_cuart_launches++;
         CU_TRY(cudaGetLastError());
     }
     return CUART_OK;
+}
+
+// mode: 0 = updates only, 1 = mixed (is_delete[i]), 2 = all deletes (vals unused).
+// opidx: original op index of each op (pre-bucketed batches), or nullptr (= position).
+cuart_status launch_update(cuart_index* h, uint32_t kind, const void* k, const uint8_t* lens,
+                           const uint64_t* vals, const uint8_t* is_delete, int mode, uint64_t n,
+                           cudaStream_t s, const uint32_t* opidx, bool bucketed, uint64_t* keep_leafref) {
+    const bool del = mode != 0;
+    const DevIndex& dx = bucketed ? h->dix_links : h->dix;
+    const uint64_t cap = n < kUpdateChunk ? n : kUpdateChunk;
+    uint64_t* leafref = keep_leafref;
+    uint64_t* slotref = nullptr;
+    cuart_status rc = CUART_OK;
+    if (!leafref) rc = scratch_alloc(h, (void**)&leafref, cap * 8, s);
+    if (rc == CUART_OK && del) rc = scratch_alloc(h, (void**)&slotref, cap * 8, s);
+    for (uint64_t base = 0; base < n && rc == CUART_OK; base += kUpdateChunk) {
+        const uint64_t m = (n - base) < kUpdateChunk ? (n - base) : kUpdateChunk;
+        if (!h->hold_epoch && (rc = next_epoch(h, s)) != CUART_OK) break;
+        rc = update_chunk(h, dx, kind, k, lens, vals, is_delete, mode, base, m, s, opidx, bucketed,
+                          keep_leafref ? keep_leafref + base : leafref, slotref);
+    }
+    if (!keep_leafref) scratch_free(h, leafref, s);
+    scratch_free(h, slotref, s);
+    return rc;
 }
 
 // Pre-bucketed update batch (a5 applied to stage 1/2): ops are reordered by bucket
@@ -719,28 +682,29 @@ static cuart_status launch_update_bucketed(cuart_index* h, const void* k, const 
     const size_t o_hist = 0, o_tot = al(hist_entries(tiles) * 4), o_q = o_tot + 1024, o_len = o_q + al(n * ks),
                  o_val = o_len + al(Key::kKind == 3 ? n : 0), o_idx = o_val + al(n * 8), total = o_idx + al(n * 4);
     uint8_t* scr = nullptr;
-    CU_TRY(cudaMallocAsync((void**)&scr, total, s));
+    cuart_status rc = scratch_alloc(h, (void**)&scr, total, s);
+    if (rc != CUART_OK) return rc;
     unsigned int* hist = (unsigned int*)(scr + o_hist);
     unsigned int* tot = (unsigned int*)(scr + o_tot);
     const uint32_t depth = (link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u) |
                            (h->bucket_shift << 8);
-    if ((uintptr_t(k) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
-    else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, depth, hist);
+    if ((uintptr_t(k) & 15) == 0) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, ByteBucket(depth), hist);
+    else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, ByteBucket(depth), hist);
     k_bscan_rows<<<kBuckets >> h->bucket_shift, kBucketThreads, 0, s>>>(hist, tiles, tot);   // rows in use only
     k_bscan<<<1, kBuckets, 0, s>>>(tot, kBuckets >> h->bucket_shift);
     k_bscatter<Key, true><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key, true>(), s>>>(
-        k, lens, n, depth, hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, nullptr, vals,
+        k, lens, n, ByteBucket(depth), hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, nullptr, vals,
         (uint64_t*)(scr + o_val), (uint32_t*)(scr + o_idx));
     g_cuart_launches += 4;
-    CU_TRY(cudaGetLastError());
-    cuart_status rc = launch_update(h, Key::kKind, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr,
-                                    (const uint64_t*)(scr + o_val), nullptr, 0, n, s, (const uint32_t*)(scr + o_idx), true);
-    if (rc != CUART_OK) return rc;
-    CU_TRY(cudaFreeAsync(scr, s));
-    return CUART_OK;
+    rc = cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+    if (rc == CUART_OK)
+        rc = launch_update(h, Key::kKind, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr,
+                           (const uint64_t*)(scr + o_val), nullptr, 0, n, s, (const uint32_t*)(scr + o_idx), true);
+    scratch_free(h, scr, s);
+    return rc;
 }
 
-static cuart_status dispatch_update(cuart_index* h, const void* k, const uint8_t* lens, const uint64_t* vals, uint64_t n,
+cuart_status dispatch_update(cuart_index* h, const void* k, const uint8_t* lens, const uint64_t* vals, uint64_t n,
                                     cudaStream_t s) {
     const bool bucket = h->prebucket == CUART_PREBUCKET_ON ? n >= kBucketTile
                       : h->prebucket == CUART_PREBUCKET_AUTO && n >= kBucketMin && h->key_kind != CUART_KEY_BYTES;
@@ -985,13 +949,6 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         return CUART_ERR_INVALID_ARGUMENT;
     }
     if (const char* pe = getenv("CUART_PREBUCKET")) h->prebucket = atoi(pe) ? CUART_PREBUCKET_ON : CUART_PREBUCKET_OFF;
-    {   // keep stream-ordered scratch mapped between calls (a5 bucketing)
-        cudaMemPool_t pool;
-        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-            uint64_t keep = ~uint64_t(0);
-            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
-        }
-    }
     cudaFuncSetAttribute(k_bscatter<KeyU64>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bscatter_smem<KeyU64>()));
     cudaFuncSetAttribute(k_bscatter<KeyU32>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bscatter_smem<KeyU32>()));
     cudaFuncSetAttribute(k_bscatter<KeyBytes>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1163,6 +1120,22 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         h->dix_links.lut32 = nullptr;
         h->dix_links.walk_wide = h->wide ? 1u : 0u;
     }
+    {   // the index's own pool for stream-ordered scratch: it keeps its memory mapped
+        // between calls (no re-mapping per batch) and is destroyed with the index, so
+        // other allocators (PyTorch's caching allocator, the device default pool) never
+        // see memory held on the index's behalf
+        cudaMemPoolProps pp = {};
+        pp.allocType = cudaMemAllocationTypePinned;
+        pp.location.type = cudaMemLocationTypeDevice;
+        pp.location.id = dev;
+        if (cudaMemPoolCreate(&h->pool, &pp) == cudaSuccess) {
+            uint64_t keep = ~uint64_t(0);
+            cudaMemPoolSetAttribute(h->pool, cudaMemPoolAttrReleaseThreshold, &keep);
+        } else {
+            cudaGetLastError();
+            h->pool = nullptr;
+        }
+    }
     *out = h;
     return CUART_OK;
 }
@@ -1184,10 +1157,9 @@ cuart_status cuart_build(const cuart_keys* keys, const uint64_t* values, size_t 
 cuart_status cuart_destroy(cuart_index* h) {
     if (!h) return CUART_OK;
     cudaSetDevice(h->device);
+    if (h->dist) dist_teardown(h);        // collective: every rank of the group destroys together
     cudaDeviceSynchronize();
     cudaFree(h->arena);
-    if (h->leafref) cudaFree(h->leafref);
-    if (h->slotref) cudaFree(h->slotref);
     drop_kevents(h);
     for (int i = 0; i < kStages; i++) {
         if (h->stage[i]) cudaFree(h->stage[i]);
@@ -1198,6 +1170,8 @@ cuart_status cuart_destroy(cuart_index* h) {
         if (h->ev_copied[i]) cudaEventDestroy(h->ev_copied[i]);
         if (h->ev_free[i]) cudaEventDestroy(h->ev_free[i]);
     }
+    if (h->ustream) cudaStreamDestroy(h->ustream);
+    if (h->pool) cudaMemPoolDestroy(h->pool);   // every scratch block was freed in stream order
     delete h;
     return CUART_OK;
 }
@@ -1300,17 +1274,21 @@ cuart_status cuart_update_long(cuart_index* h, const uint8_t* data, const uint64
     uint64_t* doff = nullptr;
     if ((rc = upload_long_batch(data, offsets, n, s, &dq, &doff)) != CUART_OK) return rc;
     uint64_t* dval = nullptr;
+    uint64_t* dref = nullptr;
     CU_TRY(cudaMallocAsync((void**)&dval, n * 8, s));
+    CU_TRY(cudaMallocAsync((void**)&dref, n * 8, s));
     CU_TRY(cudaMemcpyAsync(dval, values, n * 8, cudaMemcpyHostToDevice, s));
-    // device leaves: the two-stage kernels; host leaves: stage 1 leaves their links in leafref
-    rc = launch_update(h, CUART_KEY_LONG, dq, (const uint8_t*)doff, dval, nullptr, 0, n, s);
-    if (rc != CUART_OK) return rc;
+    // device leaves: the two-stage kernels; host leaves: stage 1 leaves their links in dref
+    rc = launch_update(h, CUART_KEY_LONG, dq, (const uint8_t*)doff, dval, nullptr, 0, n, s, nullptr, false, dref);
     std::vector<uint64_t> ref(n);
-    CU_TRY(cudaMemcpyAsync(ref.data(), h->leafref, n * 8, cudaMemcpyDeviceToHost, s));
-    CU_TRY(cudaFreeAsync(dq, s));
-    CU_TRY(cudaFreeAsync(doff, s));
-    CU_TRY(cudaFreeAsync(dval, s));
+    if (rc == CUART_OK && cudaMemcpyAsync(ref.data(), dref, n * 8, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+        rc = CUART_ERR_CUDA;
+    cudaFreeAsync(dq, s);
+    cudaFreeAsync(doff, s);
+    cudaFreeAsync(dval, s);
+    cudaFreeAsync(dref, s);
     CU_TRY(cudaStreamSynchronize(s));
+    if (rc != CUART_OK) return rc;
     // host leaves in op order: sequential semantics, the last op on a key wins
     for (size_t i = 0; i < n; i++) {
         const uint64_t l = ref[i];
@@ -1319,23 +1297,6 @@ cuart_status cuart_update_long(cuart_index* h, const uint8_t* data, const uint64
         if (long_key_equal(h, idx, data + offsets[i], offsets[i + 1] - offsets[i])) h->long_vals[idx] = values[i];
     }
     return CUART_OK;
-}
-
-cuart_status cuart_lookup_segmented(const cuart_index* h, const cuart_keys* q, size_t n, uint32_t nseg,
-                                    const uint64_t* seg_start, uint64_t* const* seg_dst, void* stream) {
-    cuart_status rc = check_keys(h, q, n);
-    if (rc != CUART_OK) return rc;
-    if (n == 0) return CUART_OK;
-    if (nseg == 0 || nseg > uint32_t(kMaxSeg) || !seg_start || !seg_dst) return CUART_ERR_INVALID_ARGUMENT;
-    SegOut so{};
-    so.nseg = nseg;
-    for (uint32_t i = 0; i <= nseg; i++) so.start[i] = seg_start[i];
-    for (uint32_t i = 0; i < nseg; i++) {
-        so.dst[i] = seg_dst[i];
-        if (so.start[i] > so.start[i + 1] || (so.start[i + 1] > so.start[i] && !so.dst[i])) return CUART_ERR_INVALID_ARGUMENT;
-    }
-    if (so.start[0] != 0 || so.start[nseg] != n) return CUART_ERR_INVALID_ARGUMENT;
-    return launch_lookup(h, h->key_kind, q->data, q->lengths, n, nullptr, (cudaStream_t)stream, &so);
 }
 
 cuart_status cuart_lookup(const cuart_index* h, const cuart_keys* q, size_t n, uint64_t* out, void* stream) {
@@ -1535,7 +1496,7 @@ cuart_status cuart_stats(const cuart_index* h, cuart_stats_t* s) {
     s->lut_format = h->lut_format;
     s->lut_exceptions = h->lut_exceptions;
     s->wide_lut = h->wide ? 1u : 0u;
-    s->arena_bytes = h->arena_bytes + h->leafref_cap * 8;
+    s->arena_bytes = h->arena_bytes;
     s->key_kind = h->key_kind;
     s->root = h->root;
     s->max_depth = h->max_depth;

@@ -12,13 +12,9 @@
 //   k_route_scatter: stable per-owner placement via warp ballots; perm[i] = slot
 //   k_unroute      : out[i] = results[perm[i]]
 //
-// Fused variant (transport "p2p"): K-ROUTE's stable scatter stores every op
-// straight into its owner's receive window on the owner GPU (CUDA IPC mappings
-// over NVLink/NVSwitch), so the partition and the all-to-all are ONE kernel; the
-// owner's lookup writes each result straight into the requester's result window
-// (cuart_lookup_segmented), so the return all-to-all is fused into the lookup's
-// last kernel.  Only the P x P count matrix travels through the collective
-// library.
+// The multi-GPU layer proper (cuart_dist_*, csrc/dist.cu) fuses routing into the
+// K-BUCKET pass; these standalone kernels remain the general partition primitive
+// (cuart_partition_by_flag splits config 5's mixed rounds, reading C7).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -125,16 +121,6 @@ __global__ void __launch_bounds__(1024) k_route_scan(uint32_t* __restrict__ hist
     }
 }
 
-// Per-owner destinations of the fused push: owner o's receive window, already
-// advanced to this source's first slot there.
-constexpr uint32_t kMaxPeers = 16;
-struct PeerDst {
-    void* keys[kMaxPeers];
-    uint8_t* lens[kMaxPeers];
-    uint64_t* vals[kMaxPeers];
-};
-
-template <bool PUSH>
 __global__ void __launch_bounds__(kRouteThreads) k_route_scatter(uint32_t kind, const void* __restrict__ keys,
                                                                  const uint8_t* __restrict__ lens,
                                                                  const uint64_t* __restrict__ values, uint64_t n,
@@ -142,15 +128,13 @@ __global__ void __launch_bounds__(kRouteThreads) k_route_scatter(uint32_t kind, 
                                                                  const uint32_t* __restrict__ offsets,
                                                                  void* __restrict__ send_keys, uint8_t* __restrict__ send_lens,
                                                                  uint64_t* __restrict__ send_values,
-                                                                 uint32_t* __restrict__ perm, PeerDst pd = PeerDst{}) {
+                                                                 uint32_t* __restrict__ perm) {
     constexpr int kWarps = kRouteThreads / 32;
     __shared__ uint32_t run[kMaxParts];             // placed so far in this block, per owner
-    __shared__ uint32_t ostart[kMaxParts];          // PUSH: first send-order slot of each owner
     __shared__ uint32_t wcnt[kWarps][kMaxParts];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     for (uint32_t o = threadIdx.x; o < nparts; o += blockDim.x) {
         run[o] = offsets[uint64_t(o) * gridDim.x + blockIdx.x];
-        if (PUSH) ostart[o] = offsets[uint64_t(o) * gridDim.x];
     }
     __syncthreads();
     const uint64_t base = uint64_t(blockIdx.x) * kRouteChunk;
@@ -172,9 +156,8 @@ __global__ void __launch_bounds__(kRouteThreads) k_route_scatter(uint32_t kind, 
             for (int w = 0; w < warp; w++) before += wcnt[w][o];
             const uint32_t slot = run[o] + before + rank;
             perm[i] = slot;
-            // PUSH: the owner's window (peer memory) at this source's base + position in the owner's run
-            const uint64_t dst = PUSH ? uint64_t(slot - ostart[o]) : uint64_t(slot);
-            void* kd = PUSH ? pd.keys[o] : send_keys;
+            const uint64_t dst = uint64_t(slot);
+            void* kd = send_keys;
             if (kind == CUART_KEY_U64) ((uint64_t*)kd)[dst] = ((const uint64_t*)keys)[i];
             else if (kind == CUART_KEY_U32) ((uint32_t*)kd)[dst] = ((const uint32_t*)keys)[i];
             else {
@@ -182,9 +165,9 @@ __global__ void __launch_bounds__(kRouteThreads) k_route_scatter(uint32_t kind, 
                 uint4* d = (uint4*)kd + 2 * dst;
                 d[0] = s[0];
                 d[1] = s[1];
-                (PUSH ? pd.lens[o] : send_lens)[dst] = lens[i];
+                send_lens[dst] = lens[i];
             }
-            if (values) (PUSH ? pd.vals[o] : send_values)[dst] = values[i];
+            if (values) send_values[dst] = values[i];
         }
         __syncthreads();
         for (uint32_t oo = threadIdx.x; oo < nparts; oo += blockDim.x) {
@@ -253,89 +236,17 @@ static cuart_status route_impl(const cuart_keys* keys, size_t n, const uint64_t*
     k_route_hist<<<unsigned(nblocks), kRouteThreads, 0, s>>>(kind, keys->data, keys->lengths, n, splitters, nparts,
                                                              flags, owner, hist);
     k_route_scan<<<1, 1024, 0, s>>>(hist, nblocks, nparts, counts);
-    k_route_scatter<false><<<unsigned(nblocks), kRouteThreads, 0, s>>>(kind, keys->data, keys->lengths, values, n,
+    k_route_scatter<<<unsigned(nblocks), kRouteThreads, 0, s>>>(kind, keys->data, keys->lengths, values, n,
                                                                        nparts, owner, hist, send_keys, send_lengths,
                                                                        send_values, perm);
     g_cuart_launches += 3;
     return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
 }
 
-// ---------------------------------------------------------------- fused p2p route
-cuart_status cuart_route_count(const cuart_keys* keys, size_t n, const uint64_t* splitters, uint32_t nparts,
-                               uint64_t* counts, void* scratch, void* stream) {
-    if (!keys || nparts == 0 || nparts > kMaxPeers || !counts) return CUART_ERR_INVALID_ARGUMENT;
-    if (nparts > 1 && !splitters) return CUART_ERR_INVALID_ARGUMENT;
-    if (n >= (uint64_t(1) << 32)) return CUART_ERR_INVALID_ARGUMENT;
-    cudaStream_t s = (cudaStream_t)stream;
-    if (n == 0) return cudaMemsetAsync(counts, 0, nparts * sizeof(uint64_t), s) == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
-    if (!keys->data || !scratch || (keys->kind == CUART_KEY_BYTES && !keys->lengths)) return CUART_ERR_INVALID_ARGUMENT;
-    const uint64_t nblocks = (n + kRouteChunk - 1) / kRouteChunk;
-    uint8_t* owner = (uint8_t*)scratch;
-    uint32_t* hist = (uint32_t*)((uint8_t*)scratch + ((n + 255) & ~size_t(255)));
-    k_route_hist<<<unsigned(nblocks), kRouteThreads, 0, s>>>(uint32_t(keys->kind), keys->data, keys->lengths, n,
-                                                             splitters, nparts, nullptr, owner, hist);
-    k_route_scan<<<1, 1024, 0, s>>>(hist, nblocks, nparts, counts);
-    g_cuart_launches += 2;
-    return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
-}
-
-cuart_status cuart_route_push(const cuart_keys* keys, size_t n, uint32_t nparts, const uint64_t* values,
-                              void* const* dst_keys, uint8_t* const* dst_lengths, uint64_t* const* dst_values,
-                              uint32_t* perm, void* scratch, void* stream) {
-    if (!keys || nparts == 0 || nparts > kMaxPeers || !dst_keys) return CUART_ERR_INVALID_ARGUMENT;
+cuart_status cuart_fill_miss(uint64_t* out, size_t n, void* stream) {
     if (n == 0) return CUART_OK;
-    if (n >= (uint64_t(1) << 32) || !keys->data || !perm || !scratch) return CUART_ERR_INVALID_ARGUMENT;
-    if (keys->kind == CUART_KEY_BYTES && (!keys->lengths || !dst_lengths)) return CUART_ERR_INVALID_ARGUMENT;
-    if (values && !dst_values) return CUART_ERR_INVALID_ARGUMENT;
-    PeerDst pd{};
-    for (uint32_t o = 0; o < nparts; o++) {
-        pd.keys[o] = dst_keys[o];
-        pd.lens[o] = dst_lengths ? dst_lengths[o] : nullptr;
-        pd.vals[o] = dst_values ? dst_values[o] : nullptr;
-    }
-    const uint64_t nblocks = (n + kRouteChunk - 1) / kRouteChunk;
-    const uint8_t* owner = (const uint8_t*)scratch;
-    const uint32_t* hist = (const uint32_t*)((const uint8_t*)scratch + ((n + 255) & ~size_t(255)));
-    k_route_scatter<true><<<unsigned(nblocks), kRouteThreads, 0, (cudaStream_t)stream>>>(
-        uint32_t(keys->kind), keys->data, keys->lengths, values, n, nparts, owner, hist, nullptr, nullptr, nullptr, perm,
-        pd);
-    g_cuart_launches += 1;
-    return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
-}
-
-// ---------------------------------------------------------------- peer windows (CUDA IPC)
-static_assert(sizeof(cudaIpcMemHandle_t) <= CUART_IPC_HANDLE_BYTES, "handle size");
-
-cuart_status cuart_ipc_alloc(size_t bytes, void** dptr) {
-    if (!dptr || bytes == 0) return CUART_ERR_INVALID_ARGUMENT;
-    const cudaError_t e = cudaMalloc(dptr, bytes);
-    return e == cudaSuccess ? CUART_OK : e == cudaErrorMemoryAllocation ? CUART_ERR_OOM : CUART_ERR_CUDA;
-}
-
-cuart_status cuart_ipc_free(void* dptr) {
-    if (!dptr) return CUART_OK;
-    return cudaFree(dptr) == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
-}
-
-cuart_status cuart_ipc_export(void* dptr, void* handle) {
-    if (!dptr || !handle) return CUART_ERR_INVALID_ARGUMENT;
-    cudaIpcMemHandle_t hd;
-    if (cudaIpcGetMemHandle(&hd, dptr) != cudaSuccess) return CUART_ERR_CUDA;
-    memset(handle, 0, CUART_IPC_HANDLE_BYTES);
-    memcpy(handle, &hd, sizeof(hd));
-    return CUART_OK;
-}
-
-cuart_status cuart_ipc_import(const void* handle, void** dptr) {
-    if (!handle || !dptr) return CUART_ERR_INVALID_ARGUMENT;
-    cudaIpcMemHandle_t hd;
-    memcpy(&hd, handle, sizeof(hd));
-    return cudaIpcOpenMemHandle(dptr, hd, cudaIpcMemLazyEnablePeerAccess) == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
-}
-
-cuart_status cuart_ipc_close(void* dptr) {
-    if (!dptr) return CUART_OK;
-    return cudaIpcCloseMemHandle(dptr) == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+    if (!out) return CUART_ERR_INVALID_ARGUMENT;
+    return cudaMemsetAsync(out, 0xFF, n * 8, (cudaStream_t)stream) == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
 }
 
 cuart_status cuart_unroute(const uint64_t* in, const uint32_t* perm, size_t n, uint64_t* out, void* stream) {

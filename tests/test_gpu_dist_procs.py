@@ -1,12 +1,13 @@
-"""The complete multi-GPU path with the CuART kernels — CudaOps (cuart_route,
-cuart_unroute, cuart_partition_by_flag, local lookups/updates) + the DistIndex
-protocol — run as 2 processes sharing cuda:0 (gloo, host-staged collectives;
-NCCL refuses duplicate devices).  Range and replica modes, lookups, updates and
-mixed rounds; results equal the single-index oracle.  "range-p2p" runs the fused
-transport: each process maps the other's receive windows through CUDA IPC (same
-device here, NVLink peers on a multi-GPU box), cuart_route_push stores ops into
-the owner's window and cuart_lookup_segmented returns results into the
-requester's window."""
+"""The complete multi-GPU path (cuart_dist_build / _lookup / _update, transport
+P2P) as 2 processes sharing cuda:0: the library's host bootstrap runs over
+torch.distributed (gloo) through the callback in cfg; each process maps the
+other's receive windows and control block with CUDA IPC (same device here,
+NVLink peers on a multi-GPU box); the fused scatter stores ops into the owner's
+window, the owner's walk stores results into the requester's window, and the
+ranks order each other with device-side flags.  (NCCL refuses two ranks on one
+device, so transport NCCL runs at one rank, tests/test_gpu_dist.py.)  Range and
+replica modes, lookups, updates and mixed rounds; results equal the single-index
+oracle."""
 import os
 import socket
 import tempfile
@@ -32,10 +33,8 @@ def _port():
 
 
 def _worker(rank, world, port, mode, outdir):
-    transport = "p2p" if mode.endswith("-p2p") else "nccl"
-    mode = mode.split("-")[0]
     import workloads as W
-    from paper_conf_icpp_koppehelggp21_b200.dist import CudaOps, DistIndex
+    from paper_conf_icpp_koppehelggp21_b200.dist import DistIndex
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -43,12 +42,13 @@ def _worker(rank, world, port, mode, outdir):
     cfg = W.Config("cX", "u64", N_KEYS, N_Q, N_U, 0.5, "")
     keys = W.u64_keys(3, N_KEYS)
     vals = W.values_for(W.SEED_VALUES + 3, np.arange(N_KEYS, dtype=np.uint64))
-    di = DistIndex(keys, vals, mode=mode, ops=CudaOps(dev), transport=transport)
+    torch.cuda.set_device(dev)
+    di = DistIndex(keys, vals, mode=mode, transport="p2p", chunk=1 << 18)
     kd = torch.from_numpy(keys.view(np.int64)).to(dev)
     q = W.lookup_batch_torch(W.CONFIGS["c3"], kd, rank * N_Q, N_Q, device=dev)
     r1 = di.lookup(q)
     uk, uv = W.update_batch_torch(W.CONFIGS["c3"], kd, rank * N_U, N_U)
-    di.update((uk, uv))
+    di.update(uk, uv)
     r2 = di.lookup(kd)
     per = ROUND // world
     k, u, v = W.mixed_ops_torch(5, N_KEYS, rank * per, per, dev)
@@ -62,7 +62,7 @@ def _worker(rank, world, port, mode, outdir):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("mode", ["range", "replica", "range-p2p"])
+@pytest.mark.parametrize("mode", ["range", "replica"])
 def test_two_processes_one_gpu(mode):
     import workloads as W
     world = 2

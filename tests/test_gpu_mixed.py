@@ -1,5 +1,6 @@
 """Config-5 semantics on one GPU: mixed lookup/update rounds (reading C7) through
-DistIndex + CudaOps (world size 1), against the oracle replay."""
+the multi-GPU layer at world size 1 (cuart_dist_* with both transports), against
+the oracle replay."""
 import os
 
 import numpy as np
@@ -23,12 +24,13 @@ def pg():
     dist.destroy_process_group()
 
 
-def test_mixed_rounds_single_gpu(pg):
-    from paper_conf_icpp_koppehelggp21_b200.dist import CudaOps, DistIndex
+@pytest.mark.parametrize("transport", ["p2p", "nccl"])
+def test_mixed_rounds_single_gpu(pg, transport):
+    from paper_conf_icpp_koppehelggp21_b200.dist import DistIndex
     n, R, rounds = 1 << 18, 1 << 20, 4
     keys = W.u64_keys(5, n)
     vals = W.values_for(W.SEED_VALUES + 5, np.arange(n, dtype=np.uint64))
-    di = DistIndex(keys, vals, mode="range", ops=CudaOps(DEV))
+    di = DistIndex(keys, vals, mode="range", transport=transport)
     o = MapOracle(keys, vals)
     for r in range(rounds):
         k, u, v = W.mixed_ops_torch(5, n, r * R, R, DEV)
