@@ -27,6 +27,8 @@
 // highest priority wins per key across chunks.
 #include <cuda_runtime.h>
 #include <nccl.h>
+#include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 #include <unistd.h>
 
@@ -42,6 +44,20 @@
 using namespace cuart;
 
 namespace {
+
+// CUART_DIST_DEBUG=1: trace the host steps of the protocol to stderr
+bool dbg_on() {
+    static const bool on = getenv("CUART_DIST_DEBUG") != nullptr;
+    return on;
+}
+#define DBG(...)                                  \
+    do {                                          \
+        if (dbg_on()) {                           \
+            fprintf(stderr, "[cuart_dist] " __VA_ARGS__); \
+            fputc('\n', stderr);                 \
+            fflush(stderr);                       \
+        }                                         \
+    } while (0)
 
 constexpr uint32_t kMaxRanks = kMaxSeg;            // 16
 enum { F_CNT = 0, F_PUSH = 1, F_RES = 2 };
@@ -630,6 +646,7 @@ cuart_status back(cuart_index* h, DistState* d, const Call& c, uint64_t ci, unsi
 
 template <class Key>
 cuart_status run_call(cuart_index* h, DistState* d, const Call& c) {
+    DBG("rank %d call %s n %llu", d->rank, c.update ? "update" : "lookup", (unsigned long long)c.n);
     // agree on the number of chunks: every rank publishes its n (one small round)
     const unsigned long long seq0 = ++d->seq;
     const uint32_t P = d->P;
@@ -685,6 +702,7 @@ cuart_status run_call(cuart_index* h, DistState* d, const Call& c) {
             if (rc != CUART_OK) break;
             const uint32_t slot = uint32_t(ci & 1);
             rc = host_wait_matrix(d, slot, base + 1 + ci);
+            DBG("rank %d chunk %llu matrix rc %d", d->rank, (unsigned long long)ci, int(rc));
             if (rc != CUART_OK) break;
             rc = owner(h, d, c, ci, base + 1 + ci, d->hmat + slot * (size_t(P) * P + 1));
             if (rc == CUART_OK) rc = back(h, d, c, ci, base + 1 + ci);
@@ -903,6 +921,7 @@ cuart_status cuart_dist_build(const cuart_dist_cfg* cfg, const cuart_keys* keys,
     if (dev >= ndev) return CUART_ERR_NO_DEVICE;
     if (cudaSetDevice(dev) != cudaSuccess) return CUART_ERR_CUDA;
     const uint32_t P = uint32_t(cfg->nranks), kind = uint32_t(keys->kind);
+    DBG("build rank %d/%u mode %u transport %u n %zu dev %d", cfg->rank, P, cfg->mode, cfg->transport, n, dev);
     DistState* d = new (std::nothrow) DistState();
     if (!d) return CUART_ERR_OOM;
     d->rank = cfg->rank;
@@ -971,6 +990,7 @@ cuart_status cuart_dist_build(const cuart_dist_cfg* cfg, const cuart_keys* keys,
             kn = sel_v.size();
         }
     }
+    DBG("local keys %zu", kn);
     cuart_keys lk{keys->kind, kd, kl};
     cuart_build_opts opts = cfg->opts;
     opts.device = dev;
@@ -980,6 +1000,7 @@ cuart_status cuart_dist_build(const cuart_dist_cfg* cfg, const cuart_keys* keys,
         free_state(d);
         return rc;
     }
+    DBG("local index built");
     h->dist = d;
     for (uint32_t j = 0; j + 1 < P; j++) d->part.sp[j] = sp[j];
     d->part.nsp = cfg->mode == CUART_DIST_RANGE ? P - 1 : 0;
@@ -1002,6 +1023,7 @@ cuart_status cuart_dist_build(const cuart_dist_cfg* cfg, const cuart_keys* keys,
     while (uint64_t(P) * C >= (uint64_t(1) << 31)) C /= 2;
     d->chunk = C;
     d->wcap = uint64_t(P) * C;
+    DBG("chunk %llu window %llu", (unsigned long long)C, (unsigned long long)d->wcap);
     set_scatter_smem<KeyU64, false>();
     set_scatter_smem<KeyU64, true>();
     set_scatter_smem<KeyU32, false>();
@@ -1009,6 +1031,7 @@ cuart_status cuart_dist_build(const cuart_dist_cfg* cfg, const cuart_keys* keys,
     set_scatter_smem<KeyBytes, false>();
     set_scatter_smem<KeyBytes, true>();
     rc = setup_buffers(h, d);
+    DBG("buffers rc %d", int(rc));
     if (rc != CUART_OK) {
         h->dist = nullptr;
         free_state(d);

@@ -210,7 +210,7 @@ class DistIndex:
         else:
             self.splitters = np.zeros(0, np.uint64)
         h = ctypes.c_void_p()
-        B._check(lib().cuart_dist_build(ctypes.byref(c), ctypes.byref(k), n, v.ctypes.data, ctypes.byref(h)),
+        B._check(lib().cuart_dist_build(ctypes.byref(c), ctypes.byref(k), v.ctypes.data, n, ctypes.byref(h)),
                  "cuart_dist_build")
         self.h = h.value
         self.index = B.Index.__new__(B.Index)       # the local part (stats, dump, timers)

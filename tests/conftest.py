@@ -4,6 +4,12 @@ import sys
 import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+# tests/test_gpu_dist.py runs up to 8 virtual ranks in ONE process, each with a user
+# stream and the library's two internal streams, whose device-side waits depend on
+# each other's kernels: every stream needs its own hardware queue (the default of 8
+# would let one rank's waiting kernel block another rank's producer queued behind it).
+# One process per GPU (the production shape) uses 3 streams.  Set before CUDA init.
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
 

@@ -97,9 +97,12 @@ def _run(P, fn):
     return res
 
 
-@pytest.mark.parametrize("transport,P", [("p2p", 1), ("p2p", 2), ("p2p", 3), ("p2p", 8), ("nccl", 1)])
-@pytest.mark.parametrize("mode", ["range", "replica"])
-@pytest.mark.parametrize("kind", ["u64", "u32", "bytes"])
+CASES = [(k, m, t, p) for k in ("u64", "u32", "bytes") for m in ("range", "replica")
+         for t, p in (("p2p", 1), ("p2p", 2), ("p2p", 3), ("nccl", 1))] + \
+        [("u64", "range", "p2p", 8), ("u64", "replica", "p2p", 8), ("bytes", "range", "p2p", 4)]
+
+
+@pytest.mark.parametrize("kind,mode,transport,P", CASES)
 def test_dist_virtual_ranks(kind, mode, transport, P):
     n = 40_000
     keys = _keyset(kind, n)
