@@ -63,6 +63,8 @@ def _args():
     p.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
                    help="range mode exchange: p2p = fused push/return over peer memory (CUDA IPC, NVLink), "
                         "nccl = route + all-to-all")
+    p.add_argument("--c5-share", type=int, default=0,
+                   help="c5 on one GPU: the per-GPU share of a P-GPU run (rank 0's keys and owned ops)")
     p.add_argument("--traffic", type=float, default=None,
                    help="ncu dram__bytes_read+write per k_lookup launch (GB), from profiles/, echoed into roofline")
     return p.parse_args()
@@ -246,12 +248,25 @@ def hbm_peak():
     return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-C5_STREAM_BYTES = 8 + (8 + 8 + 2) + (8 + 8) + (8 + 2 + 8)   # bhist, bscatter, walk I/O, bgather (u64)
+def tree_bytes_touched(stats, hits):
+    """Estimated compulsory DRAM bytes of the tree a batch reads once: every inner
+    node (a uniform batch of this size reaches all of them) plus the leaves the hits
+    touch (1 - exp(-hits / leaves) of them: uniform picks with replacement)."""
+    inner = sum(stats[t + "_bytes"] for t in ("n4", "n16", "n48", "n256"))
+    leaves = stats["leaf8"] + stats["leaf16"] + stats["leaf32"]
+    leaf_b = sum(stats[t + "_bytes"] for t in ("leaf8", "leaf16", "leaf32"))
+    frac = 1.0 - float(np.exp(-hits / max(1, leaves)))
+    return inner + leaf_b * frac, frac
 
 
 def run_c5(args, world, rank, local, dev):
     """A step = one round of the mixed stream: this rank's 1/P slice of 2^29 global ops
-    (strong scaling: the round is fixed), lookups then updates (reading C7)."""
+    (strong scaling: the round is fixed), lookups then updates (reading C7).
+
+    --c5-share P (one GPU): the per-GPU share of a P-GPU run -- rank 0's key range
+    (byte0 in [0, 256/P): 2^30 / P keys) and the round's ops that rank 0 owns (~2^29/P),
+    served by the same multi-GPU layer at one rank (no exchange: the local part of
+    what every GPU of the P-GPU run does per round)."""
     import torch
     import torch.distributed as dist
 
@@ -259,31 +274,38 @@ def run_c5(args, world, rank, local, dev):
     from paper_conf_icpp_koppehelggp21_b200.dist import DistIndex
     if world & (world - 1):
         raise SystemExit("c5 needs a power-of-two GPU count")
+    share = args.c5_share if world == 1 else 0
+    if share and share & (share - 1):
+        raise SystemExit("--c5-share needs a power of two")
     t0 = time.perf_counter()
-    keys, vals, sp = c5_local_keys(world, rank, dev)
-    di = DistIndex(keys, vals, mode="range", transport=args.transport, lut_bytes=args.lut, splitters=sp,
-                   keys_local=True, rank=rank, world=world)
+    keys, vals, sp = c5_local_keys(share or world, rank, dev)
+    di = DistIndex(keys, vals, mode="range", transport=args.transport, lut_bytes=args.lut,
+                   splitters=sp if world > 1 else None, keys_local=world > 1, rank=rank, world=world)
     build_s = time.perf_counter() - t0
     stats = di.index.stats()
     R, per = W.C5_ROUND, W.C5_ROUND // world
-    rounds = [W.mixed_ops_torch(5, W.C5.n_keys, r * R + rank * per, per, dev) for r in range(2)]
+    rounds = []
+    for r in range(2):
+        k, u, v = W.mixed_ops_torch(5, W.C5.n_keys, r * R + rank * per, per, dev)
+        if share:                                   # rank 0's ops of the round (top log2(P) key bits = 0)
+            mine = W._t_srl(k, 64 - (share.bit_length() - 1)) == 0
+            k, u, v = k[mine].contiguous(), u[mine].contiguous(), v[mine].contiguous()
+        rounds.append((k, u, v))
     torch.cuda.synchronize()
     stream = torch.cuda.current_stream()
+    n_ops = int(sum(r[0].shape[0] for r in rounds) // 2)
+    n_look = int(sum(int((r[1] == 0).sum().item()) for r in rounds) // len(rounds))
 
     def step(i, ev=None):
         k, u, v = rounds[i % 2]
-        if ev is not None:
-            ev[0].record(stream)
-        di.mixed_round(k, v, u)
-        if ev is not None:
-            ev[1].record(stream)
+        di.mixed_round(k, v, u, events=ev)
 
     for i in range(args.warmup):
         step(i)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(args.steps)]
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.3)
@@ -303,35 +325,53 @@ def run_c5(args, world, rank, local, dev):
     if world > 1:
         dist.barrier()
     clk = clocks.stop()
-    tt = torch.tensor([t_start.elapsed_time(t_end), ktot / args.steps], dtype=torch.float64, device=dev)
+    phases = [float(np.mean([e[p].elapsed_time(e[p + 1]) for e in evs])) for p in range(4)]
+    tt = torch.tensor([t_start.elapsed_time(t_end), ktot / args.steps] + phases, dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-    total_ms, kern_ms = tt.tolist()
+    total_ms, kern_ms, part_ms, look_ms, upd_ms, unr_ms = tt.tolist()
     ms_step = total_ms / args.steps
-    value = R / (ms_step * 1e-3) / 1e6
-    n_look = int(sum(int((r[1] == 0).sum().item()) for r in rounds) // len(rounds))
+    value = (world * n_ops if share == 0 else n_ops) / (ms_step * 1e-3) / 1e6
     peak, peak_src = hbm_peak()
-    c5_achieved = C5_STREAM_BYTES * n_look / (kern_ms * 1e-3) / 1e9
+    served = kq / max(1, args.steps)                  # lookups this rank's owner walks served per step
+    tree_b, leaf_frac = tree_bytes_touched(stats, served * 0.5)
+    bpl = 16.0 + tree_b / max(1.0, served)            # key in + result out + the tree read once per round
+    achieved = bpl * served / (kern_ms * 1e-3) / 1e9
+    traffic = None
+    tfile = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tfile):
+        with open(tfile) as f:
+            traffic = json.load(f).get(f"c5{'_share' + str(share) if share else ''}/walk")
     if rank == 0:
         print(json.dumps({
             "metric": METRIC, "value": round(value, 3), "unit": "Mops/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True, "scaling": "strong",
+            "warmup": args.warmup, "ms_per_step": round(ms_step, 4), "higher_is_better": True,
+            "scaling": "strong" if not share else "share",
             "vs_baseline": None, "dtype": "u64",
             "data": "synthetic (seeded splitmix64, SURVEY §8(d) c5 recipe)",
-            "config": {"workload": f"c5: {W.C5.description}", "keys": W.C5.n_keys, "round_ops": R,
-                       "ops_per_rank_per_step": per, "update_fraction": W.C5_UPDATE_P, "mode": "range",
-                       "transport": args.transport if world > 1 else None,
-                       "parallelism": f"range{world}", "local_keys_rank0": int(keys.shape[0]),
-                       "build_s": round(build_s, 2), "lut_format": stats["lut_format"]},
-            "roofline": {"bound": "hbm", "achieved": round(c5_achieved, 1), "peak": peak, "unit": "GB/s",
-                         "frac": round(c5_achieved / peak, 4), "traffic": None,
-                         "kernel": "cuart_lookup (local, pre-bucketed: k_bhist .. k_lookup .. k_bgather)",
-                         "kernel_ms": round(kern_ms, 4), "lookups_per_launch": n_look,
-                         "bytes_per_lookup": C5_STREAM_BYTES,
-                         "bytes_model": "lower bound: the bucketed call's streaming key/result/permutation bytes "
-                                        "(8+18+16+18 B per u64 lookup); tree reads not counted",
-                         "peak_source": peak_src,
-                         "note": "per-rank local lookup call of a round; the c3 line carries the walk kernel's roofline"},
+            "config": {"workload": f"c5: {W.C5.description}" + (f" -- per-GPU share of a {share}-GPU run" if share else ""),
+                       "keys": W.C5.n_keys, "round_ops": R, "ops_per_rank_per_step": n_ops,
+                       "lookups_per_rank_per_step": n_look, "update_fraction": W.C5_UPDATE_P, "mode": "range",
+                       "transport": args.transport, "parallelism": f"range{world}" if not share else f"share-of-{share}",
+                       "local_keys_rank0": int(keys.shape[0]), "build_s": round(build_s, 2),
+                       "lut_format": stats["lut_format"], "tree_bytes": int(sum(stats[t + "_bytes"] for t in (
+                           "n4", "n16", "n48", "n256", "leaf8", "leaf16", "leaf32")))},
+            "phases_ms": {"partition_by_flag": round(part_ms, 4), "dist_lookup": round(look_ms, 4),
+                          "dist_update": round(upd_ms, 4), "unroute": round(unr_ms, 4)},
+            "lookup": {"mlookups_per_s": round(world * n_look / (look_ms * 1e-3) / 1e6, 3), "ms": round(look_ms, 4)},
+            "update": {"mupdates_per_s": round(world * (n_ops - n_look) / (upd_ms * 1e-3) / 1e6, 3),
+                       "ms": round(upd_ms, 4)},
+            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(achieved / peak, 4), "traffic": traffic,
+                         "kernel": ("k_lookup_wq<KeyU64>" if stats.get("wide_lut") else "k_lookup<KeyU64>")
+                         + " (owner walk of the multi-GPU layer, fused return)",
+                         "kernel_ms": round(kern_ms, 4), "lookups_per_step": int(served),
+                         "launches_per_step": round(klaunch / max(1, args.steps), 2),
+                         "bytes_per_lookup": round(bpl, 3),
+                         "bytes_model": "key in + result out (16 B) + the tree read once per round: every inner "
+                                        f"node + the touched fraction of the leaves ({leaf_frac:.3f} for "
+                                        f"{int(served * 0.5)} hits)",
+                         "peak_source": peak_src},
             "e2e": None, "cpu_baseline": None, "gpu_launches": int(launches), "clocks": clk}), flush=True)
     di.close()
     if world > 1:

@@ -506,12 +506,15 @@ cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const voi
         return CUART_OK;
     }
     if (so) {                                          // fused return: the default policy only
+        cudaEvent_t ev0, ev1;
+        ktimer_begin(h, s, ev0, ev1);
         switch (kind) {
         case CUART_KEY_U64: k_lookup<KeyU64, 5, true><<<grid, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
         case CUART_KEY_U32: k_lookup<KeyU32, 5, true><<<grid, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
         default: k_lookup<KeyBytes, 5, true><<<grid, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
         }
         g_cuart_launches++;
+        ktimer_end(h, s, ev0, ev1, n);
         CU_TRY(cudaGetLastError());
         return CUART_OK;
     }

@@ -234,10 +234,14 @@ class DistIndex:
         B._check(lib().cuart_dist_update(self.h, ctypes.byref(k), values.data_ptr(), n, B._stream_ptr(stream)),
                  "cuart_dist_update")
 
-    def mixed_round(self, keys, values, is_update, lens=None, stream=None):
+    def mixed_round(self, keys, values, is_update, lens=None, stream=None, events=None):
         """One round of a mixed op stream (reading C7): every lookup sees the state
         before the round; the round's updates then apply in global (rank-major, op)
-        order.  Returns per op the lookup result, CUART_MISS for update ops."""
+        order.  Returns per op the lookup result, CUART_MISS for update ops.
+        events: optional 5 CUDA events recorded on the stream around the four calls
+        (partition, lookup, update, unroute) -- measurement only."""
+        rec = (lambda i: events[i].record()) if events else (lambda i: None)
+        rec(0)
         n = keys.shape[0]
         ok, ol, ov = torch.empty_like(keys), (torch.empty_like(lens) if lens is not None else None), torch.empty_like(values)
         perm = torch.empty(n, dtype=torch.int32, device=keys.device)
@@ -249,13 +253,17 @@ class DistIndex:
                                                  ok.data_ptr(), ol.data_ptr() if ol is not None else None,
                                                  ov.data_ptr(), perm.data_ptr(), counts.data_ptr(), scratch.data_ptr(),
                                                  sp), "cuart_partition_by_flag")
+        rec(1)
         n_l = int(counts[0].item())                  # host needs the split to size the two calls
         res = torch.empty(n, dtype=torch.int64, device=keys.device)
         B._check(B.lib().cuart_fill_miss(res.data_ptr() + 8 * n_l, n - n_l, sp), "cuart_fill_miss")
         self.lookup((ok[:n_l], ol[:n_l]) if ol is not None else ok[:n_l], res[:n_l], stream)
+        rec(2)
         self.update((ok[n_l:], ol[n_l:]) if ol is not None else ok[n_l:], ov[n_l:], stream)
+        rec(3)
         out = torch.empty_like(res)
         B._check(B.lib().cuart_unroute(res.data_ptr(), perm.data_ptr(), n, out.data_ptr(), sp), "cuart_unroute")
+        rec(4)
         return out
 
     def last(self):
