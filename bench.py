@@ -63,6 +63,8 @@ def _args():
     p.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
                    help="range mode exchange: p2p = fused push/return over peer memory (CUDA IPC, NVLink), "
                         "nccl = route + all-to-all")
+    p.add_argument("--l2-persist", type=int, default=0,
+                   help="cuart_build_opts.l2_persist: persisting L2 window over the root tables")
     p.add_argument("--c5-share", type=int, default=0,
                    help="c5 on one GPU: the per-GPU share of a P-GPU run (rank 0's keys and owned ops)")
     p.add_argument("--traffic", type=float, default=None,
@@ -413,7 +415,8 @@ def main():
     keys, vals, keys_d = make_keys(cfg, dev)
     if world == 1:
         layout = C.Layout(keys, vals, lut_bytes=args.lut)
-        ix = C.Index.from_layout(layout, device=local, lut_format=LUT_FORMATS[args.lut_format])
+        ix = C.Index.from_layout(layout, device=local, lut_format=LUT_FORMATS[args.lut_format],
+                                 l2_persist=args.l2_persist)
         di = None
     else:
         di = DistIndex(keys, vals, mode=mode, transport=args.transport, lut_bytes=args.lut)

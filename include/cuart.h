@@ -150,6 +150,7 @@ typedef struct {
     uint32_t lut_format;         /* CUART_LUT_* in use on the device */
     uint64_t lut_exceptions;     /* RANK: entries served by the 64-bit link table */
     uint32_t wide_lut;           /* 1: pre-bucketed walks start from the wide root table */
+    uint64_t l2_window_bytes;    /* l2_persist: bytes under the persisting access-policy window */
 } cuart_stats_t;
 
 typedef struct cuart_index cuart_index;    /* device-resident index (opaque) */

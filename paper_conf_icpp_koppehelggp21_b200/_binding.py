@@ -34,7 +34,7 @@ class _Stats(ctypes.Structure):
                 ("lut_entries", ctypes.c_uint64), ("lut_bytes_total", ctypes.c_uint64),
                 ("arena_bytes", ctypes.c_uint64), ("lut_bytes", ctypes.c_uint32), ("key_kind", ctypes.c_uint32),
                 ("root", ctypes.c_uint64), ("max_depth", ctypes.c_uint32), ("lut_format", ctypes.c_uint32),
-                ("lut_exceptions", ctypes.c_uint64), ("wide_lut", ctypes.c_uint32)]
+                ("lut_exceptions", ctypes.c_uint64), ("wide_lut", ctypes.c_uint32), ("l2_window_bytes", ctypes.c_uint64)]
 
 
 class _View(ctypes.Structure):
@@ -321,7 +321,8 @@ def _stats_dict(s):
     d.update({f"{names[t]}_bytes": int(s.bytes[t]) for t in names})
     d.update(n_keys=int(s.n_keys), lut_bytes=int(s.lut_bytes), lut_entries=int(s.lut_entries),
              arena_bytes=int(s.arena_bytes), root=int(s.root), max_depth=int(s.max_depth), key_kind=int(s.key_kind),
-             lut_format=int(s.lut_format), lut_exceptions=int(s.lut_exceptions), wide_lut=int(s.wide_lut))
+             lut_format=int(s.lut_format), lut_exceptions=int(s.lut_exceptions), wide_lut=int(s.wide_lut),
+             l2_window_bytes=int(s.l2_window_bytes))
     return d
 
 

@@ -721,6 +721,32 @@ cuart_status dispatch_update(cuart_index* h, const void* k, const uint8_t* lens,
     return launch_update(h, h->key_kind, k, lens, vals, nullptr, 0, n, s);
 }
 
+// l2_persist: the caller's stream carries the persisting window for the launches of
+// one call, then gets its previous policy back (attributes are captured per launch).
+struct L2Window {
+    cudaStream_t s = nullptr;
+    bool set = false;
+    cudaStreamAttrValue old{};
+    L2Window(const cuart_index* h, cudaStream_t st) : s(st) {
+        if (!h->l2_bytes) return;
+        if (cudaStreamGetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &old) != cudaSuccess) {
+            cudaGetLastError();
+            return;
+        }
+        cudaStreamAttrValue v{};
+        v.accessPolicyWindow.base_ptr = h->l2_base;
+        v.accessPolicyWindow.num_bytes = h->l2_bytes;
+        v.accessPolicyWindow.hitRatio = h->l2_hit;
+        v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        set = cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v) == cudaSuccess;
+        if (!set) cudaGetLastError();
+    }
+    ~L2Window() {
+        if (set) cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &old);
+    }
+};
+
 // ============================================================================ C ABI
 extern "C" {
 
@@ -1139,6 +1165,23 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
             h->pool = nullptr;
         }
     }
+    if (opts && opts->l2_persist && h->lutw_off + lutw.size() * 8 > h->lut_off) {
+        // the root tables the walks start from (LINKS + compact/rank + wide), contiguous in
+        // the arena: persisting lines up to the device's persisting-L2 limit
+        int maxp = 0, maxw = 0;
+        cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
+        cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev);
+        const size_t span = h->lutw_off + lutw.size() * 8 - h->lut_off;
+        if (maxp > 0 && maxw > 0) {
+            h->l2_base = h->arena + h->lut_off;
+            h->l2_bytes = span < size_t(maxw) ? span : size_t(maxw);
+            h->l2_hit = float(maxp) >= float(h->l2_bytes) ? 1.f : float(maxp) / float(h->l2_bytes);
+            if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, size_t(maxp)) != cudaSuccess) {
+                cudaGetLastError();
+                h->l2_bytes = 0;
+            }
+        }
+    }
     *out = h;
     return CUART_OK;
 }
@@ -1307,6 +1350,7 @@ cuart_status cuart_lookup(const cuart_index* h, const cuart_keys* q, size_t n, u
     if (rc != CUART_OK) return rc;
     if (n == 0) return CUART_OK;
     if (!out) return CUART_ERR_INVALID_ARGUMENT;
+    L2Window w(h, (cudaStream_t)stream);
     return launch_lookup(h, h->key_kind, q->data, q->lengths, n, out, (cudaStream_t)stream);
 }
 
@@ -1315,6 +1359,7 @@ cuart_status cuart_update(cuart_index* h, const cuart_keys* k, const uint64_t* v
     if (rc != CUART_OK) return rc;
     if (n == 0) return CUART_OK;
     if (!v) return CUART_ERR_INVALID_ARGUMENT;
+    L2Window w(h, (cudaStream_t)stream);
     return dispatch_update(h, k->data, k->lengths, v, n, (cudaStream_t)stream);
 }
 
@@ -1499,6 +1544,7 @@ cuart_status cuart_stats(const cuart_index* h, cuart_stats_t* s) {
     s->lut_format = h->lut_format;
     s->lut_exceptions = h->lut_exceptions;
     s->wide_lut = h->wide ? 1u : 0u;
+    s->l2_window_bytes = h->l2_bytes;
     s->arena_bytes = h->arena_bytes;
     s->key_kind = h->key_kind;
     s->root = h->root;

@@ -49,6 +49,10 @@ struct cuart_index {
     // on the hot path, released in cuart_destroy
     cudaMemPool_t pool = nullptr;
     bool hold_epoch = false;           // dist updates: every chunk of a batch shares one epoch
+    // l2_persist (§3.2.2): persisting access-policy window over the root tables
+    void* l2_base = nullptr;
+    size_t l2_bytes = 0;
+    float l2_hit = 0.f;
     DistState* dist = nullptr;         // multi-GPU state (cuart_dist_build), else nullptr
     uint64_t free_off = 0;             // free-leaf list (u32 ids) + its counter
     // host-pipeline staging

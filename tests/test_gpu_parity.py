@@ -564,3 +564,27 @@ def test_prebucket_updates_equal_direct(kind):
     on.close()
     off.close()
     wide.close()
+
+
+@pytest.mark.parametrize("on_stream", [False, True])
+def test_l2_persist_window_results_identical(on_stream):
+    """cuart_build_opts.l2_persist (keep the merged upper layers cached) sets a
+    persisting access-policy window over the root tables for the launches of each
+    call; it changes performance only: results equal the oracle, on the legacy and on
+    a created stream (whose previous policy is restored)."""
+    cfg = W.CONFIGS["c1"]
+    keys, vals = W.build_set(cfg)
+    ix = C.Index(keys, vals, lut_bytes=3, l2_persist=1, prebucket=C.PREBUCKET_ON)
+    assert ix.stats()["l2_window_bytes"] > 0
+    o = MapOracle(keys, vals)
+    q = W.lookup_batch(cfg, keys)
+    s = torch.cuda.Stream() if on_stream else torch.cuda.current_stream()
+    with torch.cuda.stream(s):
+        got = _lookup(ix, q)
+        uk, uv = W.update_batch(cfg, keys)
+        ix.update(_t(uk), _t(uv))
+        got2 = _lookup(ix, keys)
+    assert np.array_equal(got, o.lookup(q))
+    o.update(uk, uv)
+    assert np.array_equal(got2, o.lookup(keys))
+    ix.close()
