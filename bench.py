@@ -126,26 +126,51 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ oracle timing (CPU)
-def oracle_timing(cfg, keys, vals, n_lookup_sample, n_update_sample, reps=1):
-    """The oracle as it stands, single-threaded on a host core: (Mops/s, detail)."""
+def oracle_timing(cfg, keys, vals, n_lookup_sample, n_update_sample, allcore_factor=8):
+    """The oracle as it stands (SURVEY §8(d) CPU-baseline plan), on this box's host cores:
+    single-threaded lookups and sequential updates pinned to one core, then the
+    read-only lookups fanned over every core (oart_lookup_batch_mt).  Returns
+    (mixed 1-core Mops/s, detail)."""
     from oracle import ArtOracle
     t0 = time.perf_counter()
-    o = ArtOracle(keys, vals)
+    if isinstance(keys, tuple):
+        o = ArtOracle(keys, vals)
+    else:   # insertion order does not change the tree (pinned); sorted inserts build faster
+        order = np.argsort(keys)
+        o = ArtOracle(keys[order], vals[order])
     build_s = time.perf_counter() - t0
     q = host_lookups(cfg, keys, 0, n_lookup_sample)
-    uk, uv = W.update_batch(cfg, keys, 0, n_update_sample) if cfg.n_updates else (None, None)
-    times = []
-    for _ in range(reps):
+    uk, uv = W.update_batch(cfg, keys, 0, n_update_sample) if cfg.n_updates and n_update_sample else (None, None)
+    cores = sorted(os.sched_getaffinity(0))
+    os.sched_setaffinity(0, {cores[0]})             # one core (taskset)
+    try:
         t0 = time.perf_counter()
         o.lookup(q)
+        t_look = time.perf_counter() - t0
+        t_upd = 0.0
         if uk is not None:
+            t0 = time.perf_counter()
             o.update(uk, uv)
-        times.append(time.perf_counter() - t0)
+            t_upd = time.perf_counter() - t0
+    finally:
+        os.sched_setaffinity(0, set(cores))
+    qa = host_lookups(cfg, keys, n_lookup_sample, n_lookup_sample * allcore_factor)
+    t0 = time.perf_counter()
+    o.lookup_mt(qa, len(cores))
+    t_all = time.perf_counter() - t0
     o.close()
-    dt = min(times)
-    ops = n_lookup_sample + (n_update_sample if uk is not None else 0)
-    return ops / dt / 1e6, {"build_s": round(build_s, 2), "sample_lookups": n_lookup_sample,
-                            "sample_updates": n_update_sample if uk is not None else 0, "seconds": round(dt, 3)}
+    nu = n_update_sample if uk is not None else 0
+    mixed = (n_lookup_sample + nu) / (t_look + t_upd) / 1e6
+    return mixed, {"build_s": round(build_s, 2), "sample_lookups": n_lookup_sample, "sample_updates": nu,
+                   "seconds": round(t_look + t_upd, 3),
+                   "oracle_lookup_mops_1core": round(n_lookup_sample / t_look / 1e6, 3),
+                   "oracle_update_mops_1core": round(nu / t_upd / 1e6, 3) if nu else None,
+                   "oracle_lookup_mops_allcores": round(qa_len(qa) / t_all / 1e6, 3),
+                   "allcore_sample_lookups": qa_len(qa), "host_cores": len(cores)}
+
+
+def qa_len(q):
+    return q[1].shape[0] if isinstance(q, tuple) else q.shape[0]
 
 
 def host_lookups(cfg, keys, start, m):
@@ -607,8 +632,11 @@ def main():
         v, det = oracle_timing(cfg, keys, vals, nls, nus)
         cpu = {"value": round(v, 3), "unit": "Mops/s", "cores": 1, "kind": "oracle",
                "sample": f"{nls} lookups + {nus} updates of the {args.config} stream (same mix), "
-                         f"single-threaded pointer ART built over all {cfg.n_keys} keys "
-                         f"(build {det['build_s']} s untimed, timed {det['seconds']} s)"}
+                         f"single-threaded pointer ART built over all {cfg.n_keys} keys, pinned to one core "
+                         f"(build {det['build_s']} s untimed, timed {det['seconds']} s); all-core lookups: "
+                         f"{det['allcore_sample_lookups']} further lookups over {det['host_cores']} threads",
+               **{k: det[k] for k in ("oracle_lookup_mops_1core", "oracle_update_mops_1core",
+                                      "oracle_lookup_mops_allcores", "host_cores")}}
 
     if rank == 0:
         line = {

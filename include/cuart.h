@@ -199,8 +199,10 @@ cuart_status cuart_erase(cuart_index* h, const cuart_keys* keys, size_t n, void*
  *   bounds[6*i + 2*(c-5) + 1] = number of class-c leaves with key <= hi[i]
  * for c = 5 (leaf8), 6 (leaf16), 7 (leaf32); the matching leaves are the records
  * [start, end) of that buffer (cuart_dump).  Deleted leaves stay in place with
- * the tombstone value CUART_MISS.  Integer key kinds only (BYTES returns
- * CUART_ERR_INVALID_ARGUMENT).  Device pointers, bounds uint64_t[6n]; async. */
+ * the tombstone value CUART_MISS.  Every key kind: integer keys live in the leaf8
+ * buffer; byte strings in all three classes, ordered lexicographically (a proper
+ * prefix first; bound bytes past their length are ignored).  Device pointers, bounds
+ * uint64_t[6n]; async. */
 cuart_status cuart_range(const cuart_index* h, const cuart_keys* lo, const cuart_keys* hi, size_t n,
                          uint64_t* bounds, void* stream);
 /* Synchronous read of the free-leaf list: *count entries exist; up to cap copied to ids (host). */
@@ -231,6 +233,10 @@ cuart_status cuart_kernel_time(cuart_index* h, double* total_ms, uint64_t* launc
  * bucketed walk with the shared-memory root-table slice (k_lookup_slice). */
 cuart_status cuart_kernel_time_ex(cuart_index* h, double* total_ms, uint64_t* launches, uint64_t* lookups,
                                   uint64_t* slice_launches);
+/* Test hook: set the update epoch (the high half of the per-leaf conflict words,
+ * §8(a) a9) so that the wrap path -- every 2^32 - 2 update batches the words are
+ * cleared and the epoch restarts at 1 -- can be exercised.  Synchronous. */
+cuart_status cuart_debug_set_epoch(cuart_index* h, uint32_t epoch);
 /* Kernel launches issued by this library since load (for launch accounting). */
 uint64_t cuart_launch_count(void);
 

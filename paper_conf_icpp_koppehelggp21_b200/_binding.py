@@ -83,6 +83,8 @@ def lib():
             f = getattr(L, name)
             f.argtypes = args
             f.restype = ctypes.c_int
+        L.cuart_debug_set_epoch.argtypes = [P, ctypes.c_uint32]
+        L.cuart_debug_set_epoch.restype = ctypes.c_int
         L.cuart_fill_miss.argtypes = [P, S, P]
         L.cuart_fill_miss.restype = ctypes.c_int
         L.cuart_launch_count.argtypes = []
@@ -469,7 +471,8 @@ class Index:
     def range(self, lo, hi, bounds=None, stream=None):
         import torch
         if bounds is None:
-            bounds = torch.empty((lo.shape[0], 6), dtype=torch.int64, device=lo.device)
+            l0 = lo[0] if isinstance(lo, tuple) else lo
+            bounds = torch.empty((l0.shape[0], 6), dtype=torch.int64, device=l0.device)
         return cuart_range(self.h, lo, hi, bounds, stream, getattr(self, "device", None))
 
     def lookup_host(self, queries, out=None):

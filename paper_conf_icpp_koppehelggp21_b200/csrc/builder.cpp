@@ -246,7 +246,10 @@ int build_host_layout(uint32_t kind, const void* data, const uint8_t* lengths, c
             L.count[t] = c[t];
             if (c[t] > kIndexMask) return CUART_ERR_TOO_LARGE;
             L.buf[t].assign(c[t] * kRecordBytes[t], 0);
+            if (kind == CUART_KEY_BYTES) L.leaf_len[t].assign(c[t], 0);
         }
+        if (kind == CUART_KEY_BYTES)
+            for (uint64_t i = 0; i < S.n; i++) L.leaf_len[leaf_type(S.len(i))][leaf_rank[i]] = uint8_t(S.len(i));
         // f4: host-resident long leaves, in lexicographic order like every leaf class
         L.long_off.assign(1, 0);
         for (uint64_t i = 0; i < S.n; i++) {

@@ -22,6 +22,9 @@ struct HostLayout {
     std::vector<uint8_t> long_bytes;       // concatenated keys
     std::vector<uint64_t> long_off;        // [count + 1] offsets into long_bytes
     std::vector<uint64_t> long_vals;
+    // BYTES: key length of every leaf, per leaf class in leaf order (range queries,
+    // the order of two keys whose zero-padded bytes agree is decided by length)
+    std::vector<uint8_t> leaf_len[8];
 };
 
 // Status codes mirror cuart_status (include/cuart.h).

@@ -951,6 +951,8 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     if (!CUART_COLOCATED_WINNER) off = align(off + h->total_leaves * 8);
     h->free_off = off;
     off = align(off + 8 + h->total_leaves * 4);
+    h->llen_off = off;                                 // BYTES: key length per leaf (range queries)
+    if (L.key_kind == CUART_KEY_BYTES) off = align(off + h->total_leaves);
     std::vector<uint32_t> lut32;
     std::vector<uint64_t> lutr;
     uint32_t fmt = opts ? opts->lut_format : CUART_LUT_FORMAT_AUTO;
@@ -1078,6 +1080,11 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && cudaMemset(h->arena + h->err_off, 0, 256) != cudaSuccess) rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && cudaMemset(h->arena + h->free_off, 0, 8) != cudaSuccess) rc = CUART_ERR_CUDA;
+    if (L.key_kind == CUART_KEY_BYTES)
+        for (int t = T_LEAF8, o = 0; t <= T_LEAF32 && rc == CUART_OK; o += int(L.count[t]), t++)
+            if (L.count[t] && cudaMemcpy(h->arena + h->llen_off + o, L.leaf_len[t].data(), L.count[t],
+                                         cudaMemcpyHostToDevice) != cudaSuccess)
+                rc = CUART_ERR_CUDA;
     if (rc != CUART_OK) {
         cudaFree(h->arena);
         delete h;
@@ -1382,14 +1389,28 @@ cuart_status cuart_erase(cuart_index* h, const cuart_keys* k, size_t n, void* st
 cuart_status cuart_range_leaf8(const uint8_t* leaves, uint64_t nleaves, uint32_t kind, const void* lo, const void* hi,
                                size_t n, uint64_t* bounds, void* stream);   // route.cu
 
+cuart_status cuart_range_bytes(const uint8_t* const* rec, const uint8_t* const* len, const uint64_t* count,
+                               const uint8_t* lo, const uint8_t* llo, const uint8_t* hi, const uint8_t* lhi, size_t n,
+                               uint64_t* bounds, void* stream);   // route.cu
+
 cuart_status cuart_range(const cuart_index* h, const cuart_keys* lo, const cuart_keys* hi, size_t n, uint64_t* bounds,
                          void* stream) {
     cuart_status rc = check_keys(h, lo, n);
     if (rc == CUART_OK) rc = check_keys(h, hi, n);
     if (rc != CUART_OK) return rc;
-    if (h->key_kind == CUART_KEY_BYTES) return CUART_ERR_INVALID_ARGUMENT;   // integer keys only
     if (n == 0) return CUART_OK;
     if (!bounds) return CUART_ERR_INVALID_ARGUMENT;
+    if (h->key_kind == CUART_KEY_BYTES) {
+        const uint8_t* rec[3];
+        const uint8_t* len[3];
+        const uint64_t cnt[3] = {h->count[T_LEAF8], h->count[T_LEAF16], h->count[T_LEAF32]};
+        for (int c = 0; c < 3; c++) {
+            rec[c] = h->dix.base[T_LEAF8 + c];
+            len[c] = h->arena + h->llen_off + h->dix.leaf_base[T_LEAF8 + c];
+        }
+        return cuart_range_bytes(rec, len, cnt, (const uint8_t*)lo->data, lo->lengths, (const uint8_t*)hi->data,
+                                 hi->lengths, n, bounds, stream);
+    }
     return cuart_range_leaf8(h->dix.base[T_LEAF8], h->count[T_LEAF8], h->key_kind, lo->data, hi->data, n, bounds,
                              stream);
 }
@@ -1423,6 +1444,14 @@ cuart_status cuart_kernel_time_ex(cuart_index* h, double* total_ms, uint64_t* la
     *lookups = h->klookups;
     *slice_launches = h->kslice;
     drop_kevents(h);
+    return CUART_OK;
+}
+
+cuart_status cuart_debug_set_epoch(cuart_index* h, uint32_t epoch) {
+    if (!h || epoch == 0 || epoch == 0xFFFFFFFFu) return CUART_ERR_INVALID_ARGUMENT;
+    CU_TRY(cudaSetDevice(h->device));
+    CU_TRY(cudaDeviceSynchronize());
+    h->epoch = epoch;
     return CUART_OK;
 }
 

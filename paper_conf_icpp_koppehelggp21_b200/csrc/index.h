@@ -55,6 +55,7 @@ struct cuart_index {
     float l2_hit = 0.f;
     DistState* dist = nullptr;         // multi-GPU state (cuart_dist_build), else nullptr
     uint64_t free_off = 0;             // free-leaf list (u32 ids) + its counter
+    uint64_t llen_off = 0;             // BYTES: key length of every leaf (global leaf id order)
     // host-pipeline staging
     void* stage[4] = {nullptr, nullptr, nullptr, nullptr};
     uint64_t* stage_out[4] = {nullptr, nullptr, nullptr, nullptr};

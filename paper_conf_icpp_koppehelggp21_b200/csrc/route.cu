@@ -315,3 +315,78 @@ extern "C" cuart_status cuart_range_leaf8(const uint8_t* leaves, uint64_t nleave
     g_cuart_launches += 1;
     return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
 }
+
+// Byte-string keys (every leaf class buffer is in lexicographic order).  The
+// zero-padded bytes decide the order of two keys unless they agree on all 32 bytes;
+// then the shorter key (a proper prefix) comes first -- for that the library keeps
+// the key length of every leaf (leaf_len, uploaded with BYTES indexes).
+namespace {
+
+struct RangeLeaves {
+    const uint8_t* rec[3];       // leaf8 / leaf16 / leaf32 records
+    const uint8_t* len[3];       // their key lengths
+    uint64_t count[3];
+};
+
+__device__ __forceinline__ int cmp_leaf(const uint8_t* rec, uint32_t width, uint32_t lk, const uint8_t* q, uint32_t lq) {
+    for (uint32_t b = 0; b < 32; b++) {
+        const uint32_t kb = b < width ? rec[b] : 0u;
+        const uint32_t qb = b < lq ? q[b] : 0u;            // query bytes past its length are ignored
+        if (kb != qb) return kb < qb ? -1 : 1;
+    }
+    return lk < lq ? -1 : (lk > lq ? 1 : 0);
+}
+
+// number of leaves of one class with key < q (le = false) or <= q (le = true)
+__device__ uint64_t rank_bytes(const RangeLeaves& L, int c, const uint8_t* q, uint32_t lq, bool le) {
+    const uint32_t width = c == 0 ? 8u : c == 1 ? 16u : 32u;
+    const uint64_t rb = cuart::record_bytes(uint32_t(cuart::T_LEAF8 + c));
+    uint64_t lo = 0, hi = L.count[c];
+    while (lo < hi) {
+        const uint64_t mid = (lo + hi) >> 1;
+        const int r = cmp_leaf(L.rec[c] + mid * rb, width, L.len[c][mid], q, lq);
+        if (r < 0 || (le && r == 0)) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+__global__ void __launch_bounds__(128) k_range_bytes(RangeLeaves L, const uint8_t* __restrict__ lo,
+                                                     const uint8_t* __restrict__ llo, const uint8_t* __restrict__ hi,
+                                                     const uint8_t* __restrict__ lhi, uint64_t n,
+                                                     uint64_t* __restrict__ bounds) {
+    const uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    uint8_t ql[32], qh[32];
+#pragma unroll
+    for (int b = 0; b < 32; b++) {
+        ql[b] = lo[32 * i + b];
+        qh[b] = hi[32 * i + b];
+    }
+    const uint32_t a = llo[i] < 32 ? llo[i] : 32u, z = lhi[i] < 32 ? lhi[i] : 32u;
+    uint64_t* out = bounds + 6 * i;
+    for (int c = 0; c < 3; c++) {
+        const uint64_t s = rank_bytes(L, c, ql, a, false);
+        uint64_t e = rank_bytes(L, c, qh, z, true);
+        out[2 * c] = s;
+        out[2 * c + 1] = e < s ? s : e;                    // empty range when hi < lo
+    }
+}
+
+}  // namespace
+
+extern "C" cuart_status cuart_range_bytes(const uint8_t* const* rec, const uint8_t* const* len, const uint64_t* count,
+                                          const uint8_t* lo, const uint8_t* llo, const uint8_t* hi,
+                                          const uint8_t* lhi, size_t n, uint64_t* bounds, void* stream) {
+    if (n == 0) return CUART_OK;
+    RangeLeaves L{};
+    for (int c = 0; c < 3; c++) {
+        L.rec[c] = rec[c];
+        L.len[c] = len[c];
+        L.count[c] = count[c];
+    }
+    const uint64_t blocks = (n + 127) / 128;
+    k_range_bytes<<<unsigned(blocks), 128, 0, (cudaStream_t)stream>>>(L, lo, llo, hi, lhi, n, bounds);
+    g_cuart_launches += 1;
+    return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+}

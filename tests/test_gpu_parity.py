@@ -588,3 +588,28 @@ def test_l2_persist_window_results_identical(on_stream):
     o.update(uk, uv)
     assert np.array_equal(got2, o.lookup(keys))
     ix.close()
+
+
+@pytest.mark.parametrize("prebucket", [1, 2])
+def test_epoch_wrap(prebucket):
+    """§8(a) a9: the conflict words carry the batch epoch in their high half, so no
+    reset pass runs between batches; every 2^32 - 2 batches the epoch wraps, the words
+    are cleared and the epoch restarts at 1.  Driven through the test hook: batches
+    before, across and after the wrap (duplicate-heavy, so stale high-priority words
+    of the last pre-wrap batch would block later winners if the clear were missing)
+    equal the sequential oracle."""
+    cfg = W.CONFIGS["c1"]
+    keys, vals = W.build_set(cfg)
+    ix = C.Index(keys, vals, lut_bytes=3, prebucket=prebucket)
+    o = MapOracle(keys, vals)
+    B = C._binding
+    B._check(B.lib().cuart_debug_set_epoch(ix.h, 0xFFFFFFFC), "cuart_debug_set_epoch")
+    rng = np.random.default_rng(17)
+    for b in range(5):
+        m = 60_000 if b % 2 == 0 else 5_000         # a small batch after a big one: low op indices
+        uk = keys[rng.integers(0, 2000, m)]           # few distinct keys, many duplicates
+        uv = rng.integers(0, 2**63, m, dtype=np.uint64)
+        ix.update(_t(uk), _t(uv))
+        o.update(uk, uv)
+        assert np.array_equal(_lookup(ix, keys), o.lookup(keys)), b
+    ix.close()

@@ -78,3 +78,64 @@ def test_range_with_deletes_keeps_positions():
     vals = leaves[:, 8:16].copy().view(np.uint64).ravel()
     assert np.all(vals[10:20] == np.uint64(2**64 - 1)) and vals[20] == 201   # tombstones in place
     ix.close()
+
+
+def test_range_bounds_byte_strings():
+    """Byte-string range queries (each leaf class buffer is lexicographically
+    ordered): per class c, start = #class-c keys < lo and end = #class-c keys <= hi in
+    true byte-string order (a proper prefix sorts first), against Python's bytes
+    ordering over the key set.  Bounds include exact keys, proper prefixes of keys
+    (the zero-padded bytes agree, the length decides), keys with a bumped last byte,
+    random strings, and empty ranges."""
+    import bisect
+    slots, lens = W.string_keys(4, 50_000, min_len=2)
+    keys = [bytes(slots[i, : lens[i]]) for i in range(lens.shape[0])]
+    vals = np.arange(lens.shape[0], dtype=np.uint64)
+    ix = C.Index((slots, lens), vals)
+    rng = np.random.default_rng(9)
+    m = 20_000
+    pick = rng.integers(0, len(keys), m)
+    lo_b, hi_b = [], []
+    for j, p in enumerate(pick):
+        k = keys[p]
+        r = j % 5
+        if r == 0:
+            a, b = k, k                                                # exactly one key
+        elif r == 1:
+            a, b = k[: max(1, len(k) // 2)], k                         # a proper prefix as the lower bound
+        elif r == 2:
+            a = k[:-1] + bytes([min(255, k[-1] + 1)])
+            b = keys[pick[(j + 1) % m]]
+        elif r == 3:
+            a = bytes(rng.integers(97, 123, rng.integers(1, 33)).astype(np.uint8))
+            b = bytes(rng.integers(97, 123, rng.integers(1, 33)).astype(np.uint8))
+        else:
+            a, b = k, k[: max(1, len(k) - 3)]                          # hi < lo: empty
+        lo_b.append(a)
+        hi_b.append(b)
+
+    def pack(xs):
+        s_ = np.zeros((len(xs), 32), np.uint8)
+        l_ = np.zeros(len(xs), np.uint8)
+        for i, x in enumerate(xs):
+            s_[i, : len(x)] = np.frombuffer(x, np.uint8)
+            l_[i] = len(x)
+        return torch.from_numpy(s_).to(DEV), torch.from_numpy(l_).to(DEV)
+
+    b = ix.range(pack(lo_b), pack(hi_b))
+    torch.cuda.synchronize()
+    b = b.cpu().numpy()
+    classes = [sorted(k for k in keys if len(k) <= 8), sorted(k for k in keys if 8 < len(k) <= 16),
+               sorted(k for k in keys if len(k) > 16)]
+    assert all(len(c) > 0 for c in classes)
+    for i in range(m):
+        for c, ks in enumerate(classes):
+            s = bisect.bisect_left(ks, lo_b[i])
+            e = max(s, bisect.bisect_right(ks, hi_b[i]))
+            assert (b[i, 2 * c], b[i, 2 * c + 1]) == (s, e), (i, c, lo_b[i], hi_b[i])
+    # the leaf records of each class are that class's keys in this order
+    view = ix.dump()
+    for c, (t, w) in enumerate(((5, 8), (6, 16), (7, 32))):
+        rec = view["buf"][t].reshape(-1, int(view["record_bytes"][t]))[:, :w]
+        assert [bytes(r).rstrip(b"\0") for r in rec[:200]] == [k.rstrip(b"\0") for k in classes[c][:200]]
+    ix.close()
