@@ -1017,7 +1017,17 @@ cuart_status cuart_dist_build(const cuart_dist_cfg* cfg, const cuart_keys* keys,
     }
     for (uint32_t r = 0; r < P; r++) d->part.depth[r] = deps[r];
     // chunk C and window capacity P*C per slot (P*C < 2^32: send-order slots are 32-bit)
-    uint64_t C = cfg->chunk ? cfg->chunk : (kind == CUART_KEY_BYTES ? (uint64_t(1) << 22) : (uint64_t(1) << 25));
+    // Default C: the largest power of two whose two window slots (P * C ops of key +
+    // length + value + priority each, plus C results) fit a 16 GiB budget
+    // (CUART_DIST_WINDOW_BYTES): 2^28 ops at one rank, 2^25 at eight (u64).  Larger
+    // chunks walk longer runs of each bucket (more reuse of its tree slice) and pay the
+    // per-chunk protocol (a count exchange, ~10 small launches) less often.
+    uint64_t budget = uint64_t(16) << 30;
+    if (const char* pe = getenv("CUART_DIST_WINDOW_BYTES")) budget = strtoull(pe, nullptr, 0);
+    const uint64_t per_op = 2 * (uint64_t(P) * (key_bytes(kind) + (kind == CUART_KEY_BYTES ? 1 : 0) + 12) + 8);
+    uint64_t C = uint64_t(1) << 20;
+    while (C < (uint64_t(1) << 29) && 2 * C * per_op <= budget) C <<= 1;
+    if (cfg->chunk) C = cfg->chunk;
     if (const char* pe = getenv("CUART_DIST_CHUNK")) C = strtoull(pe, nullptr, 0);
     C = std::max<uint64_t>(kBucketTile, (C + kBucketTile - 1) / kBucketTile * kBucketTile);
     while (uint64_t(P) * C >= (uint64_t(1) << 31)) C /= 2;
