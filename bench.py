@@ -483,17 +483,9 @@ def main():
     sec = layout.sectors(samp, wide=bool(bucketed and stats.get("wide_lut", 0))).astype(np.float64)
     io_bytes = {"u64": 8, "u32": 4, "bytes": 33}[cfg.kind] + 8
     random_bytes_per_lookup = 32.0 * sec.mean() + io_bytes
-    # Algorithmic DRAM bytes per lookup of the dominant kernel:
-    # direct path: every sector of the query's path is a random DRAM read (S x 32 B + I/O);
-    # pre-bucketed path (auto for >= 2^22 queries): the walk runs over one bucket's slice
-    # of the tree at a time, L2-resident by construction, so the compulsory traffic is the
-    # I/O plus each tree record once per batch (SURVEY §8(d) S_DRAM excludes L2-resident data).
-    tree_bytes = sum(stats[t + "_bytes"] for t in ("n4", "n16", "n48", "n256", "leaf8", "leaf16", "leaf32"))
-    served_est = nl           # range mode: each rank serves ~nl routed lookups (its share of every rank's batch)
-    bytes_per_lookup = (io_bytes + tree_bytes / served_est) if bucketed else random_bytes_per_lookup
     # whole lookup call (bucket histogram + scatter + walk + gather), streaming bytes per query
     ks = io_bytes - 8
-    pipeline_bytes = (ks + (ks + ks + 2) + (ks + 8) + (8 + 2 + 8)) + tree_bytes / served_est if bucketed else random_bytes_per_lookup
+    stream_bytes = (ks + (ks + ks + 2) + (ks + 8) + (8 + 2 + 8)) if bucketed else io_bytes
     del samp
 
     stream = torch.cuda.current_stream()
@@ -547,8 +539,9 @@ def main():
     upd_ms = float(np.mean([e[1].elapsed_time(e[2]) for e in evs])) if nu else 0.0
     ktot, klaunch, kq, kslice = C.cuart_kernel_time_ex(ix.h)
     C.cuart_kernel_timer(ix.h, False)
-    kern_ms = ktot / max(1, klaunch)
-    served = kq / max(1, klaunch)
+    kern_ms = ktot / args.steps                # the walk's time per step (every launch of the step)
+    served = kq / args.steps                   # lookups the walk served per step
+    launches_per_step = klaunch / args.steps
     tt = torch.tensor([total_ms, look_ms, upd_ms], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -558,7 +551,17 @@ def main():
     ops_per_step = world * nl + world * nu
     value = ops_per_step / (ms_step * 1e-3) / 1e6
 
-    # roofline of the dominant kernel (k_lookup on this rank), HBM-bound random gathers
+    out_now = out if di is None else di.lookup(q, out)
+    hit = float((out_now[: 1 << 24] != -1).float().mean().item())
+    del out_now
+    # Algorithmic (compulsory) DRAM bytes of the dominant kernel, the walk (
+    # S_DRAM excludes what is L2-resident by construction): key in + result
+    # out, plus every tree record the batch needs read once -- all inner nodes and the
+    # touched fraction of the leaves.  ncu's measured DRAM bytes ("traffic") above this
+    # are re-reads the walk's access order causes.
+    tree_b, leaf_frac = tree_bytes_touched(stats, served * hit)
+    bytes_per_lookup = io_bytes + tree_b / max(1.0, served)
+    pipeline_bytes = stream_bytes + tree_b / max(1.0, served)
     peak, peak_src = hbm_peak()
     achieved = served * bytes_per_lookup / (kern_ms * 1e-3) / 1e9
     pipe_achieved = nl * pipeline_bytes / (look_ms * 1e-3) / 1e9
@@ -570,9 +573,6 @@ def main():
     if traffic is None and os.path.exists(tfile):
         with open(tfile) as f:
             traffic = json.load(f).get(f"{args.config}/{'bucketed' if bucketed else 'direct'}")
-    out_now = out if di is None else di.lookup(q, out)
-    hit = float((out_now[: 1 << 24] != -1).float().mean().item())
-    del out_now
 
     # end-to-end through the public API with HOST buffers (pinned), copies inside the timed region
     e2e = None
@@ -659,11 +659,12 @@ def main():
                          "frac": round(achieved / peak, 4), "traffic": traffic,
                          "kernel": ("k_lookup_slice" if kslice else "k_lookup_wq" if wq else "k_lookup")
                          + {"u64": "<KeyU64>", "u32": "<KeyU32>", "bytes": "<KeyBytes>"}[cfg.kind],
-                         "kernel_ms": round(kern_ms, 4), "lookups_per_launch": int(served),
+                         "kernel_ms": round(kern_ms, 4), "lookups_per_step": int(served),
+                         "launches_per_step": round(launches_per_step, 2),
                          "lookup_call_ms": round(look_ms, 4), "prebucket": "on" if bucketed else "off",
                          "bytes_per_lookup": round(bytes_per_lookup, 3),
-                         "bytes_model": "bucketed: key+result I/O + tree records once per batch" if bucketed
-                         else "direct: 32 B x sectors on the path + key+result I/O",
+                         "bytes_model": "compulsory: key in + result out + every inner node and the touched "
+                                        f"fraction of the leaves ({leaf_frac:.3f}) read once per batch",
                          "sectors_per_lookup": round(float(sec.mean()), 4),
                          "random_path_bytes_per_lookup": round(random_bytes_per_lookup, 3),
                          "peak_source": peak_src, "random_access_ceiling": RANDOM_CEILING,
