@@ -65,6 +65,8 @@ def _args():
                         "nccl = route + all-to-all")
     p.add_argument("--l2-persist", type=int, default=0,
                    help="cuart_build_opts.l2_persist: persisting L2 window over the root tables")
+    p.add_argument("--c5-fused", type=int, default=1,
+                   help="c5 rounds through cuart_dist_mixed (1) or partition + lookup + update + unroute (0)")
     p.add_argument("--c5-share", type=int, default=0,
                    help="c5 on one GPU: the per-GPU share of a P-GPU run (rank 0's keys and owned ops)")
     p.add_argument("--traffic", type=float, default=None,
@@ -325,7 +327,7 @@ def run_c5(args, world, rank, local, dev):
 
     def step(i, ev=None):
         k, u, v = rounds[i % 2]
-        di.mixed_round(k, v, u, events=ev)
+        di.mixed_round(k, v, u, events=ev, fused=args.c5_fused == 1)
 
     for i in range(args.warmup):
         step(i)
@@ -352,7 +354,10 @@ def run_c5(args, world, rank, local, dev):
     if world > 1:
         dist.barrier()
     clk = clocks.stop()
-    phases = [float(np.mean([e[p].elapsed_time(e[p + 1]) for e in evs])) for p in range(4)]
+    if args.c5_fused:        # one cuart_dist_mixed call: only its total is bracketed
+        phases = [0.0, float(np.mean([e[0].elapsed_time(e[4]) for e in evs])), 0.0, 0.0]
+    else:
+        phases = [float(np.mean([e[p].elapsed_time(e[p + 1]) for e in evs])) for p in range(4)]
     tt = torch.tensor([t_start.elapsed_time(t_end), ktot / args.steps] + phases, dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -383,11 +388,13 @@ def run_c5(args, world, rank, local, dev):
                        "local_keys_rank0": int(keys.shape[0]), "build_s": round(build_s, 2),
                        "lut_format": stats["lut_format"], "tree_bytes": int(sum(stats[t + "_bytes"] for t in (
                            "n4", "n16", "n48", "n256", "leaf8", "leaf16", "leaf32")))},
-            "phases_ms": {"partition_by_flag": round(part_ms, 4), "dist_lookup": round(look_ms, 4),
-                          "dist_update": round(upd_ms, 4), "unroute": round(unr_ms, 4)},
-            "lookup": {"mlookups_per_s": round(world * n_look / (look_ms * 1e-3) / 1e6, 3), "ms": round(look_ms, 4)},
-            "update": {"mupdates_per_s": round(world * (n_ops - n_look) / (upd_ms * 1e-3) / 1e6, 3),
-                       "ms": round(upd_ms, 4)},
+            "phases_ms": ({"dist_mixed (lookup pass + update pass)": round(look_ms, 4)} if args.c5_fused else
+                          {"partition_by_flag": round(part_ms, 4), "dist_lookup": round(look_ms, 4),
+                           "dist_update": round(upd_ms, 4), "unroute": round(unr_ms, 4)}),
+            "lookup": None if args.c5_fused else {
+                "mlookups_per_s": round(world * n_look / (look_ms * 1e-3) / 1e6, 3), "ms": round(look_ms, 4)},
+            "update": None if args.c5_fused else {
+                "mupdates_per_s": round(world * (n_ops - n_look) / (upd_ms * 1e-3) / 1e6, 3), "ms": round(upd_ms, 4)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
                          "kernel": ("k_lookup_wq<KeyU64>" if stats.get("wide_lut") else "k_lookup<KeyU64>")

@@ -410,6 +410,14 @@ cuart_status cuart_dist_lookup(cuart_index* h, const cuart_keys* queries, size_t
  * sticky error flag of the owner's index (reading C5).  n <= 2^32 / nranks. */
 cuart_status cuart_dist_update(cuart_index* h, const cuart_keys* keys, const uint64_t* new_values, size_t n,
                                void* stream);
+/* Collective mixed batch (config 5's rounds, reading C7; RANGE mode): op i is an update
+ * iff is_update[i] != 0 (device uint8_t[n]).  Every lookup of the call, on every rank,
+ * sees the state before the call; then the call's updates apply in global rank-major
+ * order.  out[i] = the lookup result, CUART_MISS for update ops.  One pass per op kind
+ * filters the batch itself (no stable partition + inverse permutation).  REPLICA mode
+ * returns CUART_ERR_INVALID_ARGUMENT (split the batch with cuart_partition_by_flag). */
+cuart_status cuart_dist_mixed(cuart_index* h, const cuart_keys* keys, const uint64_t* values, const uint8_t* is_update,
+                              size_t n, uint64_t* out, void* stream);
 /* Host-only planning (no GPU): the splitters the build uses (RANGE; nranks-1 entries)
  * and the owner of each key (owner[i], may be NULL).  With a bootstrap in cfg the
  * splitters are all-gathered and compared across ranks (INVALID_ARGUMENT on mismatch). */

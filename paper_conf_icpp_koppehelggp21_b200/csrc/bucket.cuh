@@ -72,8 +72,10 @@ __device__ __forceinline__ uint32_t bucket_at(const void* q, const uint8_t* lens
 // routed batch: owner o's ops are one contiguous run of the send order, already
 // bucketed for o's walk.
 struct ByteBucket {
+    static constexpr bool kFilter = false;
     uint32_t depth;
     __host__ __device__ ByteBucket(uint32_t d = 0) : depth(d) {}
+    __device__ __forceinline__ bool skip(uint64_t) const { return false; }
     template <class Key>
     __device__ __forceinline__ uint32_t of(const Key& k) const { return bucket_of(k, depth); }
     template <class Key>
@@ -90,10 +92,12 @@ __device__ __forceinline__ uint64_t key_prefix8(const Key& k) {
 }
 
 struct OwnerPart {
+    static constexpr bool kFilter = false;
     uint32_t nsp;                      // number of splitters (ranks - 1)
     uint32_t lbpo;                     // bucket bits per owner
     uint64_t sp[kMaxSeg - 1];          // ascending splitters over the 8-byte prefix
     uint8_t depth[kMaxSeg];            // every owner's root branch depth
+    __device__ __forceinline__ bool skip(uint64_t) const { return false; }
     template <class Key>
     __device__ __forceinline__ uint32_t owner(const Key& k) const {
         const uint64_t p = key_prefix8(k);
@@ -114,6 +118,18 @@ struct OwnerPart {
         return of(Key::template load<true>(q, lens, i));
     }
 };
+
+// OwnerPart over one kind of op of a mixed batch (config 5's rounds, reading C7):
+// ops whose flag differs from `want` are skipped -- not counted, not staged, and a
+// skipped lookup's jpos is kSkipPos, for which the gather writes CUART_MISS.  One
+// pass per kind replaces the stable partition of the batch and its inverse.
+struct FilteredOwnerPart : OwnerPart {
+    static constexpr bool kFilter = true;
+    const uint8_t* flags;
+    uint32_t want;
+    __device__ __forceinline__ bool skip(uint64_t i) const { return (__ldcs(flags + i) != 0) != (want != 0); }
+};
+constexpr uint16_t kSkipPos = 0xFFFF;
 
 // Fused push of the multi-GPU exchange (transport p2p): the staged runs of k_bscatter
 // are stored straight into the receive windows of their owners (peer memory mapped
@@ -174,16 +190,17 @@ __global__ void __launch_bounds__(kBucketThreads) k_bhist(const void* __restrict
             const uint64_t i = base + uint64_t(PER) * (uint64_t(r) * kBucketThreads + threadIdx.x);
             if (i + PER <= n) {
                 if (Key::kKind == 2) {
-                    atomicAdd(&h[pf.of(KeyU64{uint64_t(v[r].x) | (uint64_t(v[r].y) << 32)})], 1u);
-                    atomicAdd(&h[pf.of(KeyU64{uint64_t(v[r].z) | (uint64_t(v[r].w) << 32)})], 1u);
+                    if (!pf.skip(i)) atomicAdd(&h[pf.of(KeyU64{uint64_t(v[r].x) | (uint64_t(v[r].y) << 32)})], 1u);
+                    if (!pf.skip(i + 1)) atomicAdd(&h[pf.of(KeyU64{uint64_t(v[r].z) | (uint64_t(v[r].w) << 32)})], 1u);
                 } else {
-                    atomicAdd(&h[pf.of(KeyU32{v[r].x})], 1u);
-                    atomicAdd(&h[pf.of(KeyU32{v[r].y})], 1u);
-                    atomicAdd(&h[pf.of(KeyU32{v[r].z})], 1u);
-                    atomicAdd(&h[pf.of(KeyU32{v[r].w})], 1u);
+                    if (!pf.skip(i)) atomicAdd(&h[pf.of(KeyU32{v[r].x})], 1u);
+                    if (!pf.skip(i + 1)) atomicAdd(&h[pf.of(KeyU32{v[r].y})], 1u);
+                    if (!pf.skip(i + 2)) atomicAdd(&h[pf.of(KeyU32{v[r].z})], 1u);
+                    if (!pf.skip(i + 3)) atomicAdd(&h[pf.of(KeyU32{v[r].w})], 1u);
                 }
             } else {
-                for (uint64_t e = i; e < n && e < i + PER; e++) atomicAdd(&h[pf.template at<Key>(q, lens, e)], 1u);
+                for (uint64_t e = i; e < n && e < i + PER; e++)
+                    if (!pf.skip(e)) atomicAdd(&h[pf.template at<Key>(q, lens, e)], 1u);
             }
         }
     } else {
@@ -191,7 +208,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bhist(const void* __restrict
 #pragma unroll
         for (int r = 0; r < kBucketItems; r++) {
             const uint64_t i = base + uint64_t(r) * kBucketThreads + threadIdx.x;
-            bk[r] = i < n ? pf.template at<Key>(q, lens, i) : 0xFFFFFFFFu;
+            bk[r] = i < n && !pf.skip(i) ? pf.template at<Key>(q, lens, i) : 0xFFFFFFFFu;
         }
 #pragma unroll
         for (int r = 0; r < kBucketItems; r++)
@@ -262,7 +279,8 @@ static __global__ void __launch_bounds__(kBucketThreads) k_bscan_rows(unsigned i
     if (threadIdx.x == 0) totals[b] = carry;
 }
 
-// totals -> exclusive bucket bases (in place), one CTA of kBuckets threads
+// totals -> exclusive bucket bases (in place), one CTA of kBuckets threads, and the
+// grand total at counts[kBuckets] (so counts needs kBuckets + 1 entries).
 // Only the first nb buckets are in use (256 >> shift): the others count 0 (their
 // totals were never written) and get base = n.
 static __global__ void __launch_bounds__(kBuckets) k_bscan(unsigned int* __restrict__ counts, uint32_t nb) {
@@ -278,6 +296,7 @@ static __global__ void __launch_bounds__(kBuckets) k_bscan(unsigned int* __restr
         __syncthreads();
     }
     counts[t] = s[t] - own;   // exclusive
+    if (t == kBuckets - 1) counts[kBuckets] = s[t];
 }
 
 template <class Key>
@@ -361,7 +380,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
     for (int r = 0; r < kBucketItems; r++) {
         const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
         br[r] = 0xFFFFFFFFu;
-        if (j < cnt) {
+        if (j < cnt && !pf.skip(base + j)) {
             uint32_t b;
             if (Key::kKind == 2) b = pf.of(KeyU64{kv[r]});
             else if (Key::kKind == 1) b = pf.of(KeyU32{uint32_t(kv[r])});
@@ -374,10 +393,15 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
     const unsigned int lb = block_excl_scan256(mine, wtot);
     loc[threadIdx.x] = lb;
     glb[threadIdx.x] = gb - lb;                                        // slot = glb[b] + staged position (mod 2^32)
+    __shared__ unsigned int staged_n;                                  // ops staged (all of them unless filtered)
+    if (threadIdx.x == kBucketThreads - 1) staged_n = lb + mine;
     __syncthreads();
+    const uint32_t scnt = PF::kFilter ? staged_n : cnt;
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
         const uint32_t jt = uint32_t(r) * kBucketThreads + threadIdx.x;   // tile-local op position
+        if (PF::kFilter && !OPS && br[r] == 0xFFFFFFFFu && jt < cnt)
+            __stcs((unsigned short*)jpos + base + jt, (unsigned short)kSkipPos);
         if (br[r] != 0xFFFFFFFFu) {
             const uint32_t b = br[r] >> 16, rk = br[r] & 0xFFFFu;
             const uint32_t j = loc[b] + rk;                            // position in the staged tile
@@ -401,7 +425,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
 #pragma unroll 4
         for (int r = 0; r < kBucketItems; r++) {
             const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
-            if (j >= cnt) continue;
+            if (j >= scnt) continue;
             const uint32_t b = sb[j];
             const uint64_t dsend = uint64_t(glb[b] + j);                  // send-order slot
             const uint32_t w0 = pd.nrep ? 0u : (b >> pd.lbpo), w1 = pd.nrep ? pd.nrep : w0 + 1;
@@ -426,7 +450,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bscatter(const void* __restr
 #pragma unroll 4
     for (int r = 0; r < kBucketItems; r++) {
         const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
-        if (j < cnt) {
+        if (j < scnt) {
             const uint64_t dst = uint64_t(glb[sb[j]] + j);                // n < 2^32: exact
             if (KS == 8) __stcs((unsigned long long*)bq + dst, (unsigned long long)((const uint64_t*)skeys)[j]);
             else if (KS == 4) __stcs((unsigned int*)bq + dst, ((const uint32_t*)skeys)[j]);
@@ -464,12 +488,15 @@ __device__ __forceinline__ void cp_async_wait_all() {
 // ms per 2^30 against 4.19 ms with register staging, tools/bucket_micro.cu), then
 // out[i] = smem[jpos[i]] (coalesced).
 // SEG: out is ignored and result i goes to so.at(i) (fused return to the requesting GPUs).
-template <bool SEG = false>
+// FILT: the batch was bucketed with a filtered part function: only nkept of its n ops
+// were staged; a skipped op (jpos == kSkipPos) gets CUART_MISS.
+template <bool SEG = false, bool FILT = false>
 __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __restrict__ res,
                                                             const uint16_t* __restrict__ jpos, uint64_t n,
                                                             const unsigned int* __restrict__ rowoff,
                                                             const unsigned int* __restrict__ bases,
-                                                            uint64_t* __restrict__ out, SegOut so = SegOut{}) {
+                                                            uint64_t* __restrict__ out, SegOut so = SegOut{},
+                                                            uint64_t nkept = 0) {
     __shared__ uint64_t sres[kBucketTile];
     __shared__ uint8_t bof[kBucketTile];                               // bucket of each staged position
     __shared__ unsigned int loc[kBuckets];
@@ -481,7 +508,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __re
     const int b = threadIdx.x;
     const unsigned int off = rowoff[hidx(b, t)];
     const unsigned int bb = bases[b];
-    const unsigned int bnext = b + 1 < kBuckets ? bases[b + 1] : unsigned(n);
+    const unsigned int bnext = b + 1 < kBuckets ? bases[b + 1] : unsigned(FILT ? nkept : n);
     const unsigned int next = t + 1 < tiles ? rowoff[hidx(b, t + 1)] : bnext - bb;
     uint16_t jp[kBucketItems];
 #pragma unroll
@@ -494,11 +521,14 @@ __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __re
     const unsigned int l_b = block_excl_scan256(c_b, wtot);
     loc[b] = l_b;
     for (unsigned int k = 0; k < c_b; k++) bof[l_b + k] = uint8_t(b);
+    __shared__ unsigned int staged_n;
+    if (FILT && b == kBuckets - 1) staged_n = l_b + c_b;
     __syncthreads();
+    const uint32_t scnt = FILT ? staged_n : cnt;
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
         const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
-        if (j < cnt) {
+        if (j < scnt) {
             const uint32_t bj = bof[j];
             cp_async8(&sres[j], res + glb[bj] + (j - loc[bj]));
         }
@@ -510,7 +540,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_bgather(const uint64_t* __re
         const uint32_t k = uint32_t(r) * kBucketThreads + threadIdx.x;
         if (k < cnt) {
             unsigned long long* dst = SEG ? (unsigned long long*)so.at(base + k) : (unsigned long long*)out + base + k;
-            __stcs(dst, (unsigned long long)sres[jp[r]]);
+            __stcs(dst, FILT && jp[r] == kSkipPos ? ~0ull : (unsigned long long)sres[jp[r]]);
         }
     }
 }

@@ -424,7 +424,7 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
     const size_t ks = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
     auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
     const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
-    const size_t o_hist = 0, o_tot = al(hist_entries(tiles) * 4), o_q = o_tot + 1024, o_len = o_q + al(n * ks),
+    const size_t o_hist = 0, o_tot = al(hist_entries(tiles) * 4), o_q = o_tot + 2048, o_len = o_q + al(n * ks),
                  o_pos = o_len + al(Key::kKind == 3 ? n : 0), o_res = o_pos + al(n * 2), total = o_res + al(n * 8);
     uint8_t* scr = nullptr;
     cuart_status rc = scratch_alloc(h, (void**)&scr, total, s);
@@ -682,7 +682,7 @@ static cuart_status launch_update_bucketed(cuart_index* h, const void* k, const 
     const size_t ks = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
     auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
     const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
-    const size_t o_hist = 0, o_tot = al(hist_entries(tiles) * 4), o_q = o_tot + 1024, o_len = o_q + al(n * ks),
+    const size_t o_hist = 0, o_tot = al(hist_entries(tiles) * 4), o_q = o_tot + 2048, o_len = o_q + al(n * ks),
                  o_val = o_len + al(Key::kKind == 3 ? n : 0), o_idx = o_val + al(n * 8), total = o_idx + al(n * 4);
     uint8_t* scr = nullptr;
     cuart_status rc = scratch_alloc(h, (void**)&scr, total, s);

@@ -114,12 +114,10 @@ __global__ void k_publish(Peers pe, uint32_t slot, const unsigned int* __restric
     Ctrl* c = pe.ctrl[o];
     for (uint32_t k = 0; k < pe.P; k++) {
         unsigned long long v = m;
-        if (!replica && pe.P > 1) {
+        if (!replica) {                                // bases[kBuckets] = ops staged (a filtered pass stages fewer than m)
             const uint64_t b0 = bases[k << lbpo];
-            const uint64_t b1 = k + 1 < pe.P ? uint64_t(bases[(k + 1) << lbpo]) : m;
-            v = b1 - b0;
-        } else if (!replica) {
-            v = m;
+            const uint64_t b1 = k + 1 < pe.P ? uint64_t(bases[(k + 1) << lbpo]) : uint64_t(bases[kBuckets]);
+            v = m ? b1 - b0 : 0;
         }
         c->cnt[slot][pe.me][k] = v;
     }
@@ -183,13 +181,13 @@ __global__ void k_row(const unsigned int* __restrict__ bases, uint64_t m, uint32
                       unsigned long long* __restrict__ row) {
     const uint32_t o = threadIdx.x;
     if (o >= P) return;
-    if (replica || P == 1) {
+    if (replica) {
         row[o] = m;
         return;
     }
     const uint64_t b0 = bases[o << lbpo];
-    const uint64_t b1 = o + 1 < P ? uint64_t(bases[(o + 1) << lbpo]) : m;
-    row[o] = b1 - b0;
+    const uint64_t b1 = o + 1 < P ? uint64_t(bases[(o + 1) << lbpo]) : uint64_t(bases[kBuckets]);
+    row[o] = m ? b1 - b0 : 0;
 }
 
 struct WinHandle {            // one exported device allocation
@@ -404,9 +402,17 @@ Peers peers_of(const DistState* d) {
 
 // ---------------------------------------------------------------- source side: K-BUCKET by (owner, bucket)
 // Histogram + scans of chunk `slot` of m ops at q (send order = part order).
+FilteredOwnerPart filtered(const DistState* d, const uint8_t* flags, uint32_t want) {
+    FilteredOwnerPart f;
+    static_cast<OwnerPart&>(f) = d->part;
+    f.flags = flags;
+    f.want = want;
+    return f;
+}
+
 template <class Key>
 cuart_status front_bucket(cuart_index* h, DistState* d, uint32_t slot, const void* q, const uint8_t* lens, uint64_t m,
-                          cudaStream_t s) {
+                          cudaStream_t s, const uint8_t* flags = nullptr, uint32_t want = 0) {
     if (m == 0) return CUART_OK;
     const uint64_t tiles = (m + kBucketTile - 1) / kBucketTile;
     const bool replica = d->mode == CUART_DIST_REPLICA;
@@ -417,6 +423,10 @@ cuart_status front_bucket(cuart_index* h, DistState* d, uint32_t slot, const voi
     if (replica) {
         if (vec) k_bhist<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, m, ByteBucket(depth), d->hist[slot]);
         else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, m, ByteBucket(depth), d->hist[slot]);
+    } else if (flags) {
+        const FilteredOwnerPart fp = filtered(d, flags, want);
+        if (vec) k_bhist<Key, true, FilteredOwnerPart><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, m, fp, d->hist[slot]);
+        else k_bhist<Key, false, FilteredOwnerPart><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, m, fp, d->hist[slot]);
     } else {
         if (vec) k_bhist<Key, true, OwnerPart><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, m, d->part, d->hist[slot]);
         else k_bhist<Key, false, OwnerPart><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, m, d->part, d->hist[slot]);
@@ -432,7 +442,8 @@ cuart_status front_bucket(cuart_index* h, DistState* d, uint32_t slot, const voi
 // send buffer (NCCL).  OPS: values and priorities travel with the keys.
 template <class Key, bool OPS>
 cuart_status front_scatter(cuart_index* h, DistState* d, uint32_t slot, const void* q, const uint8_t* lens,
-                           const uint64_t* vals, uint64_t m, uint32_t prio_base, cudaStream_t s) {
+                           const uint64_t* vals, uint64_t m, uint32_t prio_base, cudaStream_t s,
+                           const uint8_t* flags = nullptr, uint32_t want = 0) {
     if (m == 0) return CUART_OK;
     const uint64_t tiles = (m + kBucketTile - 1) / kBucketTile;
     const bool replica = d->mode == CUART_DIST_REPLICA;
@@ -455,6 +466,10 @@ cuart_status front_scatter(cuart_index* h, DistState* d, uint32_t slot, const vo
             k_bscatter<Key, OPS, ByteBucket, true><<<T, kBucketThreads, smem, s>>>(
                 q, lens, m, ByteBucket(depth), d->hist[slot], d->tot[slot], nullptr, nullptr, d->jpos[slot], vals, nullptr,
                 nullptr, prio_base, pd);
+        else if (flags)
+            k_bscatter<Key, OPS, FilteredOwnerPart, true><<<T, kBucketThreads, smem, s>>>(
+                q, lens, m, filtered(d, flags, want), d->hist[slot], d->tot[slot], nullptr, nullptr, d->jpos[slot], vals,
+                nullptr, nullptr, prio_base, pd);
         else
             k_bscatter<Key, OPS, OwnerPart, true><<<T, kBucketThreads, smem, s>>>(
                 q, lens, m, d->part, d->hist[slot], d->tot[slot], nullptr, nullptr, d->jpos[slot], vals, nullptr, nullptr,
@@ -464,6 +479,11 @@ cuart_status front_scatter(cuart_index* h, DistState* d, uint32_t slot, const vo
             k_bscatter<Key, OPS, ByteBucket, false><<<T, kBucketThreads, smem, s>>>(
                 q, lens, m, ByteBucket(depth), d->hist[slot], d->tot[slot], d->buf[B_SEND][slot], d->buf[B_SENDL][slot],
                 d->jpos[slot], vals, (uint64_t*)d->buf[B_SENDV][slot], (uint32_t*)d->buf[B_SENDP][slot], prio_base);
+        else if (flags)
+            k_bscatter<Key, OPS, FilteredOwnerPart, false><<<T, kBucketThreads, smem, s>>>(
+                q, lens, m, filtered(d, flags, want), d->hist[slot], d->tot[slot], d->buf[B_SEND][slot],
+                d->buf[B_SENDL][slot], d->jpos[slot], vals, (uint64_t*)d->buf[B_SENDV][slot],
+                (uint32_t*)d->buf[B_SENDP][slot], prio_base);
         else
             k_bscatter<Key, OPS, OwnerPart, false><<<T, kBucketThreads, smem, s>>>(
                 q, lens, m, d->part, d->hist[slot], d->tot[slot], d->buf[B_SEND][slot], d->buf[B_SENDL][slot],
@@ -476,6 +496,10 @@ cuart_status front_scatter(cuart_index* h, DistState* d, uint32_t slot, const vo
 
 template <class Key, bool OPS>
 void set_scatter_smem() {
+    cudaFuncSetAttribute(k_bscatter<Key, OPS, FilteredOwnerPart, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         int(bscatter_smem<Key, OPS>()));
+    cudaFuncSetAttribute(k_bscatter<Key, OPS, FilteredOwnerPart, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         int(bscatter_smem<Key, OPS>()));
     cudaFuncSetAttribute(k_bscatter<Key, OPS, ByteBucket, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          int(bscatter_smem<Key, OPS>()));
     cudaFuncSetAttribute(k_bscatter<Key, OPS, OwnerPart, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -494,6 +518,8 @@ struct Call {
     uint64_t* out;            // lookups
     uint64_t n;
     bool update;
+    const uint8_t* flags = nullptr;   // mixed batch: op i is an update iff flags[i] != 0; this pass
+                                      // serves the updates (update) or the lookups (!update) only
 };
 
 template <class Key>
@@ -503,12 +529,14 @@ cuart_status front(cuart_index* h, DistState* d, const Call& c, uint64_t ci, uns
     const uint64_t m = b0 < c.n ? std::min<uint64_t>(d->chunk, c.n - b0) : 0;
     const void* q = (const uint8_t*)c.q + b0 * d->ks;
     const uint8_t* l = c.lens ? c.lens + b0 : nullptr;
+    const uint8_t* fl = c.flags ? c.flags + b0 : nullptr;
+    const uint32_t want = c.update ? 1u : 0u;
     const bool replica = d->mode == CUART_DIST_REPLICA;
     cudaStream_t s = d->S;
-    cuart_status rc = front_bucket<Key>(h, d, slot, q, l, m, s);
+    cuart_status rc = front_bucket<Key>(h, d, slot, q, l, m, s, fl, want);
     if (rc != CUART_OK) return rc;
     // tot[slot] holds the send-order bases (k_bscan); an empty chunk has none
-    if (m == 0) D_TRY(cudaMemsetAsync(d->tot[slot], 0, kBuckets * 4, s));
+    if (m == 0) D_TRY(cudaMemsetAsync(d->tot[slot], 0, (kBuckets + 1) * 4, s));
     const uint32_t prio_base = uint32_t(uint64_t(d->rank) * ((uint64_t(1) << 32) / d->P) + b0);
     if (d->transport == CUART_TRANSPORT_P2P) {
         const Peers pe = peers_of(d);
@@ -517,8 +545,8 @@ cuart_status front(cuart_index* h, DistState* d, const Call& c, uint64_t ci, uns
                                        replica ? 1u : 0u, d->adj[slot], d->hmat + slot * (size_t(d->P) * d->P + 1));
         g_cuart_launches += 2;
         D_TRY(cudaGetLastError());
-        if (c.update) rc = front_scatter<Key, true>(h, d, slot, q, l, c.vals + b0, m, prio_base, s);
-        else rc = front_scatter<Key, false>(h, d, slot, q, l, nullptr, m, 0, s);
+        if (c.update) rc = front_scatter<Key, true>(h, d, slot, q, l, c.vals + b0, m, prio_base, s, fl, want);
+        else rc = front_scatter<Key, false>(h, d, slot, q, l, nullptr, m, 0, s, fl, want);
         if (rc != CUART_OK) return rc;
         k_signal<<<1, 32, 0, s>>>(pe, F_PUSH, seq);
         g_cuart_launches++;
@@ -526,8 +554,8 @@ cuart_status front(cuart_index* h, DistState* d, const Call& c, uint64_t ci, uns
         return CUART_OK;
     }
     // NCCL: scatter into the local send buffer, then the counts
-    if (c.update) rc = front_scatter<Key, true>(h, d, slot, q, l, c.vals + b0, m, prio_base, s);
-    else rc = front_scatter<Key, false>(h, d, slot, q, l, nullptr, m, 0, s);
+    if (c.update) rc = front_scatter<Key, true>(h, d, slot, q, l, c.vals + b0, m, prio_base, s, fl, want);
+    else rc = front_scatter<Key, false>(h, d, slot, q, l, nullptr, m, 0, s, fl, want);
     if (rc != CUART_OK) return rc;
     k_row<<<1, 32, 0, s>>>(d->tot[slot], m, d->P, d->lbpo, replica ? 1u : 0u, d->row);
     g_cuart_launches++;
@@ -624,7 +652,8 @@ cuart_status owner(cuart_index* h, DistState* d, const Call& c, uint64_t ci, uns
 }
 
 // Source role, after the owners: wait for the results (P2P), gather into query order.
-cuart_status back(cuart_index* h, DistState* d, const Call& c, uint64_t ci, unsigned long long seq) {
+cuart_status back(cuart_index* h, DistState* d, const Call& c, uint64_t ci, unsigned long long seq,
+                  const unsigned long long* M) {
     (void)h;
     const uint32_t slot = uint32_t(ci & 1);
     const uint64_t b0 = ci * d->chunk;
@@ -636,8 +665,17 @@ cuart_status back(cuart_index* h, DistState* d, const Call& c, uint64_t ci, unsi
     }
     if (!c.update && m) {
         const uint64_t tiles = (m + kBucketTile - 1) / kBucketTile;
-        k_bgather<false><<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint64_t*)d->buf[B_RES][slot], d->jpos[slot],
-                                                                   m, d->hist[slot], d->tot[slot], c.out + b0);
+        if (c.flags) {                                // a mixed batch's lookups: update ops get CUART_MISS
+            uint64_t kept = 0;
+            for (uint32_t o = 0; o < d->P; o++) kept += M[uint64_t(d->rank) * d->P + o];
+            k_bgather<false, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(
+                (const uint64_t*)d->buf[B_RES][slot], d->jpos[slot], m, d->hist[slot], d->tot[slot], c.out + b0,
+                SegOut{}, kept);
+        } else {
+            k_bgather<false><<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint64_t*)d->buf[B_RES][slot],
+                                                                       d->jpos[slot], m, d->hist[slot], d->tot[slot],
+                                                                       c.out + b0);
+        }
         g_cuart_launches++;
     }
     D_TRY(cudaGetLastError());
@@ -693,7 +731,7 @@ cuart_status run_call(cuart_index* h, DistState* d, const Call& c) {
         for (uint64_t ci = 0; ci < nc && rc == CUART_OK; ci++) {
             rc = front<Key>(h, d, c, ci, base + 1 + ci);
             if (rc == CUART_OK) rc = owner(h, d, c, ci, base + 1 + ci, d->hrow);
-            if (rc == CUART_OK) rc = back(h, d, c, ci, base + 1 + ci);
+            if (rc == CUART_OK) rc = back(h, d, c, ci, base + 1 + ci, d->hrow);
         }
     } else {
         rc = front<Key>(h, d, c, 0, base + 1);
@@ -705,7 +743,7 @@ cuart_status run_call(cuart_index* h, DistState* d, const Call& c) {
             DBG("rank %d chunk %llu matrix rc %d", d->rank, (unsigned long long)ci, int(rc));
             if (rc != CUART_OK) break;
             rc = owner(h, d, c, ci, base + 1 + ci, d->hmat + slot * (size_t(P) * P + 1));
-            if (rc == CUART_OK) rc = back(h, d, c, ci, base + 1 + ci);
+            if (rc == CUART_OK) rc = back(h, d, c, ci, base + 1 + ci, d->hmat + slot * (size_t(P) * P + 1));
         }
     }
     h->hold_epoch = false;
@@ -713,7 +751,7 @@ cuart_status run_call(cuart_index* h, DistState* d, const Call& c) {
 }
 
 cuart_status dist_call(cuart_index* h, const cuart_keys* k, const uint64_t* vals, uint64_t* out, size_t n, void* stream,
-                       bool update) {
+                       bool update, const uint8_t* flags = nullptr) {
     if (!h || !h->dist || !k) return CUART_ERR_INVALID_ARGUMENT;
     DistState* d = h->dist;
     if (d->failed) return CUART_ERR_INTERNAL;
@@ -727,6 +765,23 @@ cuart_status dist_call(cuart_index* h, const cuart_keys* k, const uint64_t* vals
     D_TRY(cudaEventRecord(d->ev_in, us));
     D_TRY(cudaStreamWaitEvent(d->S, d->ev_in, 0));
     D_TRY(cudaStreamWaitEvent(d->O, d->ev_in, 0));
+    if (flags) {                                    // a mixed round: all lookups, then all updates (reading C7)
+        if (d->mode != CUART_DIST_RANGE || (n > 0 && (!vals || !out))) return CUART_ERR_INVALID_ARGUMENT;
+        Call cl{k->data, k->lengths, nullptr, out, uint64_t(n), false, flags};
+        Call cu{k->data, k->lengths, vals, nullptr, uint64_t(n), true, flags};
+        cuart_status rc;
+        switch (h->key_kind) {
+        case CUART_KEY_U64: rc = run_call<KeyU64>(h, d, cl); if (rc == CUART_OK) rc = run_call<KeyU64>(h, d, cu); break;
+        case CUART_KEY_U32: rc = run_call<KeyU32>(h, d, cl); if (rc == CUART_OK) rc = run_call<KeyU32>(h, d, cu); break;
+        default: rc = run_call<KeyBytes>(h, d, cl); if (rc == CUART_OK) rc = run_call<KeyBytes>(h, d, cu); break;
+        }
+        if (rc != CUART_OK) d->failed = true;
+        D_TRY(cudaEventRecord(d->ev_s, d->S));
+        D_TRY(cudaEventRecord(d->ev_o, d->O));
+        D_TRY(cudaStreamWaitEvent(us, d->ev_s, 0));
+        D_TRY(cudaStreamWaitEvent(us, d->ev_o, 0));
+        return rc;
+    }
     Call c{k->data, k->lengths, vals, out, uint64_t(n), update};
     if (!update && d->mode == CUART_DIST_REPLICA) {   // replicas: served locally, no exchange
         cuart_status rc = launch_lookup(h, h->key_kind, k->data, k->lengths, n, out, d->S);
@@ -773,7 +828,7 @@ cuart_status setup_buffers(cuart_index* h, DistState* d) {
     for (int sl = 0; sl < 2; sl++) {
         if ((rc = dalloc(d, &p, hist_entries(tiles) * 4)) != CUART_OK) return rc;
         d->hist[sl] = (unsigned int*)p;
-        if ((rc = dalloc(d, &p, 1024)) != CUART_OK) return rc;
+        if ((rc = dalloc(d, &p, 2048)) != CUART_OK) return rc;
         d->tot[sl] = (unsigned int*)p;
         if ((rc = dalloc(d, &p, C * 2)) != CUART_OK) return rc;
         d->jpos[sl] = (uint16_t*)p;
@@ -1058,6 +1113,13 @@ cuart_status cuart_dist_lookup(cuart_index* h, const cuart_keys* q, size_t n, ui
 
 cuart_status cuart_dist_update(cuart_index* h, const cuart_keys* k, const uint64_t* v, size_t n, void* stream) {
     return dist_call(h, k, v, nullptr, n, stream, true);
+}
+
+cuart_status cuart_dist_mixed(cuart_index* h, const cuart_keys* k, const uint64_t* v, const uint8_t* is_update, size_t n,
+                              uint64_t* out, void* stream) {
+    if (n > 0 && !is_update) return CUART_ERR_INVALID_ARGUMENT;
+    static const uint8_t none = 0;
+    return dist_call(h, k, v, out, n, stream, false, n ? is_update : &none);
 }
 
 cuart_status cuart_dist_last(const cuart_index* h, uint64_t* recv_ops, uint64_t* chunks) {

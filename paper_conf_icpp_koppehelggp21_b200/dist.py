@@ -49,7 +49,7 @@ def _sig(L):
     for name, args in {"cuart_dist_unique_id": [P], "cuart_dist_build": [P, P, P, S, P],
                        "cuart_dist_lookup": [P, P, S, P, P], "cuart_dist_update": [P, P, P, S, P],
                        "cuart_dist_partition": [P, P, S, P, P], "cuart_dist_chunk_plan": [U32, U32, P, P, P, P],
-                       "cuart_dist_last": [P, P, P]}.items():
+                       "cuart_dist_last": [P, P, P], "cuart_dist_mixed": [P, P, P, P, S, P, P]}.items():
         f = getattr(L, name)
         if f.argtypes is None:
             f.argtypes = args
@@ -234,12 +234,26 @@ class DistIndex:
         B._check(lib().cuart_dist_update(self.h, ctypes.byref(k), values.data_ptr(), n, B._stream_ptr(stream)),
                  "cuart_dist_update")
 
-    def mixed_round(self, keys, values, is_update, lens=None, stream=None, events=None):
+    def mixed_round(self, keys, values, is_update, lens=None, stream=None, events=None, fused=True):
         """One round of a mixed op stream (reading C7): every lookup sees the state
         before the round; the round's updates then apply in global (rank-major, op)
         order.  Returns per op the lookup result, CUART_MISS for update ops.
-        events: optional 5 CUDA events recorded on the stream around the four calls
-        (partition, lookup, update, unroute) -- measurement only."""
+        Range mode: one cuart_dist_mixed call (each pass filters its op kind).
+        Replica mode (or fused=False): cuart_partition_by_flag, cuart_dist_lookup,
+        cuart_dist_update, cuart_unroute; events: optional 5 CUDA events recorded
+        around those four calls -- measurement only."""
+        if fused and self.mode == "range":
+            kk, n, keep = B.make_keys((keys, lens) if lens is not None else keys)
+            out = torch.empty(n, dtype=torch.int64, device=keys.device)
+            B._check_dev(values, self.device, "values")
+            B._check_dev(is_update, self.device, "is_update")
+            if events:
+                events[0].record()
+            B._check(lib().cuart_dist_mixed(self.h, ctypes.byref(kk), values.data_ptr(), is_update.data_ptr(), n,
+                                            out.data_ptr(), B._stream_ptr(stream)), "cuart_dist_mixed")
+            if events:
+                events[-1].record()
+            return out
         rec = (lambda i: events[i].record()) if events else (lambda i: None)
         rec(0)
         n = keys.shape[0]

@@ -144,11 +144,13 @@ def _len(k):
     return k[1].shape[0] if isinstance(k, tuple) else k.shape[0]
 
 
+@pytest.mark.parametrize("fused", [True, False])
 @pytest.mark.parametrize("P", [1, 2, 4])
-def test_dist_mixed_rounds_p_independent(P):
+def test_dist_mixed_rounds_p_independent(P, fused):
     """Config 5's recipe (reading C7) at 2^16 keys: rounds of mixed ops, rank r
     originating the r-th 1/P slice of each round; outputs equal the single-stream
-    oracle replay, so they do not depend on P."""
+    oracle replay, so they do not depend on P.  fused: one cuart_dist_mixed call per
+    round (filtered passes); else partition + dist lookup + dist update + unroute."""
     n, R, rounds = 1 << 16, 1 << 17, 3
     keys = W.u64_keys(5, n)
     vals = W.values_for(W.SEED_VALUES + 5, np.arange(n, dtype=np.uint64))
@@ -159,7 +161,7 @@ def test_dist_mixed_rounds_p_independent(P):
         outs = []
         for rd in range(rounds):
             k, u, v = W.mixed_ops_torch(5, n, rd * R + r * per, per, DEV)
-            outs.append(_u64(di.mixed_round(k, v, u)))
+            outs.append(_u64(di.mixed_round(k, v, u, fused=fused)))
         di.close()
         return np.concatenate(outs)
 
