@@ -33,7 +33,10 @@
  *    only enqueue work on `stream` (a cudaStream_t passed as void*, NULL =
  *    legacy default stream) and never synchronise the host.
  *    cuart_lookup_host / cuart_update_host take HOST pointers (pinned for full
- *    speed) and run a chunked H2D -> kernel -> D2H pipeline; they return when
+ *    speed) and run a chunked H2D -> kernel -> D2H pipeline on the index's own
+ *    streams; they start after every operation already queued on the legacy
+ *    default stream (and so on every blocking stream) -- work on other
+ *    non-blocking streams must be synchronised by the caller -- and return when
  *    the results are in host memory.
  *  - Ordering: lookups may run concurrently on several streams; updates on
  *    one index must not overlap each other (the conflict scratch is per index).

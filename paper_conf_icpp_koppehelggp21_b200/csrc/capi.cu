@@ -1224,6 +1224,7 @@ cuart_status cuart_destroy(cuart_index* h) {
         if (h->ev_free[i]) cudaEventDestroy(h->ev_free[i]);
     }
     if (h->ustream) cudaStreamDestroy(h->ustream);
+    if (h->ev_join) cudaEventDestroy(h->ev_join);
     if (h->pool) cudaMemPoolDestroy(h->pool);   // every scratch block was freed in stream order
     delete h;
     return CUART_OK;
@@ -1491,6 +1492,18 @@ static cuart_status ensure_stage(cuart_index* h) {
 }
 
 static size_t key_stride(uint32_t kind) { return kind == CUART_KEY_U64 ? 8 : kind == CUART_KEY_U32 ? 4 : 32; }
+
+// The host pipelines run on the index's own non-blocking streams, which do not
+// synchronise with the legacy default stream: order them after every operation
+// already queued there (and, through the legacy stream's implicit synchronisation,
+// on every blocking stream), e.g. a cuart_update(h, ..., NULL) just before.
+static cuart_status join_legacy_stream(cuart_index* h) {
+    if (!h->ev_join) CU_TRY(cudaEventCreateWithFlags(&h->ev_join, cudaEventDisableTiming));
+    CU_TRY(cudaEventRecord(h->ev_join, 0));
+    for (int i = 0; i < kStages; i++) CU_TRY(cudaStreamWaitEvent(h->streams[i], h->ev_join, 0));
+    CU_TRY(cudaStreamWaitEvent(h->ustream, h->ev_join, 0));
+    return CUART_OK;
+}
 // ops per host-pipeline chunk: kStageChunk, or CUART_STAGE_CHUNK read when the
 // handle's staging buffers are first allocated (a tuning / test knob)
 static size_t stage_chunk() {
@@ -1507,6 +1520,7 @@ cuart_status cuart_lookup_host(const cuart_index* hc, const cuart_keys* q, size_
     if (!out) return CUART_ERR_INVALID_ARGUMENT;
     CU_TRY(cudaSetDevice(h->device));
     if ((rc = ensure_stage(h)) != CUART_OK) return rc;
+    if ((rc = join_legacy_stream(h)) != CUART_OK) return rc;
     const size_t ks = key_stride(h->key_kind);
     size_t c = 0;
     const size_t chunk = h->stage_cap;
@@ -1531,6 +1545,7 @@ cuart_status cuart_update_host(cuart_index* h, const cuart_keys* k, const uint64
     if (!v) return CUART_ERR_INVALID_ARGUMENT;
     CU_TRY(cudaSetDevice(h->device));
     if ((rc = ensure_stage(h)) != CUART_OK) return rc;
+    if ((rc = join_legacy_stream(h)) != CUART_OK) return rc;
     const size_t ks = key_stride(h->key_kind);
     // The kernels of all chunks run in op order on ONE stream (sequential semantics
     // across chunks); the H2D copies of the next chunks run on the staging sets' own

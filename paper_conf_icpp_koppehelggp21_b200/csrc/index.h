@@ -64,6 +64,7 @@ struct cuart_index {
     size_t stage_cap = 0;
     cudaStream_t streams[4] = {nullptr, nullptr, nullptr, nullptr};   // host-pipeline streams
     cudaStream_t ustream = nullptr;                                   // update pipeline: the kernels, in op order
+    cudaEvent_t ev_join = nullptr;                                    // host pipelines start after the legacy stream
     cudaEvent_t ev_copied[4] = {nullptr, nullptr, nullptr, nullptr};  // staging set s filled
     cudaEvent_t ev_free[4] = {nullptr, nullptr, nullptr, nullptr};    // staging set s consumed
     int policy = 5;                    // cache-policy variant of the kernels (kernels.cuh Loader)

@@ -613,3 +613,26 @@ def test_epoch_wrap(prebucket):
         o.update(uk, uv)
         assert np.array_equal(_lookup(ix, keys), o.lookup(keys)), b
     ix.close()
+
+
+def test_host_pipeline_orders_after_async_update():
+    """the host-buffer calls run on the index's non-blocking streams; an
+    asynchronous cuart_update enqueued just before on the legacy stream must be
+    visible to them (they join the legacy stream at entry)."""
+    cfg = W.CONFIGS["c1"]
+    keys, vals = W.build_set(cfg)
+    ix = C.Index(keys, vals, lut_bytes=3)
+    o = MapOracle(keys, vals)
+    for rep in range(3):
+        uk, uv = W.update_batch(cfg, keys, rep * 100_000, 100_000)
+        ix.update(_t(uk), _t(uv), stream=0)           # async, legacy stream, no synchronisation
+        o.update(uk, uv)
+        assert np.array_equal(ix.lookup_host(keys), o.lookup(keys)), rep
+        uk2, uv2 = W.update_batch(cfg, keys, 10**6 + rep * 50_000, 50_000)
+        ix.update_host(uk2, uv2)
+        o.update(uk2, uv2)
+    out = torch.empty(keys.shape[0], dtype=torch.int64, device=DEV)
+    ix.lookup(_t(keys), out, stream=0)
+    torch.cuda.synchronize()
+    assert np.array_equal(_u64(out), o.lookup(keys))
+    ix.close()
