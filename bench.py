@@ -65,7 +65,7 @@ def _args():
                         "nccl = route + all-to-all")
     p.add_argument("--l2-persist", type=int, default=0,
                    help="cuart_build_opts.l2_persist: persisting L2 window over the root tables")
-    p.add_argument("--c5-fused", type=int, default=1,
+    p.add_argument("--c5-fused", type=int, default=0,
                    help="c5 rounds through cuart_dist_mixed (1) or partition + lookup + update + unroute (0)")
     p.add_argument("--c5-share", type=int, default=0,
                    help="c5 on one GPU: the per-GPU share of a P-GPU run (rank 0's keys and owned ops)")

@@ -234,14 +234,15 @@ class DistIndex:
         B._check(lib().cuart_dist_update(self.h, ctypes.byref(k), values.data_ptr(), n, B._stream_ptr(stream)),
                  "cuart_dist_update")
 
-    def mixed_round(self, keys, values, is_update, lens=None, stream=None, events=None, fused=True):
+    def mixed_round(self, keys, values, is_update, lens=None, stream=None, events=None, fused=False):
         """One round of a mixed op stream (reading C7): every lookup sees the state
         before the round; the round's updates then apply in global (rank-major, op)
         order.  Returns per op the lookup result, CUART_MISS for update ops.
-        Range mode: one cuart_dist_mixed call (each pass filters its op kind).
-        Replica mode (or fused=False): cuart_partition_by_flag, cuart_dist_lookup,
-        cuart_dist_update, cuart_unroute; events: optional 5 CUDA events recorded
-        around those four calls -- measurement only."""
+        Default: cuart_partition_by_flag, cuart_dist_lookup, cuart_dist_update,
+        cuart_unroute (events: optional 5 CUDA events recorded around those four
+        calls -- measurement only).  fused=True (range mode): one cuart_dist_mixed
+        call whose two passes filter their op kind -- measured slower on c5
+        (DESIGN.md §10), kept as an API."""
         if fused and self.mode == "range":
             kk, n, keep = B.make_keys((keys, lens) if lens is not None else keys)
             out = torch.empty(n, dtype=torch.int64, device=keys.device)

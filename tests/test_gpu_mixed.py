@@ -85,7 +85,7 @@ def test_c5_full_size_rounds():
     outs = []
     for rnd in range(2):
         k, u, v = W.mixed_ops_torch(5, n, rnd * R, R, DEV)
-        outs.append(di.mixed_round(k, v, u))
+        outs.append(di.mixed_round(k, v, u, fused=rnd == 1))      # round 1 through cuart_dist_mixed
         del k, u, v
     rng = np.random.default_rng(55)
     probe = np.sort(rng.choice(n, 1_000_000, replace=False))
