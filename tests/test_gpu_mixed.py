@@ -54,16 +54,19 @@ def _c5_keys(n, dev, chunk=1 << 27):
     return torch.cat(ks).numpy().view(np.uint64), torch.cat(vs).numpy().view(np.uint64)
 
 
-def _c5_updates_on(keyset, rnd, n, R, chunk=1 << 25):
+def _c5_updates_on(keyset, rnd, n, R, chunk=1 << 26):
     """(keys, values) of round `rnd`'s update ops whose key is in `keyset` (sorted
-    u64), in global op order -- the only ops of the round that can change those keys."""
+    u64), in global op order -- the only ops of the round that can change those keys.
+    The ops are drawn with the generator's torch twin on the device (pinned bit for
+    bit to the numpy generator, tests/test_workloads.py) and only selected there;
+    the replay itself is the CPU oracle's."""
+    ks_d = torch.from_numpy(keyset.view(np.int64)).to(DEV)
     ks, vs = [], []
     for s0 in range(rnd * R, (rnd + 1) * R, chunk):
-        k, u, v = W.mixed_ops(5, n, np.arange(s0, s0 + chunk, dtype=np.uint64))
-        pos = np.minimum(np.searchsorted(keyset, k), keyset.shape[0] - 1)
-        m = (u == 1) & (keyset[pos] == k)
-        ks.append(k[m])
-        vs.append(v[m])
+        k, u, v = W.mixed_ops_torch(5, n, s0, chunk, DEV)
+        m = (u == 1) & torch.isin(k, ks_d)
+        ks.append(k[m].cpu().numpy().view(np.uint64))
+        vs.append(v[m].cpu().numpy().view(np.uint64))
     return np.concatenate(ks), np.concatenate(vs)
 
 

@@ -76,3 +76,14 @@ def test_mixed_ops_twin_and_mix():
     present = np.isin(k, keys)
     assert present[u == 1].all()                                   # updates target the set
     assert abs(present[u == 0].mean() - 0.5) < 0.02                # lookups: 50% hit
+
+
+def test_torch_helper_twins():
+    """The torch helpers the full-size tests use agree with the numpy generator."""
+    cfg = W.CONFIGS["c4"]
+    n = 30_000
+    idx = W.string_lookup_index_torch(cfg, n, 500, 4000, "cpu", W.zipf_cdf_torch(n, "cpu"),
+                                      W.rank_permutation_torch(cfg, n, "cpu"))
+    assert np.array_equal(idx.numpy(), W.string_lookup_at(cfg, n, np.arange(500, 4500)))
+    v = W.values_torch(W.SEED_VALUES + 5, 123, 5000, "cpu")
+    assert np.array_equal(v.numpy().view(np.uint64), W.values_for(W.SEED_VALUES + 5, np.arange(123, 5123, dtype=np.uint64)))
