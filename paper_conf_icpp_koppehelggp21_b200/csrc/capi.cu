@@ -74,37 +74,6 @@ __global__ void __launch_bounds__(TPB) k_lookup(DevIndex ix, const void* __restr
     }
 }
 
-// The direct walk with two queries per thread (kernels.cuh find_leaf2): query j of
-// the thread is i0 + j * TPB (coalesced key loads and result stores), and the two
-// walks advance in lockstep with their requests in flight together.  Same results
-// as k_lookup.  SEG: result i goes to so.at(i) (multi-GPU owner walk).
-template <class Key, int POL, bool SEG = false, int TPB = 256>
-__global__ void __launch_bounds__(TPB) k_lookup2(DevIndex ix, const void* __restrict__ q,
-                                                 const uint8_t* __restrict__ lens, uint64_t n,
-                                                 uint64_t* __restrict__ out, SegOut so = SegOut{}) {
-    const Loader<POL> ld;
-    const uint64_t i0 = uint64_t(blockIdx.x) * (TPB * 2) + threadIdx.x;
-    Key k[2];
-    uint64_t link[2], leaf[2], val[2];
-#pragma unroll
-    for (int j = 0; j < 2; j++) {
-        const uint64_t i = i0 + uint64_t(j) * TPB;
-        if (i < n) k[j] = Key::template load<POL != 0>(q, lens, i);
-    }
-#pragma unroll
-    for (int j = 0; j < 2; j++) link[j] = i0 + uint64_t(j) * TPB < n ? start_link(ix, ld, k[j]) : 0;
-    find_leaf2(ix, ld, k, link, leaf, val);
-#pragma unroll
-    for (int j = 0; j < 2; j++) {
-        const uint64_t i = i0 + uint64_t(j) * TPB;
-        if (i >= n) continue;
-        const uint64_t r = leaf[j] ? val[j] : kMiss;
-        uint64_t* dst = SEG ? so.at(i) : out + i;
-        if (POL != 0) __stcs((unsigned long long*)dst, (unsigned long long)r);
-        else *dst = r;
-    }
-}
-
 // Pre-bucketed walk from the wide root table with Q queries per thread in lockstep
 // phases (integer keys): all Q keys, then all Q wide entries, then all Q leaf
 // records are requested before any of them is used, so a thread keeps Q
@@ -539,13 +508,7 @@ cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const voi
     if (so) {                                          // fused return: the default policy only
         cudaEvent_t ev0, ev1;
         ktimer_begin(h, s, ev0, ev1);
-        const unsigned g2 = unsigned((n + 511) / 512);
-        if (h->direct_ilp >= 2) switch (kind) {
-        case CUART_KEY_U64: k_lookup2<KeyU64, 5, true><<<g2, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
-        case CUART_KEY_U32: k_lookup2<KeyU32, 5, true><<<g2, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
-        default: k_lookup2<KeyBytes, 5, true><<<g2, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
-        }
-        else switch (kind) {
+        switch (kind) {
         case CUART_KEY_U64: k_lookup<KeyU64, 5, true><<<grid, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
         case CUART_KEY_U32: k_lookup<KeyU32, 5, true><<<grid, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
         default: k_lookup<KeyBytes, 5, true><<<grid, 256, 0, s>>>(dx, q, lens, n, nullptr, *so); break;
@@ -574,18 +537,6 @@ cuart_status launch_lookup_direct(const cuart_index* h, uint32_t kind, const voi
         if (kind == CUART_KEY_U64) { CUART_WQ(KeyU64) } else { CUART_WQ(KeyU32) }
 #undef CUART_WQ
 #undef CUART_WQ_Q
-        g_cuart_launches++;
-        ktimer_end(h, s, ev0, ev1, n);
-        CU_TRY(cudaGetLastError());
-        return CUART_OK;
-    }
-    if (h->direct_ilp >= 2 && h->policy == 5 && n >= (uint64_t(1) << 16)) {   // two walks per thread
-        const unsigned g2 = unsigned((n + 511) / 512);
-        switch (kind) {
-        case CUART_KEY_U64: k_lookup2<KeyU64, 5><<<g2, 256, 0, s>>>(dx, q, lens, n, out); break;
-        case CUART_KEY_U32: k_lookup2<KeyU32, 5><<<g2, 256, 0, s>>>(dx, q, lens, n, out); break;
-        default: k_lookup2<KeyBytes, 5><<<g2, 256, 0, s>>>(dx, q, lens, n, out); break;
-        }
         g_cuart_launches++;
         ktimer_end(h, s, ev0, ev1, n);
         CU_TRY(cudaGetLastError());
@@ -1023,7 +974,6 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     if (const char* pe = getenv("CUART_LOOKUP_TPB")) h->lk_tpb = unsigned(atoi(pe));
     if (const char* pe = getenv("CUART_UPD2_TPB")) h->upd2_tpb = unsigned(atoi(pe));
     if (const char* pe = getenv("CUART_WQ_LEAFPOL")) h->wq_lp = atoi(pe);
-    if (const char* pe = getenv("CUART_DIRECT_ILP")) h->direct_ilp = atoi(pe);
     h->prebucket = opts ? opts->prebucket : CUART_PREBUCKET_AUTO;
     if (h->prebucket > CUART_PREBUCKET_ON) {
         delete h;

@@ -410,178 +410,6 @@ __device__ __forceinline__ uint64_t find_leaf(const DevIndex& ix, const Loader<P
     }
 }
 
-// ----------------------------------------------------------------------------- two walks per thread
-// The direct walk is a chain of dependent loads: a thread that follows one
-// query waits a full memory round trip per node.  find_leaf2 advances TWO queries
-// in lockstep and splits every node step at its dependent load, so the loads of
-// both queries are in flight together: phase A issues each query's first request
-// of its current record (the N256 child slot, the N48 index byte, the N16 keys, the
-// N4 block, the leaf record), phase B consumes it and issues the second request
-// where the node type has one (N48 child, N16 child, N4 child[3]).  Results are
-// those of find_leaf (same loads, same compares).
-struct LeafRaw {
-    U8x32 a;      // first (or only) request
-    uint4 b;      // leaf32: the second request
-};
-
-template <class Key, class LD>
-__device__ __forceinline__ void leaf_load_raw(const LD& ld, const uint8_t* rec, uint32_t t, LeafRaw& r) {
-    if (t == T_LEAF8) {
-        const uint4 v = ld.leafv4(rec);
-        r.a.w[0] = v.x; r.a.w[1] = v.y; r.a.w[2] = v.z; r.a.w[3] = v.w;
-    } else if (t == T_LEAF16) {
-        r.a = ld.leafv8(rec);
-    } else {
-        const bool odd = (uintptr_t(rec) & 16) != 0;
-        r.b = ld.leafv4(odd ? rec : rec + 32);
-        r.a = ld.leafv8(odd ? rec + 16 : rec);
-    }
-}
-
-// The compare of Key::leaf_match on already loaded leaf bytes.
-template <class Key>
-__device__ __forceinline__ bool leaf_cmp_raw(const Key& key, const uint8_t* rec, uint32_t t, uint32_t aux,
-                                             const LeafRaw& r, uint64_t& val) {
-    if (Key::kKind == 2) {
-        val = uint64_t(r.a.w[2]) | (uint64_t(r.a.w[3]) << 32);
-        return aux == 8 && (uint64_t(r.a.w[0]) | (uint64_t(r.a.w[1]) << 32)) == bswap64(((const KeyU64&)key).k);
-    }
-    if (Key::kKind == 1) {
-        val = uint64_t(r.a.w[2]) | (uint64_t(r.a.w[3]) << 32);
-        return aux == 4 && r.a.w[1] == 0 && r.a.w[0] == __byte_perm(((const KeyU32&)key).k, 0, 0x0123);
-    }
-    const KeyBytes& kb = (const KeyBytes&)key;
-    if (t == T_LEAF8) {
-        val = uint64_t(r.a.w[2]) | (uint64_t(r.a.w[3]) << 32);
-        return aux == kb.l && (uint64_t(r.a.w[0]) | (uint64_t(r.a.w[1]) << 32)) == kb.w[0];
-    }
-    if (t == T_LEAF16) {
-        val = uint64_t(r.a.w[4]) | (uint64_t(r.a.w[5]) << 32);
-        return aux == kb.l && (uint64_t(r.a.w[0]) | (uint64_t(r.a.w[1]) << 32)) == kb.w[0] &&
-               (uint64_t(r.a.w[2]) | (uint64_t(r.a.w[3]) << 32)) == kb.w[1];
-    }
-    const bool odd = (uintptr_t(rec) & 16) != 0;
-    uint32_t k[8];
-#pragma unroll
-    for (int j = 0; j < 4; j++) {
-        k[j] = odd ? (&r.b.x)[j] : r.a.w[j];
-        k[4 + j] = odd ? r.a.w[j] : r.a.w[4 + j];
-    }
-    val = odd ? (uint64_t(r.a.w[4]) | (uint64_t(r.a.w[5]) << 32)) : (uint64_t(r.b.x) | (uint64_t(r.b.y) << 32));
-    bool eq = aux == kb.l;
-#pragma unroll
-    for (int j = 0; j < 4; j++) eq &= (uint64_t(k[2 * j]) | (uint64_t(k[2 * j + 1]) << 32)) == kb.w[j];
-    return eq;
-}
-
-// Phase A: first request of the record `link` points to.  Returns false when the
-// walk ends without a request (null link, key too short).
-template <class Key, int POL>
-__device__ __forceinline__ bool walk_a(const DevIndex& ix, const Loader<POL>& ld, const Key& key, uint64_t link,
-                                       LeafRaw& r) {
-    const uint32_t t = link_type(link), aux = link_aux(link);
-    const uint8_t* rec = ix.base[t] + link_index(link) * record_bytes(t);
-    if (t >= T_LEAF8 && t <= T_LEAF32) {
-        leaf_load_raw<Key>(ld, rec, t, r);
-        return true;
-    }
-    if (t == T_NULL || t > T_N256 || aux >= key.len()) return false;
-    const uint32_t b = key.byte(aux);
-    if (t == T_N256) {
-        const uint64_t c = ld.node64(rec + kN256Child + 8 * b);
-        r.a.w[0] = uint32_t(c);
-        r.a.w[1] = uint32_t(c >> 32);
-    } else if (t == T_N48) {
-        r.a.w[0] = ld.node8(rec + kN48Index + b);
-    } else if (t == T_N16) {
-        const uint4 k4 = ld.nodev4(rec + kN16Keys);
-        r.a.w[0] = k4.x; r.a.w[1] = k4.y; r.a.w[2] = k4.z; r.a.w[3] = k4.w;
-    } else {
-        r.a = ld.nodev8(rec);
-    }
-    return true;
-}
-
-// Phase B1: consume the first request.  Returns the address of the second request
-// (a child link), or 0 when the step is complete: then `next` is the next link and
-// `fin` says whether the walk ended (leaf compared, or a miss).
-template <class Key>
-__device__ __forceinline__ const uint8_t* walk_b(const DevIndex& ix, const Key& key, uint64_t link, const LeafRaw& r,
-                                                 uint64_t& next, bool& fin, uint64_t& hit_leaf, uint64_t& val) {
-    const uint32_t t = link_type(link), aux = link_aux(link);
-    const uint8_t* rec = ix.base[t] + link_index(link) * record_bytes(t);
-    fin = false;
-    if (t >= T_LEAF8) {
-        fin = true;
-        hit_leaf = leaf_cmp_raw(key, rec, t, aux, r, val) ? link : 0;
-        return nullptr;
-    }
-    const uint32_t b = key.byte(aux);
-    if (t == T_N256) {
-        next = uint64_t(r.a.w[0]) | (uint64_t(r.a.w[1]) << 32);
-        return nullptr;
-    }
-    if (t == T_N48) {
-        if (r.a.w[0] == kN48Empty) {
-            fin = true;
-            return nullptr;
-        }
-        return rec + kN48Child + 8 * r.a.w[0];
-    }
-    if (t == T_N16) {
-        const int c = find_key16(r.a.w[0], r.a.w[1], r.a.w[2], r.a.w[3], b);
-        if (c < 0) {
-            fin = true;
-            return nullptr;
-        }
-        return rec + kN16Child + 8 * c;
-    }
-    const int c = find_key4(r.a.w[0], b);                     // N4: keys + children 0..2 in the 32-B block
-    if (c < 0) {
-        fin = true;
-        return nullptr;
-    }
-    if (c == 3) return rec + kN4Child + 24;
-    const uint32_t lo = c == 0 ? r.a.w[2] : c == 1 ? r.a.w[4] : r.a.w[6];
-    const uint32_t hi = c == 0 ? r.a.w[3] : c == 1 ? r.a.w[5] : r.a.w[7];
-    next = uint64_t(lo) | (uint64_t(hi) << 32);
-    return nullptr;
-}
-
-// Two walks in lockstep; leaf[j] = the matching leaf link (value in val[j]) or 0.
-template <class Key, int POL>
-__device__ __forceinline__ void find_leaf2(const DevIndex& ix, const Loader<POL>& ld, const Key (&key)[2],
-                                           uint64_t (&link)[2], uint64_t (&leaf)[2], uint64_t (&val)[2]) {
-    bool act[2];
-#pragma unroll
-    for (int j = 0; j < 2; j++) {
-        act[j] = link[j] != 0;
-        leaf[j] = 0;
-    }
-#pragma unroll 1
-    while (act[0] || act[1]) {
-        LeafRaw r[2];
-#pragma unroll
-        for (int j = 0; j < 2; j++)                            // phase A: both first requests in flight
-            if (act[j]) act[j] = walk_a(ix, ld, key[j], link[j], r[j]);
-        const uint8_t* a2[2] = {nullptr, nullptr};
-#pragma unroll
-        for (int j = 0; j < 2; j++) {
-            if (!act[j]) continue;
-            bool fin;
-            a2[j] = walk_b(ix, key[j], link[j], r[j], link[j], fin, leaf[j], val[j]);
-            if (fin) act[j] = false;
-        }
-        uint64_t c[2];
-#pragma unroll
-        for (int j = 0; j < 2; j++)                            // phase B2: both second requests in flight
-            if (a2[j]) c[j] = ld.node64(a2[j]);
-#pragma unroll
-        for (int j = 0; j < 2; j++)
-            if (a2[j]) link[j] = c[j];
-    }
-}
-
 // Compact 32-bit LUT entry (integer keys only; layout.h): [31:29] type; leaves
 // [28:0] index; inner nodes [28:26] branch depth - k, [25:0] index.
 __device__ __forceinline__ uint64_t expand_lut32(uint32_t e, uint32_t k, uint32_t leaf_len) {
