@@ -146,6 +146,15 @@ struct PushDst {
     uint32_t nrep;
 };
 
+#ifndef CUART_SCATTER_MIN_BLOCKS
+#define CUART_SCATTER_MIN_BLOCKS 1
+#endif
+constexpr int kScatterMinBlocks = CUART_SCATTER_MIN_BLOCKS;   // register cap of the lookup scatter (A/B knob)
+#ifndef CUART_HIST_MIN_BLOCKS
+#define CUART_HIST_MIN_BLOCKS 1
+#endif
+constexpr int kHistMinBlocks = CUART_HIST_MIN_BLOCKS;
+
 // Block-wide exclusive scan of one value per thread (kBucketThreads == kBuckets == 256).
 // Contains one __syncthreads; the caller syncs before reusing wtot.
 __device__ __forceinline__ unsigned int block_excl_scan256(unsigned int v, unsigned int* wtot) {
@@ -169,7 +178,7 @@ __device__ __forceinline__ unsigned int block_excl_scan256(unsigned int v, unsig
 // integer keys arrive in 16-B loads (2 u64 / 4 u32 keys per load): 1.27 ms per
 // 2^30 u64 keys (6.8 TB/s) against 2.08 ms with 8-B loads (tools/bucket_micro.cu).
 template <class Key, bool VEC, class PF = ByteBucket>
-__global__ void __launch_bounds__(kBucketThreads) k_bhist(const void* __restrict__ q, const uint8_t* __restrict__ lens,
+__global__ void __launch_bounds__(kBucketThreads, kHistMinBlocks) k_bhist(const void* __restrict__ q, const uint8_t* __restrict__ lens,
                                                           uint64_t n, PF pf, unsigned int* __restrict__ hist) {
     __shared__ unsigned int h[kBuckets];
     h[threadIdx.x] = 0;
@@ -324,13 +333,8 @@ __device__ __forceinline__ void copy_key_to_smem(const void* q, uint64_t i, uint
 // prio_base (OPS): the priority written with an op is prio_base + its index in the
 // batch (the multi-GPU layer numbers ops globally, rank-major, reading C7).
 // PUSH: the runs go to the owners' receive windows (PushDst), not to bq/blens/bvals/bidx.
-// ONEPASS (default): the tile's per-bucket counts come from the histogram pass
-// (rowoff of this tile and the next, bases), so the staged offsets are known before
-// any key is ranked: each key is ranked (one shared atomic) and staged right away,
-// and no bucket/rank array is held in registers across a barrier (measured: see
-// DESIGN.md §5).  !ONEPASS: rank all keys, scan the tile's own counts, then stage.
-template <class Key, bool OPS = false, class PF = ByteBucket, bool PUSH = false, bool ONEPASS = true>
-__global__ void __launch_bounds__(kBucketThreads, ONEPASS && !OPS && Key::kKind != 3 ? 5 : 1) k_bscatter(const void* __restrict__ q, const uint8_t* __restrict__ lens,
+template <class Key, bool OPS = false, class PF = ByteBucket, bool PUSH = false>
+__global__ void __launch_bounds__(kBucketThreads, !OPS && Key::kKind != 3 ? kScatterMinBlocks : 1) k_bscatter(const void* __restrict__ q, const uint8_t* __restrict__ lens,
                                                              uint64_t n, PF pf,
                                                              const unsigned int* __restrict__ rowoff,
                                                              const unsigned int* __restrict__ bases,
@@ -370,59 +374,6 @@ __global__ void __launch_bounds__(kBucketThreads, ONEPASS && !OPS && Key::kKind 
     const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
     __shared__ unsigned int staged_n;                                  // ops staged (all of them unless filtered)
     uint32_t scnt = cnt;
-    if (ONEPASS) {
-        // this tile's count of bucket b from the histogram pass's offsets (as k_bgather)
-        const uint32_t b = threadIdx.x;
-        const uint64_t t = blockIdx.x, tiles = gridDim.x;
-        const unsigned int off = rowoff[hidx(b, t)];
-        const unsigned int bb = bases[b];
-        const unsigned int next = t + 1 < tiles ? rowoff[hidx(b, t + 1)] : bases[b + 1] - bb;   // bases[kBuckets] = total
-        const unsigned int c_b = next - off;
-        const unsigned int lb = block_excl_scan256(c_b, wtot);
-        loc[b] = lb;
-        glb[b] = gb - lb;
-        if (b == kBuckets - 1) staged_n = lb + c_b;
-        __syncthreads();
-        scnt = staged_n;
-        uint64_t kv[kBucketItems];
-        uint64_t vv[OPS ? kBucketItems : 1];
-#pragma unroll
-        for (int r = 0; r < kBucketItems; r++) {                       // all loads first
-            const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
-            kv[r] = 0;
-            if (j < cnt && Key::kKind != 3)
-                kv[r] = Key::kKind == 2 ? uint64_t(__ldcs((const unsigned long long*)q + base + j))
-                                        : uint64_t(__ldcs((const unsigned int*)q + base + j));
-            if (OPS) vv[OPS ? r : 0] = j < cnt ? uint64_t(__ldcs((const unsigned long long*)vals + base + j)) : 0ull;
-        }
-#pragma unroll
-        for (int r = 0; r < kBucketItems; r++) {                       // rank + stage each key at once
-            const uint32_t jt = uint32_t(r) * kBucketThreads + threadIdx.x;
-            if (jt >= cnt) continue;
-            if (pf.skip(base + jt)) {
-                if (PF::kFilter && !OPS) __stcs((unsigned short*)jpos + base + jt, (unsigned short)kSkipPos);
-                continue;
-            }
-            uint32_t bk;
-            if (Key::kKind == 2) bk = pf.of(KeyU64{kv[r]});
-            else if (Key::kKind == 1) bk = pf.of(KeyU32{uint32_t(kv[r])});
-            else bk = pf.template at<Key>(q, lens, base + jt);
-            const uint32_t j = loc[bk] + atomicAdd(&h[bk], 1u);         // position in the staged tile
-            sb[j] = uint8_t(bk);
-            if (Key::kKind == 2) ((uint64_t*)skeys)[j] = kv[r];
-            else if (Key::kKind == 1) ((uint32_t*)skeys)[j] = uint32_t(kv[r]);
-            else {
-                copy_key_to_smem<Key>(q, base + jt, skeys, j);
-                slens[j] = lens[base + jt];
-            }
-            if (OPS) {
-                svals[j] = vv[OPS ? r : 0];
-                sidx[j] = uint16_t(jt);
-            } else {
-                __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
-            }
-        }
-    } else {
     __syncthreads();
     uint32_t br[kBucketItems];                                         // bucket << 16 | rank (0xFFFFFFFF = none)
     uint64_t kv[kBucketItems];                                         // integer keys kept in registers
@@ -479,7 +430,6 @@ __global__ void __launch_bounds__(kBucketThreads, ONEPASS && !OPS && Key::kKind 
             }
         }
     }
-    }   // !ONEPASS
     __syncthreads();
     if (PUSH) {                                                        // fused route: runs -> owner windows
 #pragma unroll 4
@@ -544,7 +494,9 @@ __device__ __forceinline__ void cp_async_wait_all() {
 #ifndef CUART_GATHER_MIN_BLOCKS
 #define CUART_GATHER_MIN_BLOCKS 5
 #endif
-constexpr int kGatherMinBlocks = CUART_GATHER_MIN_BLOCKS;   // 5 CTAs/SM: <= 51 registers (64 at 1)
+// 5 CTAs/SM: <= 51 registers instead of 63, occupancy 62% instead of 50%; measured
+// c3 gather 3.79 -> 3.54 ms per 2^30 (profiles/r02/ab_scatter_gather.txt)
+constexpr int kGatherMinBlocks = CUART_GATHER_MIN_BLOCKS;
 
 // Per tile: the tile's results sit in 256 contiguous runs of the bucketed result
 // array (one per bucket, located exactly as k_bscatter placed them).  The run

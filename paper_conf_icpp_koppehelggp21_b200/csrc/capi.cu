@@ -437,12 +437,8 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
     else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, lens, n, ByteBucket(depth), hist);
     k_bscan_rows<<<kBuckets >> h->bucket_shift, kBucketThreads, 0, s>>>(hist, tiles, tot);   // rows in use only
     k_bscan<<<1, kBuckets, 0, s>>>(tot, kBuckets >> h->bucket_shift);
-    if (h->scatter_onepass)
-        k_bscatter<Key><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key>(), s>>>(
-            q, lens, n, ByteBucket(depth), hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, (uint16_t*)(scr + o_pos));
-    else
-        k_bscatter<Key, false, ByteBucket, false, false><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key>(), s>>>(
-            q, lens, n, ByteBucket(depth), hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, (uint16_t*)(scr + o_pos));
+    k_bscatter<Key><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key>(), s>>>(
+        q, lens, n, ByteBucket(depth), hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, (uint16_t*)(scr + o_pos));
     g_cuart_launches += 4;
     if (cudaGetLastError() != cudaSuccess) {
         scratch_free(h, scr, s);
@@ -699,14 +695,9 @@ static cuart_status launch_update_bucketed(cuart_index* h, const void* k, const 
     else k_bhist<Key, false><<<unsigned(tiles), kBucketThreads, 0, s>>>(k, lens, n, ByteBucket(depth), hist);
     k_bscan_rows<<<kBuckets >> h->bucket_shift, kBucketThreads, 0, s>>>(hist, tiles, tot);   // rows in use only
     k_bscan<<<1, kBuckets, 0, s>>>(tot, kBuckets >> h->bucket_shift);
-    if (h->scatter_onepass)
-        k_bscatter<Key, true><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key, true>(), s>>>(
-            k, lens, n, ByteBucket(depth), hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, nullptr, vals,
-            (uint64_t*)(scr + o_val), (uint32_t*)(scr + o_idx));
-    else
-        k_bscatter<Key, true, ByteBucket, false, false><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key, true>(), s>>>(
-            k, lens, n, ByteBucket(depth), hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, nullptr, vals,
-            (uint64_t*)(scr + o_val), (uint32_t*)(scr + o_idx));
+    k_bscatter<Key, true><<<unsigned(tiles), kBucketThreads, bscatter_smem<Key, true>(), s>>>(
+        k, lens, n, ByteBucket(depth), hist, tot, scr + o_q, Key::kKind == 3 ? scr + o_len : nullptr, nullptr, vals,
+        (uint64_t*)(scr + o_val), (uint32_t*)(scr + o_idx));
     g_cuart_launches += 4;
     rc = cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
     if (rc == CUART_OK)
@@ -983,25 +974,12 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     if (const char* pe = getenv("CUART_LOOKUP_TPB")) h->lk_tpb = unsigned(atoi(pe));
     if (const char* pe = getenv("CUART_UPD2_TPB")) h->upd2_tpb = unsigned(atoi(pe));
     if (const char* pe = getenv("CUART_WQ_LEAFPOL")) h->wq_lp = atoi(pe);
-    if (const char* pe = getenv("CUART_SCATTER_ONEPASS")) h->scatter_onepass = atoi(pe) != 0;
     h->prebucket = opts ? opts->prebucket : CUART_PREBUCKET_AUTO;
     if (h->prebucket > CUART_PREBUCKET_ON) {
         delete h;
         return CUART_ERR_INVALID_ARGUMENT;
     }
     if (const char* pe = getenv("CUART_PREBUCKET")) h->prebucket = atoi(pe) ? CUART_PREBUCKET_ON : CUART_PREBUCKET_OFF;
-    cudaFuncSetAttribute(k_bscatter<KeyU64, false, ByteBucket, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         int(bscatter_smem<KeyU64>()));
-    cudaFuncSetAttribute(k_bscatter<KeyU32, false, ByteBucket, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         int(bscatter_smem<KeyU32>()));
-    cudaFuncSetAttribute(k_bscatter<KeyBytes, false, ByteBucket, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         int(bscatter_smem<KeyBytes>()));
-    cudaFuncSetAttribute(k_bscatter<KeyU64, true, ByteBucket, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         int(bscatter_smem<KeyU64, true>()));
-    cudaFuncSetAttribute(k_bscatter<KeyU32, true, ByteBucket, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         int(bscatter_smem<KeyU32, true>()));
-    cudaFuncSetAttribute(k_bscatter<KeyBytes, true, ByteBucket, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         int(bscatter_smem<KeyBytes, true>()));
     cudaFuncSetAttribute(k_bscatter<KeyU64>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bscatter_smem<KeyU64>()));
     cudaFuncSetAttribute(k_bscatter<KeyU32>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bscatter_smem<KeyU32>()));
     cudaFuncSetAttribute(k_bscatter<KeyBytes>, cudaFuncAttributeMaxDynamicSharedMemorySize,

@@ -80,7 +80,6 @@ struct cuart_index {
     unsigned lk_tpb = 256;             // k_lookup threads per CTA (CUART_LOOKUP_TPB: 64 / 128 / 256)
     unsigned upd2_tpb = 256;           // k_upd2 threads per CTA (CUART_UPD2_TPB: 64 / 256)
     int wq_lp = 3;                     // k_lookup_wq leaf-load cache policy (CUART_WQ_LEAFPOL, kernels.cuh leafv4_b)
-    bool scatter_onepass = true;       // k_bscatter ranks + stages in one pass (CUART_SCATTER_ONEPASS=0: two)
     // K-BUCKET on the root byte >> shift: 256 >> shift buckets (CUART_BUCKET_SHIFT).  Set
     // at upload: 64 buckets when a bucket's slice of the walked records stays within
     // 64 MB (c2, c3: runs of ~64 keys per tile cut the run-scattered traffic of scatter
