@@ -63,6 +63,8 @@ def _args():
     p.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
                    help="range mode exchange: p2p = fused push/return over peer memory (CUDA IPC, NVLink), "
                         "nccl = route + all-to-all")
+    p.add_argument("--dist", action="store_true",
+                   help="N = 1 through the multi-GPU layer (cuart_dist_*, one rank): its protocol overhead")
     p.add_argument("--l2-persist", type=int, default=0,
                    help="cuart_build_opts.l2_persist: persisting L2 window over the root tables")
     p.add_argument("--c5-fused", type=int, default=0,
@@ -437,7 +439,7 @@ def main():
         # multi-rank path with several ranks sharing one GPU (host-staged collectives)
         backend = os.environ.get("CUART_DIST_BACKEND", "nccl")
         dist.init_process_group(backend, device_id=dev if backend == "nccl" else None)
-    mode = "single" if world == 1 else args.mode
+    mode = "single" if world == 1 and not args.dist else args.mode
     if args.config == "c5":
         run_c5(args, world, rank, local, dev)
         return
@@ -445,13 +447,13 @@ def main():
     cfg = W.CONFIGS[args.config]
     t0 = time.perf_counter()
     keys, vals, keys_d = make_keys(cfg, dev)
-    if world == 1:
+    if world == 1 and not args.dist:
         layout = C.Layout(keys, vals, lut_bytes=args.lut)
         ix = C.Index.from_layout(layout, device=local, lut_format=LUT_FORMATS[args.lut_format],
                                  l2_persist=args.l2_persist)
         di = None
     else:
-        di = DistIndex(keys, vals, mode=mode, transport=args.transport, lut_bytes=args.lut)
+        di = DistIndex(keys, vals, mode=mode, transport=args.transport, lut_bytes=args.lut, rank=rank, world=world)
         ix = di.index
         layout = None
     build_s = time.perf_counter() - t0
@@ -655,8 +657,8 @@ def main():
             "config": {"workload": f"{args.config}: {cfg.description}", "keys": cfg.n_keys,
                        "lookups_per_rank": nl, "updates_per_rank": nu, "key_kind": cfg.kind,
                        "lut_bytes": args.lut, "lut_format": stats["lut_format"], "mode": mode,
-                       "transport": args.transport if world > 1 and mode == "range" else None,
-                       "parallelism": f"{mode}{world}" if world > 1 else "single",
+                       "transport": args.transport if (world > 1 or args.dist) and mode == "range" else None,
+                       "parallelism": f"{mode}{world}" if world > 1 or args.dist else "single",
                        "l2": f"inputs ({q_bytes / 2**30:.1f} GiB of queries per step) larger than L2; no flush",
                        "measured_hit_ratio": round(hit, 4), "build_s": round(build_s, 2)},
             "lookup": {"mlookups_per_s": round(world * nl / (look_ms * 1e-3) / 1e6, 3), "ms": round(look_ms, 4)},
