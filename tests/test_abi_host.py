@@ -65,6 +65,40 @@ def test_cuart_build_without_device_fails_loudly():
     assert e.value.status == 8
 
 
+def test_dist_cfg_validation_without_gpu():
+    """cuart_dist_build / cuart_dist_partition / cuart_dist_chunk_plan reject bad
+    configurations before touching a device; a valid one reaches the device check."""
+    import ctypes
+    import torch
+    from paper_conf_icpp_koppehelggp21_b200 import dist as D
+    keys = np.arange(1000, dtype=np.uint64) * np.uint64(7919)
+    vals = np.arange(1000, dtype=np.uint64)
+    k, n, keep = C._binding.make_keys(keys)
+
+    def build(**kw):
+        c, keep2 = D._cfg(kw.get("rank", 0), kw.get("world", 2), "range", "p2p", None,
+                          splitters=kw.get("splitters"), keys_local=kw.get("keys_local", False))
+        for f in ("nranks", "mode", "transport"):
+            if f in kw:
+                setattr(c, f, kw[f])
+        h = ctypes.c_void_p()
+        return D.lib().cuart_dist_build(ctypes.byref(c), ctypes.byref(k), vals.ctypes.data, n, ctypes.byref(h))
+
+    assert build(rank=2) == 1                                   # rank out of range
+    assert build(nranks=17) == 1                                # more ranks than CUART_DIST_MAX_RANKS
+    assert build(mode=7) == 1 and build(transport=9) == 1
+    assert build(world=3, splitters=np.array([5, 3], np.uint64)) == 1        # descending splitters
+    assert build(keys_local=True) == 1                          # a local share needs its splitters
+    if not torch.cuda.is_available():
+        assert build(world=1) == 8                              # valid: CUART_ERR_NO_DEVICE here
+    M = np.ones((2, 2), np.uint64)
+    bad = np.zeros(3, np.uint64)
+    assert D.lib().cuart_dist_chunk_plan(2, 2, M.ctypes.data, bad.ctypes.data, bad.ctypes.data, bad.ctypes.data) == 1
+    assert D.lib().cuart_dist_chunk_plan(0, 0, M.ctypes.data, bad.ctypes.data, bad.ctypes.data, bad.ctypes.data) == 1
+    sp, own = D.partition(keys, 0, 4)
+    assert np.all(np.diff(sp.astype(np.float64)) >= 0) and set(own.tolist()) == {0, 1, 2, 3}
+
+
 def _strings(keys):
     slots = np.zeros((len(keys), 32), np.uint8)
     lens = np.zeros(len(keys), np.uint8)
