@@ -492,9 +492,18 @@ def main():
     sec = layout.sectors(samp, wide=bool(bucketed and stats.get("wide_lut", 0))).astype(np.float64)
     io_bytes = {"u64": 8, "u32": 4, "bytes": 33}[cfg.kind] + 8
     random_bytes_per_lookup = 32.0 * sec.mean() + io_bytes
-    # whole lookup call (bucket histogram + scatter + walk + gather), streaming bytes per query
+    # tile form of K-BUCKET (cuart_build_opts.bucket_form, default): single-index integer
+    # lookups; the multi-GPU owner walks (fused return) keep the global form
+    tile = bucketed and di is None and os.environ.get("CUART_BUCKET_FORM", "2") != "1" and \
+        os.environ.get("CUART_SLICE", "0") != "2"
+    # whole lookup call, streaming bytes per query: global form = histogram + scatter +
+    # walk I/O + gather; tile form = tile sort + walk I/O + tile gather (run padding,
+    # ~2%, not counted)
     ks = io_bytes - 8
-    stream_bytes = (ks + (ks + ks + 2) + (ks + 8) + (8 + 2 + 8)) if bucketed else io_bytes
+    if tile:
+        stream_bytes = (ks + ks + 2) + (ks + 8) + (8 + 2 + 8)
+    else:
+        stream_bytes = (ks + (ks + ks + 2) + (ks + 8) + (8 + 2 + 8)) if bucketed else io_bytes
     del samp
 
     stream = torch.cuda.current_stream()
@@ -581,7 +590,7 @@ def main():
     tfile = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if traffic is None and os.path.exists(tfile):
         with open(tfile) as f:
-            traffic = json.load(f).get(f"{args.config}/{'bucketed' if bucketed else 'direct'}")
+            traffic = json.load(f).get(f"{args.config}/{'tile' if tile else 'bucketed' if bucketed else 'direct'}")
 
     # end-to-end through the public API with HOST buffers (pinned), copies inside the timed region
     e2e = None
@@ -666,7 +675,8 @@ def main():
                        "ms": round(upd_ms, 4)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
-                         "kernel": ("k_lookup_slice" if kslice else "k_lookup_wq" if wq else "k_lookup")
+                         "kernel": ("k_lookup_slice" if kslice else "k_lookup_wt" if tile else "k_lookup_wq" if wq
+                                    else "k_lookup")
                          + {"u64": "<KeyU64>", "u32": "<KeyU32>", "bytes": "<KeyBytes>"}[cfg.kind],
                          "kernel_ms": round(kern_ms, 4), "lookups_per_step": int(served),
                          "launches_per_step": round(launches_per_step, 2),
@@ -686,7 +696,8 @@ def main():
                              "achieved": round(ns_achieved, 1), "frac": round(ns_achieved / peak, 4)},
                          "lookup_call": {"ms": round(look_ms, 4), "bytes_per_lookup": round(pipeline_bytes, 3),
                                          "achieved": round(pipe_achieved, 1), "frac": round(pipe_achieved / peak, 4),
-                                         "kernels": "k_bhist, k_bscan_rows, k_bscan, k_bscatter, "
+                                         "kernels": "k_tsort, k_lookup_wt, k_tgather" if tile else
+                                         "k_bhist, k_bscan_rows, k_bscan, k_bscatter, "
                                          + ("k_lookup_slice" if kslice else "k_lookup_wq" if wq else "k_lookup") + ", k_bgather"
                                          if bucketed else "k_lookup"}},
             "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": int(launches), "clocks": clk,

@@ -122,7 +122,19 @@ typedef struct {
                                     most entries lead to an N4/N16 or a full N256 of
                                     leaves), CUART_WIDE_OFF, CUART_WIDE_ON.  Results are
                                     identical.                                             */
+    uint32_t bucket_form;        /* layout of a pre-bucketed integer-key lookup batch (a5):
+                                    CUART_BUCKET_TILE sorts every 4096-query tile by bucket in
+                                    place and walks bucket b's runs of all tiles together
+                                    (no histogram pass, no global scatter: 52 streaming B per
+                                    u64 query); CUART_BUCKET_GLOBAL scatters the batch into
+                                    one contiguous run per bucket (60 B per query).
+                                    CUART_BUCKET_FORM_AUTO = tile.  Multi-GPU owner walks
+                                    (fused return) and byte-string batches use the global
+                                    form.  Results are identical.                          */
 } cuart_build_opts;
+#define CUART_BUCKET_FORM_AUTO 0u
+#define CUART_BUCKET_GLOBAL 1u
+#define CUART_BUCKET_TILE 2u
 #define CUART_WIDE_AUTO 0u
 #define CUART_WIDE_OFF 1u
 #define CUART_WIDE_ON 2u

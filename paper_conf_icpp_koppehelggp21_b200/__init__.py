@@ -18,5 +18,6 @@ from ._binding import (  # noqa: F401
     cuart_stats, cuart_status_string, cuart_update, cuart_update_host, cuart_upload, lib,
     cuart_update_ex, cuart_erase, cuart_free_leaves, cuart_range,
     PREBUCKET_AUTO, PREBUCKET_OFF, PREBUCKET_ON, SLICE_AUTO, SLICE_OFF, SLICE_ON, WIDE_AUTO, WIDE_OFF, WIDE_ON,
+    BUCKET_FORM_AUTO, BUCKET_GLOBAL, BUCKET_TILE,
     cuart_kernel_timer, cuart_kernel_time, cuart_kernel_time_ex, LongIndex, pack_long,
 )

@@ -26,7 +26,8 @@ class _Keys(ctypes.Structure):
 
 class _Opts(ctypes.Structure):
     _fields_ = [("lut_bytes", ctypes.c_uint32), ("l2_persist", ctypes.c_uint32),
-                ("device", ctypes.c_int32), ("lut_format", ctypes.c_uint32), ("prebucket", ctypes.c_uint32), ("slice_lut", ctypes.c_uint32), ("wide_lut", ctypes.c_uint32)]
+                ("device", ctypes.c_int32), ("lut_format", ctypes.c_uint32), ("prebucket", ctypes.c_uint32), ("slice_lut", ctypes.c_uint32), ("wide_lut", ctypes.c_uint32),
+                ("bucket_form", ctypes.c_uint32)]
 
 
 class _Stats(ctypes.Structure):
@@ -175,10 +176,12 @@ def make_keys(keys, lengths=None):
 PREBUCKET_AUTO, PREBUCKET_OFF, PREBUCKET_ON = 0, 1, 2
 SLICE_AUTO, SLICE_OFF, SLICE_ON = 0, 1, 2
 WIDE_AUTO, WIDE_OFF, WIDE_ON = 0, 1, 2
+BUCKET_FORM_AUTO, BUCKET_GLOBAL, BUCKET_TILE = 0, 1, 2
 
 
-def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0, wide_lut=0):
-    return _Opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut)
+def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0, wide_lut=0,
+          bucket_form=0):
+    return _Opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form)
 
 
 def _stream_ptr(stream):
@@ -192,14 +195,14 @@ def _stream_ptr(stream):
 
 # ------------------------------------------------------------------ hot path
 def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0,
-                slice_lut=0, wide_lut=0):
+                slice_lut=0, wide_lut=0, bucket_form=0):
     """Build + upload (host buffers).  Returns an opaque handle (int)."""
     k, n, keep = make_keys(keys)
     v = np.ascontiguousarray(values, dtype=np.uint64)
     if v.shape[0] != n:
         raise ValueError("values length mismatch")
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut)
+    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form)
     _check(lib().cuart_build(ctypes.byref(k), _ptr(v), n, ctypes.byref(o), ctypes.byref(h)), "cuart_build")
     return h.value
 
@@ -379,9 +382,10 @@ def cuart_layout_sectors(l, queries, threads=0, wide=False):
     return out
 
 
-def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0, wide_lut=0):
+def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0, wide_lut=0,
+                 bucket_form=0):
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut)
+    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form)
     _check(lib().cuart_upload(l, ctypes.byref(o), ctypes.byref(h)), "cuart_upload")
     return h.value
 
@@ -436,16 +440,17 @@ class Index:
     """Device-resident CuART index on one GPU."""
 
     def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0,
-                 slice_lut=0, wide_lut=0):
-        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut)
+                 slice_lut=0, wide_lut=0, bucket_form=0):
+        self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut,
+                             bucket_form)
         self.device = _torch_device(device)
 
     @classmethod
     def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0,
-                    wide_lut=0):
+                    wide_lut=0, bucket_form=0):
         """Upload an already-built host layout (keeps the host copy usable)."""
         self = cls.__new__(cls)
-        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut)
+        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form)
         self.device = _torch_device(device)
         return self
 

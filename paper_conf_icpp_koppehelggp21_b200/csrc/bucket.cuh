@@ -562,4 +562,140 @@ __global__ void __launch_bounds__(kBucketThreads, kGatherMinBlocks) k_bgather(co
     }
 }
 
+// ============================================================================ tile form
+// K-BUCKET without a global scatter.  The global form above needs every tile's
+// per-bucket counts before any key moves (k_bhist reads the whole batch once more
+// than the copy does) and writes each tile into up to 256 separate runs.  The tile
+// form sorts each tile by bucket in place:
+//
+//   k_tsort      : per tile: rank in shared memory, tq[tile] = the tile's keys in
+//                  bucket order (one contiguous, coalesced store), jpos[i] = sorted
+//                  position of query i, toff[tidx(b, t)] = start | length << 16 of
+//                  bucket b's run in tile t
+//   k_lookup_wt  : (capi.cu) CTA (bucket b, group of tiles) walks b's runs of its
+//                  tiles; CTAs are numbered bucket-major, so the CTAs resident at a
+//                  time share one bucket's slice of the tree as in the global form
+//   k_tgather    : per tile: out[i] = tres[tile][jpos[i]], every access coalesced
+//
+// Every run starts on a 32-B boundary (padded to kRunAlign bytes): a run is walked
+// at a different time than its neighbours in the same tile, so a sector shared by
+// two runs would be read twice from DRAM and written partially twice (a partial
+// sector costs a read-modify-write); the walk writes its padding slots too, so every
+// result sector it touches is written whole.  Streaming bytes per u64 query: 8 read
+// + 10 written (sort), 8 + 8 (walk I/O), 10 read + 8 written (gather) = 52 B plus
+// the padding (~1.5 slots per run), against 60 B for hist + scatter + walk + gather.
+constexpr uint32_t kRunAlign = 32;
+template <uint32_t KS>
+__host__ __device__ constexpr uint32_t run_align_keys() { return kRunAlign / KS; }
+// slots per tile region: 4096 keys + at most (A - 1) padding slots per bucket
+template <uint32_t KS>
+__host__ __device__ constexpr uint32_t tile_stride() { return uint32_t(kBucketTile) + kBuckets * (run_align_keys<KS>() - 1); }
+// run table: [group of 8 tiles][bucket < nb][tile in group], u32 start | len << 16
+__device__ __forceinline__ uint64_t tidx(uint32_t b, uint64_t t, uint32_t nb) {
+    return ((t / kHistGroup) * nb + b) * kHistGroup + (t % kHistGroup);
+}
+__host__ __device__ constexpr uint64_t tidx_entries(uint64_t tiles, uint32_t nb) {
+    return ((tiles + kHistGroup - 1) / kHistGroup) * kHistGroup * nb;
+}
+
+template <class Key>
+__global__ void __launch_bounds__(kBucketThreads) k_tsort(const void* __restrict__ q, uint64_t n, ByteBucket pf,
+                                                        uint32_t nb, void* __restrict__ tq,
+                                                        uint16_t* __restrict__ jpos, uint32_t* __restrict__ toff) {
+    static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
+    constexpr uint32_t KS = Key::kKind == 2 ? 8 : 4;
+    constexpr uint32_t A = run_align_keys<KS>();
+    constexpr uint32_t TS = tile_stride<KS>();
+    __shared__ __align__(16) uint8_t skeys[TS * KS];
+    __shared__ unsigned int h[kBuckets];
+    __shared__ unsigned int loc[kBuckets];
+    __shared__ unsigned int wtot[kBucketThreads / 32];
+    __shared__ unsigned int ptot;
+    h[threadIdx.x] = 0;
+    const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
+    __syncthreads();
+    uint64_t kv[kBucketItems];
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {                           // all loads first
+        const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
+        kv[r] = 0;
+        if (j < cnt)
+            kv[r] = Key::kKind == 2 ? uint64_t(__ldcs((const unsigned long long*)q + base + j))
+                                    : uint64_t(__ldcs((const unsigned int*)q + base + j));
+    }
+    uint32_t br[kBucketItems];                                         // bucket << 16 | rank
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
+        br[r] = 0xFFFFFFFFu;
+        if (j < cnt) {
+            const uint32_t b = Key::kKind == 2 ? pf.of(KeyU64{kv[r]}) : pf.of(KeyU32{uint32_t(kv[r])});
+            br[r] = (b << 16) | atomicAdd(&h[b], 1u);
+        }
+    }
+    __syncthreads();
+    const unsigned int c = h[threadIdx.x];
+    const unsigned int pc = (c + A - 1) & ~(A - 1);                     // padded run
+    const unsigned int lb = block_excl_scan256(pc, wtot);
+    loc[threadIdx.x] = lb;
+    if (threadIdx.x < nb) toff[tidx(threadIdx.x, blockIdx.x, nb)] = lb | (c << 16);
+    if (threadIdx.x == kBucketThreads - 1) ptot = lb + pc;
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t jt = uint32_t(r) * kBucketThreads + threadIdx.x;
+        if (br[r] != 0xFFFFFFFFu) {
+            const uint32_t j = loc[br[r] >> 16] + (br[r] & 0xFFFFu);
+            if (Key::kKind == 2) ((uint64_t*)skeys)[j] = kv[r];
+            else ((uint32_t*)skeys)[j] = uint32_t(kv[r]);
+            __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
+        }
+    }
+    __syncthreads();
+    // the sorted, padded tile -> tq in 16-B stores (every run and the region are
+    // 32-B aligned; padding slots carry stale shared memory, never read as keys)
+    const uint32_t nv = ptot * KS / 16;
+    uint4* dst = (uint4*)((uint8_t*)tq + uint64_t(blockIdx.x) * TS * KS);
+#pragma unroll 4
+    for (uint32_t v = threadIdx.x; v < nv; v += kBucketThreads) __stcs(dst + v, ((const uint4*)skeys)[v]);
+}
+
+// Per tile: the tile's padded, sorted results (written by k_lookup_wt) -> shared
+// memory in 16-B cp.async copies, then out[i] = sres[jpos[i]] (coalesced).
+__device__ __forceinline__ void cp_async16(void* smem, const void* g) {
+    const unsigned sa = unsigned(__cvta_generic_to_shared(smem));
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(g));
+}
+template <uint32_t KS>
+__global__ void __launch_bounds__(kBucketThreads) k_tgather(const uint64_t* __restrict__ tres,
+                                                          const uint16_t* __restrict__ jpos,
+                                                          const uint32_t* __restrict__ toff, uint32_t nb, uint64_t n,
+                                                          uint64_t* __restrict__ out) {
+    constexpr uint32_t TS = tile_stride<KS>();
+    constexpr uint32_t A = run_align_keys<KS>();
+    __shared__ __align__(16) uint64_t sres[TS];
+    const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
+    uint16_t jp[kBucketItems];
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t k = uint32_t(r) * kBucketThreads + threadIdx.x;
+        jp[r] = k < cnt ? __ldcs(jpos + base + k) : 0;
+    }
+    const uint32_t e = toff[tidx(nb - 1, blockIdx.x, nb)];             // last run: start | len << 16
+    const uint32_t ptot = (e & 0xFFFFu) + (((e >> 16) + A - 1) & ~(A - 1));
+    const uint64_t* src = tres + uint64_t(blockIdx.x) * TS;
+    const uint32_t nv = (ptot + 1) / 2;                                 // ptot is a multiple of A (even)
+#pragma unroll 4
+    for (uint32_t v = threadIdx.x; v < nv; v += kBucketThreads) cp_async16(&sres[2 * v], src + 2 * v);
+    cp_async_wait_all();
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t k = uint32_t(r) * kBucketThreads + threadIdx.x;
+        if (k < cnt) __stcs((unsigned long long*)out + base + k, (unsigned long long)sres[jp[r]]);
+    }
+}
+
 }  // namespace cuart

@@ -84,19 +84,10 @@ __global__ void __launch_bounds__(TPB) k_lookup(DevIndex ix, const void* __restr
 // warp ends); LP = leaf-load cache policy: evict_last by default, since in the
 // bucketed walk a leaf is re-read by the hit queries of its bucket window (c3:
 // 8.91 -> 8.42 ms per 2^30 against the direct walk's evict_first + L2::64B).
-template <class Key, int POL, int Q, int TPB = 256, bool SEG = false, int LP = 3>
-__global__ void __launch_bounds__(TPB) k_lookup_wq(DevIndex ix, const void* __restrict__ q,
-                                                   const uint8_t* __restrict__ lens, uint64_t n,
-                                                   uint64_t* __restrict__ out, SegOut so = SegOut{}) {
-    static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
-    const Loader<POL> ld;
-    const uint64_t i0 = uint64_t(blockIdx.x) * (TPB * Q) + threadIdx.x;
-    Key k[Q];
-#pragma unroll
-    for (int j = 0; j < Q; j++) {
-        const uint64_t i = i0 + uint64_t(j) * TPB;
-        k[j] = i < n ? Key::template load<true>(q, lens, i) : Key{0};
-    }
+// The lockstep walk of Q already-loaded integer keys from the wide root table
+// (shared by k_lookup_wq and the tile-form walk k_lookup_wt).
+template <class Key, int POL, int Q, int LP>
+__device__ __forceinline__ void wq_walk(const DevIndex& ix, const Loader<POL>& ld, const Key (&k)[Q], uint64_t (&res)[Q]) {
     U8x32 e[Q];
 #pragma unroll
     for (int j = 0; j < Q; j++) e[j] = ld.lutv8(ix.lutw + k[j].prefix(ix.lut_bytes) * 4);
@@ -127,19 +118,122 @@ __global__ void __launch_bounds__(TPB) k_lookup_wq(DevIndex ix, const void* __re
         if (link_type(link[j]) == T_LEAF8) r[j] = ld.template leafv4_b<LP>(ix.base[T_LEAF8] + link_index(link[j]) * record_bytes(T_LEAF8));
 #pragma unroll
     for (int j = 0; j < Q; j++) {
-        const uint64_t i = i0 + uint64_t(j) * TPB;
-        if (i >= n) continue;
-        uint64_t res = kMiss;
+        res[j] = kMiss;
         if (link_type(link[j]) == T_LEAF8) {
             const uint64_t kb = Key::kKind == 2 ? bswap64(uint64_t(k[j].k)) : uint64_t(__byte_perm(uint32_t(k[j].k), 0, 0x0123));
             if (link_aux(link[j]) == k[j].len() && (uint64_t(r[j].x) | (uint64_t(r[j].y) << 32)) == kb)
-                res = uint64_t(r[j].z) | (uint64_t(r[j].w) << 32);
+                res[j] = uint64_t(r[j].z) | (uint64_t(r[j].w) << 32);
         } else if (link[j]) {
             uint64_t val = kMiss;
-            if (find_leaf(ix, ld, k[j], link[j], val)) res = val;
+            if (find_leaf(ix, ld, k[j], link[j], val)) res[j] = val;
         }
+    }
+}
+
+template <class Key, int POL, int Q, int TPB = 256, bool SEG = false, int LP = 3>
+__global__ void __launch_bounds__(TPB) k_lookup_wq(DevIndex ix, const void* __restrict__ q,
+                                                   const uint8_t* __restrict__ lens, uint64_t n,
+                                                   uint64_t* __restrict__ out, SegOut so = SegOut{}) {
+    static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
+    const Loader<POL> ld;
+    const uint64_t i0 = uint64_t(blockIdx.x) * (TPB * Q) + threadIdx.x;
+    Key k[Q];
+#pragma unroll
+    for (int j = 0; j < Q; j++) {
+        const uint64_t i = i0 + uint64_t(j) * TPB;
+        k[j] = i < n ? Key::template load<true>(q, lens, i) : Key{0};
+    }
+    uint64_t res[Q];
+    wq_walk<Key, POL, Q, LP>(ix, ld, k, res);
+#pragma unroll
+    for (int j = 0; j < Q; j++) {
+        const uint64_t i = i0 + uint64_t(j) * TPB;
+        if (i >= n) continue;
         uint64_t* dst = SEG ? so.at(i) : out + i;
-        __stcs((unsigned long long*)dst, (unsigned long long)res);
+        __stcs((unsigned long long*)dst, (unsigned long long)res[j]);
+    }
+}
+
+// Tile-form K-BUCKET walk (bucket.cuh k_tsort): CTA (b, g) walks bucket b's runs of
+// the tg tiles of group g -- the padded runs are concatenated in tile order, thread p
+// of a round takes position p of the concatenation (a binary search over the run
+// prefix in shared memory gives its tile), and the result goes to the same
+// tile-sorted position, which k_tgather returns to query order; a padding position
+// writes CUART_MISS so that every result sector is written whole.  CTAs are numbered
+// bucket-major, so the CTAs resident at a time walk one bucket's slice of the tree
+// (the locality of the global bucketed order) without a global scatter.  WIDE: the
+// lockstep wide-table walk of k_lookup_wq; else the generic walk from the LINKS root
+// table.  No barrier inside the round loop: each warp runs its rounds independently.
+template <class Key, int Q, int TPB, int LP, bool WIDE, int MINB = 1>
+__global__ void __launch_bounds__(TPB, MINB) k_lookup_wt(DevIndex ix, const void* __restrict__ tq,
+                                                         const uint32_t* __restrict__ toff, uint64_t n, uint32_t nb,
+                                                         uint32_t tg, uint32_t ngroups, uint64_t* __restrict__ tres) {
+    static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
+    constexpr uint32_t KS = Key::kKind == 2 ? 8 : 4;
+    constexpr uint32_t A = run_align_keys<KS>();
+    constexpr uint32_t TS = tile_stride<KS>();
+    __shared__ uint32_t pre[33];                       // run start in the concatenation; pre[32]: sentinel
+    __shared__ uint2 de[32];                           // {slot - position, end of the live part of the run}
+    __shared__ uint32_t total;
+    const uint32_t b = blockIdx.x / ngroups, g = blockIdx.x - b * ngroups;
+    const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
+    const uint64_t gbase = uint64_t(g) * tg * TS;      // first slot of the group (tg * TS < 2^18)
+    if (threadIdx.x < 32) {
+        const uint32_t lane = threadIdx.x;
+        const uint64_t t = uint64_t(g) * tg + lane;
+        uint32_t e = 0;
+        const bool valid = lane < tg && t < tiles;
+        if (valid) e = toff[tidx(b, t, nb)];
+        const uint32_t len = e >> 16, plen = (len + A - 1) & ~(A - 1);
+        uint32_t x = plen;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
+            if (lane >= uint32_t(d)) x += y;
+        }
+        const uint32_t p_run = x - plen;
+        pre[lane] = valid ? p_run : 0xFFFFFFFFu;        // invalid lanes are never selected
+        de[lane] = make_uint2(lane * TS + (e & 0xFFFFu) - p_run, p_run + len);
+        if (lane == 31) {
+            total = x;
+            pre[32] = 0xFFFFFFFFu;
+        }
+    }
+    __syncthreads();
+    const uint32_t T = total;
+    uint32_t lo = 0;                                   // tile of the thread's last position (only moves forward)
+    const Key* kq = (const Key*)tq + gbase;
+    unsigned long long* rq = (unsigned long long*)tres + gbase;
+    constexpr uint32_t kDead = 0x80000000u;            // padding slot: no walk, CUART_MISS written
+#pragma unroll 1
+    for (uint32_t p0 = 0; p0 < T; p0 += TPB * Q) {
+        uint32_t rel[Q];                               // slot relative to gbase | kDead, or ~0 (past the end)
+        Key k[Q];
+#pragma unroll
+        for (int j = 0; j < Q; j++) {
+            const uint32_t p = p0 + uint32_t(j) * TPB + threadIdx.x;
+            // largest tile whose run starts at or before p: positions grow by TPB per
+            // step and runs average 4096 / nb slots, so this is 0-2 steps forward
+#pragma unroll 1
+            while (pre[lo + 1] <= p) lo++;
+            const uint2 d = de[lo];
+            rel[j] = p >= T ? ~0u : (p + d.x) | (p < d.y ? 0u : kDead);
+            k[j] = rel[j] < kDead ? Key::template load<true>(kq, nullptr, rel[j]) : Key{0};
+        }
+        const Loader<5> ld;                            // per round: the policies are not held across rounds
+        uint64_t res[Q];
+        if (WIDE) {
+            wq_walk<Key, 5, Q, LP>(ix, ld, k, res);
+        } else {
+#pragma unroll
+            for (int j = 0; j < Q; j++) {
+                uint64_t val = kMiss;
+                res[j] = rel[j] < kDead && find_leaf(ix, ld, k[j], start_link(ix, ld, k[j]), val) ? val : kMiss;
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < Q; j++)
+            if (rel[j] != ~0u) __stcs(rq + (rel[j] & ~kDead), (unsigned long long)(rel[j] < kDead ? res[j] : kMiss));
     }
 }
 
@@ -470,6 +564,60 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
     return rc;
 }
 
+// a5 pre-bucketing, tile form (bucket.cuh k_tsort / k_tgather, capi.cu k_lookup_wt):
+// sort every tile by bucket in place -> walk bucket-major over the tiles' runs ->
+// per-tile gather.  Integer keys, results to `out` (no fused multi-GPU return).
+template <class Key>
+static cuart_status launch_tiled(const cuart_index* h, const void* q, uint64_t n, uint64_t* out, cudaStream_t s) {
+    constexpr uint32_t KS = Key::kKind == 2 ? 8 : 4;
+    constexpr uint32_t TS = tile_stride<KS>();
+    auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
+    const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
+    const uint32_t nb = kBuckets >> h->bucket_shift;
+    const size_t o_off = 0, o_q = al(tidx_entries(tiles, nb) * 4), o_pos = o_q + al(tiles * TS * KS),
+                 o_res = o_pos + al(n * 2), total = o_res + al(tiles * TS * 8);
+    uint8_t* scr = nullptr;
+    cuart_status rc = scratch_alloc(h, (void**)&scr, total, s);
+    if (rc != CUART_OK) return rc;
+    uint32_t* toff = (uint32_t*)(scr + o_off);
+    const uint32_t depth = (link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u) |
+                           (h->bucket_shift << 8);
+    k_tsort<Key><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, n, ByteBucket(depth), nb, scr + o_q,
+                                                           (uint16_t*)(scr + o_pos), toff);
+    g_cuart_launches++;
+    if (cudaGetLastError() != cudaSuccess) {
+        scratch_free(h, scr, s);
+        return CUART_ERR_CUDA;
+    }
+    // tiles per walk CTA: bucket runs average 4096 / nb keys; ~2048 queries per CTA
+    // (16 rounds of 64 threads x 2 queries), at most 32 (one warp builds the prefix).
+    // c3 walk per 2^30: 12.3 / 10.8 / 9.7 / 9.4 ms at 4 / 8 / 16 / 32 tiles (the
+    // table prologue is paid per CTA)
+    uint32_t tg = uint32_t((2048 * uint64_t(nb)) / kBucketTile);
+    tg = tg < 1 ? 1 : tg > 32 ? 32 : tg;
+    if (h->tile_group) tg = h->tile_group;
+    const uint32_t ngroups = uint32_t((tiles + tg - 1) / tg);
+    const DevIndex& dx = h->dix_links;
+    const bool wide = dx.walk_wide && h->policy == 5 && h->ilp > 1;
+    cudaEvent_t ev0, ev1;
+    ktimer_begin(h, s, ev0, ev1);
+    const unsigned g = nb * ngroups;
+    uint64_t* tres = (uint64_t*)(scr + o_res);
+    // 20 CTAs/SM (48 registers instead of 52, no spill): c3 walk 9.42 -> 9.07 ms per 2^30
+    // (profiles/r02/tile_form.txt); 24 CTAs/SM spills (40 registers + 24 B stack)
+    if (wide && h->wt_minb == 1) k_lookup_wt<Key, 2, 64, 3, true, 1><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+    else if (wide && h->wt_minb == 24) k_lookup_wt<Key, 2, 64, 3, true, 24><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+    else if (wide) k_lookup_wt<Key, 2, 64, 3, true, 20><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+    else k_lookup_wt<Key, 2, 64, 3, false><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+    g_cuart_launches++;
+    ktimer_end(h, s, ev0, ev1, n);
+    k_tgather<KS><<<unsigned(tiles), kBucketThreads, 0, s>>>(tres, (const uint16_t*)(scr + o_pos), toff, nb, n, out);
+    g_cuart_launches++;
+    rc = cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+    scratch_free(h, scr, s);
+    return rc;
+}
+
 static constexpr uint64_t kBucketMin = uint64_t(1) << 22;   // below this the batch is too small to reorder
 
 cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const void* q, const uint8_t* lens, uint64_t n,
@@ -480,6 +628,9 @@ cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const void* q, c
     const bool bucket = h->prebucket == CUART_PREBUCKET_ON ? n >= kBucketTile
                       : h->prebucket == CUART_PREBUCKET_AUTO && n >= kBucketMin && kind != CUART_KEY_BYTES;
     if (bucket && n < (uint64_t(1) << 32)) {
+        const bool tiled = h->bucket_form == CUART_BUCKET_TILE && !so && h->slice_lut != CUART_SLICE_ON;
+        if (tiled && kind == CUART_KEY_U64) return launch_tiled<KeyU64>(h, q, n, out, s);
+        if (tiled && kind == CUART_KEY_U32) return launch_tiled<KeyU32>(h, q, n, out, s);
         switch (kind) {
         case CUART_KEY_U64: return launch_bucketed<KeyU64>(h, q, lens, n, out, s, so);
         case CUART_KEY_U32: return launch_bucketed<KeyU32>(h, q, lens, n, out, s, so);
@@ -980,6 +1131,20 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         return CUART_ERR_INVALID_ARGUMENT;
     }
     if (const char* pe = getenv("CUART_PREBUCKET")) h->prebucket = atoi(pe) ? CUART_PREBUCKET_ON : CUART_PREBUCKET_OFF;
+    {
+        const uint32_t bf = opts ? opts->bucket_form : CUART_BUCKET_FORM_AUTO;
+        if (bf > CUART_BUCKET_TILE) {
+            delete h;
+            return CUART_ERR_INVALID_ARGUMENT;
+        }
+        h->bucket_form = bf == CUART_BUCKET_GLOBAL ? CUART_BUCKET_GLOBAL : CUART_BUCKET_TILE;
+        if (const char* pe = getenv("CUART_WT_MINB")) h->wt_minb = uint32_t(atoi(pe));
+        if (const char* pe = getenv("CUART_TILE_GROUP")) {
+            const int v = atoi(pe);
+            h->tile_group = v < 1 ? 1u : v > 32 ? 32u : uint32_t(v);
+        }
+        if (const char* pe = getenv("CUART_BUCKET_FORM")) h->bucket_form = atoi(pe) == 1 ? CUART_BUCKET_GLOBAL : CUART_BUCKET_TILE;
+    }
     cudaFuncSetAttribute(k_bscatter<KeyU64>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bscatter_smem<KeyU64>()));
     cudaFuncSetAttribute(k_bscatter<KeyU32>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(bscatter_smem<KeyU32>()));
     cudaFuncSetAttribute(k_bscatter<KeyBytes>, cudaFuncAttributeMaxDynamicSharedMemorySize,

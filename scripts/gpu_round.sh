@@ -8,4 +8,5 @@ timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smok
 timeout 1200 python bench.py > gpurun_out/bench_c3.log 2>&1; echo "bench rc=$?" >> gpurun_out/bench_c3.log
 timeout 900 python bench.py --impl reference --steps 2 --warmup 3 > gpurun_out/bench_ref.log 2>&1
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sectors_srcunit_tex_op_read.sum,lts__t_sector_hit_rate.pct --clock-control none -k regex:'k_' --csv --log-file gpurun_out/launches_c3.csv python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu-baseline > gpurun_out/ncu_launch.log 2>&1
-timeout 1500 ncu --set full --import-source on --clock-control none -k regex:'k_lookup_wq|k_bscatter|k_bgather|k_upd1_wq|k_upd2|k_bhist' -c 7 -o gpurun_out/c3_full python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > gpurun_out/ncu_full.log 2>&1
+timeout 1500 ncu --set full --import-source on --clock-control none -k regex:'k_tsort|k_lookup_wt|k_tgather|k_bscatter|k_upd1_wq|k_upd2|k_bhist' -c 7 -o gpurun_out/c3_full python bench.py --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > gpurun_out/ncu_full.log 2>&1
+for c in c2 c4; do timeout 900 python bench.py --config $c --no-e2e --no-cpu-baseline > gpurun_out/bench_$c.log 2>&1; done

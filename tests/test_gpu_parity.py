@@ -263,15 +263,21 @@ def test_host_pipeline_many_chunks(kind, monkeypatch):
     ix.close()
 
 
+@pytest.mark.parametrize("form,tg", [("tile", None), ("tile", "1"), ("tile", "32"), ("global", None)])
 @pytest.mark.parametrize("shift", ["0", "2", "3"])
-def test_prebucket_bucket_counts_and_skew(shift, monkeypatch):
+def test_prebucket_bucket_counts_and_skew(shift, form, tg, monkeypatch):
     """K-BUCKET with 256 / 64 / 32 buckets (CUART_BUCKET_SHIFT, read at upload) on
     skewed batches: every query in one bucket, queries in two buckets, and a ragged
-    uniform batch; lookups and a bucketed update batch must equal the plain map."""
+    uniform batch; lookups and a bucketed update batch must equal the plain map.
+    Both batch forms; the tile form also with 1 and 32 tiles per walk CTA
+    (CUART_TILE_GROUP), i.e. the smallest and the largest run prefix."""
     monkeypatch.setenv("CUART_BUCKET_SHIFT", shift)
+    if tg:
+        monkeypatch.setenv("CUART_TILE_GROUP", tg)
     rng = np.random.default_rng(int(shift) + 40)
     keys, vals = W.build_set(W.CONFIGS["c1"])
-    ix = C.Index(keys, vals, lut_bytes=3, prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_ON)
+    ix = C.Index(keys, vals, lut_bytes=3, prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_ON,
+                 bucket_form=C.BUCKET_TILE if form == "tile" else C.BUCKET_GLOBAL)
     mp = MapOracle(keys, vals)
     top = keys >> np.uint64(56)
     one = keys[top == top[0]]
@@ -519,6 +525,10 @@ def test_prebucket_equals_direct(kind):
         variants.append(C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, slice_lut=C.SLICE_ON))
         variants.append(C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_ON))
         variants.append(C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_OFF))
+        # the global K-BUCKET form (hist + scatter) beside the default tile form
+        for wl in (C.WIDE_ON, C.WIDE_OFF):
+            variants.append(C.Index(keys, vals, lut_bytes=lut, prebucket=C.PREBUCKET_ON, wide_lut=wl,
+                                    bucket_form=C.BUCKET_GLOBAL))
     # 2048 * 4096 + 4097 spans more than one pass of k_bscan_rows (2048 tiles per pass)
     sizes = (4095, 4096, 4097, 100_003, 1 << 20) + ((2048 * 4096 + 4097,) if kind == "u64" else ())
     for m in sizes:
