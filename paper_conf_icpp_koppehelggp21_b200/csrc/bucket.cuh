@@ -598,8 +598,12 @@ __host__ __device__ constexpr uint64_t tidx_entries(uint64_t tiles, uint32_t nb)
     return ((tiles + kHistGroup - 1) / kHistGroup) * kHistGroup * nb;
 }
 
-template <class Key>
-__global__ void __launch_bounds__(kBucketThreads) k_tsort(const void* __restrict__ q, uint64_t n, ByteBucket pf,
+// VEC (batch 16-B aligned; the default): keys arrive in 16-B loads, a thread's keys
+// are pairs (u64) / quads (u32) of consecutive queries, and their sorted slots leave
+// as one 4-B / 8-B jpos store; capped at 64 registers (4 CTAs/SM).  c3: 3.46 -> 3.26
+// ms per 2^30 against the strided 8-B-load variant (profiles/r02/tile_form.txt).
+template <class Key, bool VEC = false>
+__global__ void __launch_bounds__(kBucketThreads, VEC ? 4 : 1) k_tsort(const void* __restrict__ q, uint64_t n, ByteBucket pf,
                                                         uint32_t nb, void* __restrict__ tq,
                                                         uint16_t* __restrict__ jpos, uint32_t* __restrict__ toff) {
     static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
@@ -615,19 +619,54 @@ __global__ void __launch_bounds__(kBucketThreads) k_tsort(const void* __restrict
     const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
     const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
     __syncthreads();
+    // item r of this thread is tile position jof(r): strided (plain) or in runs of PER
+    constexpr uint32_t PER = VEC ? 16 / KS : 1;
+    auto jof = [](int r) -> uint32_t {
+        return VEC ? (uint32_t(r / PER) * kBucketThreads + threadIdx.x) * PER + uint32_t(r % PER)
+                   : uint32_t(r) * kBucketThreads + threadIdx.x;
+    };
     uint64_t kv[kBucketItems];
+    if (VEC) {
 #pragma unroll
-    for (int r = 0; r < kBucketItems; r++) {                           // all loads first
-        const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
-        kv[r] = 0;
-        if (j < cnt)
-            kv[r] = Key::kKind == 2 ? uint64_t(__ldcs((const unsigned long long*)q + base + j))
-                                    : uint64_t(__ldcs((const unsigned int*)q + base + j));
+        for (int r = 0; r < kBucketItems; r += PER) {                  // all loads first
+            const uint32_t j = jof(r);
+            uint4 v = make_uint4(0, 0, 0, 0);
+            if (j + PER <= cnt) v = __ldcs((const uint4*)((const uint8_t*)q + (base + j) * KS));
+            else
+                for (uint32_t e = 0; e < PER; e++)
+                    if (j + e < cnt) {                                 // ragged end of the batch
+                        if (KS == 8) {
+                            const uint64_t x = __ldcs((const unsigned long long*)q + base + j + e);
+                            (&v.x)[2 * e] = uint32_t(x);
+                            (&v.x)[2 * e + 1] = uint32_t(x >> 32);
+                        } else {
+                            (&v.x)[e] = __ldcs((const unsigned int*)q + base + j + e);
+                        }
+                    }
+            if (KS == 8) {
+                kv[r] = uint64_t(v.x) | (uint64_t(v.y) << 32);
+                kv[r + 1] = uint64_t(v.z) | (uint64_t(v.w) << 32);
+            } else {
+                kv[r] = v.x;
+                kv[r + 1] = v.y;
+                kv[r + 2] = v.z;
+                kv[r + 3] = v.w;
+            }
+        }
+    } else {
+#pragma unroll
+        for (int r = 0; r < kBucketItems; r++) {                       // all loads first
+            const uint32_t j = jof(r);
+            kv[r] = 0;
+            if (j < cnt)
+                kv[r] = Key::kKind == 2 ? uint64_t(__ldcs((const unsigned long long*)q + base + j))
+                                        : uint64_t(__ldcs((const unsigned int*)q + base + j));
+        }
     }
     uint32_t br[kBucketItems];                                         // bucket << 16 | rank
 #pragma unroll
     for (int r = 0; r < kBucketItems; r++) {
-        const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
+        const uint32_t j = jof(r);
         br[r] = 0xFFFFFFFFu;
         if (j < cnt) {
             const uint32_t b = Key::kKind == 2 ? pf.of(KeyU64{kv[r]}) : pf.of(KeyU32{uint32_t(kv[r])});
@@ -643,13 +682,30 @@ __global__ void __launch_bounds__(kBucketThreads) k_tsort(const void* __restrict
     if (threadIdx.x == kBucketThreads - 1) ptot = lb + pc;
     __syncthreads();
 #pragma unroll
-    for (int r = 0; r < kBucketItems; r++) {
-        const uint32_t jt = uint32_t(r) * kBucketThreads + threadIdx.x;
-        if (br[r] != 0xFFFFFFFFu) {
-            const uint32_t j = loc[br[r] >> 16] + (br[r] & 0xFFFFu);
-            if (Key::kKind == 2) ((uint64_t*)skeys)[j] = kv[r];
-            else ((uint32_t*)skeys)[j] = uint32_t(kv[r]);
-            __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
+    for (int r0 = 0; r0 < kBucketItems; r0 += PER) {
+        uint32_t js[PER];
+#pragma unroll
+        for (int e = 0; e < int(PER); e++) {
+            const int r = r0 + e;
+            js[e] = 0;
+            if (br[r] != 0xFFFFFFFFu) {
+                const uint32_t j = loc[br[r] >> 16] + (br[r] & 0xFFFFu);
+                if (Key::kKind == 2) ((uint64_t*)skeys)[j] = kv[r];
+                else ((uint32_t*)skeys)[j] = uint32_t(kv[r]);
+                js[e] = j;
+                if (!VEC) __stcs((unsigned short*)jpos + base + jof(r), (unsigned short)j);
+            }
+        }
+        if (VEC) {
+            const uint32_t j = jof(r0);
+            if (j + PER <= cnt) {
+                if (PER == 2) __stcs((unsigned int*)(jpos + base + j), js[0] | (js[PER > 1 ? 1 : 0] << 16));
+                else __stcs((uint2*)(jpos + base + j), make_uint2(js[0] | (js[PER > 1 ? 1 : 0] << 16),
+                                                                  js[PER > 2 ? 2 : 0] | (js[PER > 3 ? 3 : 0] << 16)));
+            } else {
+                for (uint32_t e = 0; e < PER; e++)
+                    if (j + e < cnt) jpos[base + j + e] = uint16_t(js[e]);
+            }
         }
     }
     __syncthreads();

@@ -582,8 +582,12 @@ static cuart_status launch_tiled(const cuart_index* h, const void* q, uint64_t n
     uint32_t* toff = (uint32_t*)(scr + o_off);
     const uint32_t depth = (link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u) |
                            (h->bucket_shift << 8);
-    k_tsort<Key><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, n, ByteBucket(depth), nb, scr + o_q,
-                                                           (uint16_t*)(scr + o_pos), toff);
+    if (h->tsort_vec && (uintptr_t(q) & 15) == 0)
+        k_tsort<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, n, ByteBucket(depth), nb, scr + o_q,
+                                                                     (uint16_t*)(scr + o_pos), toff);
+    else
+        k_tsort<Key><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, n, ByteBucket(depth), nb, scr + o_q,
+                                                               (uint16_t*)(scr + o_pos), toff);
     g_cuart_launches++;
     if (cudaGetLastError() != cudaSuccess) {
         scratch_free(h, scr, s);
@@ -605,7 +609,9 @@ static cuart_status launch_tiled(const cuart_index* h, const void* q, uint64_t n
     uint64_t* tres = (uint64_t*)(scr + o_res);
     // 20 CTAs/SM (48 registers instead of 52, no spill): c3 walk 9.42 -> 9.07 ms per 2^30
     // (profiles/r02/tile_form.txt); 24 CTAs/SM spills (40 registers + 24 B stack)
-    if (wide && h->wt_minb == 1) k_lookup_wt<Key, 2, 64, 3, true, 1><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+    if (wide && h->wt_tpb == 128) k_lookup_wt<Key, 2, 128, 3, true, 10><<<g, 128, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+    else if (wide && h->wt_tpb == 256) k_lookup_wt<Key, 2, 256, 3, true, 5><<<g, 256, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+    else if (wide && h->wt_minb == 1) k_lookup_wt<Key, 2, 64, 3, true, 1><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
     else if (wide && h->wt_minb == 24) k_lookup_wt<Key, 2, 64, 3, true, 24><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
     else if (wide) k_lookup_wt<Key, 2, 64, 3, true, 20><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
     else k_lookup_wt<Key, 2, 64, 3, false><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
@@ -1139,6 +1145,8 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         }
         h->bucket_form = bf == CUART_BUCKET_GLOBAL ? CUART_BUCKET_GLOBAL : CUART_BUCKET_TILE;
         if (const char* pe = getenv("CUART_WT_MINB")) h->wt_minb = uint32_t(atoi(pe));
+        if (const char* pe = getenv("CUART_WT_TPB")) h->wt_tpb = uint32_t(atoi(pe));
+        if (const char* pe = getenv("CUART_TSORT_VEC")) h->tsort_vec = uint32_t(atoi(pe));
         if (const char* pe = getenv("CUART_TILE_GROUP")) {
             const int v = atoi(pe);
             h->tile_group = v < 1 ? 1u : v > 32 ? 32u : uint32_t(v);
