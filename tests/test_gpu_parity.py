@@ -321,6 +321,36 @@ def test_prebucket_gather_misaligned_out(n):
     ix.close()
 
 
+@pytest.mark.parametrize("kind", ["u64", "u32"])
+def test_prebucket_misaligned_queries(kind):
+    """The tile sort loads keys in 16-B vectors only from a 16-B-aligned batch; a
+    query view 4 / 8 B into its buffer takes the strided 8-B path.  Both equal the
+    plain map, with a ragged tail tile."""
+    rng = np.random.default_rng(77)
+    if kind == "u64":
+        keys, vals = W.build_set(W.CONFIGS["c1"])
+        q = np.where(rng.random(70_003) < 0.5, keys[rng.integers(0, keys.shape[0], 70_003)],
+                     rng.integers(0, 2**64, 70_003, dtype=np.uint64))
+        tdt = torch.int64
+    else:
+        keys = np.unique((np.arange(1 << 17, dtype=np.uint32) * 29) & np.uint32(0xFFFFFF))
+        vals = np.arange(keys.shape[0], dtype=np.uint64) + 1
+        q = rng.integers(0, 1 << 24, 70_003, dtype=np.uint32)
+        tdt = torch.int32
+    ix = C.Index(keys, vals, lut_bytes=3, prebucket=C.PREBUCKET_ON, wide_lut=C.WIDE_ON)
+    mp = MapOracle(keys, vals)
+    want = mp.lookup(q)
+    for off in (0, 1):
+        buf = torch.zeros(q.shape[0] + 1, dtype=tdt, device=DEV)
+        qv = buf[off:off + q.shape[0]]
+        qv.copy_(torch.from_numpy(q.view(np.int64 if kind == "u64" else np.int32)).to(DEV))
+        out = torch.empty(q.shape[0], dtype=torch.int64, device=DEV)
+        ix.lookup(qv, out)
+        torch.cuda.synchronize()
+        assert np.array_equal(out.cpu().numpy().view(np.uint64), want), off
+    ix.close()
+
+
 def test_c2_full_size_sampled():
     """Config 2 at full size (2^24 dense u32 keys, LUT over the first 3 bytes):
     2^28 lookups in the bench's launch configuration; sampled outputs vs the
