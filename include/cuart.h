@@ -128,9 +128,11 @@ typedef struct {
                                     (no histogram pass, no global scatter: 52 streaming B per
                                     u64 query); CUART_BUCKET_GLOBAL scatters the batch into
                                     one contiguous run per bucket (60 B per query).
-                                    CUART_BUCKET_FORM_AUTO = tile.  Multi-GPU owner walks
-                                    (fused return) and byte-string batches use the global
-                                    form.  Results are identical.                          */
+                                    CUART_BUCKET_FORM_AUTO = tile.  Byte-string batches
+                                    (bucketed only with CUART_PREBUCKET_ON) take the tile
+                                    form too; multi-GPU owner walks (fused return) and
+                                    update batches use the global form.  Results are
+                                    identical.                                             */
 } cuart_build_opts;
 #define CUART_BUCKET_FORM_AUTO 0u
 #define CUART_BUCKET_GLOBAL 1u

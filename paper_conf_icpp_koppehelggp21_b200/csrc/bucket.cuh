@@ -717,6 +717,61 @@ __global__ void __launch_bounds__(kBucketThreads, VEC ? 4 : 1) k_tsort(const voi
     for (uint32_t v = threadIdx.x; v < nv; v += kBucketThreads) __stcs(dst + v, ((const uint4*)skeys)[v]);
 }
 
+// Tile sort of a byte-string batch (32-B slots + lengths).  A key is exactly one
+// 32-B sector, so no staging is needed: pass 1 reads each query's length and the
+// one key byte its bucket needs and ranks it in shared memory; pass 2 copies the
+// whole slot (an L2 hit: pass 1 brought its sector in) to its sorted slot -- a
+// full-sector store -- with its length and jpos.  Runs need no padding (A = 1).
+static __global__ void __launch_bounds__(kBucketThreads) k_tsort_bytes(const uint8_t* __restrict__ q,
+                                                                     const uint8_t* __restrict__ lens, uint64_t n,
+                                                                     ByteBucket pf, uint32_t nb, uint8_t* __restrict__ tq,
+                                                                     uint8_t* __restrict__ tlen, uint16_t* __restrict__ jpos,
+                                                                     uint32_t* __restrict__ toff) {
+    constexpr uint32_t TS = tile_stride<32>();
+    __shared__ unsigned int h[kBuckets];
+    __shared__ unsigned int loc[kBuckets];
+    __shared__ unsigned int wtot[kBucketThreads / 32];
+    h[threadIdx.x] = 0;
+    const uint64_t base = uint64_t(blockIdx.x) * kBucketTile;
+    const uint32_t cnt = uint32_t(n - base < uint64_t(kBucketTile) ? n - base : kBucketTile);
+    __syncthreads();
+    uint32_t br[kBucketItems];                                         // bucket << 16 | rank
+    const uint32_t d = pf.depth & 0xFFu, sh = pf.depth >> 8;
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++) {
+        // plain loads (not evict-first): the key's sector must still be in L2 for pass 2
+        const uint32_t j = uint32_t(r) * kBucketThreads + threadIdx.x;
+        br[r] = 0xFFFFFFFFu;
+        if (j < cnt) {
+            const uint32_t l = lens[base + j];
+            br[r] = d < l ? uint32_t(q[(base + j) * 32 + d]) >> sh : 0u;
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < kBucketItems; r++)
+        if (br[r] != 0xFFFFFFFFu) br[r] = (br[r] << 16) | atomicAdd(&h[br[r]], 1u);
+    __syncthreads();
+    const unsigned int c = h[threadIdx.x];
+    const unsigned int lb = block_excl_scan256(c, wtot);
+    loc[threadIdx.x] = lb;
+    if (threadIdx.x < nb) toff[tidx(threadIdx.x, blockIdx.x, nb)] = lb | (c << 16);
+    __syncthreads();
+    uint8_t* dq = tq + uint64_t(blockIdx.x) * TS * 32;
+    uint8_t* dl = tlen + uint64_t(blockIdx.x) * TS;
+#pragma unroll 4
+    for (int r = 0; r < kBucketItems; r++) {
+        const uint32_t jt = uint32_t(r) * kBucketThreads + threadIdx.x;
+        if (br[r] == 0xFFFFFFFFu) continue;
+        const uint32_t j = loc[br[r] >> 16] + (br[r] & 0xFFFFu);
+        const uint4* src = (const uint4*)(q + (base + jt) * 32);
+        const uint4 a = __ldcs(src), b = __ldcs(src + 1);
+        __stcs((uint4*)(dq + uint64_t(j) * 32), a);
+        __stcs((uint4*)(dq + uint64_t(j) * 32) + 1, b);
+        dl[j] = lens[base + jt];
+        __stcs((unsigned short*)jpos + base + jt, (unsigned short)j);
+    }
+}
+
 // Per tile: the tile's padded, sorted results (written by k_lookup_wt) -> shared
 // memory in 16-B cp.async copies, then out[i] = sres[jpos[i]] (coalesced).
 __device__ __forceinline__ void cp_async16(void* smem, const void* g) {

@@ -167,9 +167,10 @@ __global__ void __launch_bounds__(TPB) k_lookup_wq(DevIndex ix, const void* __re
 template <class Key, int Q, int TPB, int LP, bool WIDE, int MINB = 1>
 __global__ void __launch_bounds__(TPB, MINB) k_lookup_wt(DevIndex ix, const void* __restrict__ tq,
                                                          const uint32_t* __restrict__ toff, uint64_t n, uint32_t nb,
-                                                         uint32_t tg, uint32_t ngroups, uint64_t* __restrict__ tres) {
-    static_assert(Key::kKind == 1 || Key::kKind == 2, "integer keys");
-    constexpr uint32_t KS = Key::kKind == 2 ? 8 : 4;
+                                                         uint32_t tg, uint32_t ngroups, uint64_t* __restrict__ tres,
+                                                         const uint8_t* __restrict__ tlen = nullptr) {
+    static_assert(Key::kKind == 1 || Key::kKind == 2 || (Key::kKind == 3 && !WIDE), "integer keys or byte strings");
+    constexpr uint32_t KS = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
     constexpr uint32_t A = run_align_keys<KS>();
     constexpr uint32_t TS = tile_stride<KS>();
     __shared__ uint32_t pre[33];                       // run start in the concatenation; pre[32]: sentinel
@@ -202,7 +203,8 @@ __global__ void __launch_bounds__(TPB, MINB) k_lookup_wt(DevIndex ix, const void
     __syncthreads();
     const uint32_t T = total;
     uint32_t lo = 0;                                   // tile of the thread's last position (only moves forward)
-    const Key* kq = (const Key*)tq + gbase;
+    const uint8_t* kq = (const uint8_t*)tq + gbase * KS;
+    const uint8_t* kl = Key::kKind == 3 ? tlen + gbase : nullptr;
     unsigned long long* rq = (unsigned long long*)tres + gbase;
     constexpr uint32_t kDead = 0x80000000u;            // padding slot: no walk, CUART_MISS written
 #pragma unroll 1
@@ -218,11 +220,12 @@ __global__ void __launch_bounds__(TPB, MINB) k_lookup_wt(DevIndex ix, const void
             while (pre[lo + 1] <= p) lo++;
             const uint2 d = de[lo];
             rel[j] = p >= T ? ~0u : (p + d.x) | (p < d.y ? 0u : kDead);
-            k[j] = rel[j] < kDead ? Key::template load<true>(kq, nullptr, rel[j]) : Key{0};
+            if (rel[j] < kDead) k[j] = Key::template load<true>(kq, kl, rel[j]);
+            else k[j] = Key{};
         }
         const Loader<5> ld;                            // per round: the policies are not held across rounds
         uint64_t res[Q];
-        if (WIDE) {
+        if constexpr (WIDE) {
             wq_walk<Key, 5, Q, LP>(ix, ld, k, res);
         } else {
 #pragma unroll
@@ -568,21 +571,26 @@ static cuart_status launch_bucketed(const cuart_index* h, const void* q, const u
 // sort every tile by bucket in place -> walk bucket-major over the tiles' runs ->
 // per-tile gather.  Integer keys, results to `out` (no fused multi-GPU return).
 template <class Key>
-static cuart_status launch_tiled(const cuart_index* h, const void* q, uint64_t n, uint64_t* out, cudaStream_t s) {
-    constexpr uint32_t KS = Key::kKind == 2 ? 8 : 4;
+static cuart_status launch_tiled(const cuart_index* h, const void* q, const uint8_t* lens, uint64_t n, uint64_t* out,
+                                 cudaStream_t s) {
+    constexpr uint32_t KS = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
     constexpr uint32_t TS = tile_stride<KS>();
     auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
     const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
     const uint32_t nb = kBuckets >> h->bucket_shift;
-    const size_t o_off = 0, o_q = al(tidx_entries(tiles, nb) * 4), o_pos = o_q + al(tiles * TS * KS),
-                 o_res = o_pos + al(n * 2), total = o_res + al(tiles * TS * 8);
+    const size_t o_off = 0, o_q = al(tidx_entries(tiles, nb) * 4), o_len = o_q + al(tiles * TS * KS),
+                 o_pos = o_len + al(Key::kKind == 3 ? tiles * TS : 0), o_res = o_pos + al(n * 2),
+                 total = o_res + al(tiles * TS * 8);
     uint8_t* scr = nullptr;
     cuart_status rc = scratch_alloc(h, (void**)&scr, total, s);
     if (rc != CUART_OK) return rc;
     uint32_t* toff = (uint32_t*)(scr + o_off);
     const uint32_t depth = (link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u) |
                            (h->bucket_shift << 8);
-    if (h->tsort_vec && (uintptr_t(q) & 15) == 0)
+    if constexpr (Key::kKind == 3)
+        k_tsort_bytes<<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint8_t*)q, lens, n, ByteBucket(depth), nb,
+                                                                scr + o_q, scr + o_len, (uint16_t*)(scr + o_pos), toff);
+    else if (h->tsort_vec && (uintptr_t(q) & 15) == 0)
         k_tsort<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, n, ByteBucket(depth), nb, scr + o_q,
                                                                      (uint16_t*)(scr + o_pos), toff);
     else
@@ -602,19 +610,27 @@ static cuart_status launch_tiled(const cuart_index* h, const void* q, uint64_t n
     if (h->tile_group) tg = h->tile_group;
     const uint32_t ngroups = uint32_t((tiles + tg - 1) / tg);
     const DevIndex& dx = h->dix_links;
-    const bool wide = dx.walk_wide && h->policy == 5 && h->ilp > 1;
+    const bool wide = Key::kKind != 3 && dx.walk_wide && h->policy == 5 && h->ilp > 1;
     cudaEvent_t ev0, ev1;
     ktimer_begin(h, s, ev0, ev1);
     const unsigned g = nb * ngroups;
     uint64_t* tres = (uint64_t*)(scr + o_res);
     // 20 CTAs/SM (48 registers instead of 52, no spill): c3 walk 9.42 -> 9.07 ms per 2^30
     // (profiles/r02/tile_form.txt); 24 CTAs/SM spills (40 registers + 24 B stack)
-    if (wide && h->wt_tpb == 128) k_lookup_wt<Key, 2, 128, 3, true, 10><<<g, 128, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
-    else if (wide && h->wt_tpb == 256) k_lookup_wt<Key, 2, 256, 3, true, 5><<<g, 256, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
-    else if (wide && h->wt_minb == 1) k_lookup_wt<Key, 2, 64, 3, true, 1><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
-    else if (wide && h->wt_minb == 24) k_lookup_wt<Key, 2, 64, 3, true, 24><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
-    else if (wide) k_lookup_wt<Key, 2, 64, 3, true, 20><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
-    else k_lookup_wt<Key, 2, 64, 3, false><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+    if constexpr (Key::kKind == 3) {
+        // byte strings: 256-thread CTAs at 8 CTAs/SM (32 registers): c4 walk 32.97 ms per
+        // 2^29 against 38.39 (64 threads, 46 registers) and 35.58 (64 threads, 24 CTAs/SM)
+        // (profiles/r02/tile_form.txt)
+        if (h->wt_tpb == 64) k_lookup_wt<Key, 1, 64, 3, false, 24><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres, scr + o_len);
+        else k_lookup_wt<Key, 1, 256, 3, false, 8><<<g, 256, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres, scr + o_len);
+    } else {
+        if (wide && h->wt_tpb == 128) k_lookup_wt<Key, 2, 128, 3, true, 10><<<g, 128, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+        else if (wide && h->wt_tpb == 256) k_lookup_wt<Key, 2, 256, 3, true, 5><<<g, 256, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+        else if (wide && h->wt_minb == 1) k_lookup_wt<Key, 2, 64, 3, true, 1><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+        else if (wide && h->wt_minb == 24) k_lookup_wt<Key, 2, 64, 3, true, 24><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+        else if (wide) k_lookup_wt<Key, 2, 64, 3, true, 20><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+        else k_lookup_wt<Key, 1, 64, 3, false><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
+    }
     g_cuart_launches++;
     ktimer_end(h, s, ev0, ev1, n);
     k_tgather<KS><<<unsigned(tiles), kBucketThreads, 0, s>>>(tres, (const uint16_t*)(scr + o_pos), toff, nb, n, out);
@@ -635,8 +651,9 @@ cuart_status launch_lookup(const cuart_index* h, uint32_t kind, const void* q, c
                       : h->prebucket == CUART_PREBUCKET_AUTO && n >= kBucketMin && kind != CUART_KEY_BYTES;
     if (bucket && n < (uint64_t(1) << 32)) {
         const bool tiled = h->bucket_form == CUART_BUCKET_TILE && !so && h->slice_lut != CUART_SLICE_ON;
-        if (tiled && kind == CUART_KEY_U64) return launch_tiled<KeyU64>(h, q, n, out, s);
-        if (tiled && kind == CUART_KEY_U32) return launch_tiled<KeyU32>(h, q, n, out, s);
+        if (tiled && kind == CUART_KEY_U64) return launch_tiled<KeyU64>(h, q, lens, n, out, s);
+        if (tiled && kind == CUART_KEY_U32) return launch_tiled<KeyU32>(h, q, lens, n, out, s);
+        if (tiled && kind == CUART_KEY_BYTES) return launch_tiled<KeyBytes>(h, q, lens, n, out, s);
         switch (kind) {
         case CUART_KEY_U64: return launch_bucketed<KeyU64>(h, q, lens, n, out, s, so);
         case CUART_KEY_U32: return launch_bucketed<KeyU32>(h, q, lens, n, out, s, so);

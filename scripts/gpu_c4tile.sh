@@ -1,0 +1,15 @@
+#!/bin/bash
+# byte-string tile form variants: c4 bench + launch lists
+mkdir -p gpurun_out
+M=gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sectors_srcunit_tex_op_read.sum
+timeout 900 python -m pytest tests/test_gpu_parity.py -m gpu -q -p no:cacheprovider -k "prebucket or misaligned" > gpurun_out/pytest_c4tile.log 2>&1; echo "rc=$?" >> gpurun_out/pytest_c4tile.log
+run() { # name env...
+  local name=$1; shift
+  env "$@" timeout 600 python bench.py --config c4 --no-e2e --no-cpu-baseline --steps 5 > gpurun_out/ab_$name.log 2>&1
+  env "$@" timeout 600 ncu --metrics $M --clock-control none -k regex:'k_' -c 4 --csv --log-file gpurun_out/ll_$name.csv python bench.py --config c4 --steps 1 --warmup 0 --no-e2e --no-cpu-baseline > /dev/null 2>&1
+}
+run c4_tile CUART_PREBUCKET=1
+run c4_tile_m24 CUART_PREBUCKET=1 CUART_WT_MINB=24
+run c4_tile_m32 CUART_PREBUCKET=1 CUART_WT_MINB=32
+run c4_tile_t256 CUART_PREBUCKET=1 CUART_WT_TPB=256
+run c4_global CUART_PREBUCKET=1 CUART_BUCKET_FORM=1
