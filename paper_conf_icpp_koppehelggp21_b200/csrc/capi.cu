@@ -587,9 +587,14 @@ static cuart_status launch_tiled(const cuart_index* h, const void* q, const uint
     uint32_t* toff = (uint32_t*)(scr + o_off);
     const uint32_t depth = (link_type(h->root) >= T_N4 && link_type(h->root) <= T_N256 ? link_aux(h->root) : 0u) |
                            (h->bucket_shift << 8);
-    if constexpr (Key::kKind == 3)
-        k_tsort_bytes<<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint8_t*)q, lens, n, ByteBucket(depth), nb,
-                                                                scr + o_q, scr + o_len, (uint16_t*)(scr + o_pos), toff);
+    if constexpr (Key::kKind == 3) {
+        if (h->tsort_b1k)
+            k_tsort_bytes1k<<<unsigned(tiles), 1024, 0, s>>>((const uint8_t*)q, lens, n, ByteBucket(depth), nb,
+                                                             scr + o_q, scr + o_len, (uint16_t*)(scr + o_pos), toff);
+        else
+            k_tsort_bytes<<<unsigned(tiles), kBucketThreads, 0, s>>>((const uint8_t*)q, lens, n, ByteBucket(depth), nb,
+                                                                    scr + o_q, scr + o_len, (uint16_t*)(scr + o_pos), toff);
+    }
     else if (h->tsort_vec && (uintptr_t(q) & 15) == 0)
         k_tsort<Key, true><<<unsigned(tiles), kBucketThreads, 0, s>>>(q, n, ByteBucket(depth), nb, scr + o_q,
                                                                      (uint16_t*)(scr + o_pos), toff);
@@ -622,6 +627,8 @@ static cuart_status launch_tiled(const cuart_index* h, const void* q, const uint
         // 2^29 against 38.39 (64 threads, 46 registers) and 35.58 (64 threads, 24 CTAs/SM)
         // (profiles/r02/tile_form.txt)
         if (h->wt_tpb == 64) k_lookup_wt<Key, 1, 64, 3, false, 24><<<g, 64, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres, scr + o_len);
+        else if (h->wt_tpb == 128) k_lookup_wt<Key, 1, 128, 3, false, 12><<<g, 128, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres, scr + o_len);
+        else if (h->wt_minb == 6) k_lookup_wt<Key, 1, 256, 3, false, 6><<<g, 256, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres, scr + o_len);
         else k_lookup_wt<Key, 1, 256, 3, false, 8><<<g, 256, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres, scr + o_len);
     } else {
         if (wide && h->wt_tpb == 128) k_lookup_wt<Key, 2, 128, 3, true, 10><<<g, 128, 0, s>>>(dx, scr + o_q, toff, n, nb, tg, ngroups, tres);
@@ -1164,6 +1171,7 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         if (const char* pe = getenv("CUART_WT_MINB")) h->wt_minb = uint32_t(atoi(pe));
         if (const char* pe = getenv("CUART_WT_TPB")) h->wt_tpb = uint32_t(atoi(pe));
         if (const char* pe = getenv("CUART_TSORT_VEC")) h->tsort_vec = uint32_t(atoi(pe));
+        if (const char* pe = getenv("CUART_TSORT_B1K")) h->tsort_b1k = uint32_t(atoi(pe));
         if (const char* pe = getenv("CUART_TILE_GROUP")) {
             const int v = atoi(pe);
             h->tile_group = v < 1 ? 1u : v > 32 ? 32u : uint32_t(v);

@@ -97,6 +97,7 @@ struct cuart_index {
     uint32_t tile_group = 0;                     // tiles per tile-form walk CTA (0 = from the bucket count)
     uint32_t wt_tpb = 0;                         // k_lookup_wt CTA size (0: 64 integer, 256 byte strings; knob CUART_WT_TPB)
     uint32_t tsort_vec = 1;                      // k_tsort with 16-B key loads when the batch is 16-B aligned (knob CUART_TSORT_VEC)
+    uint32_t tsort_b1k = 0;                      // byte-string tile sort: 1024 threads, keys in registers (knob CUART_TSORT_B1K)
     uint32_t wt_minb = 20;                       // k_lookup_wt min CTAs/SM (register cap; A/B knob CUART_WT_MINB: 1, 20, 24)
     uint32_t slice_lut = CUART_SLICE_AUTO;       // bucketed walk with the bucket's LUT slice in smem
     bool slice_ok = false;                       // RANK table, integer keys, root branch depth + 2 <= k
