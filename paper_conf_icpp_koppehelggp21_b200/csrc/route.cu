@@ -185,6 +185,166 @@ __global__ void __launch_bounds__(256) k_unroute(const uint64_t* __restrict__ in
     for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) out[i] = in[perm[i]];
 }
 
+// ---- two-way stable partition by flag (cuart_partition_by_flag) ------------
+// Ops with flag 0 first, then flag != 0, each in op order.  A thread owns 16
+// CONSECUTIVE ops of a 4096-op tile, so one block scan of the per-thread counts
+// ranks the whole tile (no per-round barriers): k_pf_count counts the tile's flag-0
+// ops (16-B flag loads), k_pf_scan turns the counts into tile offsets, k_pf_scatter
+// places every op at (flag 0) off0[tile] + rank or (flag 1) L + (tile base - off0[tile])
+// + rank.  Streaming bytes per u64 op: 1 (count) + 1 + 8 + 8 read, 8 + 8 + 4 written.
+constexpr int kPfPer = kRouteChunk / kRouteThreads;     // 16 consecutive ops per thread
+
+__device__ __forceinline__ uint32_t zero_flag_count16(uint4 v) {
+    uint32_t c = 0;
+#pragma unroll
+    for (int w = 0; w < 4; w++) {
+        const uint32_t x = (&v.x)[w];
+#pragma unroll
+        for (int b = 0; b < 4; b++) c += ((x >> (8 * b)) & 0xFFu) == 0 ? 1u : 0u;
+    }
+    return c;
+}
+
+// block-wide exclusive scan of one value per thread (256 threads); total -> *tot
+__device__ __forceinline__ uint32_t pf_block_scan(uint32_t v, uint32_t* wsum, uint32_t* tot) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t x = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
+        if (lane >= d) x += y;
+    }
+    if (lane == 31) wsum[warp] = x;
+    __syncthreads();
+    uint32_t before = 0, all = 0;
+#pragma unroll
+    for (int w = 0; w < kRouteThreads / 32; w++) {
+        before += w < warp ? wsum[w] : 0u;
+        all += wsum[w];
+    }
+    if (tot) *tot = all;
+    return before + x - v;
+}
+
+__device__ __forceinline__ uint4 pf_flags16(const uint8_t* flags, uint64_t i, uint64_t n) {
+    if (i + kPfPer <= n && (uintptr_t(flags + i) & 15) == 0) return *(const uint4*)(flags + i);
+    uint4 v = make_uint4(0x01010101u, 0x01010101u, 0x01010101u, 0x01010101u);   // past the end: "flag 1", never placed
+    for (int e = 0; e < kPfPer; e++)
+        if (i + e < n) {
+            const uint32_t sh = 8 * (e & 3);
+            uint32_t& w = (&v.x)[e >> 2];
+            w = (w & ~(0xFFu << sh)) | (uint32_t(flags[i + e]) << sh);
+        }
+    return v;
+}
+
+__global__ void __launch_bounds__(kRouteThreads) k_pf_count(const uint8_t* __restrict__ flags, uint64_t n,
+                                                            uint32_t* __restrict__ cnt0) {
+    __shared__ uint32_t wsum[kRouteThreads / 32];
+    __shared__ uint32_t tot;
+    const uint64_t i = uint64_t(blockIdx.x) * kRouteChunk + uint64_t(threadIdx.x) * kPfPer;
+    const uint32_t c = i < n ? zero_flag_count16(pf_flags16(flags, i, n)) : 0u;
+    pf_block_scan(c, wsum, threadIdx.x == 0 ? &tot : nullptr);
+    if (threadIdx.x == 0) cnt0[blockIdx.x] = tot;
+}
+
+// One CTA: exclusive scan of the per-tile flag-0 counts (in place) + counts[0..1].
+__global__ void __launch_bounds__(1024) k_pf_scan(uint32_t* __restrict__ cnt0, uint64_t ntiles, uint64_t n,
+                                                  uint64_t* __restrict__ counts) {
+    __shared__ uint64_t wsum[32];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint64_t per = (ntiles + 1023) / 1024;
+    const uint64_t t0 = uint64_t(threadIdx.x) * per;
+    uint64_t s = 0;
+    for (uint64_t t = t0; t < t0 + per && t < ntiles; t++) s += cnt0[t];
+    uint64_t x = s;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint64_t y = __shfl_up_sync(0xffffffffu, x, d);
+        if (lane >= d) x += y;
+    }
+    if (lane == 31) wsum[warp] = x;
+    __syncthreads();
+    uint64_t before = 0, all = 0;
+    for (int w = 0; w < 32; w++) {
+        before += w < warp ? wsum[w] : 0;
+        all += wsum[w];
+    }
+    uint64_t run = before + x - s;
+    for (uint64_t t = t0; t < t0 + per && t < ntiles; t++) {
+        const uint32_t c = cnt0[t];
+        cnt0[t] = uint32_t(run);
+        run += c;
+    }
+    if (threadIdx.x == 0) {
+        counts[0] = all;
+        counts[1] = n - all;
+    }
+}
+
+__global__ void __launch_bounds__(kRouteThreads) k_pf_scatter(uint32_t kind, const void* __restrict__ keys,
+                                                              const uint8_t* __restrict__ lens,
+                                                              const uint64_t* __restrict__ values, uint64_t n,
+                                                              const uint8_t* __restrict__ flags,
+                                                              const uint32_t* __restrict__ off0,
+                                                              const uint64_t* __restrict__ counts,
+                                                              void* __restrict__ out_keys, uint8_t* __restrict__ out_lens,
+                                                              uint64_t* __restrict__ out_values,
+                                                              uint32_t* __restrict__ perm) {
+    __shared__ uint32_t wsum[kRouteThreads / 32];
+    __shared__ uint32_t sdst[kRouteChunk];                            // destination slot of every op of the tile
+    const uint64_t tb = uint64_t(blockIdx.x) * kRouteChunk;
+    const uint64_t i0 = tb + uint64_t(threadIdx.x) * kPfPer;
+    const uint4 fv = pf_flags16(flags, i0, n);
+    const uint32_t c0 = i0 < n ? zero_flag_count16(fv) : 0u;
+    const uint32_t r0 = pf_block_scan(c0, wsum, nullptr);             // flag-0 ops before mine in the tile
+    const uint64_t L = counts[0];
+    const uint64_t b0 = off0[blockIdx.x];                              // flag-0 ops before this tile
+    // slots relative to the partition's flag-0 / flag-1 bases fit 32 bits (n < 2^32)
+    uint32_t p0 = uint32_t(b0 + r0);                                   // next flag-0 slot
+    uint32_t p1 = uint32_t(L + (tb - b0) + (uint64_t(threadIdx.x) * kPfPer - r0));   // next flag-1 slot
+#pragma unroll
+    for (int e = 0; e < kPfPer; e++) {
+        const bool f = (((&fv.x)[e >> 2] >> (8 * (e & 3))) & 0xFFu) != 0;
+        sdst[threadIdx.x * kPfPer + e] = f ? p1++ : p0++;
+    }
+    __syncthreads();
+    // the copy: op j of the tile in coalesced order; runs of equal flags land in
+    // consecutive slots, so the stores are coalesced too
+#pragma unroll 4
+    for (int r = 0; r < kPfPer; r++) {
+        const uint32_t j = uint32_t(r) * kRouteThreads + threadIdx.x;
+        const uint64_t i = tb + j;
+        if (i >= n) break;
+        const uint64_t dst = sdst[j];
+        perm[i] = uint32_t(dst);
+        if (kind == CUART_KEY_U64) ((uint64_t*)out_keys)[dst] = ((const uint64_t*)keys)[i];
+        else if (kind == CUART_KEY_U32) ((uint32_t*)out_keys)[dst] = ((const uint32_t*)keys)[i];
+        else {
+            const uint4* src = (const uint4*)keys + 2 * i;
+            uint4* d = (uint4*)out_keys + 2 * dst;
+            d[0] = src[0];
+            d[1] = src[1];
+            out_lens[dst] = lens[i];
+        }
+        if (values) out_values[dst] = values[i];
+    }
+}
+
+// out[i] = in[perm[i]], 4 ops per thread (16-B perm loads and 32-B stores when aligned)
+__global__ void __launch_bounds__(256) k_unroute4(const uint64_t* __restrict__ in, const uint32_t* __restrict__ perm,
+                                                  uint64_t n, uint64_t* __restrict__ out) {
+    const uint64_t i = (uint64_t(blockIdx.x) * 256 + threadIdx.x) * 4;
+    if (i + 4 <= n) {
+        const uint4 p = __ldcs((const uint4*)(perm + i));
+        const uint64_t a = in[p.x], b = in[p.y], c = in[p.z], d = in[p.w];
+        __stcs((ulonglong2*)(out + i), make_ulonglong2(a, b));
+        __stcs((ulonglong2*)(out + i) + 1, make_ulonglong2(c, d));
+    } else {
+        for (uint64_t j = i; j < n; j++) out[j] = in[perm[j]];
+    }
+}
+
 }  // namespace
 
 extern std::atomic<uint64_t> g_cuart_launches;
@@ -212,8 +372,22 @@ cuart_status cuart_partition_by_flag(const cuart_keys* keys, size_t n, const uin
                                      void* out_keys, uint8_t* out_lengths, uint64_t* out_values, uint32_t* perm,
                                      uint64_t* counts, void* scratch, void* stream) {
     if (n > 0 && !flags) return CUART_ERR_INVALID_ARGUMENT;
-    return route_impl(keys, n, nullptr, flags, 2, values, out_keys, out_lengths, out_values, perm, counts, scratch,
-                      stream);
+    if (!keys || !counts) return CUART_ERR_INVALID_ARGUMENT;
+    if (n >= (uint64_t(1) << 32)) return CUART_ERR_INVALID_ARGUMENT;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (n == 0) return cudaMemsetAsync(counts, 0, 2 * sizeof(uint64_t), s) == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+    if (!keys->data || !out_keys || !perm || !scratch) return CUART_ERR_INVALID_ARGUMENT;
+    if (keys->kind == CUART_KEY_BYTES && (!keys->lengths || !out_lengths)) return CUART_ERR_INVALID_ARGUMENT;
+    if (values && !out_values) return CUART_ERR_INVALID_ARGUMENT;
+    const uint64_t ntiles = (n + kRouteChunk - 1) / kRouteChunk;
+    uint32_t* cnt0 = (uint32_t*)((uint8_t*)scratch + ((n + 255) & ~size_t(255)));   // the route histogram's space
+    const uint32_t kind = uint32_t(keys->kind);
+    k_pf_count<<<unsigned(ntiles), kRouteThreads, 0, s>>>(flags, n, cnt0);
+    k_pf_scan<<<1, 1024, 0, s>>>(cnt0, ntiles, n, counts);
+    k_pf_scatter<<<unsigned(ntiles), kRouteThreads, 0, s>>>(kind, keys->data, keys->lengths, values, n, flags, cnt0,
+                                                            counts, out_keys, out_lengths, out_values, perm);
+    g_cuart_launches += 3;
+    return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
 }
 
 static cuart_status route_impl(const cuart_keys* keys, size_t n, const uint64_t* splitters, const uint8_t* flags,
@@ -252,6 +426,11 @@ cuart_status cuart_fill_miss(uint64_t* out, size_t n, void* stream) {
 cuart_status cuart_unroute(const uint64_t* in, const uint32_t* perm, size_t n, uint64_t* out, void* stream) {
     if (n == 0) return CUART_OK;
     if (!in || !perm || !out) return CUART_ERR_INVALID_ARGUMENT;
+    if ((uintptr_t(perm) & 15) == 0 && (uintptr_t(out) & 15) == 0 && (n + 1023) / 1024 < (uint64_t(1) << 31)) {
+        k_unroute4<<<unsigned((n + 1023) / 1024), 256, 0, (cudaStream_t)stream>>>(in, perm, n, out);
+        g_cuart_launches += 1;
+        return cudaGetLastError() == cudaSuccess ? CUART_OK : CUART_ERR_CUDA;
+    }
     uint64_t blocks = (n + 255) / 256;
     if (blocks > (uint64_t(1) << 31) - 1) blocks = (uint64_t(1) << 31) - 1;
     k_unroute<<<unsigned(blocks), 256, 0, (cudaStream_t)stream>>>(in, perm, n, out);

@@ -97,3 +97,58 @@ def test_route_matches_stable_partition(kind, nparts, n):
     assert np.array_equal(sv.cpu().numpy().view(np.uint64), vals[order])
     back = _unroute(sv, perm)
     assert np.array_equal(back.cpu().numpy().view(np.uint64), vals)
+
+
+@pytest.mark.parametrize("kind", ["u64", "u32", "bytes"])
+@pytest.mark.parametrize("n,p", [(1, 0.5), (4095, 0.1), (4096 * 3 + 17, 0.1), (200_003, 0.5), (70_001, 0.0),
+                                 (70_001, 1.0)])
+def test_partition_by_flag_matches_stable_partition(kind, n, p):
+    """cuart_partition_by_flag (the two-way partition that splits config 5's mixed
+    rounds, reading C7): flag-0 ops first, then flag-1 ops, each in op order, with
+    the values carried along; perm[i] = slot of op i and cuart_unroute inverts it.
+    Ragged tails, all-lookup and all-update batches, and a flags view 1 byte into
+    its buffer (unaligned 16-B flag loads fall back to scalar loads)."""
+    rng = np.random.default_rng(n + int(p * 10))
+    if kind == "u64":
+        keys = rng.integers(0, 2**64, n, dtype=np.uint64)
+        lens = None
+    elif kind == "u32":
+        keys = rng.integers(0, 2**32, n, dtype=np.uint32)
+        lens = None
+    else:
+        keys = rng.integers(1, 256, (n, 32), dtype=np.uint8)
+        lens = rng.integers(1, 33, n, dtype=np.uint8)
+    vals = rng.integers(0, 2**63, n, dtype=np.uint64)
+    flags = (rng.random(n) < p).astype(np.uint8)
+    order = np.argsort(flags, kind="stable")
+    want_perm = np.empty(n, np.int64)
+    want_perm[order] = np.arange(n)
+    for off in (0, 1):
+        fbuf = torch.zeros(n + 1, dtype=torch.uint8, device=DEV)
+        fv = fbuf[off:off + n]
+        fv.copy_(torch.from_numpy(flags).to(DEV))
+        kt = _t(keys)
+        lt = _t(lens) if lens is not None else None
+        vt = _t(vals)
+        ok, ov = torch.empty_like(kt), torch.empty_like(vt)
+        ol = torch.empty_like(lt) if lt is not None else None
+        perm = torch.empty(n, dtype=torch.int32, device=DEV)
+        counts = torch.empty(2, dtype=torch.int64, device=DEV)
+        scratch = torch.empty(max(1, B.lib().cuart_route_scratch_bytes(n, 2)), dtype=torch.uint8, device=DEV)
+        k, _, keep = B.make_keys((kt, lt) if lt is not None else kt)
+        stream = torch.cuda.current_stream().cuda_stream
+        B._check(B.lib().cuart_partition_by_flag(ctypes.byref(k), n, fv.data_ptr(), vt.data_ptr(), ok.data_ptr(),
+                                                 ol.data_ptr() if ol is not None else None, ov.data_ptr(),
+                                                 perm.data_ptr(), counts.data_ptr(), scratch.data_ptr(), stream),
+                 "cuart_partition_by_flag")
+        torch.cuda.synchronize()
+        nl = int((flags == 0).sum())
+        assert counts.cpu().tolist() == [nl, n - nl]
+        assert np.array_equal(perm.cpu().numpy().astype(np.int64), want_perm)
+        got_k = ok.cpu().numpy()
+        assert np.array_equal(got_k.view(keys.dtype) if kind != "bytes" else got_k, keys[order])
+        if lens is not None:
+            assert np.array_equal(ol.cpu().numpy(), lens[order])
+        assert np.array_equal(ov.cpu().numpy().view(np.uint64), vals[order])
+        back = _unroute(ov, perm)
+        assert np.array_equal(back.cpu().numpy().view(np.uint64), vals)
