@@ -54,6 +54,8 @@ def _args():
     p.add_argument("--config", default="c3", choices=["c1", "c2", "c3", "c4", "c5"])
     p.add_argument("--impl", default="cuart", choices=["cuart", "reference"])
     p.add_argument("--lut", type=int, default=3)
+    p.add_argument("--skip-log2", type=int, default=0,
+                   help="byte-string skip table cap (cuart_build_opts.skip_log2; 0 = library choice)")
     p.add_argument("--lut-format", default="auto", choices=["auto", "links", "compact32", "rank"],
                    help="device form of the root table (cuart_build_opts.lut_format)")
     p.add_argument("--no-e2e", action="store_true")
@@ -449,7 +451,7 @@ def main():
     keys, vals, keys_d = make_keys(cfg, dev)
     if world == 1 and not args.dist:
         layout = C.Layout(keys, vals, lut_bytes=args.lut)
-        ix = C.Index.from_layout(layout, device=local, lut_format=LUT_FORMATS[args.lut_format],
+        ix = C.Index.from_layout(layout, device=local, lut_format=LUT_FORMATS[args.lut_format], skip_log2=args.skip_log2,
                                  l2_persist=args.l2_persist)
         di = None
     else:
@@ -666,6 +668,7 @@ def main():
             "config": {"workload": f"{args.config}: {cfg.description}", "keys": cfg.n_keys,
                        "lookups_per_rank": nl, "updates_per_rank": nu, "key_kind": cfg.kind,
                        "lut_bytes": args.lut, "lut_format": stats["lut_format"], "mode": mode,
+                       "skip_table": {"prefix_bytes": stats.get("skip_prefix", 0), "slots": stats.get("skip_slots", 0)},
                        "transport": args.transport if (world > 1 or args.dist) and mode == "range" else None,
                        "parallelism": f"{mode}{world}" if world > 1 or args.dist else "single",
                        "l2": f"inputs ({q_bytes / 2**30:.1f} GiB of queries per step) larger than L2; no flush",

@@ -133,6 +133,13 @@ typedef struct {
                                     form too; multi-GPU owner walks (fused return) and
                                     update batches use the global form.  Results are
                                     identical.                                             */
+    uint32_t skip_log2;          /* byte-string indexes: skip table over the first D key bytes
+                                    ("merged upper layers", where the first bytes do not
+                                    discriminate): D = the longest prefix (<= 16 B) with at most
+                                    2^skip_log2 distinct values among the keys; a lookup starts at
+                                    the node covering its D-byte prefix.  0 = library choice
+                                    (2^20: table <= 64 MB, L2-resident); 1..26 explicit; the
+                                    env CUART_SKIP=0 disables it.  Results are identical.     */
 } cuart_build_opts;
 #define CUART_BUCKET_FORM_AUTO 0u
 #define CUART_BUCKET_GLOBAL 1u
@@ -168,6 +175,8 @@ typedef struct {
     uint64_t lut_exceptions;     /* RANK: entries served by the 64-bit link table */
     uint32_t wide_lut;           /* 1: pre-bucketed walks start from the wide root table */
     uint64_t l2_window_bytes;    /* l2_persist: bytes under the persisting access-policy window */
+    uint32_t skip_prefix;        /* byte strings: prefix length D of the skip table (0 = none) */
+    uint64_t skip_slots;         /* its slots (32 B each; at most half of them used)          */
 } cuart_stats_t;
 
 typedef struct cuart_index cuart_index;    /* device-resident index (opaque) */

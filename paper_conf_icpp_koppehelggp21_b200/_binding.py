@@ -27,7 +27,7 @@ class _Keys(ctypes.Structure):
 class _Opts(ctypes.Structure):
     _fields_ = [("lut_bytes", ctypes.c_uint32), ("l2_persist", ctypes.c_uint32),
                 ("device", ctypes.c_int32), ("lut_format", ctypes.c_uint32), ("prebucket", ctypes.c_uint32), ("slice_lut", ctypes.c_uint32), ("wide_lut", ctypes.c_uint32),
-                ("bucket_form", ctypes.c_uint32)]
+                ("bucket_form", ctypes.c_uint32), ("skip_log2", ctypes.c_uint32)]
 
 
 class _Stats(ctypes.Structure):
@@ -35,7 +35,8 @@ class _Stats(ctypes.Structure):
                 ("lut_entries", ctypes.c_uint64), ("lut_bytes_total", ctypes.c_uint64),
                 ("arena_bytes", ctypes.c_uint64), ("lut_bytes", ctypes.c_uint32), ("key_kind", ctypes.c_uint32),
                 ("root", ctypes.c_uint64), ("max_depth", ctypes.c_uint32), ("lut_format", ctypes.c_uint32),
-                ("lut_exceptions", ctypes.c_uint64), ("wide_lut", ctypes.c_uint32), ("l2_window_bytes", ctypes.c_uint64)]
+                ("lut_exceptions", ctypes.c_uint64), ("wide_lut", ctypes.c_uint32), ("l2_window_bytes", ctypes.c_uint64),
+                ("skip_prefix", ctypes.c_uint32), ("skip_slots", ctypes.c_uint64)]
 
 
 class _View(ctypes.Structure):
@@ -180,8 +181,8 @@ BUCKET_FORM_AUTO, BUCKET_GLOBAL, BUCKET_TILE = 0, 1, 2
 
 
 def _opts(lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0, wide_lut=0,
-          bucket_form=0):
-    return _Opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form)
+          bucket_form=0, skip_log2=0):
+    return _Opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form, skip_log2)
 
 
 def _stream_ptr(stream):
@@ -195,14 +196,14 @@ def _stream_ptr(stream):
 
 # ------------------------------------------------------------------ hot path
 def cuart_build(keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0,
-                slice_lut=0, wide_lut=0, bucket_form=0):
+                slice_lut=0, wide_lut=0, bucket_form=0, skip_log2=0):
     """Build + upload (host buffers).  Returns an opaque handle (int)."""
     k, n, keep = make_keys(keys)
     v = np.ascontiguousarray(values, dtype=np.uint64)
     if v.shape[0] != n:
         raise ValueError("values length mismatch")
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form)
+    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form, skip_log2)
     _check(lib().cuart_build(ctypes.byref(k), _ptr(v), n, ctypes.byref(o), ctypes.byref(h)), "cuart_build")
     return h.value
 
@@ -327,7 +328,7 @@ def _stats_dict(s):
     d.update(n_keys=int(s.n_keys), lut_bytes=int(s.lut_bytes), lut_entries=int(s.lut_entries),
              arena_bytes=int(s.arena_bytes), root=int(s.root), max_depth=int(s.max_depth), key_kind=int(s.key_kind),
              lut_format=int(s.lut_format), lut_exceptions=int(s.lut_exceptions), wide_lut=int(s.wide_lut),
-             l2_window_bytes=int(s.l2_window_bytes))
+             l2_window_bytes=int(s.l2_window_bytes), skip_prefix=int(s.skip_prefix), skip_slots=int(s.skip_slots))
     return d
 
 
@@ -383,9 +384,9 @@ def cuart_layout_sectors(l, queries, threads=0, wide=False):
 
 
 def cuart_upload(l, lut_bytes=0, l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0, wide_lut=0,
-                 bucket_form=0):
+                 bucket_form=0, skip_log2=0):
     h = ctypes.c_void_p()
-    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form)
+    o = _opts(lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form, skip_log2)
     _check(lib().cuart_upload(l, ctypes.byref(o), ctypes.byref(h)), "cuart_upload")
     return h.value
 
@@ -440,17 +441,18 @@ class Index:
     """Device-resident CuART index on one GPU."""
 
     def __init__(self, keys, values, lut_bytes=CUART_LUT_AUTO, l2_persist=0, device=-1, lut_format=0, prebucket=0,
-                 slice_lut=0, wide_lut=0, bucket_form=0):
+                 slice_lut=0, wide_lut=0, bucket_form=0, skip_log2=0):
         self.h = cuart_build(keys, values, lut_bytes, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut,
-                             bucket_form)
+                             bucket_form, skip_log2)
         self.device = _torch_device(device)
 
     @classmethod
     def from_layout(cls, layout: "Layout", l2_persist=0, device=-1, lut_format=0, prebucket=0, slice_lut=0,
-                    wide_lut=0, bucket_form=0):
+                    wide_lut=0, bucket_form=0, skip_log2=0):
         """Upload an already-built host layout (keeps the host copy usable)."""
         self = cls.__new__(cls)
-        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form)
+        self.h = cuart_upload(layout.h, 0, l2_persist, device, lut_format, prebucket, slice_lut, wide_lut, bucket_form,
+                              skip_log2)
         self.device = _torch_device(device)
         return self
 

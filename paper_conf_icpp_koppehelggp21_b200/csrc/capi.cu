@@ -58,7 +58,7 @@ static void drop_kevents(cuart_index* h) {
 // ============================================================================ kernels
 // SEG: out is ignored, result i goes to so.at(i) (fused multi-GPU return, §8(e)).
 template <class Key, int POL, bool SEG = false, int TPB = 256>
-__global__ void __launch_bounds__(TPB) k_lookup(DevIndex ix, const void* __restrict__ q,
+__global__ void __launch_bounds__(TPB, Key::kKind == 3 && TPB == 256 ? 8 : 1) k_lookup(DevIndex ix, const void* __restrict__ q,
                                                 const uint8_t* __restrict__ lens, uint64_t n,
                                                 uint64_t* __restrict__ out, SegOut so = SegOut{}) {
     const Loader<POL> ld;
@@ -1058,6 +1058,113 @@ static uint64_t expand_lut32_host(uint32_t e, uint32_t k, uint32_t leaf_len) {
 // index is base[type] + (number of earlier entries of that type in the block).
 // Leaves (lexicographically numbered, so not consecutive) and everything else are
 // exceptions read from the full 64-bit table.  Integer keys only.
+// ---- skip table (byte strings; kernels.cuh skip_start) -----------------------
+// The node covering every key with the D-byte prefix P: walk from the root table (or
+// the root) following P's bytes until a leaf or an inner node branching at depth >= D.
+static uint64_t skip_cover(const HostLayout& L, const uint8_t* P, uint32_t D) {
+    uint64_t link = L.root;
+    if (L.lut_bytes && D >= L.lut_bytes && !L.lut.empty()) {
+        uint64_t p = 0;
+        for (uint32_t b = 0; b < L.lut_bytes; b++) p = (p << 8) | P[b];
+        link = L.lut[p];
+    }
+    for (;;) {
+        const uint32_t t = link_type(link), aux = link_aux(link);
+        if (t == T_NULL || t >= T_LEAF8 || aux >= D) return link;
+        const uint8_t* rec = L.buf[t].data() + link_index(link) * record_bytes(t);
+        const uint32_t b = P[aux];
+        uint64_t child = 0;
+        if (t == T_N4 || t == T_N16) {
+            const uint8_t* keys = rec + (t == T_N4 ? kN4Keys : kN16Keys);
+            const int nk = t == T_N4 ? 4 : 16;
+            int c = -1;
+            for (int i = 0; i < nk; i++)
+                if (keys[i] == b) {
+                    c = i;
+                    break;
+                }
+            if (c < 0) return 0;
+            memcpy(&child, rec + (t == T_N4 ? kN4Child : kN16Child) + 8 * c, 8);
+        } else if (t == T_N48) {
+            const uint8_t s = rec[kN48Index + b];
+            if (s == kN48Empty) return 0;
+            memcpy(&child, rec + kN48Child + 8 * s, 8);
+        } else {
+            memcpy(&child, rec + kN256Child + 8 * b, 8);
+        }
+        link = child;
+    }
+}
+
+// D = the largest prefix length in [lut_bytes + 2, 16] whose distinct prefixes (an
+// upper bound: counted per leaf class, each sorted) number at most 2^18, so the
+// table (2 slots per prefix, 32 B each: <= 16 MB) stays L2-resident.  Returns false
+// (no table) for integer keys or when no such D exists.
+static bool build_skip_table(const HostLayout& L, std::vector<uint64_t>& tab, uint32_t& D, uint64_t& mask,
+                             uint32_t max_log2) {
+    if (L.key_kind != CUART_KEY_BYTES || L.root == 0) return false;
+    uint64_t cnt[17] = {0};
+    for (int t = T_LEAF8; t <= T_LEAF32; t++) {
+        const uint64_t m = L.count[t];
+        const uint32_t kb = kLeafKeyBytes[t];
+        for (uint64_t i = 0; i < m; i++) {
+            const uint8_t* k = L.buf[t].data() + i * record_bytes(t);
+            const uint32_t len = L.leaf_len[t].empty() ? kb : L.leaf_len[t][i];
+            uint32_t lcp = 0, plen = 0;
+            if (i > 0) {
+                const uint8_t* pk = k - record_bytes(t);
+                plen = L.leaf_len[t].empty() ? kb : L.leaf_len[t][i - 1];
+                while (lcp < 16 && lcp < kb && pk[lcp] == k[lcp]) lcp++;
+            }
+            for (uint32_t d = 1; d <= 16 && d <= len; d++)
+                if (i == 0 || lcp < d || plen < d) cnt[d]++;
+        }
+    }
+    D = 0;
+    for (uint32_t d = 16; d >= L.lut_bytes + 2 && d >= 2; d--)
+        if (cnt[d] > 0 && cnt[d] <= (uint64_t(1) << max_log2)) {
+            D = d;
+            break;
+        }
+    if (D == 0) return false;
+    uint64_t slots = 1;
+    while (slots < 2 * cnt[D]) slots <<= 1;
+    mask = slots - 1;
+    tab.assign(slots * 4, 0);
+    for (int t = T_LEAF8; t <= T_LEAF32; t++) {
+        const uint64_t m = L.count[t];
+        const uint32_t kb = kLeafKeyBytes[t];
+        for (uint64_t i = 0; i < m; i++) {
+            const uint8_t* k = L.buf[t].data() + i * record_bytes(t);
+            const uint32_t len = L.leaf_len[t].empty() ? kb : L.leaf_len[t][i];
+            if (len < D) continue;
+            uint8_t P[16] = {0};
+            memcpy(P, k, D < kb ? D : kb);
+            uint64_t p0, p1;
+            memcpy(&p0, P, 8);
+            memcpy(&p1, P + 8, 8);
+            p0 &= low_bytes_mask(D < 8 ? D : 8u);
+            p1 = D > 8 ? p1 & low_bytes_mask(D - 8) : 0ull;
+            uint64_t h = skip_hash(p0, p1) & mask;
+            bool present = false;
+            while (tab[4 * h + 2] != 0) {
+                if (tab[4 * h] == p0 && tab[4 * h + 1] == p1) {
+                    present = true;
+                    break;
+                }
+                h = (h + 1) & mask;
+            }
+            if (present) continue;
+            const uint64_t link = skip_cover(L, P, D);
+            if (link == 0) continue;                       // cannot happen for a stored key
+            tab[4 * h] = p0;
+            tab[4 * h + 1] = p1;
+            tab[4 * h + 2] = link;
+        }
+    }
+    return true;
+}
+
 static bool rank_lut(const HostLayout& L, std::vector<uint64_t>& blocks, uint64_t& n_exc) {
     if (L.lut.empty() || L.key_kind == CUART_KEY_BYTES) return false;
     const uint32_t k = L.lut_bytes;
@@ -1243,6 +1350,18 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     }
     h->lutw_off = off;
     off = align(off + lutw.size() * 8);
+    std::vector<uint64_t> skipt;
+    uint32_t skip_d = 0;
+    uint64_t skip_mask = 0;
+    {
+        const char* pe = getenv("CUART_SKIP");
+        uint32_t lg = opts && opts->skip_log2 ? opts->skip_log2 : 20u;
+        if (const char* pl = getenv("CUART_SKIP_LOG2")) lg = uint32_t(atoi(pl));
+        lg = lg > 26 ? 26u : lg;
+        if (!(pe && atoi(pe) == 0)) build_skip_table(L, skipt, skip_d, skip_mask, lg);
+    }
+    h->skip_off = off;
+    off = align(off + skipt.size() * 8);
     h->err_off = off;
     off = align(off + 256);
     h->arena_bytes = off;
@@ -1269,6 +1388,9 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && !lutr.empty() &&
         cudaMemcpy(h->arena + h->lutc_off, lutr.data(), lutr.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
+        rc = CUART_ERR_CUDA;
+    if (rc == CUART_OK && !skipt.empty() &&
+        cudaMemcpy(h->arena + h->skip_off, skipt.data(), skipt.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
         rc = CUART_ERR_CUDA;
     if (rc == CUART_OK && !lutw.empty() &&
         cudaMemcpy(h->arena + h->lutw_off, lutw.data(), lutw.size() * 8, cudaMemcpyHostToDevice) != cudaSuccess)
@@ -1348,6 +1470,11 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
     d.lutw = h->wide ? (uint64_t*)(h->arena + h->lutw_off) : nullptr;
     d.lut_entries = L.lut.size();
     d.walk_wide = 0;
+    d.skip = skipt.empty() ? nullptr : (const uint64_t*)(h->arena + h->skip_off);
+    d.skip_mask = skip_mask;
+    d.skip_d = skip_d;
+    h->skip_d = skip_d;
+    h->skip_entries = skipt.size() / 4;
     h->dix_links = d;
     if (d.lut) {
         h->dix_links.lutr = nullptr;
@@ -1787,6 +1914,8 @@ cuart_status cuart_stats(const cuart_index* h, cuart_stats_t* s) {
     s->lut_exceptions = h->lut_exceptions;
     s->wide_lut = h->wide ? 1u : 0u;
     s->l2_window_bytes = h->l2_bytes;
+    s->skip_prefix = h->skip_d;
+    s->skip_slots = h->skip_entries;
     s->arena_bytes = h->arena_bytes;
     s->key_kind = h->key_kind;
     s->root = h->root;

@@ -71,6 +71,9 @@ struct cuart_index {
     uint32_t lut_format = CUART_LUT_LINKS;
     uint64_t lutc_off = 0;             // compact / rank LUT region
     uint64_t lutw_off = 0;             // wide LUT region (32 B/entry), 0 bytes if absent
+    uint64_t skip_off = 0;             // skip table region (byte strings), 0 bytes if absent
+    uint32_t skip_d = 0;               // its prefix length (0: no table)
+    uint64_t skip_entries = 0;         // its slots
     bool wide = false;
     uint64_t lut_exceptions = 0;       // RANK: entries served by the 64-bit table
     int grid_ctas_per_sm = 0;          // 0 = default grid (one op per thread); else persistent grid

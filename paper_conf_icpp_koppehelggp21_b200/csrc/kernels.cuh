@@ -30,6 +30,11 @@ struct DevIndex {
     uint64_t* lutw;               // wide root table (32 B/entry: link + the target N4/N16's keys), or nullptr
     uint64_t lut_entries;         // 2^(8 lut_bytes)
     uint32_t walk_wide;           // 1: lookups start from lutw (pre-bucketed walks, whose lutw slice is L2-resident)
+    // byte strings: skip table over the first skip_d key bytes (32-B entries {prefix
+    // words p0, p1, link of the node covering that prefix, 0}, open addressing), or nullptr
+    const uint64_t* skip;
+    uint64_t skip_mask;
+    uint32_t skip_d;
 };
 
 // Segmented output (multi-GPU fused return, §8(e)): result i goes to
@@ -482,9 +487,35 @@ __device__ __forceinline__ uint64_t start_wide(const DevIndex& ix, const Loader<
     return decode_wide(ix, ld, key, ld.lutv8(ix.lutw + p * 4));
 }
 
+// Skip table ("merged upper layers", for byte strings whose first bytes do
+// not discriminate: c4's keys share 6-byte segments, so the 3-byte root table skips
+// one level only).  Entry = the node covering every key with a given D-byte prefix
+// (the first node on the path whose branch depth is >= D, or the leaf), so a walk
+// can start there; a prefix absent from the table belongs to no key of length >= D.
+// One 32-B request (the table is small and L2-resident) replaces the top levels.
+template <int POL>
+__device__ __forceinline__ uint64_t skip_start(const DevIndex& ix, const Loader<POL>& ld, const KeyBytes& key) {
+    const uint32_t D = ix.skip_d;
+    const uint64_t p0 = key.w[0] & low_bytes_mask(D < 8 ? D : 8u);
+    const uint64_t p1 = D > 8 ? key.w[1] & low_bytes_mask(D - 8) : 0ull;
+    uint64_t h = skip_hash(p0, p1) & ix.skip_mask;
+#pragma unroll 1
+    for (;;) {
+        const U8x32 e = ld.lutv8(ix.skip + 4 * h);
+        const uint64_t link = uint64_t(e.w[4]) | (uint64_t(e.w[5]) << 32);
+        if (link == 0) return 0;
+        if ((uint64_t(e.w[0]) | (uint64_t(e.w[1]) << 32)) == p0 && (uint64_t(e.w[2]) | (uint64_t(e.w[3]) << 32)) == p1)
+            return link;
+        h = (h + 1) & ix.skip_mask;
+    }
+}
+
 template <class Key, int POL, bool TRACK = false>
 __device__ __forceinline__ uint64_t start_link(const DevIndex& ix, const Loader<POL>& ld, const Key& key,
                                                uint64_t* slot = nullptr) {
+    if constexpr (Key::kKind == 3 && !TRACK) {
+        if (ix.skip && key.len() >= ix.skip_d) return skip_start(ix, ld, key);
+    }
     if (TRACK) *slot = 0;
     if (ix.lut_bytes && key.len() >= ix.lut_bytes) {
         const uint64_t p = key.prefix(ix.lut_bytes);
