@@ -173,18 +173,21 @@ __global__ void __launch_bounds__(TPB, MINB) k_lookup_wt(DevIndex ix, const void
     constexpr uint32_t KS = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
     constexpr uint32_t A = run_align_keys<KS>();
     constexpr uint32_t TS = tile_stride<KS>();
-    __shared__ uint32_t pre[33];                       // run start in the concatenation; pre[32]: sentinel
-    __shared__ uint2 de[32];                           // {slot - position, end of the live part of the run}
+    // up to kTgMax tiles per CTA; the first two warps scan their run lengths
+    constexpr uint32_t kTgMax = 64;
+    static_assert(TPB >= kTgMax, "two warps build the run table");
+    __shared__ uint32_t pre[kTgMax + 1];               // run start in the concatenation; pre[tg..]: sentinel
+    __shared__ uint2 de[kTgMax];                       // {slot - position, end of the live part of the run}
+    __shared__ uint32_t wtot[2];
     __shared__ uint32_t total;
     const uint32_t b = blockIdx.x / ngroups, g = blockIdx.x - b * ngroups;
     const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
-    const uint64_t gbase = uint64_t(g) * tg * TS;      // first slot of the group (tg * TS < 2^18)
-    if (threadIdx.x < 32) {
-        const uint32_t lane = threadIdx.x;
-        const uint64_t t = uint64_t(g) * tg + lane;
-        uint32_t e = 0;
-        const bool valid = lane < tg && t < tiles;
-        if (valid) e = toff[tidx(b, t, nb)];
+    const uint64_t gbase = uint64_t(g) * tg * TS;      // first slot of the group (tg * TS < 2^19)
+    const uint32_t i = threadIdx.x;
+    const bool valid = i < tg && uint64_t(g) * tg + i < tiles;
+    if (i < kTgMax) {
+        const uint32_t lane = i & 31;
+        const uint32_t e = valid ? toff[tidx(b, uint64_t(g) * tg + i, nb)] : 0u;
         const uint32_t len = e >> 16, plen = (len + A - 1) & ~(A - 1);
         uint32_t x = plen;
 #pragma unroll
@@ -192,12 +195,19 @@ __global__ void __launch_bounds__(TPB, MINB) k_lookup_wt(DevIndex ix, const void
             const uint32_t y = __shfl_up_sync(0xffffffffu, x, d);
             if (lane >= uint32_t(d)) x += y;
         }
-        const uint32_t p_run = x - plen;
-        pre[lane] = valid ? p_run : 0xFFFFFFFFu;        // invalid lanes are never selected
-        de[lane] = make_uint2(lane * TS + (e & 0xFFFFu) - p_run, p_run + len);
-        if (lane == 31) {
-            total = x;
-            pre[32] = 0xFFFFFFFFu;
+        if (lane == 31) wtot[i >> 5] = x;
+        pre[i] = x - plen;                             // exclusive within the warp (fixed up below)
+        de[i] = make_uint2(i * TS + (e & 0xFFFFu), len);
+    }
+    __syncthreads();
+    if (i < kTgMax) {
+        const uint32_t p_run = pre[i] + (i >= 32 ? wtot[0] : 0u);
+        const uint2 r = de[i];
+        pre[i] = valid ? p_run : 0xFFFFFFFFu;           // invalid lanes are never selected
+        de[i] = make_uint2(r.x - p_run, p_run + r.y);
+        if (i == 0) {
+            total = wtot[0] + wtot[1];
+            pre[kTgMax] = 0xFFFFFFFFu;
         }
     }
     __syncthreads();
@@ -611,7 +621,7 @@ static cuart_status launch_tiled(const cuart_index* h, const void* q, const uint
     // c3 walk per 2^30: 12.3 / 10.8 / 9.7 / 9.4 ms at 4 / 8 / 16 / 32 tiles (the
     // table prologue is paid per CTA)
     uint32_t tg = uint32_t((2048 * uint64_t(nb)) / kBucketTile);
-    tg = tg < 1 ? 1 : tg > 32 ? 32 : tg;
+    tg = tg < 1 ? 1 : tg > 64 ? 64 : tg;
     if (h->tile_group) tg = h->tile_group;
     const uint32_t ngroups = uint32_t((tiles + tg - 1) / tg);
     const DevIndex& dx = h->dix_links;
@@ -1281,7 +1291,7 @@ cuart_status cuart_upload(const cuart_layout* lay, const cuart_build_opts* opts,
         if (const char* pe = getenv("CUART_TSORT_B1K")) h->tsort_b1k = uint32_t(atoi(pe));
         if (const char* pe = getenv("CUART_TILE_GROUP")) {
             const int v = atoi(pe);
-            h->tile_group = v < 1 ? 1u : v > 32 ? 32u : uint32_t(v);
+            h->tile_group = v < 1 ? 1u : v > 64 ? 64u : uint32_t(v);
         }
         if (const char* pe = getenv("CUART_BUCKET_FORM")) h->bucket_form = atoi(pe) == 1 ? CUART_BUCKET_GLOBAL : CUART_BUCKET_TILE;
     }

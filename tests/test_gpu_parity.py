@@ -263,14 +263,14 @@ def test_host_pipeline_many_chunks(kind, monkeypatch):
     ix.close()
 
 
-@pytest.mark.parametrize("form,tg", [("tile", None), ("tile", "1"), ("tile", "32"), ("global", None)])
+@pytest.mark.parametrize("form,tg", [("tile", None), ("tile", "1"), ("tile", "33"), ("tile", "64"), ("global", None)])
 @pytest.mark.parametrize("shift", ["0", "2", "3"])
 def test_prebucket_bucket_counts_and_skew(shift, form, tg, monkeypatch):
     """K-BUCKET with 256 / 64 / 32 buckets (CUART_BUCKET_SHIFT, read at upload) on
     skewed batches: every query in one bucket, queries in two buckets, and a ragged
     uniform batch; lookups and a bucketed update batch must equal the plain map.
     Both batch forms; the tile form also with 1 and 32 tiles per walk CTA
-    (CUART_TILE_GROUP), i.e. the smallest and the largest run prefix."""
+    (CUART_TILE_GROUP) and 33 / 64 (the run table spans both scanning warps)."""
     monkeypatch.setenv("CUART_BUCKET_SHIFT", shift)
     if tg:
         monkeypatch.setenv("CUART_TILE_GROUP", tg)
