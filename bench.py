@@ -175,6 +175,31 @@ def oracle_timing(cfg, keys, vals, n_lookup_sample, n_update_sample, allcore_fac
                    "allcore_sample_lookups": qa_len(qa), "host_cores": len(cores)}
 
 
+def layout_engine_timing(cfg, keys, layout, n1, det, allcore_factor=8):
+    """§8 f3 (§4.2, Fig. 7): the paper's CPU lookup engine over the flat CuART
+    layout (cuart_layout_lookup, product code; OpenMP) on the same query samples as
+    the oracle's 1-core and all-core lookups, so the two CPU rates compare the flat
+    type-segregated layout against the pointer ART on this host."""
+    cores = sorted(os.sched_getaffinity(0))
+    q1 = host_lookups(cfg, keys, 0, n1)
+    os.sched_setaffinity(0, {cores[0]})
+    try:
+        t0 = time.perf_counter()
+        layout.lookup(q1, threads=1)
+        t1 = time.perf_counter() - t0
+    finally:
+        os.sched_setaffinity(0, set(cores))
+    qa = host_lookups(cfg, keys, n1, n1 * allcore_factor)
+    t0 = time.perf_counter()
+    layout.lookup(qa, threads=len(cores))
+    ta = time.perf_counter() - t0
+    r1, ra = n1 / t1 / 1e6, qa_len(qa) / ta / 1e6
+    return {"kind": "cuart_layout_lookup (flat layout, CPU)", "lookup_mops_1core": round(r1, 3),
+            "lookup_mops_allcores": round(ra, 3), "threads": len(cores),
+            "vs_oracle_1core": round(r1 / det["oracle_lookup_mops_1core"], 3),
+            "vs_oracle_allcores": round(ra / det["oracle_lookup_mops_allcores"], 3)}
+
+
 def qa_len(q):
     return q[1].shape[0] if isinstance(q, tuple) else q.shape[0]
 
@@ -657,6 +682,8 @@ def main():
                          f"{det['allcore_sample_lookups']} further lookups over {det['host_cores']} threads",
                **{k: det[k] for k in ("oracle_lookup_mops_1core", "oracle_update_mops_1core",
                                       "oracle_lookup_mops_allcores", "host_cores")}}
+        if layout is not None:
+            cpu["f3_layout_engine"] = layout_engine_timing(cfg, keys, layout, nls, det)
 
     if rank == 0:
         line = {
