@@ -516,7 +516,8 @@ def main():
     wq = bucketed and bool(stats.get("wide_lut", 0)) and os.environ.get("CUART_ILP", "2") != "1"
     # sectors of the path the walk kernel takes: the pre-bucketed walk starts from the
     # wide root table when the index has one (stats["wide_lut"]), else the plain path
-    sec = layout.sectors(samp, wide=bool(bucketed and stats.get("wide_lut", 0))).astype(np.float64)
+    sec = layout.sectors(samp, wide=bool(bucketed and stats.get("wide_lut", 0)),
+                         skip_prefix=int(stats.get("skip_prefix", 0))).astype(np.float64)
     io_bytes = {"u64": 8, "u32": 4, "bytes": 33}[cfg.kind] + 8
     random_bytes_per_lookup = 32.0 * sec.mean() + io_bytes
     # tile form of K-BUCKET (cuart_build_opts.bucket_form, default): single-index integer

@@ -284,8 +284,12 @@ cuart_status cuart_layout_lookup(const cuart_layout* l, const cuart_keys* querie
 cuart_status cuart_layout_sectors(const cuart_layout* l, const cuart_keys* queries, size_t n,
                                   uint32_t* sectors, int threads);
 /* As cuart_layout_sectors for the walk of a given variant: flags CUART_SECTORS_WIDE =
- * the pre-bucketed walk starting from the wide root table (cuart_build_opts.wide_lut). */
+ * the pre-bucketed walk starting from the wide root table (cuart_build_opts.wide_lut);
+ * CUART_SECTORS_SKIP(D) = byte-string walks starting from a skip table over D-byte
+ * prefixes (one 32-B probe, then the walk below the covering node; cuart_stats
+ * skip_prefix gives D). */
 #define CUART_SECTORS_WIDE 1u
+#define CUART_SECTORS_SKIP(d) ((uint32_t)(d) << 8)
 cuart_status cuart_layout_sectors_ex(const cuart_layout* l, const cuart_keys* queries, size_t n,
                                      uint32_t* sectors, int threads, uint32_t flags);
 cuart_status cuart_upload(const cuart_layout* l, const cuart_build_opts* opts, cuart_index** out);

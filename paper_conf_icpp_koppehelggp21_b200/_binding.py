@@ -375,10 +375,11 @@ def cuart_layout_lookup(l, queries, threads=0):
     return out
 
 
-def cuart_layout_sectors(l, queries, threads=0, wide=False):
+def cuart_layout_sectors(l, queries, threads=0, wide=False, skip_prefix=0):
     q, n, keep = make_keys(queries)
     out = np.empty(n, dtype=np.uint32)
-    _check(lib().cuart_layout_sectors_ex(l, ctypes.byref(q), n, _ptr(out), threads, 1 if wide else 0),
+    flags = (1 if wide else 0) | ((int(skip_prefix) & 0xFF) << 8)
+    _check(lib().cuart_layout_sectors_ex(l, ctypes.byref(q), n, _ptr(out), threads, flags),
            "cuart_layout_sectors_ex")
     return out
 
@@ -411,8 +412,8 @@ class Layout:
     def view(self):
         return cuart_layout_view_get(self.h)
 
-    def sectors(self, queries, threads=0, wide=False):
-        return cuart_layout_sectors(self.h, queries, threads, wide)
+    def sectors(self, queries, threads=0, wide=False, skip_prefix=0):
+        return cuart_layout_sectors(self.h, queries, threads, wide, skip_prefix)
 
     def close(self):
         cuart_layout_free(self.h)

@@ -404,12 +404,47 @@ inline uint32_t sectors(uint64_t off, uint32_t bytes) { return uint32_t((off + b
 // 64-B record; leaves 16 / 32 / 48 B.
 // wide: the walk starts from the 32-B wide root-table entry (link + the target
 // N4/N16's keys, kernels.cuh start_wide) and reads that node's child link directly.
-uint64_t walk_one(const HostLayout& L, const uint8_t* key, uint32_t len, uint32_t* sec = nullptr, bool wide = false) {
+uint64_t walk_one(const HostLayout& L, const uint8_t* key, uint32_t len, uint32_t* sec = nullptr, bool wide = false,
+                  uint32_t skip_d = 0) {
     if (len == 0 || len > kMaxKey) return kMiss;
     uint32_t s = 0;
     uint64_t link = L.root;
     struct Guard { uint32_t* dst; uint32_t* s; ~Guard() { if (dst) *dst = *s; } } guard{sec, &s};
-    if (L.lut_bytes && len >= L.lut_bytes) {
+    if (skip_d && len >= skip_d && L.key_kind == CUART_KEY_BYTES) {
+        // the device's skip table (capi.cu build_skip_table): one 32-B probe yields the
+        // node covering the query's first skip_d bytes; the levels above it are not read
+        s += 1;
+        if (L.lut_bytes && skip_d >= L.lut_bytes) {
+            uint64_t p = 0;
+            for (uint32_t b = 0; b < L.lut_bytes; b++) p = (p << 8) | key[b];
+            link = L.lut[p];
+        }
+        for (;;) {
+            const uint32_t t = link_type(link);
+            if (t == T_NULL) return kMiss;
+            if (t >= T_LEAF8 || link_aux(link) >= skip_d) break;
+            const uint8_t* rec = L.buf[t].data() + link_index(link) * kRecordBytes[t];
+            const uint8_t b = key[link_aux(link)];
+            uint64_t child = 0;
+            if (t == T_N256) memcpy(&child, rec + kN256Child + 8 * b, 8);
+            else if (t == T_N48) {
+                if (rec[kN48Index + b] == kN48Empty) return kMiss;
+                memcpy(&child, rec + kN48Child + 8 * rec[kN48Index + b], 8);
+            } else {
+                const uint8_t* keys = rec + (t == T_N4 ? kN4Keys : kN16Keys);
+                const uint32_t nk = t == T_N4 ? 4 : 16;
+                uint32_t c = nk;
+                for (uint32_t j = 0; j < nk; j++)
+                    if (keys[j] == b) {
+                        c = j;
+                        break;
+                    }
+                if (c == nk) return kMiss;
+                memcpy(&child, rec + (t == T_N4 ? kN4Child : kN16Child) + 8 * c, 8);
+            }
+            link = child;
+        }
+    } else if (L.lut_bytes && len >= L.lut_bytes) {
         uint64_t p = 0;
         for (uint32_t b = 0; b < L.lut_bytes; b++) p = (p << 8) | key[b];
         link = L.lut[p];
@@ -477,7 +512,7 @@ uint64_t walk_one(const HostLayout& L, const uint8_t* key, uint32_t len, uint32_
 }  // namespace
 
 void host_layout_sectors(const HostLayout& L, uint32_t kind, const void* queries, const uint8_t* lengths, uint64_t n,
-                         uint32_t* sec, int threads, bool wide) {
+                         uint32_t* sec, int threads, bool wide, uint32_t skip_d) {
     QView q{kind, queries, lengths};
     if (threads <= 0) threads = omp_get_max_threads();
 #pragma omp parallel for schedule(static) num_threads(threads)
@@ -485,7 +520,7 @@ void host_layout_sectors(const HostLayout& L, uint32_t kind, const void* queries
         uint8_t key[kMaxKey];
         q.bytes(i, key);
         sec[i] = 0;
-        walk_one(L, key, q.len(i), &sec[i], wide);
+        walk_one(L, key, q.len(i), &sec[i], wide, skip_d);
     }
 }
 

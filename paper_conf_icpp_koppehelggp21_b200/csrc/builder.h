@@ -39,6 +39,6 @@ void host_layout_lookup(const HostLayout& L, uint32_t kind, const void* queries,
 
 // Per-query count of the 32-byte sectors the GPU lookup reads (algorithmic bytes).
 void host_layout_sectors(const HostLayout& L, uint32_t kind, const void* queries, const uint8_t* lengths,
-                         uint64_t n, uint32_t* sectors, int threads, bool wide = false);
+                         uint64_t n, uint32_t* sectors, int threads, bool wide = false, uint32_t skip_d = 0);
 
 }  // namespace cuart

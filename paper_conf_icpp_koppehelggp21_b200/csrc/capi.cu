@@ -1021,7 +1021,7 @@ cuart_status cuart_layout_sectors_ex(const cuart_layout* l, const cuart_keys* q,
     if (q->kind == CUART_KEY_BYTES && n > 0 && !q->lengths) return CUART_ERR_INVALID_ARGUMENT;
     if (uint32_t(q->kind) != l->L.key_kind) return CUART_ERR_INVALID_ARGUMENT;
     host_layout_sectors(l->L, l->L.key_kind, q->data, q->lengths, n, sectors, threads,
-                        (flags & CUART_SECTORS_WIDE) && !l->L.lut.empty());
+                        (flags & CUART_SECTORS_WIDE) && !l->L.lut.empty(), (flags >> 8) & 0xFFu);
     return CUART_OK;
 }
 

@@ -287,3 +287,33 @@ def test_sector_walker_wide_root_table():
     assert lay.sectors(q).tolist() == [3, 1, 3]
     assert lay.sectors(q, wide=True).tolist() == [2, 1, 2]
     lay.close()
+
+
+def test_sector_walker_skip_table_path():
+    """cuart_layout_sectors_ex(SKIP(D)) counts the byte-string walk that starts from
+    the skip table: one 32-B probe, then only the levels below the node covering the
+    query's first D bytes.  Hand case: keys "aaaaaaa" + x + "b" (x in 0..4, length 9)
+    and "zz" (length 2): the root N4 branches at byte 0; under "a" an N16 (5 children)
+    branches at depth 7 over leaf16 records.  Plain walk = root N4 (1 sector) + N16 keys
+    and child (2) + leaf16 (1) = 4; skip D = 8: probe (1) + leaf (1) = 2; D = 4: probe +
+    N16 (2) + leaf = 4 (the N16 branches at depth 7 >= 4, so it covers "aaaa"); a query
+    shorter than D takes the plain walk (zz: root N4 + leaf8 = 2); "aaaabbbbb" has the
+    prefix but misses at the N16's keys (probe + 1 = 2); "qqqqq" has no 4-byte prefix in
+    the tree and stops at the probe (1)."""
+    names = [b"aaaaaaa" + bytes([0x30 + x]) + b"b" for x in range(5)] + [b"zz"]
+    slots = np.zeros((len(names), 32), np.uint8)
+    for i, s in enumerate(names):
+        slots[i, :len(s)] = np.frombuffer(s, np.uint8)
+    lens = np.array([len(s) for s in names], np.uint8)
+    lay = C.Layout((slots, lens), np.arange(len(names), dtype=np.uint64) + 1, lut_bytes=0)
+    q_names = [names[2], b"zz", b"aaaabbbbb", b"qqqqq"]
+    qs = np.zeros((4, 32), np.uint8)
+    for i, s in enumerate(q_names):
+        qs[i, :len(s)] = np.frombuffer(s, np.uint8)
+    ql = np.array([len(s) for s in q_names], np.uint8)
+    assert lay.lookup((qs, ql)).tolist()[:2] == [3, 6]
+    plain = lay.sectors((qs, ql)).tolist()
+    assert plain[:2] == [4, 2]
+    assert lay.sectors((qs, ql), skip_prefix=8).tolist()[:2] == [2, 2]
+    assert lay.sectors((qs, ql), skip_prefix=4).tolist() == [4, 2, 2, 1]
+    lay.close()
