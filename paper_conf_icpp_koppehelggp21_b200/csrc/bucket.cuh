@@ -590,6 +590,10 @@ __host__ __device__ constexpr uint32_t run_align_keys() { return kRunAlign / KS;
 // slots per tile region: 4096 keys + at most (A - 1) padding slots per bucket
 template <uint32_t KS>
 __host__ __device__ constexpr uint32_t tile_stride() { return uint32_t(kBucketTile) + kBuckets * (run_align_keys<KS>() - 1); }
+// the stride a batch with nb buckets needs (scratch is sized by it; kernels keep the
+// 256-bucket maximum for their shared-memory staging)
+template <uint32_t KS>
+__host__ __device__ constexpr uint32_t tile_stride_rt(uint32_t nb) { return uint32_t(kBucketTile) + nb * (run_align_keys<KS>() - 1); }
 // run table: [group of 8 tiles][bucket < nb][tile in group], u32 start | len << 16
 __device__ __forceinline__ uint64_t tidx(uint32_t b, uint64_t t, uint32_t nb) {
     return ((t / kHistGroup) * nb + b) * kHistGroup + (t % kHistGroup);
@@ -712,7 +716,8 @@ __global__ void __launch_bounds__(kBucketThreads, VEC ? 4 : 1) k_tsort(const voi
     // the sorted, padded tile -> tq in 16-B stores (every run and the region are
     // 32-B aligned; padding slots carry stale shared memory, never read as keys)
     const uint32_t nv = ptot * KS / 16;
-    uint4* dst = (uint4*)((uint8_t*)tq + uint64_t(blockIdx.x) * TS * KS);
+    const uint32_t ts = tile_stride_rt<KS>(nb);                        // this batch's tile stride
+    uint4* dst = (uint4*)((uint8_t*)tq + uint64_t(blockIdx.x) * ts * KS);
 #pragma unroll 4
     for (uint32_t v = threadIdx.x; v < nv; v += kBucketThreads) __stcs(dst + v, ((const uint4*)skeys)[v]);
 }
@@ -881,7 +886,7 @@ __global__ void __launch_bounds__(kBucketThreads) k_tgather(const uint64_t* __re
     }
     const uint32_t e = toff[tidx(nb - 1, blockIdx.x, nb)];             // last run: start | len << 16
     const uint32_t ptot = (e & 0xFFFFu) + (((e >> 16) + A - 1) & ~(A - 1));
-    const uint64_t* src = tres + uint64_t(blockIdx.x) * TS;
+    const uint64_t* src = tres + uint64_t(blockIdx.x) * tile_stride_rt<KS>(nb);
     const uint32_t nv = (ptot + 1) / 2;                                 // ptot is a multiple of A (even)
 #pragma unroll 4
     for (uint32_t v = threadIdx.x; v < nv; v += kBucketThreads) cp_async16(&sres[2 * v], src + 2 * v);

@@ -182,7 +182,8 @@ __global__ void __launch_bounds__(TPB, MINB) k_lookup_wt(DevIndex ix, const void
     __shared__ uint32_t total;
     const uint32_t b = blockIdx.x / ngroups, g = blockIdx.x - b * ngroups;
     const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
-    const uint64_t gbase = uint64_t(g) * tg * TS;      // first slot of the group (tg * TS < 2^19)
+    const uint32_t ts = tile_stride_rt<KS>(nb);       // tile stride of this batch (<= TS)
+    const uint64_t gbase = uint64_t(g) * tg * ts;      // first slot of the group (tg * ts < 2^19)
     const uint32_t i = threadIdx.x;
     const bool valid = i < tg && uint64_t(g) * tg + i < tiles;
     if (i < kTgMax) {
@@ -197,7 +198,7 @@ __global__ void __launch_bounds__(TPB, MINB) k_lookup_wt(DevIndex ix, const void
         }
         if (lane == 31) wtot[i >> 5] = x;
         pre[i] = x - plen;                             // exclusive within the warp (fixed up below)
-        de[i] = make_uint2(i * TS + (e & 0xFFFFu), len);
+        de[i] = make_uint2(i * ts + (e & 0xFFFFu), len);
     }
     __syncthreads();
     if (i < kTgMax) {
@@ -584,10 +585,10 @@ template <class Key>
 static cuart_status launch_tiled(const cuart_index* h, const void* q, const uint8_t* lens, uint64_t n, uint64_t* out,
                                  cudaStream_t s) {
     constexpr uint32_t KS = Key::kKind == 2 ? 8 : Key::kKind == 1 ? 4 : 32;
-    constexpr uint32_t TS = tile_stride<KS>();
     auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
     const uint64_t tiles = (n + kBucketTile - 1) / kBucketTile;
     const uint32_t nb = kBuckets >> h->bucket_shift;
+    const uint64_t TS = tile_stride_rt<KS>(nb);       // c3 (64 buckets): 4288 slots per 4096-query tile
     const size_t o_off = 0, o_q = al(tidx_entries(tiles, nb) * 4), o_len = o_q + al(tiles * TS * KS),
                  o_pos = o_len + al(Key::kKind == 3 ? tiles * TS : 0), o_res = o_pos + al(n * 2),
                  total = o_res + al(tiles * TS * 8);
