@@ -103,7 +103,8 @@ typedef struct {
                                     >= 2^22 ops, lookups and plain updates),
                                     CUART_PREBUCKET_OFF, CUART_PREBUCKET_ON.  Results are
                                     identical; it reorders the batch so concurrent warps
-                                    share subtrees (stream-ordered scratch ~18 B/query). */
+                                    share subtrees (stream-ordered scratch from the index's pool: ~19 B per u64
+                                    query in the tile form, ~18 B in the global form). */
     uint32_t slice_lut;          /* pre-bucketed lookups with a RANK root table: every
                                     CTA walks its share of each bucket with the bucket's slice
                                     of the table staged in shared memory (64 KiB at k=3),
